@@ -1,0 +1,181 @@
+/*
+ * ns.h -- C ABI of libneuroscaler.so: the data-parallel enhancement hot path of
+ * NeuroScaler (SIGCOMM '22), B200-native (sm_100a).
+ *
+ * "NeuroScaler takes an ingest stream and a DNN pair and outputs a
+ *  high-resolution stream" (§4).  Per stream and per chunk the
+ * library (1) scores frames from codec metadata and selects anchor frames
+ * without inference (§5.1, Alg. 1), (2) runs the
+ * stream's content-aware SR DNN on the anchors only (§6.2), and (3)
+ * rebuilds every other frame by reusing cached SR frames guided by reference
+ * index, motion vector and residual (§2, §6.1).  Many streams
+ * are batched per call, so one kernel serves many streams without GPU
+ * context switches (§6.2).
+ *
+ * Conventions (all calls):
+ *  - Every pointer inside ns_chunk / ns_sr_job and every output array is a
+ *    DEVICE pointer owned by the caller, unless a comment says "host".
+ *  - Every call is asynchronous on `stream` (a cudaStream_t; NULL = legacy
+ *    default stream).  The library performs no host synchronisation on the
+ *    hot path and no device allocation after ns_ctx_create (memory
+ *    pre-allocation, App. A): working memory is carved
+ *    from the context pool.
+ *  - Arguments are validated on the host before anything is enqueued; on any
+ *    error nothing is launched, the call returns a negative ns_status and
+ *    ns_last_error() describes the problem.
+ *  - A context is bound to one device and is not thread-safe; use one context
+ *    per device per host thread.
+ *
+ * Data layout:
+ *  - LR frames u8, 3 full-resolution planes [n][3][h][w]; residual int16
+ *    [n][3][h][w] with values in [-255, 255]; HR frames u8 [3][s*h][s*w].
+ *  - Motion: one ns_block_mv per 8x8 LR block, [n][h/8][w/8], MVs in 1/8 LR
+ *    pel, pred(x) = ref(x + mv) (reading Z14).
+ */
+#ifndef NEUROSCALER_NS_H
+#define NEUROSCALER_NS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define NS_API __attribute__((visibility("default")))
+#else
+#define NS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    NS_OK = 0,
+    NS_EINVAL = -1,        /* invalid argument (see ns_last_error)              */
+    NS_ECUDA = -2,         /* a CUDA runtime error; message includes its string */
+    NS_ENOMEM = -3,        /* the context pool is too small for the request     */
+    NS_EUNSUPPORTED = -4   /* device is not sm_100 / shape not supported        */
+} ns_status;
+
+/* Frame types exported by the decoder (G_key, G_altref, G_normal). */
+typedef enum { NS_KEY = 0, NS_ALTREF = 1, NS_NORMAL = 2 } ns_frame_type;
+
+/* Reference index of a block ("reference index"). */
+typedef enum { NS_REF_LAST = 0, NS_REF_GOLDEN = 1, NS_REF_INTRA = 2 } ns_ref;
+
+/* One 8x8 LR block's motion vector (1/8 LR pel) and reference. 8 bytes. */
+typedef struct {
+    int16_t mvx, mvy;
+    uint8_t ref;        /* ns_ref */
+    uint8_t pad[3];
+} ns_block_mv;
+
+typedef struct ns_ctx ns_ctx;
+typedef struct ns_model ns_model;
+
+/* One stream's chunk (= GOP of n_frames frames) as the decoder exports it
+   (frame type and residual; reference index, MV). */
+typedef struct {
+    int32_t w, h;              /* LR size; w % 8 == 0, h % 8 == 0, w,h >= 8         */
+    int32_t scale;             /* SR factor s in {2, 3, 4}; must equal model scale   */
+    int32_t n_frames;          /* 1 <= n <= 256                                      */
+    const uint8_t *lr;         /* [n][3][h][w] decoded LR frames                     */
+    const int16_t *res;        /* [n][3][h][w] decoded residual                      */
+    const ns_block_mv *mv;     /* [n][h/8][w/8]                                      */
+    const uint8_t *type;       /* [n] ns_frame_type                                  */
+    const uint32_t *res_size;  /* [n] optional encoded-size proxy or NULL    */
+    const ns_model *model;     /* this stream's content-aware DNN             */
+    uint8_t *hr_last;          /* [3][s*h][s*w] LAST reference entering the chunk;
+                                  overwritten with HR[n-1] at chunk end. May be NULL
+                                  if no frame references LAST before a KEY frame.  */
+    uint8_t *hr_golden;        /* [3][s*h][s*w] GOLDEN reference entering the chunk;
+                                  overwritten with the chunk's last KEY/ALTREF HR.
+                                  May be NULL under the same condition.            */
+    const uint8_t *gt;         /* optional [n][3][s*h][s*w] ground truth for stats   */
+} ns_chunk;
+
+/* Anchor selection mode (§5.1 top-k per chunk; §5.2 global budget). */
+enum { NS_TOPK_PER_STREAM = 0, NS_GLOBAL_BUDGET = 1 };
+/* Residual carried from the G_altref pass into the G_normal pass (reading Z2,
+   default) or recomputed per group (literal Alg. 1 line 2). */
+enum { NS_CARRY = 0, NS_FRESH = 1 };
+
+typedef struct {
+    int32_t mode;              /* NS_TOPK_PER_STREAM | NS_GLOBAL_BUDGET              */
+    int32_t k;                 /* top-k mode: anchors per stream, 0 <= k <= n         */
+    int64_t budget;            /* global mode: T_intv * M in cost units       */
+    const int64_t *cost;       /* HOST [S]: T_DNN of one anchor of stream s, >= 1     */
+    int32_t group_residual;    /* NS_CARRY | NS_FRESH                                 */
+    int32_t use_res_size;      /* 1: score = res_size (P:191 proxy) when non-NULL     */
+} ns_select_params;
+
+/* One anchor-SR job: HR = SR_model(LR) (O5). */
+typedef struct {
+    const ns_model *model;
+    const uint8_t *lr;         /* [3][h][w] */
+    int32_t w, h;
+    uint8_t *hr_out;           /* [3][s*h][s*w] */
+} ns_sr_job;
+
+/* Creates a context on `device` with a device memory pool of pool_bytes
+   ("pre-allocates ... and construct a memory pool when a program
+   launches").  NS_EUNSUPPORTED if the device is not compute capability 10.0.
+   *out receives the context (host object). */
+NS_API ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out);
+NS_API ns_status ns_ctx_destroy(ns_ctx *ctx);
+
+/* Reserves a model slot (weights + packed kernel operands) from the pool.
+   n_blocks >= 1, n_ch in {16, 32}, scale in {2, 3, 4} (8 blocks, 32
+   channels, scale 3).  The kernels are shape-specialised on (n_ch, scale) at
+   build time; weights are runtime data ("model pre-optimization"). */
+NS_API ns_status ns_model_create(ns_ctx *ctx, int n_blocks, int n_ch, int scale, ns_model **out);
+
+/* Refits the model with a bf16 weight blob (uint16 bit patterns, DEVICE or
+   HOST pointer -- detected) of exactly ns_model_blob_len() entries, in the
+   order head, blocks x (conv1, conv2), end, up, tail; each [Cout][Cin][3][3]
+   followed by bias[Cout] (head Cin = 3, up Cout = s*s*C, tail Cout = 3).
+   Repacks into the kernels' operand layout on `stream`; no re-planning. */
+NS_API ns_status ns_model_set_weights(ns_model *m, const uint16_t *bf16_blob, size_t n, void *stream);
+NS_API size_t ns_model_blob_len(int n_blocks, int n_ch, int scale);
+NS_API ns_status ns_model_destroy(ns_model *m);
+
+/* Anchor scoring + zero-inference selection for S streams (§5.1).
+   chunks: HOST array [S]; all chunks must have the same n_frames.
+   Outputs (DEVICE, [S][n]): gain (KEY frames: INT64_MAX, "equal anchor gain"
+   P:170-176), rank (position in the per-stream priority order, or in the
+   global order in NS_GLOBAL_BUDGET mode), is_anchor (0/1). */
+NS_API ns_status ns_select_anchors(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
+                            int64_t *gain, int32_t *rank, uint8_t *is_anchor, void *stream);
+
+/* SR on a host-supplied job list (jobs: HOST array [n_jobs]).  Jobs may mix
+   models and resolutions; they are grouped by shape internally. */
+NS_API ns_status ns_sr_anchors(ns_ctx *ctx, const ns_sr_job *jobs, int n_jobs, void *stream);
+
+/* Reuse-based reconstruction of every non-anchor frame of S chunks (§2, §6.1).
+   is_anchor: DEVICE [S][n].  hr_out: HOST table [S*n] of DEVICE pointers, each
+   [3][s*h][s*w]; anchors' entries must already hold the SR output (e.g. from
+   ns_sr_anchors).  hr_out[s][f] must not alias hr_out[s][f-1], hr_last or
+   hr_golden of the same stream (checked) nor the frame serving as GOLDEN
+   (not checked).  Writes hr_last / hr_golden at chunk end. */
+NS_API ns_status ns_reconstruct_chunk(ns_ctx *ctx, const ns_chunk *chunks, int S, const uint8_t *is_anchor,
+                               uint8_t *const *hr_out, void *stream);
+
+/* The whole hot path for S streams: select -> SR on anchors (grouped across
+   streams) -> reconstruct.  hr_out: HOST table [S*n] of DEVICE pointers.
+   is_anchor_out (DEVICE [S][n]) may be NULL.  stats: DEVICE [S][8] fp64 or
+   NULL: {frames, anchors, sum anchor score, total score, SSE vs gt (or -1),
+   PSNR vs gt (or -1), 0, 0}. */
+NS_API ns_status ns_enhance_streams(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
+                             uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream);
+
+/* Number of this library's kernel launches enqueued by the calling thread
+   since the last reset (for the bench's gpu_launches claim). */
+NS_API uint64_t ns_launch_count(int reset);
+
+/* Thread-local description of the last error (includes cudaGetErrorString for
+   NS_ECUDA).  Never NULL. */
+NS_API const char *ns_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NEUROSCALER_NS_H */

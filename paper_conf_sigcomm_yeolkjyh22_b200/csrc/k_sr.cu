@@ -1,0 +1,455 @@
+// k_sr.cu -- anchor SR DNN (NAS "high" EDSR-style net, 8
+// residual blocks, 32 channels, x3) as implicit-GEMM 3x3 convolutions on the
+// 5th-generation tensor cores (tcgen05.mma, accumulators in TMEM), fed by TMA.
+//
+// Formulation: one UMMA M tile = 128 consecutive
+// output pixels of one row; N = output channels; K = 9 taps x Cin.  Input rows
+// live in shared memory as K-major "interleaved" core matrices
+// [Cin/8][130 px][8 ch] bf16 (exactly the TMA box of the activation layout
+// [job][H][C/8][W][8]); the 3x3 taps are pure descriptor offsets: tap (dy, dx)
+// reads ring slot (row y+dy-1) at start + dx*16 B, because consecutive pixels
+// are 16 B apart inside a channel group (SBO = 128 B per 8 rows).  No im2col,
+// zero padding comes from TMA out-of-bounds fill.  A CTA walks a strip of rows
+// with a 6-slot TMA ring, double-buffered TMEM accumulators, and a fused
+// epilogue (bias, ReLU, residual add, pixel shuffle, or the HR tail with the
+// integer bilinear skip, round and clamp to u8).
+#include <cuda_bf16.h>
+#include <cstdio>
+#include "ns_internal.h"
+#include "ptx.cuh"
+
+namespace ns {
+
+enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4 };
+constexpr int kSlots = 6;
+constexpr int kRows = 32;   // rows per CTA strip
+
+struct ConvArgs {
+    int H, W;               // conv spatial dims (input == output)
+    int n_xtiles, rows_per_cta;
+    int j0;                 // first job of the batch
+    const SrJob *jobs;
+    const int32_t *job_count;
+    size_t b_off, bias_off; // this launch's B operand / bias offsets in the packed model
+    uint16_t *out;          // bf16 activation out (EPI_STORE/RELU/RESID/SHUFFLE)
+    const uint16_t *resid;  // EPI_RESID
+    int C;                  // channels of the output activation (shuffle: per sub-pixel)
+    int s;                  // scale (shuffle / tail)
+    int sub0;               // shuffle: first sub-pixel of this launch
+    int lr_h, lr_w;         // tail: LR dims of the bilinear skip
+};
+
+__host__ __device__ constexpr uint32_t round_up(uint32_t v, uint32_t a) { return (v + a - 1) / a * a; }
+__host__ __device__ constexpr uint32_t tmem_cols_for(uint32_t c) {
+    return c <= 32 ? 32 : c <= 64 ? 64 : c <= 128 ? 128 : c <= 256 ? 256 : 512;
+}
+
+template <int CIN, int NT, int NSPLIT>
+struct ConvCfg {
+    static constexpr int NTOT = NT * NSPLIT;
+    static constexpr int KC = CIN / 16;
+    static constexpr uint32_t B_BYTES = 9u * CIN * NTOT * 2u;
+    static constexpr uint32_t BIAS_BYTES = NTOT * 4u;
+    static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
+    static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    static constexpr int ACCB = (NTOT <= 256) ? 2 : 1;
+    static constexpr uint32_t TMEM_COLS = tmem_cols_for(ACCB * NTOT);
+    static constexpr uint32_t SMEM = W_REGION + kSlots * SLOT + 128;
+    static_assert(NT % 16 == 0 && NT >= 16 && NT <= 256, "UMMA M=128 needs N % 16 == 0, 16..256");
+    static_assert(CIN % 16 == 0, "Cin multiple of 16");
+    static_assert(SMEM <= 232448, "shared memory");
+};
+
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+    __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
+    return *reinterpret_cast<uint32_t *>(&v);
+}
+__device__ __forceinline__ float bf_lo(uint32_t u) { return __uint_as_float(u << 16); }
+__device__ __forceinline__ float bf_hi(uint32_t u) { return __uint_as_float(u & 0xFFFF0000u); }
+
+// O6 tap of the fixed-point bilinear upsample (half-pixel centres, Q7).
+__device__ __forceinline__ void up_tap(int X, int s, int len, int &i0, int &i1, int &w1) {
+    int u = 2 * X + 1 - s;
+    int x0 = (u >= 0) ? u / (2 * s) : -((-u + 2 * s - 1) / (2 * s));
+    int rem = u - 2 * s * x0;
+    w1 = (128 * rem + s) / (2 * s);
+    i0 = min(max(x0, 0), len - 1);
+    i1 = min(max(x0 + 1, 0), len - 1);
+}
+
+template <int CIN, int NT, int NSPLIT, int EPI>
+__global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+    using Cfg = ConvCfg<CIN, NT, NSPLIT>;
+    constexpr int NTOT = Cfg::NTOT;
+    constexpr int ACCB = Cfg::ACCB;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *s_w = smem;
+    const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
+    uint8_t *s_ring = smem + Cfg::W_REGION;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + kSlots * Cfg::SLOT);  // [0,6) ring, 6 w, 7-8 mma
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 10);
+
+    const int slot_job = blockIdx.z;
+    const int job = a.j0 + slot_job;
+    if (a.job_count && job >= *a.job_count) return;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int x0 = blockIdx.x * kTile;
+    const int y0 = blockIdx.y * a.rows_per_cta;
+    const int y1 = min(y0 + a.rows_per_cta, a.H);
+    const int nrows = y1 - y0;
+    const int n_loads = nrows + 2;  // rows y0-1 .. y1
+
+    if (tid == 0) {
+        for (int i = 0; i < 9; i++) mbar_init(&bars[i], 1);
+        fence_mbar_init();
+    }
+    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *s_tmem;
+    const SrJob J = a.jobs[job];
+
+    if (tid == 0) {
+        prefetch_tmap(&tm_in);
+        mbar_arrive_expect_tx(&bars[6], Cfg::B_BYTES + Cfg::BIAS_BYTES);
+        bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[6]);
+        bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[6]);
+        for (int q = 0; q < 4 && q < n_loads; q++) {
+            mbar_arrive_expect_tx(&bars[q % kSlots], Cfg::SLOT_BYTES);
+            tma_load_5d(s_ring + (q % kSlots) * Cfg::SLOT, &tm_in, &bars[q % kSlots], 0, x0 - 1, 0, y0 - 1 + q,
+                        slot_job);
+        }
+    }
+
+    const uint32_t idesc = idesc_bf16_f32(128, NT);
+    auto issue = [&](int r) {  // MMAs of output row y0 + r (thread 0 only)
+        for (int d = 0; d < 3; d++) {
+            const int q = r + d;
+            mbar_wait(&bars[q % kSlots], (q / kSlots) & 1);
+        }
+        tc_fence_after();
+        const uint32_t acc = tmem + (uint32_t)((r % ACCB) * NTOT);
+        const uint32_t wbase = smem_u32(s_w);
+#pragma unroll
+        for (int sp = 0; sp < NSPLIT; sp++) {
+#pragma unroll
+            for (int tap = 0; tap < 9; tap++) {
+                const int dy = tap / 3, dx = tap % 3;
+                const uint32_t abase = smem_u32(s_ring + ((r + dy) % kSlots) * Cfg::SLOT);
+#pragma unroll
+                for (int kc = 0; kc < Cfg::KC; kc++) {
+                    const uint64_t ad = smem_desc(abase + (uint32_t)(2 * kc * kHalo * 16 + dx * 16), kHalo * 16, 128);
+                    const uint64_t bd =
+                        smem_desc(wbase + (uint32_t)(((sp * 9 + tap) * Cfg::KC + kc) * 2 * NT * 16), NT * 16, 128);
+                    umma_bf16(acc + sp * NT, ad, bd, idesc, (tap | kc) != 0 ? 1u : 0u);
+                }
+            }
+        }
+        umma_commit(&bars[7 + (r % ACCB)]);
+    };
+
+    mbar_wait(&bars[6], 0);  // weights + bias resident (all threads: epilogue reads the bias)
+    if (tid == 0 && ACCB == 2) issue(0);
+
+    const int p = warp * 32 + lane;  // TMEM lane == pixel of the tile
+    const int x = x0 + p;
+    for (int r = 0; r < nrows; r++) {
+        if (tid == 0) {
+            const int q = r + 4;  // prefetch row y0 + r + 3 into the slot freed by MMA(r - 2)
+            if (q < n_loads) {
+                mbar_arrive_expect_tx(&bars[q % kSlots], Cfg::SLOT_BYTES);
+                tma_load_5d(s_ring + (q % kSlots) * Cfg::SLOT, &tm_in, &bars[q % kSlots], 0, x0 - 1, 0,
+                            y0 - 1 + q, slot_job);
+            }
+            if (ACCB == 1) issue(r);
+            else if (r + 1 < nrows) issue(r + 1);
+        }
+        __syncwarp();
+        mbar_wait(&bars[7 + (r % ACCB)], (r / ACCB) & 1);
+        tc_fence_after();
+        const uint32_t acc = tmem + (uint32_t)((r % ACCB) * NTOT) + ((uint32_t)(warp * 32) << 16);
+        const int y = y0 + r;
+
+        if constexpr (EPI == EPI_STORE || EPI == EPI_RELU || EPI == EPI_RESID) {
+            static_assert(NSPLIT == 1, "");
+            constexpr int C = NT;
+            uint32_t v[C];
+            if constexpr (C == 32) {
+                uint32_t (&vv)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
+                tmem_ld32(acc, vv);
+            } else {
+                uint32_t (&vv)[16] = *reinterpret_cast<uint32_t(*)[16]>(v);
+                tmem_ld16(acc, vv);
+            }
+            tmem_wait_ld();
+            if (x < a.W) {
+                const size_t rowbase = ((size_t)slot_job * a.H + y) * (C / 8);
+#pragma unroll
+                for (int cg = 0; cg < C / 8; cg++) {
+                    float f[8];
+#pragma unroll
+                    for (int i = 0; i < 8; i++) {
+                        f[i] = __uint_as_float(v[cg * 8 + i]) + s_bias[cg * 8 + i];
+                        if (EPI == EPI_RELU) f[i] = fmaxf(f[i], 0.f);
+                    }
+                    const size_t off = ((rowbase + cg) * a.W + x) * 8;
+                    if (EPI == EPI_RESID) {
+                        const uint4 rr = *reinterpret_cast<const uint4 *>(a.resid + off);
+                        f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
+                        f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
+                        f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
+                        f[6] += bf_lo(rr.w); f[7] += bf_hi(rr.w);
+                    }
+                    uint4 o;
+                    o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
+                    o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
+                    *reinterpret_cast<uint4 *>(a.out + off) = o;
+                }
+            }
+        } else if constexpr (EPI == EPI_SHUFFLE) {
+            // D column n' = (i*s + j) * C + c  <->  upsampler channel c*s*s + i*s + j
+            // (rows permuted at repack) -> HR pixel (s*y + i, s*x + j), channel c.
+            const int C = a.C, s = a.s;
+            const int Hs = a.H * s, Ws = a.W * s;
+            const int nsub = NTOT / C;
+            for (int sub = 0; sub < nsub; sub++) {
+                const int gsub = a.sub0 + sub;
+                const int i = gsub / s, j = gsub % s;
+                const size_t rowbase = ((size_t)slot_job * Hs + (size_t)(s * y + i)) * (C / 8);
+                if (C == 32) {
+                    uint32_t v[32];
+                    tmem_ld32(acc + sub * 32, v);
+                    tmem_wait_ld();
+                    if (x < a.W) {
+#pragma unroll
+                        for (int cg = 0; cg < 4; cg++) {
+                            const float *b = s_bias + sub * 32 + cg * 8;
+                            uint4 o;
+                            o.x = pack_bf16(__uint_as_float(v[cg * 8 + 0]) + b[0], __uint_as_float(v[cg * 8 + 1]) + b[1]);
+                            o.y = pack_bf16(__uint_as_float(v[cg * 8 + 2]) + b[2], __uint_as_float(v[cg * 8 + 3]) + b[3]);
+                            o.z = pack_bf16(__uint_as_float(v[cg * 8 + 4]) + b[4], __uint_as_float(v[cg * 8 + 5]) + b[5]);
+                            o.w = pack_bf16(__uint_as_float(v[cg * 8 + 6]) + b[6], __uint_as_float(v[cg * 8 + 7]) + b[7]);
+                            *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * Ws + (size_t)(s * x + j)) * 8) = o;
+                        }
+                    }
+                } else {
+                    uint32_t v[16];
+                    tmem_ld16(acc + sub * 16, v);
+                    tmem_wait_ld();
+                    if (x < a.W) {
+#pragma unroll
+                        for (int cg = 0; cg < 2; cg++) {
+                            const float *b = s_bias + sub * 16 + cg * 8;
+                            uint4 o;
+                            o.x = pack_bf16(__uint_as_float(v[cg * 8 + 0]) + b[0], __uint_as_float(v[cg * 8 + 1]) + b[1]);
+                            o.y = pack_bf16(__uint_as_float(v[cg * 8 + 2]) + b[2], __uint_as_float(v[cg * 8 + 3]) + b[3]);
+                            o.z = pack_bf16(__uint_as_float(v[cg * 8 + 4]) + b[4], __uint_as_float(v[cg * 8 + 5]) + b[5]);
+                            o.w = pack_bf16(__uint_as_float(v[cg * 8 + 6]) + b[6], __uint_as_float(v[cg * 8 + 7]) + b[7]);
+                            *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * Ws + (size_t)(s * x + j)) * 8) = o;
+                        }
+                    }
+                }
+            }
+        } else {  // EPI_TAIL: out = clamp(floor(up_s(LR) + t + 0.5), 0, 255), u8 planar HR
+            static_assert(NT == 16 && NSPLIT == 1, "");
+            uint32_t v[16];
+            tmem_ld16(acc, v);
+            tmem_wait_ld();
+            if (x < a.W) {
+                const int s = a.s, lh = a.lr_h, lw = a.lr_w;
+                int ya, yb, wy, xa, xb, wx;
+                up_tap(y, s, lh, ya, yb, wy);
+                up_tap(x, s, lw, xa, xb, wx);
+                const size_t plane = (size_t)lh * lw, hplane = (size_t)a.H * a.W;
+#pragma unroll
+                for (int c = 0; c < 3; c++) {
+                    const uint8_t *L = J.lr + c * plane;
+                    const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
+                    const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
+                    const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
+                    const int U = (vv + 8192) >> 14;
+                    const float t = __uint_as_float(v[c]) + s_bias[c];
+                    const float o = floorf((float)U + t + 0.5f);
+                    J.hr[c * hplane + (size_t)y * a.W + x] = (uint8_t)fminf(fmaxf(o, 0.f), 255.f);
+                }
+            }
+        }
+        tc_fence_before();
+        __syncthreads();
+    }
+    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
+}
+
+// LR u8 planar [3][h][w] -> bf16 [h][2][w][8]: channels 0..2 = LR - 128 (Z13), 3..15 = 0.
+__global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0) {
+    const int slot = blockIdx.y, job = j0 + slot;
+    if (job_count && job >= *job_count) return;
+    const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= h * w) return;
+    const int y = idx / w, x = idx % w;
+    const uint8_t *L = jobs[job].lr;
+    const size_t plane = (size_t)h * w;
+    const float r = (float)L[idx] - 128.f, g = (float)L[plane + idx] - 128.f, b = (float)L[2 * plane + idx] - 128.f;
+    uint4 o0, z;
+    o0.x = pack_bf16(r, g);
+    o0.y = pack_bf16(b, 0.f);
+    o0.z = 0; o0.w = 0;
+    z.x = z.y = z.z = z.w = 0;
+    uint16_t *base = x0 + (((size_t)slot * h + y) * 2) * (size_t)w * 8;
+    *reinterpret_cast<uint4 *>(base + (size_t)x * 8) = o0;
+    *reinterpret_cast<uint4 *>(base + ((size_t)w + x) * 8) = z;
+}
+
+// ------------------------------------------------------------------ host side
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                     const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                     CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+static PFN_encodeTiled get_encode() {
+    static PFN_encodeTiled fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<PFN_encodeTiled>(p);
+    }
+    return fn;
+}
+
+// Activation tensor [nb][H][C/8][W][8] bf16 viewed as 5-D (8, W, C/8, H, nb); box (8, 130, C/8, 1, 1).
+static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int nb) {
+    PFN_encodeTiled enc = get_encode();
+    if (!enc) return -1;
+    cuuint64_t dims[5] = {8, (cuuint64_t)W, (cuuint64_t)(C / 8), (cuuint64_t)H, (cuuint64_t)nb};
+    cuuint64_t strides[4] = {16, (cuuint64_t)W * 16, (cuuint64_t)(C / 8) * W * 16, (cuuint64_t)H * (C / 8) * W * 16};
+    cuuint32_t box[5] = {8, kHalo, (cuuint32_t)(C / 8), 1, 1};
+    cuuint32_t estr[5] = {1, 1, 1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, base, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : -2;
+}
+
+size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
+    const size_t px = (size_t)h * w * nb;
+    size_t b = px * 16 * 2;                  // x0
+    b += 3 * px * C * 2;                     // h0, hb, tb
+    b += px * s * s * C * 2;                 // u (HR)
+    return b + 5 * 256;
+}
+
+int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) {
+    a->h = h; a->w = w; a->C = C; a->s = s; a->nb = nb;
+    const size_t px = (size_t)h * w * nb;
+    auto take = [&](size_t bytes) {
+        uint8_t *p = mem;
+        mem += (bytes + 255) / 256 * 256;
+        return reinterpret_cast<uint16_t *>(p);
+    };
+    a->x0 = take(px * 16 * 2);
+    a->h0 = take(px * C * 2);
+    a->hb = take(px * C * 2);
+    a->tb = take(px * C * 2);
+    a->u = take(px * s * s * C * 2);
+    int rc = 0;
+    rc |= make_act_map(&a->tm_x0, a->x0, h, w, 16, nb);
+    rc |= make_act_map(&a->tm_h0, a->h0, h, w, C, nb);
+    rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb);
+    rc |= make_act_map(&a->tm_tb, a->tb, h, w, C, nb);
+    rc |= make_act_map(&a->tm_u, a->u, h * s, w * s, C, nb);
+    return rc;
+}
+
+template <int CIN, int NT, int NSPLIT, int EPI>
+static cudaError_t conv(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+    using Cfg = ConvCfg<CIN, NT, NSPLIT>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_conv3x3<CIN, NT, NSPLIT, EPI>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    args.n_xtiles = (args.W + kTile - 1) / kTile;
+    args.rows_per_cta = kRows;
+    dim3 grid(args.n_xtiles, (args.H + kRows - 1) / kRows, nj);
+    k_conv3x3<CIN, NT, NSPLIT, EPI><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
+    return cudaGetLastError();
+}
+
+template <int C>
+static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
+                           const int32_t *job_count, cudaStream_t st) {
+    const int h = a->h, w = a->w, s = a->s;
+    cudaError_t e;
+    {
+        dim3 g((h * w + 255) / 256, nj);
+        k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0);
+        count_launch();
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
+    ConvArgs base{};
+    base.H = h; base.W = w; base.j0 = j0; base.jobs = jobs; base.job_count = job_count; base.C = C; base.s = s;
+    auto L = [&](int l) { return model_layer(n_blocks, C, s, l); };
+    {   // head: conv(x; W_head) -> h0
+        ConvArgs g = base; LayerShape ls = L(0);
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
+        if ((e = conv<16, C, 1, EPI_STORE>(a->tm_x0, g, nj, st)) != cudaSuccess) return e;
+    }
+    for (int b = 0; b < n_blocks; b++) {
+        const CUtensorMap &hin = (b == 0) ? a->tm_h0 : a->tm_hb;
+        const uint16_t *hres = (b == 0) ? a->h0 : a->hb;
+        ConvArgs g = base; LayerShape l1 = L(1 + 2 * b), l2 = L(2 + 2 * b);
+        g.b_off = l1.b_off; g.bias_off = l1.bias_off; g.out = a->tb;
+        if ((e = conv<C, C, 1, EPI_RELU>(hin, g, nj, st)) != cudaSuccess) return e;
+        g = base; g.b_off = l2.b_off; g.bias_off = l2.bias_off; g.out = a->hb; g.resid = hres;
+        if ((e = conv<C, C, 1, EPI_RESID>(a->tm_tb, g, nj, st)) != cudaSuccess) return e;
+    }
+    {   // end: h0 + conv(h; W_end) -> tb
+        ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 1);
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->tb; g.resid = a->h0;
+        if ((e = conv<C, C, 1, EPI_RESID>(n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
+    }
+    {   // upsampler conv + pixel shuffle -> u (HR)
+        LayerShape ls = L(2 * n_blocks + 2);
+        ConvArgs g = base; g.out = a->u;
+        const int ntot = s * s * C;
+        if (ntot <= 256) {
+            g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
+            if (C == 16 && s == 2) e = conv<C, 64, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
+            else if (C == 16 && s == 3) e = conv<C, 144, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
+            else if (C == 16 && s == 4) e = conv<C, 256, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
+            else e = conv<C, (C == 32 ? 128 : 64), 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);  // C=32, s=2
+        } else if (ntot == 288) {  // C = 32, s = 3: two N tiles of 144 in one launch
+            g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
+            e = conv<C, 144, 2, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
+        } else {                   // C = 32, s = 4: two launches of N = 256
+            for (int sp = 0; sp < 2 && e == cudaSuccess; sp++) {
+                ConvArgs g2 = g;
+                g2.b_off = ls.b_off + (size_t)sp * 9 * C * 256 * 2;
+                g2.bias_off = ls.bias_off + (size_t)sp * 256 * 4;
+                g2.sub0 = sp * 8;
+                e = conv<C, 256, 1, EPI_SHUFFLE>(a->tm_tb, g2, nj, st);
+            }
+        }
+        if (e != cudaSuccess) return e;
+    }
+    {   // HR tail + integer bilinear skip -> u8 planar
+        ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 3);
+        g.H = h * s; g.W = w * s; g.lr_h = h; g.lr_w = w;
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off;
+        if ((e = conv<C, 16, 1, EPI_TAIL>(a->tm_u, g, nj, st)) != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
+cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
+                         const int32_t *job_count, cudaStream_t st) {
+    if (a->C == 32) return run_net<32>(a, n_blocks, jobs, j0, nj, job_count, st);
+    return run_net<16>(a, n_blocks, jobs, j0, nj, job_count, st);
+}
+
+}  // namespace ns

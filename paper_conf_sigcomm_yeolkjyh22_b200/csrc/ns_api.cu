@@ -1,0 +1,596 @@
+// ns_api.cu -- host side of the C ABI declared in include/ns.h: argument
+// validation, the pre-allocated context pool (App. A),
+// model slots + weight refit, descriptor staging and the
+// multi-stream batcher that drives the kernels.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <atomic>
+#include <algorithm>
+#include <map>
+#include <tuple>
+#include <vector>
+#include "ns_internal.h"
+
+using namespace ns;
+
+// ------------------------------------------------------------------ errors / counters
+static thread_local char g_err[512] = "";
+static std::atomic<uint64_t> g_launches{0};
+
+static ns_status fail(ns_status st, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return st;
+}
+static ns_status cuda_fail(cudaError_t e, const char *where) {
+    return fail(NS_ECUDA, "%s: %s (%s)", where, cudaGetErrorString(e), cudaGetErrorName(e));
+}
+#define NS_CUDA(call)                                           \
+    do {                                                        \
+        cudaError_t _e = (call);                                \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call);     \
+    } while (0)
+
+namespace ns {
+void count_launch(int n) { g_launches.fetch_add((uint64_t)n, std::memory_order_relaxed); }
+
+// ------------------------------------------------------------------ model layout
+int model_num_layers(int n_blocks) { return 2 * n_blocks + 4; }
+
+static size_t align128(size_t v) { return (v + 127) / 128 * 128; }
+
+LayerShape model_layer(int n_blocks, int C, int s, int L) {
+    LayerShape ls{};
+    if (L == 0) {
+        ls.cin = 16; ls.cin_real = 3; ls.ntot = C; ls.cout_real = C;
+    } else if (L <= 2 * n_blocks + 1) {
+        ls.cin = C; ls.cin_real = C; ls.ntot = C; ls.cout_real = C;
+    } else if (L == 2 * n_blocks + 2) {
+        ls.cin = C; ls.cin_real = C; ls.ntot = s * s * C; ls.cout_real = s * s * C; ls.perm = 1;
+    } else {
+        ls.cin = C; ls.cin_real = C; ls.ntot = 16; ls.cout_real = 3;
+    }
+    ls.nsplit = ls.ntot > 256 ? 2 : 1;
+    size_t off = 0;
+    for (int l = 0; l < L; l++) off += model_layer(n_blocks, C, s, l).bytes;
+    ls.b_off = off;
+    ls.bias_off = off + align128((size_t)9 * ls.cin * ls.ntot * 2);
+    ls.bytes = align128((size_t)9 * ls.cin * ls.ntot * 2) + align128((size_t)ls.ntot * 4);
+    return ls;
+}
+
+size_t model_packed_bytes(int n_blocks, int C, int s) {
+    size_t t = 0;
+    for (int l = 0; l < model_num_layers(n_blocks); l++) t += model_layer(n_blocks, C, s, l).bytes;
+    return t;
+}
+}  // namespace ns
+
+// ------------------------------------------------------------------ context
+namespace {
+constexpr int kStageSlots = 4;
+constexpr size_t kStageBytes = 8u << 20;
+constexpr int kMaxSN = 1 << 20;           // max streams x frames per call
+constexpr int kMaxJobs = 1 << 20;
+
+struct ArenaEntry {
+    int h, w, C, s;
+    SrArena a;
+};
+}  // namespace
+
+struct ns_model {
+    ns_ctx *ctx;
+    int n_blocks, C, s;
+    uint8_t *packed;
+    size_t bytes;
+    bool has_weights;
+};
+
+struct ns_ctx {
+    int device;
+    uint8_t *pool = nullptr;
+    size_t pool_bytes = 0, used = 0;
+    uint8_t *stage_host[kStageSlots] = {};
+    uint8_t *stage_dev[kStageSlots] = {};
+    cudaEvent_t stage_ev[kStageSlots] = {};
+    bool stage_used[kStageSlots] = {};
+    int stage_next = 0;
+    // device scratch (capacity kMaxSN)
+    int64_t *score, *gain;
+    int32_t *rank, *order, *grank, *pos_stream, *cut, *job_count;
+    uint8_t *anchor;
+    int16_t *gold;
+    SrJob *jobs;
+    uint16_t *blob_stage;  // device staging for host weight blobs
+    size_t blob_stage_elems;
+    int sr_batch = 16;
+    std::vector<ArenaEntry> arenas;
+};
+
+static uint8_t *pool_take(ns_ctx *c, size_t bytes) {
+    size_t off = (c->used + 255) / 256 * 256;
+    if (off + bytes > c->pool_bytes) return nullptr;
+    c->used = off + bytes;
+    return c->pool + off;
+}
+
+// Stage a host buffer of `bytes` into device memory on `st`; returns the device address.
+static ns_status stage_begin(ns_ctx *c, uint8_t **host, uint8_t **dev, int *slot) {
+    const int i = c->stage_next;
+    c->stage_next = (c->stage_next + 1) % kStageSlots;
+    if (c->stage_used[i]) NS_CUDA(cudaEventSynchronize(c->stage_ev[i]));
+    *host = c->stage_host[i];
+    *dev = c->stage_dev[i];
+    *slot = i;
+    return NS_OK;
+}
+static ns_status stage_end(ns_ctx *c, int slot, size_t bytes, cudaStream_t st) {
+    if (bytes) NS_CUDA(cudaMemcpyAsync(c->stage_dev[slot], c->stage_host[slot], bytes, cudaMemcpyHostToDevice, st));
+    return NS_OK;
+}
+static ns_status stage_release(ns_ctx *c, int slot, cudaStream_t st) {
+    NS_CUDA(cudaEventRecord(c->stage_ev[slot], st));
+    c->stage_used[slot] = true;
+    return NS_OK;
+}
+
+extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) {
+    if (!out) return fail(NS_EINVAL, "ns_ctx_create: out is NULL");
+    *out = nullptr;
+    int ndev = 0;
+    NS_CUDA(cudaGetDeviceCount(&ndev));
+    if (device < 0 || device >= ndev) return fail(NS_EINVAL, "ns_ctx_create: device %d out of range (%d)", device, ndev);
+    cudaDeviceProp prop;
+    NS_CUDA(cudaGetDeviceProperties(&prop, device));
+    if (prop.major != 10 || prop.minor != 0)
+        return fail(NS_EUNSUPPORTED, "ns_ctx_create: device %d is sm_%d%d, this build targets sm_100a", device,
+                    prop.major, prop.minor);
+    NS_CUDA(cudaSetDevice(device));
+    ns_ctx *c = new ns_ctx();
+    c->device = device;
+    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2) + (size_t)kMaxJobs * sizeof(SrJob) +
+                         kStageSlots * kStageBytes + (64u << 20) + 64 * 1024;
+    if (pool_bytes < fixed + (64u << 20)) {
+        delete c;
+        return fail(NS_EINVAL, "ns_ctx_create: pool_bytes %zu too small (need >= %zu)", pool_bytes,
+                    fixed + (64u << 20));
+    }
+    cudaError_t e = cudaMalloc(&c->pool, pool_bytes);
+    if (e != cudaSuccess) {
+        delete c;
+        return cuda_fail(e, "cudaMalloc(pool)");
+    }
+    c->pool_bytes = pool_bytes;
+    c->score = (int64_t *)pool_take(c, sizeof(int64_t) * kMaxSN);
+    c->gain = (int64_t *)pool_take(c, sizeof(int64_t) * kMaxSN);
+    c->rank = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
+    c->order = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
+    c->grank = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
+    c->pos_stream = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
+    c->anchor = (uint8_t *)pool_take(c, kMaxSN);
+    c->gold = (int16_t *)pool_take(c, sizeof(int16_t) * (kMaxSN + 4096));
+    c->cut = (int32_t *)pool_take(c, 256);
+    c->job_count = (int32_t *)pool_take(c, sizeof(int32_t) * 4096);
+    c->jobs = (SrJob *)pool_take(c, sizeof(SrJob) * kMaxJobs);
+    c->blob_stage_elems = (64u << 20) / 2;
+    c->blob_stage = (uint16_t *)pool_take(c, 64u << 20);
+    for (int i = 0; i < kStageSlots; i++) {
+        c->stage_dev[i] = pool_take(c, kStageBytes);
+        if ((e = cudaHostAlloc(&c->stage_host[i], kStageBytes, cudaHostAllocDefault)) != cudaSuccess ||
+            (e = cudaEventCreateWithFlags(&c->stage_ev[i], cudaEventDisableTiming)) != cudaSuccess) {
+            ns_ctx_destroy(c);
+            return cuda_fail(e, "staging");
+        }
+    }
+    *out = c;
+    return NS_OK;
+}
+
+extern "C" ns_status ns_ctx_destroy(ns_ctx *c) {
+    if (!c) return fail(NS_EINVAL, "ns_ctx_destroy: NULL");
+    cudaSetDevice(c->device);
+    cudaDeviceSynchronize();
+    for (int i = 0; i < kStageSlots; i++) {
+        if (c->stage_host[i]) cudaFreeHost(c->stage_host[i]);
+        if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
+    }
+    if (c->pool) cudaFree(c->pool);
+    delete c;
+    return NS_OK;
+}
+
+// ------------------------------------------------------------------ models
+extern "C" size_t ns_model_blob_len(int B, int C, int s) {
+    size_t n = (size_t)C * 3 * 9 + C;
+    n += (size_t)2 * B * ((size_t)C * C * 9 + C);
+    n += (size_t)C * C * 9 + C;
+    n += (size_t)s * s * C * C * 9 + (size_t)s * s * C;
+    n += (size_t)3 * C * 9 + 3;
+    return n;
+}
+
+extern "C" ns_status ns_model_create(ns_ctx *c, int n_blocks, int n_ch, int scale, ns_model **out) {
+    if (!c || !out) return fail(NS_EINVAL, "ns_model_create: NULL argument");
+    if (n_blocks < 1 || n_blocks > 64) return fail(NS_EINVAL, "ns_model_create: n_blocks %d not in [1, 64]", n_blocks);
+    if (n_ch != 16 && n_ch != 32) return fail(NS_EUNSUPPORTED, "ns_model_create: n_ch %d not in {16, 32}", n_ch);
+    if (scale < 2 || scale > 4) return fail(NS_EINVAL, "ns_model_create: scale %d not in {2, 3, 4}", scale);
+    const size_t bytes = model_packed_bytes(n_blocks, n_ch, scale);
+    uint8_t *p = pool_take(c, bytes);
+    if (!p) return fail(NS_ENOMEM, "ns_model_create: pool exhausted (%zu bytes needed)", bytes);
+    ns_model *m = new ns_model{c, n_blocks, n_ch, scale, p, bytes, false};
+    *out = m;
+    return NS_OK;
+}
+
+extern "C" ns_status ns_model_set_weights(ns_model *m, const uint16_t *blob, size_t n, void *stream) {
+    if (!m || !blob) return fail(NS_EINVAL, "ns_model_set_weights: NULL argument");
+    const size_t need = ns_model_blob_len(m->n_blocks, m->C, m->s);
+    if (n != need) return fail(NS_EINVAL, "ns_model_set_weights: blob has %zu entries, model needs %zu", n, need);
+    ns_ctx *c = m->ctx;
+    cudaStream_t st = (cudaStream_t)stream;
+    NS_CUDA(cudaSetDevice(c->device));
+    cudaPointerAttributes at;
+    const uint16_t *src = blob;
+    if (cudaPointerGetAttributes(&at, blob) != cudaSuccess || at.type != cudaMemoryTypeDevice) {
+        cudaGetLastError();
+        if (need > c->blob_stage_elems) return fail(NS_ENOMEM, "ns_model_set_weights: blob larger than staging");
+        NS_CUDA(cudaMemcpyAsync(c->blob_stage, blob, need * 2, cudaMemcpyHostToDevice, st));
+        src = c->blob_stage;
+    }
+    NS_CUDA(launch_repack(src, m->n_blocks, m->C, m->s, m->packed, st));
+    if (src == c->blob_stage) NS_CUDA(cudaStreamSynchronize(st));  // host blob / staging reuse (not hot path)
+    m->has_weights = true;
+    return NS_OK;
+}
+
+extern "C" ns_status ns_model_destroy(ns_model *m) {
+    if (!m) return fail(NS_EINVAL, "ns_model_destroy: NULL");
+    // pool memory is released with the context (bump allocator, P:625 fragments)
+    delete m;
+    return NS_OK;
+}
+
+extern "C" uint64_t ns_launch_count(int reset) {
+    return reset ? g_launches.exchange(0) : g_launches.load();
+}
+extern "C" const char *ns_last_error(void) { return g_err; }
+
+// ------------------------------------------------------------------ validation
+static bool al16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+
+static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n_out) {
+    if (!ch) return fail(NS_EINVAL, "chunks is NULL");
+    if (S < 1) return fail(NS_EINVAL, "S = %d < 1", S);
+    const int n = ch[0].n_frames;
+    if (n < 1 || n > kMaxFrames) return fail(NS_EINVAL, "n_frames %d not in [1, %d]", n, kMaxFrames);
+    if ((size_t)S * n > (size_t)kMaxSN) return fail(NS_EINVAL, "S * n = %zu exceeds %d", (size_t)S * n, kMaxSN);
+    for (int s = 0; s < S; s++) {
+        const ns_chunk &c = ch[s];
+        if (c.n_frames != n) return fail(NS_EINVAL, "chunk %d: n_frames %d differs from chunk 0 (%d)", s, c.n_frames, n);
+        if (c.w < 8 || c.h < 8 || c.w % 8 || c.h % 8)
+            return fail(NS_EINVAL, "chunk %d: w=%d h=%d must be positive multiples of 8", s, c.w, c.h);
+        if (c.w > 8192 || c.h > 8192) return fail(NS_EINVAL, "chunk %d: w/h > 8192", s);
+        if (c.scale < 2 || c.scale > 4) return fail(NS_EINVAL, "chunk %d: scale %d not in {2,3,4}", s, c.scale);
+        if (!c.lr || !c.res || !c.mv || !c.type) return fail(NS_EINVAL, "chunk %d: lr/res/mv/type must be non-NULL", s);
+        if (!al16(c.res) || !al16(c.lr) || !al16(c.mv)) return fail(NS_EINVAL, "chunk %d: lr/res/mv must be 16-B aligned", s);
+        if (c.gt && !al16(c.gt)) return fail(NS_EINVAL, "chunk %d: gt must be 16-B aligned", s);
+        if ((c.hr_last && !al16(c.hr_last)) || (c.hr_golden && !al16(c.hr_golden)))
+            return fail(NS_EINVAL, "chunk %d: hr_last/hr_golden must be 16-B aligned", s);
+        if (c.hr_last && c.hr_last == c.hr_golden) return fail(NS_EINVAL, "chunk %d: hr_last aliases hr_golden", s);
+        if (need_model) {
+            if (!c.model) return fail(NS_EINVAL, "chunk %d: model is NULL", s);
+            if (c.model->s != c.scale) return fail(NS_EINVAL, "chunk %d: model scale %d != chunk scale %d", s, c.model->s, c.scale);
+            if (!c.model->has_weights) return fail(NS_EINVAL, "chunk %d: model has no weights (ns_model_set_weights)", s);
+        }
+    }
+    *n_out = n;
+    return NS_OK;
+}
+
+static ns_status check_hr_table(const ns_chunk *ch, int S, int n, uint8_t *const *hr) {
+    if (!hr) return fail(NS_EINVAL, "hr_out table is NULL");
+    for (int s = 0; s < S; s++)
+        for (int f = 0; f < n; f++) {
+            uint8_t *p = hr[(size_t)s * n + f];
+            if (!p || !al16(p)) return fail(NS_EINVAL, "hr_out[%d][%d] is NULL or not 16-B aligned", s, f);
+            if (f > 0 && p == hr[(size_t)s * n + f - 1]) return fail(NS_EINVAL, "hr_out[%d][%d] aliases hr_out[%d][%d]", s, f, s, f - 1);
+            if (p == ch[s].hr_last || p == ch[s].hr_golden)
+                return fail(NS_EINVAL, "hr_out[%d][%d] aliases the stream's hr_last/hr_golden", s, f);
+        }
+    return NS_OK;
+}
+
+// Builds StreamDesc[S] (+ optional hr table) into a staging slot.
+struct Staged {
+    int slot;
+    uint8_t *host, *dev;
+    size_t used;
+    StreamDesc *d_sd;
+    uint8_t **d_hr;
+    int64_t *d_cost;
+};
+
+static size_t a256(size_t v) { return (v + 255) / 256 * 256; }
+
+static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint8_t *const *hr, const int64_t *cost,
+                               const int *group, const int *job_base, bool use_res_size, Staged *out) {
+    Staged g{};
+    ns_status r = stage_begin(c, &g.host, &g.dev, &g.slot);
+    if (r != NS_OK) return r;
+    size_t off = 0;
+    const size_t sd_bytes = a256(sizeof(StreamDesc) * S);
+    const size_t hr_bytes = hr ? a256(sizeof(uint8_t *) * (size_t)S * n) : 0;
+    const size_t cost_bytes = cost ? a256(sizeof(int64_t) * S) : 0;
+    if (sd_bytes + hr_bytes + cost_bytes > kStageBytes) return fail(NS_EINVAL, "too many streams for one call (staging)");
+    StreamDesc *sd = reinterpret_cast<StreamDesc *>(g.host);
+    for (int s = 0; s < S; s++) {
+        const ns_chunk &k = ch[s];
+        StreamDesc d{};
+        d.lr = k.lr; d.res = k.res; d.mv = k.mv; d.type = k.type; d.res_size = k.res_size;
+        d.hr_last = k.hr_last; d.hr_golden = k.hr_golden; d.gt = k.gt;
+        d.wts = k.model ? k.model->packed : nullptr;
+        d.w = k.w; d.h = k.h; d.s = k.scale; d.n = k.n_frames;
+        d.hr_base = s * n;
+        d.group = group ? group[s] : 0;
+        d.job_base = job_base ? job_base[s] : 0;
+        d.use_res_size = use_res_size ? 1 : 0;
+        sd[s] = d;
+    }
+    g.d_sd = reinterpret_cast<StreamDesc *>(g.dev);
+    off = sd_bytes;
+    if (hr) {
+        memcpy(g.host + off, hr, sizeof(uint8_t *) * (size_t)S * n);
+        g.d_hr = reinterpret_cast<uint8_t **>(g.dev + off);
+        off += hr_bytes;
+    }
+    if (cost) {
+        memcpy(g.host + off, cost, sizeof(int64_t) * S);
+        g.d_cost = reinterpret_cast<int64_t *>(g.dev + off);
+        off += cost_bytes;
+    }
+    g.used = off;
+    *out = g;
+    return NS_OK;
+}
+
+static ns_status check_params(const ns_select_params *p, int S, int n) {
+    if (!p) return fail(NS_EINVAL, "params is NULL");
+    if (p->group_residual != NS_CARRY && p->group_residual != NS_FRESH)
+        return fail(NS_EINVAL, "group_residual %d invalid", p->group_residual);
+    if (p->mode == NS_TOPK_PER_STREAM) {
+        if (p->k < 0 || p->k > n) return fail(NS_EINVAL, "k = %d not in [0, n = %d]", p->k, n);
+    } else if (p->mode == NS_GLOBAL_BUDGET) {
+        if (!p->cost) return fail(NS_EINVAL, "global mode needs cost[S]");
+        if (p->budget < 0) return fail(NS_EINVAL, "budget < 0");
+        for (int s = 0; s < S; s++)
+            if (p->cost[s] < 1) return fail(NS_EINVAL, "cost[%d] = %lld < 1", s, (long long)p->cost[s]);
+    } else {
+        return fail(NS_EINVAL, "mode %d invalid", p->mode);
+    }
+    return NS_OK;
+}
+
+// select into (gain, rank, is_anchor); order/score in ctx scratch
+static ns_status run_select(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n, const ns_select_params *p,
+                            int64_t *gain, int32_t *rank, uint8_t *is_anchor, cudaStream_t st) {
+    int maxv = 0;
+    for (int s = 0; s < S; s++) maxv = std::max(maxv, 3 * ch[s].h * ch[s].w / 8);
+    NS_CUDA(launch_score(g.d_sd, S, n, maxv, c->score, st));
+    const bool global = p->mode == NS_GLOBAL_BUDGET;
+    NS_CUDA(launch_select(g.d_sd, c->score, S, n, global ? -1 : p->k, p->group_residual == NS_FRESH, gain, rank,
+                          is_anchor, global ? c->order : nullptr, st));
+    if (global)
+        NS_CUDA(launch_global(g.d_sd, S, n, gain, c->order, g.d_cost, p->budget, c->grank, c->pos_stream, c->cut,
+                              rank, is_anchor, st));
+    return NS_OK;
+}
+
+extern "C" ns_status ns_select_anchors(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
+                                       int64_t *gain, int32_t *rank, uint8_t *is_anchor, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_select_anchors: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, false, &n);
+    if (r != NS_OK) return r;
+    if ((r = check_params(p, S, n)) != NS_OK) return r;
+    if (!gain || !rank || !is_anchor) return fail(NS_EINVAL, "ns_select_anchors: outputs must be non-NULL");
+    cudaStream_t st = (cudaStream_t)stream;
+    NS_CUDA(cudaSetDevice(c->device));
+    Staged g;
+    if ((r = stage_streams(c, ch, S, n, nullptr, p->mode == NS_GLOBAL_BUDGET ? p->cost : nullptr, nullptr, nullptr,
+                           p->use_res_size != 0, &g)) != NS_OK)
+        return r;
+    if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
+    r = run_select(c, g, ch, S, n, p, gain, rank, is_anchor, st);
+    stage_release(c, g.slot, st);
+    return r;
+}
+
+// ------------------------------------------------------------------ SR
+static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, const SrArena **out) {
+    for (auto &e : c->arenas)
+        if (e.h == h && e.w == w && e.C == C && e.s == s) {
+            *out = &e.a;
+            return NS_OK;
+        }
+    const size_t bytes = sr_arena_bytes(h, w, C, s, c->sr_batch);
+    uint8_t *mem = pool_take(c, bytes);
+    if (!mem)
+        return fail(NS_ENOMEM, "SR arena for %dx%d C%d x%d (%d jobs) needs %zu bytes; pool has %zu free", w, h, C, s,
+                    c->sr_batch, bytes, c->pool_bytes - c->used);
+    ArenaEntry e{h, w, C, s, {}};
+    if (sr_arena_init(&e.a, h, w, C, s, c->sr_batch, mem) != 0)
+        return fail(NS_ECUDA, "cuTensorMapEncodeTiled failed for the SR arena");
+    c->arenas.push_back(e);
+    *out = &c->arenas.back().a;
+    return NS_OK;
+}
+
+// jobs (device table) [0, max_jobs) of one shape; job_count (device) may be NULL
+static ns_status run_sr_group(ns_ctx *c, int h, int w, int C, int s, int B, const SrJob *d_jobs, int max_jobs,
+                              const int32_t *job_count, cudaStream_t st) {
+    const SrArena *a = nullptr;
+    ns_status r = get_arena(c, h, w, C, s, &a);
+    if (r != NS_OK) return r;
+    for (int j0 = 0; j0 < max_jobs; j0 += a->nb) {
+        const int nj = std::min(a->nb, max_jobs - j0);
+        NS_CUDA(sr_run_batch(a, B, d_jobs, j0, nj, job_count, st));
+    }
+    return NS_OK;
+}
+
+extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_sr_anchors: ctx is NULL");
+    if (n_jobs < 0 || (n_jobs > 0 && !jobs)) return fail(NS_EINVAL, "ns_sr_anchors: bad job list");
+    if (n_jobs == 0) return NS_OK;
+    for (int j = 0; j < n_jobs; j++) {
+        const ns_sr_job &J = jobs[j];
+        if (!J.model || !J.lr || !J.hr_out) return fail(NS_EINVAL, "job %d: NULL model/lr/hr_out", j);
+        if (!J.model->has_weights) return fail(NS_EINVAL, "job %d: model has no weights", j);
+        if (J.w < 8 || J.h < 8 || J.w % 8 || J.h % 8) return fail(NS_EINVAL, "job %d: w=%d h=%d must be multiples of 8", j, J.w, J.h);
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    NS_CUDA(cudaSetDevice(c->device));
+    // group by shape
+    std::map<std::tuple<int, int, int, int, int>, std::vector<int>> groups;
+    for (int j = 0; j < n_jobs; j++)
+        groups[std::make_tuple(jobs[j].h, jobs[j].w, jobs[j].model->C, jobs[j].model->s, jobs[j].model->n_blocks)]
+            .push_back(j);
+    ns_status r = NS_OK;
+    for (auto &kv : groups) {
+        const auto &idx = kv.second;
+        if (idx.size() * sizeof(SrJob) > kStageBytes) return fail(NS_EINVAL, "too many SR jobs in one call");
+        uint8_t *host, *dev;
+        int slot;
+        if ((r = stage_begin(c, &host, &dev, &slot)) != NS_OK) return r;
+        SrJob *hj = reinterpret_cast<SrJob *>(host);
+        for (size_t i = 0; i < idx.size(); i++) {
+            const ns_sr_job &J = jobs[idx[i]];
+            hj[i] = SrJob{J.lr, J.hr_out, J.model->packed};
+        }
+        if ((r = stage_end(c, slot, idx.size() * sizeof(SrJob), st)) != NS_OK) return r;
+        int h, w, C, s, B;
+        std::tie(h, w, C, s, B) = kv.first;
+        r = run_sr_group(c, h, w, C, s, B, reinterpret_cast<const SrJob *>(dev), (int)idx.size(), nullptr, st);
+        stage_release(c, slot, st);
+        if (r != NS_OK) return r;
+    }
+    return NS_OK;
+}
+
+// ------------------------------------------------------------------ reconstruct
+static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n,
+                                 const uint8_t *is_anchor, cudaStream_t st) {
+    int maxW8 = 0, maxH = 0;
+    size_t maxhr = 0;
+    for (int s = 0; s < S; s++) {
+        maxW8 = std::max(maxW8, ch[s].w * ch[s].scale / 8);
+        maxH = std::max(maxH, ch[s].h * ch[s].scale);
+        maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
+    }
+    NS_CUDA(launch_golden_index(g.d_sd, S, n, c->gold, st));
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(g.d_sd, S, n, f, maxW8, maxH, is_anchor, g.d_hr, c->gold, st));
+    NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, maxhr, st));
+    return NS_OK;
+}
+
+extern "C" ns_status ns_reconstruct_chunk(ns_ctx *c, const ns_chunk *ch, int S, const uint8_t *is_anchor,
+                                          uint8_t *const *hr_out, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_reconstruct_chunk: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, false, &n);
+    if (r != NS_OK) return r;
+    if (!is_anchor) return fail(NS_EINVAL, "ns_reconstruct_chunk: is_anchor is NULL");
+    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    cudaStream_t st = (cudaStream_t)stream;
+    NS_CUDA(cudaSetDevice(c->device));
+    Staged g;
+    if ((r = stage_streams(c, ch, S, n, hr_out, nullptr, nullptr, nullptr, false, &g)) != NS_OK) return r;
+    if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
+    r = run_reconstruct(c, g, ch, S, n, is_anchor, st);
+    stage_release(c, g.slot, st);
+    return r;
+}
+
+// ------------------------------------------------------------------ the whole path
+extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
+                                        uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_enhance_streams: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, true, &n);
+    if (r != NS_OK) return r;
+    if ((r = check_params(p, S, n)) != NS_OK) return r;
+    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    cudaStream_t st = (cudaStream_t)stream;
+    NS_CUDA(cudaSetDevice(c->device));
+    const bool topk = p->mode == NS_TOPK_PER_STREAM;
+    // SR shape groups and job slots (multi-stream batcher)
+    std::map<std::tuple<int, int, int, int, int>, int> gid;
+    std::vector<std::tuple<int, int, int, int, int>> gkey;
+    std::vector<int> group(S), job_base(S), gcount, goff;
+    std::vector<int> gstreams;
+    int64_t min_cost = INT64_MAX;
+    if (!topk)
+        for (int s = 0; s < S; s++) min_cost = std::min(min_cost, p->cost[s]);
+    for (int s = 0; s < S; s++) {
+        auto key = std::make_tuple(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks);
+        auto it = gid.find(key);
+        if (it == gid.end()) {
+            it = gid.emplace(key, (int)gkey.size()).first;
+            gkey.push_back(key);
+            gstreams.push_back(0);
+        }
+        group[s] = it->second;
+        gstreams[it->second]++;
+    }
+    const int G = (int)gkey.size();
+    gcount.resize(G);
+    goff.resize(G);
+    int total = 0;
+    for (int gi = 0; gi < G; gi++) {
+        int64_t mx = topk ? (int64_t)gstreams[gi] * p->k : (int64_t)gstreams[gi] * n;
+        if (!topk) mx = std::min<int64_t>(mx, p->budget / std::max<int64_t>(min_cost, 1));
+        gcount[gi] = (int)mx;
+        goff[gi] = total;
+        total += (int)mx;
+    }
+    if (total > kMaxJobs) return fail(NS_EINVAL, "too many SR jobs (%d)", total);
+    {
+        std::vector<int> local(G, 0);
+        for (int s = 0; s < S; s++) {
+            const int gi = group[s];
+            job_base[s] = topk ? goff[gi] + local[gi]++ * p->k : goff[gi];
+        }
+    }
+    Staged g;
+    if ((r = stage_streams(c, ch, S, n, hr_out, topk ? nullptr : p->cost, group.data(), job_base.data(),
+                           p->use_res_size != 0, &g)) != NS_OK)
+        return r;
+    if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
+    uint8_t *anchor = is_anchor_out ? is_anchor_out : c->anchor;
+    do {
+        if ((r = run_select(c, g, ch, S, n, p, c->gain, c->rank, anchor, st)) != NS_OK) break;
+        if (total > 0) {
+            cudaError_t e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, topk, p->k, st);
+            if (e != cudaSuccess) { r = cuda_fail(e, "compact"); break; }
+            for (int gi = 0; gi < G && r == NS_OK; gi++) {
+                int h, w, C, s, B;
+                std::tie(h, w, C, s, B) = gkey[gi];
+                r = run_sr_group(c, h, w, C, s, B, c->jobs + goff[gi], gcount[gi], topk ? nullptr : c->job_count + gi, st);
+            }
+            if (r != NS_OK) break;
+        }
+        if ((r = run_reconstruct(c, g, ch, S, n, anchor, st)) != NS_OK) break;
+        if (stats) {
+            size_t maxhr = 0;
+            for (int s = 0; s < S; s++) maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
+            cudaError_t e = launch_stats(g.d_sd, S, n, anchor, c->score, g.d_hr, maxhr, stats, st);
+            if (e != cudaSuccess) { r = cuda_fail(e, "stats"); break; }
+        }
+    } while (0);
+    stage_release(c, g.slot, st);
+    return r;
+}

@@ -1,0 +1,106 @@
+// ns_internal.h -- shared host/device definitions of libneuroscaler (not ABI).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstddef>
+#include "../../include/ns.h"
+
+namespace ns {
+
+constexpr int kMaxFrames = 256;
+constexpr int kTile = 128;        // output pixels per UMMA M tile (one row segment)
+constexpr int kHalo = kTile + 2;  // input pixels per tile row (3x3 halo)
+
+// Device-side per-stream descriptor (built by the host from ns_chunk).
+struct StreamDesc {
+    const uint8_t *lr;
+    const int16_t *res;
+    const ns_block_mv *mv;
+    const uint8_t *type;
+    const uint32_t *res_size;
+    uint8_t *hr_last;
+    uint8_t *hr_golden;
+    const uint8_t *gt;
+    const uint8_t *wts;    // packed model operands (see model layout below)
+    int32_t w, h, s, n;
+    int32_t hr_base;       // index of hr_out[s][0] in the device hr table
+    int32_t group;         // SR shape group index (ns_enhance_streams)
+    int32_t job_base;      // first SR job slot of this stream in its group
+    int32_t use_res_size;
+};
+
+// One anchor-SR job (device).
+struct SrJob {
+    const uint8_t *lr;     // [3][h][w]
+    uint8_t *hr;           // [3][s*h][s*w]
+    const uint8_t *wts;    // packed model operands
+};
+
+// Packed model: per layer L a UMMA B operand (bf16, K-major core matrices)
+// [split][tap 9][kc CIN/16][kh 2][n NT][8] followed by fp32 bias[NTOT],
+// each region 128-B aligned.  Layers: 0 head (CIN 16, 3 real), 1..2B body,
+// 2B+1 end, 2B+2 up (NTOT = s*s*C, rows permuted to (i, j, c) order for the
+// fused pixel shuffle), 2B+3 tail (NTOT = 16, 3 real).
+struct LayerShape {
+    int cin, cin_real, ntot, nsplit, cout_real;
+    int perm;              // 0 none, 1 pixel-shuffle permutation
+    size_t b_off, bias_off, bytes;  // offsets from the model base
+};
+
+int model_num_layers(int n_blocks);
+LayerShape model_layer(int n_blocks, int C, int s, int L);
+size_t model_packed_bytes(int n_blocks, int C, int s);
+
+// ------------------------------------------------------------ launch wrappers
+// Every launch goes through these (kernels live in k_*.cu); each returns the
+// cudaError_t of the launch.  `st` is the stream.
+cudaError_t launch_score(const StreamDesc *d_sd, int S, int n, int max_frame_vec8, int64_t *score,
+                         cudaStream_t st);
+cudaError_t launch_select(const StreamDesc *d_sd, const int64_t *score, int S, int n, int k, int fresh,
+                          int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order, cudaStream_t st);
+cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *gain, const int32_t *order,
+                          const int64_t *cost, int64_t budget, int32_t *grank, int32_t *pos_stream,
+                          int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st);
+cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
+                           uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups,
+                           int topk, int k, cudaStream_t st);
+cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st);
+cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, int maxW8, int maxH,
+                              const uint8_t *is_anchor, uint8_t *const *d_hr_table, const int16_t *gold_idx,
+                              cudaStream_t st);
+cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
+                              const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st);
+cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
+                         uint8_t *const *d_hr_table, size_t max_hr_bytes, double *stats, cudaStream_t st);
+cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint8_t *packed, cudaStream_t st);
+
+// SR (k_sr.cu)
+struct SrArena {
+    int h, w, C, s, nb;        // shape and batch capacity (jobs per batch)
+    uint16_t *x0, *h0, *hb, *tb, *u;   // bf16 activations, layout [job][H][C/8][W][8]
+    CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_u;
+};
+size_t sr_arena_bytes(int h, int w, int C, int s, int nb);
+int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);  // 0 ok
+// Runs the whole net on jobs [j0, j0+nj) of a device job table (all of one
+// shape).  job_count (device) may be NULL; otherwise CTAs of jobs >= *job_count exit.
+cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
+                         const int32_t *job_count, cudaStream_t st);
+
+// Kernel families for ns_launch_count / ns_profile_read.
+enum Fam { F_SCORE = 0, F_SELECT, F_GLOBAL, F_COMPACT, F_SR_PREP, F_SR_HEAD, F_SR_BODY, F_SR_END, F_SR_UP,
+           F_SR_TAIL, F_RECON, F_STATE, F_STATS, F_REPACK, F_COUNT };
+const char *fam_name(int fam);
+
+// Wraps the launch(es) of one kernel family on stream `st`: counts launches
+// and, when profiling is enabled, brackets them with CUDA events.
+struct KScope {
+    int fam, n;
+    cudaStream_t st;
+    void *rec;
+    KScope(int fam, cudaStream_t st, int n = 1);
+    ~KScope();
+};
+
+}  // namespace ns
