@@ -1,0 +1,415 @@
+#!/usr/bin/env python3
+"""bench.py -- NeuroScaler enhancement hot path on B200: enhanced 4K frames/s.
+
+A step = one chunk (60-frame GOP) of every stream on this GPU through the whole
+hot path (ns_enhance_streams: score -> Alg. 1 selection -> SR DNN on anchors ->
+reuse reconstruction -> state -> stats).  Default workload = BASELINE.json
+configs[3] "c4": 64 concurrent 720p->4K x3 streams on one B200, NAS "high"
+model (8 blocks, 32 channels), 8% anchors (k = 5 of 60), one content-aware
+model per stream.  N GPUs (torchrun) = N independent shards of 64 streams
+(weak scaling, no collective on the hot path; NCCL only gathers stats after
+timing).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config 4]
+  python bench.py --impl reference ...   # the CPU oracle on a bounded sample
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "enhanced 4K frames/s per B200 & 8×B200; anchor-SR tensor util; reuse HBM GB/s"
+UNIT = "4K frames/s"
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return dict(hbm=float(d["hbm_gbs"]), bf16=float(d["bf16_tflops"]),
+                    bf16_sus=float(d.get("bf16_tflops_sustained", d["bf16_tflops"])), src="measured")
+    return dict(hbm=6650.0, bf16=1590.0, bf16_sus=1400.0, src="fallback (B200_PROFILING.md)")
+
+
+# ---------------------------------------------------------------- workload
+def cfg_of(args):
+    c = dict(synth.CONFIGS[args.config])
+    if args.config == 5:
+        raise SystemExit("config 5 is the multi-GPU sharding of 512 streams: run config 4 per GPU (weak scaling)")
+    c["streams"] = args.streams or c.get("streams", 1)
+    return c
+
+
+def _gen(a):
+    seed, w, h, s, n, alt = a
+    return synth.make_chunk(seed, w, h, s, n, types=synth.default_types(n, alt))
+
+
+def gen_pool(cfg, n_distinct, rank):
+    seeds = [1000 * 4 + rank * 100000 + i for i in range(n_distinct)]
+    args = [(sd, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"]) for sd in seeds]
+    procs = min(len(args), max(1, (os.cpu_count() or 1)))
+    if procs > 1:
+        import multiprocessing as mp
+        with mp.get_context("fork").Pool(procs) as pool:
+            return pool.map(_gen, args)
+    return [_gen(a) for a in args]
+
+
+# ---------------------------------------------------------------- clocks
+class Clocks:
+    FIELDS = "clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown," \
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                       "-i", str(self.idx), "-lms", "200"], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if not self.p:
+            return None
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except Exception:
+            self.p.kill()
+            out, _ = self.p.communicate()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- CPU oracle
+def cpu_sample(cfg, chunk, blob):
+    """Times the oracle as it stands on a bounded sample of one stream-chunk and
+    converts to the metric: chunk time = score+select (whole chunk) + k x SR
+    frame (timed on a row strip, scaled by pixels) + (n-k) x reconstruction of a
+    non-anchor frame (timed on 2 frames)."""
+    import oracle
+    B, C, s, n, k = cfg["n_blocks"], cfg["n_ch"], cfg["scale"], cfg["n"], cfg["k"]
+    h, w = chunk.h, chunk.w
+    t0 = time.perf_counter()
+    sc = oracle.score(chunk.res)
+    oracle.select_topk(list(chunk.type), [int(v) for v in sc], k)
+    t_sel = time.perf_counter() - t0
+    rows = min(h, 48)
+    t0 = time.perf_counter()
+    oracle.sr_forward(np.ascontiguousarray(chunk.lr[0][:, :rows]), blob, B, C, s)
+    t_sr = (time.perf_counter() - t0) * h / rows
+    sub = synth.Chunk(w=w, h=h, scale=s, lr=chunk.lr[:3], res=chunk.res[:3], mv=chunk.mv[:3],
+                      type=chunk.type[:3].copy(), res_size=chunk.res_size[:3])
+    hr = np.zeros((3, 3, s * h, s * w), np.uint8)
+    t0 = time.perf_counter()
+    oracle.reconstruct(sub, [1, 0, 0], hr)
+    t_rec = (time.perf_counter() - t0) / 2
+    t_chunk = t_sel + k * t_sr + (n - k) * t_rec
+    threads = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
+    return dict(value=n / t_chunk, unit=UNIT, cores=threads, kind="oracle",
+                sample=f"1 stream-chunk of {cfg['name']} ({w}x{h}->x{s}, n={n}, k={k}): score+select on the full "
+                       f"chunk ({t_sel:.2f}s), SR on a {w}x{rows} LR strip scaled by pixels ({t_sr:.1f}s/frame, fp64 "
+                       f"OpenMP), reconstruction of 2 non-anchor frames ({t_rec:.2f}s/frame, 1 thread)",
+                seconds=dict(select=t_sel, sr_frame=t_sr, recon_frame=t_rec))
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle, as it stands, on this arm's workload."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    cfg = cfg_of(args)
+    chunk = _gen((4000, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"]))
+    blob = synth.make_weights(4000, cfg["n_blocks"], cfg["n_ch"], cfg["scale"])
+    vals = []
+    for i in range(args.warmup + args.steps):
+        r = cpu_sample(cfg, chunk, blob)
+        if i >= args.warmup:
+            vals.append(r["value"])
+    v = float(np.mean(vals))
+    ms = 1000.0 * cfg["n"] / v
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{cfg['name']} (one stream-chunk sample per step)"},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["cores"], "kind": "oracle", "sample": r["sample"]},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- GPU arm
+def algorithmic(cfg, types, ia, S, n):
+    """Algorithmic FLOPs / bytes per kernel family over one step (DESIGN.md
+    "Roofline"): the defined convs only; reconstruct = ref 3 B + write 3 B +
+    residual 6/s^2 B + MV 0.125/s^2 B per HR pixel of a non-anchor inter frame,
+    LR 3/s^2 B + write 3 B for a non-anchor KEY frame."""
+    B, C, s, h, w = cfg["n_blocks"], cfg["n_ch"], cfg["scale"], cfg["h"], cfg["w"]
+    px, hpx = h * w, h * w * s * s
+    anchors = int(ia.sum())
+    conv = lambda cin, cout: 2.0 * 9 * cin * cout
+    fl = {"sr_head": anchors * px * conv(3, C), "sr_body": anchors * px * conv(C, C) * 2 * B,
+          "sr_end": anchors * px * conv(C, C), "sr_up": anchors * px * conv(C, s * s * C),
+          "sr_tail": anchors * hpx * conv(C, 3)}
+    rec_bytes = 0.0
+    for si in range(S):
+        for f in range(n):
+            if ia[si, f]:
+                continue
+            if types[si][f] == synth.NS_KEY:
+                rec_bytes += hpx * 3 + px * 3
+            else:
+                rec_bytes += hpx * 6 + px * 6 + px * 8 / 64.0
+    by = {"recon": rec_bytes, "score": S * n * px * 6.0, "state": S * 2 * 2 * hpx * 3.0,
+          "sr_prep": anchors * px * (3 + 32)}
+    return fl, by
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", type=int, default=4)
+    ap.add_argument("--streams", type=int, default=0)
+    ap.add_argument("--distinct", type=int, default=8, help="distinct generated streams (replicated on device)")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--sr-batch", type=int, default=16)
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sigcomm_yeolkjyh22_b200 as ns
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    cfg = cfg_of(args)
+    S, n, k, s = cfg["streams"], cfg["n"], cfg["k"], cfg["scale"]
+    B, C, h, w = cfg["n_blocks"], cfg["n_ch"], cfg["h"], cfg["w"]
+    H, W = s * h, s * w
+    P = min(args.distinct, S)
+
+    t_gen = time.time()
+    pool = gen_pool(cfg, P, rank)
+    t_gen = time.time() - t_gen
+
+    ctx = ns.Context(local, pool_bytes=int((1.2 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)))
+    # per-stream content-aware models: distinct weights per stream
+    models = []
+    for si in range(S):
+        m = ctx.model(B, C, s)
+        m.set_weights(synth.make_weights(4000 + rank * 100000 + si, B, C, s))
+        models.append(m)
+    # device inputs: P generated chunks, copied to S distinct device buffers
+    lr_d = torch.empty((S, n, 3, h, w), dtype=torch.uint8, device=dev)
+    res_d = torch.empty((S, n, 3, h, w), dtype=torch.int16, device=dev)
+    mv_d = torch.empty((S, n, h // 8, w // 8, 8), dtype=torch.uint8, device=dev)
+    ty_d = torch.empty((S, n), dtype=torch.uint8, device=dev)
+    for si in range(P):
+        c = pool[si]
+        lr_d[si].copy_(torch.from_numpy(c.lr))
+        res_d[si].copy_(torch.from_numpy(c.res))
+        mv_d[si].copy_(torch.from_numpy(np.ascontiguousarray(c.mv).view(np.uint8).reshape(n, h // 8, w // 8, 8)))
+        ty_d[si].copy_(torch.from_numpy(c.type))
+    for si in range(P, S):
+        lr_d[si].copy_(lr_d[si % P]); res_d[si].copy_(res_d[si % P])
+        mv_d[si].copy_(mv_d[si % P]); ty_d[si].copy_(ty_d[si % P])
+    hr = torch.empty((S, n, 3, H, W), dtype=torch.uint8, device=dev)
+    state = torch.zeros((S, 2, 3, H, W), dtype=torch.uint8, device=dev)
+    chunks = [ns.DeviceChunk(w=w, h=h, scale=s, lr=lr_d[si], res=res_d[si], mv=mv_d[si], type=ty_d[si],
+                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1]) for si in range(S)]
+    hr_out = [[hr[si, f] for f in range(n)] for si in range(S)]
+    ia = torch.zeros((S, n), dtype=torch.uint8, device=dev)
+    stats = torch.zeros((S, 8), dtype=torch.float64, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def step():
+        ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, k=k, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    clocks = Clocks(int(os.environ.get("CUDA_VISIBLE_DEVICES", str(local)).split(",")[local])
+                    if os.environ.get("CUDA_VISIBLE_DEVICES") else local)
+    clocks.start()
+    ns.launch_count(reset=True)
+    ns.profile_enable(True)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize(dev)
+    e0.record(stream)
+    for _ in range(args.steps):
+        step()
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    ns.profile_enable(False)
+    launches = ns.launch_count()
+    ms = e0.elapsed_time(e1)
+    clk = clocks.stop()
+    prof = ns.profile_read()
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        dist.barrier()
+    frames = world * S * n * args.steps
+    value = frames / (ms / 1000.0)
+
+    # stats gather (the only collective; off the timed region)
+    st = stats.clone()
+    if world > 1:
+        allst = [torch.zeros_like(st) for _ in range(world)]
+        dist.all_gather(allst, st)
+        st = torch.cat(allst)
+    st = st.cpu().numpy()
+    ia_np = ia.cpu().numpy()
+    types = [pool[si % P].type for si in range(S)]
+
+    # rooflines from the live per-family event timing
+    pk = peaks()
+    fl, by = algorithmic(cfg, types, ia_np, S, n)
+    rl = {}
+    for fam, (nl, ng, tms) in prof.items():
+        if nl == 0 or tms <= 0:
+            continue
+        tot = tms / args.steps
+        ent = {"launches_per_step": nl / args.steps, "ms_per_step": tot, "share": tms / ms if world == 1 else None}
+        if fam in fl:
+            a = fl[fam] / (tot / 1000.0) / 1e12
+            ent.update(bound="tensor", achieved=a, unit="TFLOP/s", peak=pk["bf16_sus"], frac=a / pk["bf16_sus"])
+        elif fam in by:
+            a = by[fam] / (tot / 1000.0) / 1e9
+            ent.update(bound="hbm", achieved=a, unit="GB/s", peak=pk["hbm"], frac=a / pk["hbm"])
+        rl[fam] = ent
+    sr_fams = [f for f in ("sr_prep", "sr_head", "sr_body", "sr_end", "sr_up", "sr_tail") if f in rl]
+    sr_ms = sum(rl[f]["ms_per_step"] for f in sr_fams)
+    sr_tf = sum(fl.values()) / (sr_ms / 1000.0) / 1e12 if sr_ms else 0.0
+    dom = max((f for f in rl if "bound" in rl[f]), key=lambda f: rl[f]["ms_per_step"])
+    d = rl[dom]
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+    per_launch = (fl.get(dom) or by.get(dom)) / max(1, d["launches_per_step"])
+    roofline = {"bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
+                "frac": d["frac"], "traffic": traffic, "kernel": dom,
+                "per_launch_algorithmic": per_launch,
+                "peak_source": f"{pk['src']} ({'bf16 sustained' if d['bound'] == 'tensor' else 'HBM copy'})"}
+
+    # e2e: host (pinned) -> device copy of every stream's inputs + the whole
+    # path + device -> host read of the step's result (stats, anchor map)
+    e2e = None
+    if args.e2e_steps > 0:
+        pin = [dict(lr=torch.from_numpy(c.lr).pin_memory(), res=torch.from_numpy(c.res).pin_memory(),
+                    mv=torch.from_numpy(np.ascontiguousarray(c.mv).view(np.uint8).reshape(n, h // 8, w // 8, 8))
+                    .pin_memory(), ty=torch.from_numpy(c.type).pin_memory()) for c in pool]
+        st_h = torch.empty((S, 8), dtype=torch.float64).pin_memory()
+        ia_h = torch.empty((S, n), dtype=torch.uint8).pin_memory()
+        h2d = sum(int(pin[si % P][kk].numel() * pin[si % P][kk].element_size()) for si in range(S)
+                  for kk in ("lr", "res", "mv", "ty"))
+        d2h = st_h.numel() * 8 + ia_h.numel()
+
+        def e2e_step():
+            for si in range(S):
+                p = pin[si % P]
+                lr_d[si].copy_(p["lr"], non_blocking=True); res_d[si].copy_(p["res"], non_blocking=True)
+                mv_d[si].copy_(p["mv"], non_blocking=True); ty_d[si].copy_(p["ty"], non_blocking=True)
+            step()
+            st_h.copy_(stats, non_blocking=True)
+            ia_h.copy_(ia, non_blocking=True)
+
+        e2e_step()
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        q1.record(stream)
+        torch.cuda.synchronize(dev)
+        ems = q0.elapsed_time(q1)
+        if world > 1:
+            t = torch.tensor([ems], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ems = float(t.item())
+        e2e = {"value": world * S * n * args.e2e_steps / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
+               "note": "H2D of every stream's LR+residual+MV+type from pinned host memory each step; D2H of the "
+                       "per-stream stats and anchor map; HR frames stay in HBM for the downstream encoder"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        r = cpu_sample(cfg, pool[0], synth.make_weights(4000, B, C, s))
+        cpu = {kk: r[kk] for kk in ("value", "unit", "cores", "kind", "sample")}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "bf16",
+                "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
+                        f"random-init per-stream weights of the NAS 'high' architecture)",
+                "config": {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{W}x{H} x{s} streams per GPU, "
+                                       f"B{B}/C{C}, n={n}, k={k} (top-k per stream)",
+                           "streams_per_gpu": S, "frames_per_step_per_gpu": S * n, "parallelism": f"streams x{world}",
+                           "l2": "inputs larger than L2 (~130 GB touched per step)", "sr_batch": args.sr_batch,
+                           "gen_s": round(t_gen, 1)},
+                "roofline": roofline, "rooflines": rl,
+                "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
+                             "anchors_per_step": int(ia_np.sum())},
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+                "quality": {"anchors": float(st[:, 1].sum()), "frames": float(st[:, 0].sum())}}
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def ns_arena_gb(cfg, nb):
+    h, w, C, s = cfg["h"], cfg["w"], cfg["n_ch"], cfg["scale"]
+    px = h * w * nb
+    return (px * 16 * 2 + 3 * px * C * 2 + px * s * s * C * 2) / (1 << 30)
+
+
+if __name__ == "__main__":
+    main()

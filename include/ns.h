@@ -171,6 +171,20 @@ NS_API ns_status ns_enhance_streams(ns_ctx *ctx, const ns_chunk *chunks, int S, 
    since the last reset (for the bench's gpu_launches claim). */
 NS_API uint64_t ns_launch_count(int reset);
 
+/* Per-kernel-family device time (profiling; off by default).  When enabled,
+   every launch wrapper brackets its kernel(s) with CUDA events on the call's
+   stream.  ns_profile_enable(1) clears and starts, (0) stops (records are kept).
+   ns_profile_read synchronises the recorded events and fills one entry per
+   family (out must hold >= 16 entries); returns the number written or < 0. */
+typedef struct {
+    char name[24];
+    uint64_t launches;     /* kernels launched                         */
+    uint64_t scopes;       /* event-bracketed launch groups             */
+    double total_ms;       /* summed device time of those groups        */
+} ns_prof_entry;
+NS_API int ns_profile_enable(int on);
+NS_API int ns_profile_read(ns_prof_entry *out, int max);
+
 /* Thread-local description of the last error (includes cudaGetErrorString for
    NS_ECUDA).  Never NULL. */
 NS_API const char *ns_last_error(void);

@@ -38,13 +38,18 @@ class NsSelectParams(ctypes.Structure):
                 ("group_residual", ctypes.c_int32), ("use_res_size", ctypes.c_int32)]
 
 
+class NsProfEntry(ctypes.Structure):
+    _fields_ = [("name", ctypes.c_char * 24), ("launches", ctypes.c_uint64), ("scopes", ctypes.c_uint64),
+                ("total_ms", ctypes.c_double)]
+
+
 class NsSrJob(ctypes.Structure):
     _fields_ = [("model", P), ("lr", P), ("w", ctypes.c_int32), ("h", ctypes.c_int32), ("hr_out", P)]
 
 
 EXPORTS = ["ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_blob_len",
            "ns_model_destroy", "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
-           "ns_launch_count", "ns_last_error"]
+           "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read"]
 
 _lib = None
 
@@ -77,6 +82,10 @@ def lib() -> ctypes.CDLL:
         L.ns_launch_count.argtypes = [i32]
         L.ns_launch_count.restype = ctypes.c_uint64
         L.ns_last_error.restype = ctypes.c_char_p
+        L.ns_profile_enable.argtypes = [i32]
+        L.ns_profile_enable.restype = i32
+        L.ns_profile_read.argtypes = [P, i32]
+        L.ns_profile_read.restype = i32
         for f in ("ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_destroy",
                   "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams"):
             getattr(L, f).restype = i32
@@ -95,6 +104,21 @@ def last_error() -> str:
 
 def launch_count(reset: bool = False) -> int:
     return int(lib().ns_launch_count(1 if reset else 0))
+
+
+def profile_enable(on: bool = True):
+    """Starts (clearing) / stops per-kernel-family event timing in the library."""
+    lib().ns_profile_enable(1 if on else 0)
+
+
+def profile_read() -> dict:
+    """{family: (launches, groups, total_ms)} over the recorded launches (syncs)."""
+    arr = (NsProfEntry * 32)()
+    n = lib().ns_profile_read(arr, 32)
+    if n < 0:
+        raise NsError(n, "ns_profile_read", last_error())
+    return {arr[i].name.decode(): (int(arr[i].launches), int(arr[i].scopes), float(arr[i].total_ms))
+            for i in range(n)}
 
 
 def _ptr(t) -> Optional[int]:

@@ -31,6 +31,7 @@ __global__ void k_golden_index(const StreamDesc *sd, int S, int n, int16_t *gold
 }
 
 cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st) {
+    KScope ks(F_RECON, st);
     k_golden_index<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, gold_idx);
     return cudaGetLastError();
 }
@@ -112,6 +113,7 @@ __global__ void __launch_bounds__(kReconThreads)
 cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, int maxW8, int maxH,
                               const uint8_t *is_anchor, uint8_t *const *d_hr_table, const int16_t *gold_idx,
                               cudaStream_t st) {
+    KScope ks(F_RECON, st);
     dim3 g((maxW8 + kReconThreads - 1) / kReconThreads, maxH, S);
     k_recon_step<<<g, kReconThreads, 0, st>>>(d_sd, n, f, is_anchor, d_hr_table, gold_idx);
     return cudaGetLastError();
@@ -142,6 +144,7 @@ __global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st) {
     const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
+    KScope ks(F_STATE, st);
     dim3 g(blocks < 1 ? 1 : (blocks > 4096 ? 4096 : blocks), S, 2);
     k_state_copy<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, gold_idx);
     return cudaGetLastError();
@@ -199,6 +202,7 @@ __global__ void k_stats_final(const StreamDesc *sd, int S, int n, double *stats)
 
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
                          uint8_t *const *d_hr_table, size_t max_hr_bytes, double *stats, cudaStream_t st) {
+    KScope ks(F_STATS, st, 3);
     k_stats_meta<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, score, stats);
     const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
     dim3 g(blocks < 1 ? 1 : (blocks > 1024 ? 1024 : blocks), S * n);
@@ -242,11 +246,11 @@ __global__ void k_repack_b(const uint16_t *blob, size_t src_off, LayerShape ls, 
 }
 
 cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint8_t *packed, cudaStream_t st) {
+    KScope ks(F_REPACK, st, model_num_layers(n_blocks));
     size_t src = 0;
     for (int l = 0; l < model_num_layers(n_blocks); l++) {
         LayerShape ls = model_layer(n_blocks, C, s, l);
         k_repack_b<<<256, 256, 0, st>>>(blob, src, ls, C, s, packed);
-        count_launch();
         src += (size_t)ls.cout_real * ls.cin_real * 9 + ls.cout_real;
     }
     return cudaGetLastError();

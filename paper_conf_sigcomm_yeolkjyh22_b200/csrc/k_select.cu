@@ -53,6 +53,7 @@ __global__ void __launch_bounds__(kScoreThreads) k_score(const StreamDesc *sd, i
 
 cudaError_t launch_score(const StreamDesc *d_sd, int S, int n, int max_frame_vec8, int64_t *score,
                          cudaStream_t st) {
+    KScope ks(F_SCORE, st);
     cudaError_t e = cudaMemsetAsync(score, 0, sizeof(int64_t) * S * n, st);
     if (e != cudaSuccess) return e;
     const int per = kScoreThreads * kScoreUnroll;
@@ -160,6 +161,7 @@ __global__ void __launch_bounds__(kSelWarps * 32)
 
 cudaError_t launch_select(const StreamDesc *d_sd, const int64_t *score, int S, int n, int k, int fresh,
                           int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order, cudaStream_t st) {
+    KScope ks(F_SELECT, st);
     k_select<<<(S + kSelWarps - 1) / kSelWarps, kSelWarps * 32, 0, st>>>(d_sd, score, S, n, k, fresh, gain, rank,
                                                                         is_anchor, order);
     return cudaGetLastError();
@@ -237,6 +239,7 @@ __global__ void k_global_mark(int N, const int32_t *grank, const int32_t *cut, i
 cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *gain, const int32_t *order,
                           const int64_t *cost, int64_t budget, int32_t *grank, int32_t *pos_stream,
                           int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st) {
+    KScope ks(F_GLOBAL, st, 3);
     const int N = S * n;
     // rank currently holds the per-stream rank (written by k_select)
     k_global_rank<<<(N + 255) / 256, 256, 0, st>>>(d_sd, S, n, gain, order, rank, grank, pos_stream);
@@ -272,6 +275,7 @@ cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *
                            uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups, int topk,
                            int k, cudaStream_t st) {
     (void)k;
+    KScope ks(F_COMPACT, st);
     if (!topk) {
         cudaError_t e = cudaMemsetAsync(job_count, 0, sizeof(int32_t) * n_groups, st);
         if (e != cudaSuccess) return e;

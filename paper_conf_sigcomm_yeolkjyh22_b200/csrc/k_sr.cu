@@ -364,7 +364,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
 }
 
 template <int CIN, int NT, int NSPLIT, int EPI>
-static cudaError_t conv(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+static cudaError_t conv(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = ConvCfg<CIN, NT, NSPLIT>;
     static bool attr = false;
     if (!attr) {
@@ -376,6 +376,7 @@ static cudaError_t conv(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream
     args.n_xtiles = (args.W + kTile - 1) / kTile;
     args.rows_per_cta = kRows;
     dim3 grid(args.n_xtiles, (args.H + kRows - 1) / kRows, nj);
+    KScope ks(fam, st);
     k_conv3x3<CIN, NT, NSPLIT, EPI><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
     return cudaGetLastError();
 }
@@ -387,8 +388,8 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     cudaError_t e;
     {
         dim3 g((h * w + 255) / 256, nj);
+        KScope ks(F_SR_PREP, st);
         k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0);
-        count_launch();
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     ConvArgs base{};
@@ -397,21 +398,21 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
-        if ((e = conv<16, C, 1, EPI_STORE>(a->tm_x0, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv<16, C, 1, EPI_STORE>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     for (int b = 0; b < n_blocks; b++) {
         const CUtensorMap &hin = (b == 0) ? a->tm_h0 : a->tm_hb;
         const uint16_t *hres = (b == 0) ? a->h0 : a->hb;
         ConvArgs g = base; LayerShape l1 = L(1 + 2 * b), l2 = L(2 + 2 * b);
         g.b_off = l1.b_off; g.bias_off = l1.bias_off; g.out = a->tb;
-        if ((e = conv<C, C, 1, EPI_RELU>(hin, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv<C, C, 1, EPI_RELU>(F_SR_BODY, hin, g, nj, st)) != cudaSuccess) return e;
         g = base; g.b_off = l2.b_off; g.bias_off = l2.bias_off; g.out = a->hb; g.resid = hres;
-        if ((e = conv<C, C, 1, EPI_RESID>(a->tm_tb, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv<C, C, 1, EPI_RESID>(F_SR_BODY, a->tm_tb, g, nj, st)) != cudaSuccess) return e;
     }
     {   // end: h0 + conv(h; W_end) -> tb
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 1);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->tb; g.resid = a->h0;
-        if ((e = conv<C, C, 1, EPI_RESID>(n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv<C, C, 1, EPI_RESID>(F_SR_END, n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
     }
     {   // upsampler conv + pixel shuffle -> u (HR)
         LayerShape ls = L(2 * n_blocks + 2);
@@ -419,20 +420,20 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         const int ntot = s * s * C;
         if (ntot <= 256) {
             g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
-            if (C == 16 && s == 2) e = conv<C, 64, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
-            else if (C == 16 && s == 3) e = conv<C, 144, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
-            else if (C == 16 && s == 4) e = conv<C, 256, 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
-            else e = conv<C, (C == 32 ? 128 : 64), 1, EPI_SHUFFLE>(a->tm_tb, g, nj, st);  // C=32, s=2
+            if (C == 16 && s == 2) e = conv<C, 64, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
+            else if (C == 16 && s == 3) e = conv<C, 144, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
+            else if (C == 16 && s == 4) e = conv<C, 256, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
+            else e = conv<C, (C == 32 ? 128 : 64), 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);  // C=32, s=2
         } else if (ntot == 288) {  // C = 32, s = 3: two N tiles of 144 in one launch
             g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
-            e = conv<C, 144, 2, EPI_SHUFFLE>(a->tm_tb, g, nj, st);
+            e = conv<C, 144, 2, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
         } else {                   // C = 32, s = 4: two launches of N = 256
             for (int sp = 0; sp < 2 && e == cudaSuccess; sp++) {
                 ConvArgs g2 = g;
                 g2.b_off = ls.b_off + (size_t)sp * 9 * C * 256 * 2;
                 g2.bias_off = ls.bias_off + (size_t)sp * 256 * 4;
                 g2.sub0 = sp * 8;
-                e = conv<C, 256, 1, EPI_SHUFFLE>(a->tm_tb, g2, nj, st);
+                e = conv<C, 256, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g2, nj, st);
             }
         }
         if (e != cudaSuccess) return e;
@@ -441,7 +442,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 3);
         g.H = h * s; g.W = w * s; g.lr_h = h; g.lr_w = w;
         g.b_off = ls.b_off; g.bias_off = ls.bias_off;
-        if ((e = conv<C, 16, 1, EPI_TAIL>(a->tm_u, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv<C, 16, 1, EPI_TAIL>(F_SR_TAIL, a->tm_u, g, nj, st)) != cudaSuccess) return e;
     }
     return cudaSuccess;
 }

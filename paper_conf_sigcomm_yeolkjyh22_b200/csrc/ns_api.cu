@@ -6,6 +6,7 @@
 #include <cstdio>
 #include <cstring>
 #include <atomic>
+#include <mutex>
 #include <algorithm>
 #include <map>
 #include <tuple>
@@ -34,8 +35,50 @@ static ns_status cuda_fail(cudaError_t e, const char *where) {
         if (_e != cudaSuccess) return cuda_fail(_e, #call);     \
     } while (0)
 
+namespace {
+struct ProfRec {
+    int fam;
+    int n;
+    cudaEvent_t e0, e1;
+};
+std::mutex g_pmu;
+std::atomic<bool> g_prof{false};
+std::vector<ProfRec> g_recs;
+std::vector<cudaEvent_t> g_evpool;
+cudaEvent_t ev_get() {
+    if (!g_evpool.empty()) {
+        cudaEvent_t e = g_evpool.back();
+        g_evpool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+const char *kFamNames[] = {"score", "select", "global", "compact", "sr_prep", "sr_head", "sr_body", "sr_end",
+                           "sr_up", "sr_tail", "recon", "state", "stats", "repack"};
+}  // namespace
+
 namespace ns {
-void count_launch(int n) { g_launches.fetch_add((uint64_t)n, std::memory_order_relaxed); }
+const char *fam_name(int fam) { return (fam >= 0 && fam < F_COUNT) ? kFamNames[fam] : "?"; }
+
+KScope::KScope(int fam_, cudaStream_t st_, int n_) : fam(fam_), n(n_), st(st_), rec(nullptr) {
+    g_launches.fetch_add((uint64_t)n, std::memory_order_relaxed);
+    if (g_prof.load(std::memory_order_relaxed)) {
+        std::lock_guard<std::mutex> lk(g_pmu);
+        ProfRec *r = new ProfRec{fam, n, ev_get(), ev_get()};
+        cudaEventRecord(r->e0, st);
+        rec = r;
+    }
+}
+KScope::~KScope() {
+    if (!rec) return;
+    ProfRec *r = static_cast<ProfRec *>(rec);
+    cudaEventRecord(r->e1, st);
+    std::lock_guard<std::mutex> lk(g_pmu);
+    g_recs.push_back(*r);
+    delete r;
+}
 
 // ------------------------------------------------------------------ model layout
 int model_num_layers(int n_blocks) { return 2 * n_blocks + 4; }
@@ -258,6 +301,38 @@ extern "C" uint64_t ns_launch_count(int reset) {
     return reset ? g_launches.exchange(0) : g_launches.load();
 }
 extern "C" const char *ns_last_error(void) { return g_err; }
+
+extern "C" int ns_profile_enable(int on) {
+    std::lock_guard<std::mutex> lk(g_pmu);
+    if (on) {  // start: drop previous records; stop: keep them for ns_profile_read
+        for (auto &r : g_recs) {
+            g_evpool.push_back(r.e0);
+            g_evpool.push_back(r.e1);
+        }
+        g_recs.clear();
+    }
+    g_prof.store(on != 0);
+    return NS_OK;
+}
+
+extern "C" int ns_profile_read(ns_prof_entry *out, int max) {
+    if (!out || max < (int)F_COUNT) return fail(NS_EINVAL, "ns_profile_read: need room for %d entries", (int)F_COUNT);
+    std::lock_guard<std::mutex> lk(g_pmu);
+    for (int f = 0; f < F_COUNT; f++) {
+        memset(&out[f], 0, sizeof(ns_prof_entry));
+        snprintf(out[f].name, sizeof(out[f].name), "%s", fam_name(f));
+    }
+    for (auto &r : g_recs) {
+        float ms = 0.f;
+        cudaError_t e = cudaEventSynchronize(r.e1);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.e0, r.e1);
+        if (e != cudaSuccess) return cuda_fail(e, "ns_profile_read");
+        out[r.fam].launches += (uint64_t)r.n;
+        out[r.fam].scopes += 1;
+        out[r.fam].total_ms += ms;
+    }
+    return (int)F_COUNT;
+}
 
 // ------------------------------------------------------------------ validation
 static bool al16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
