@@ -3,6 +3,7 @@
 // (K10) and the model weight repack (model pre-optimisation, §6.2).
 #include <cstdint>
 #include "ns_internal.h"
+#include "ptx.cuh"
 
 namespace ns {
 
@@ -36,27 +37,299 @@ cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *g
     return cudaGetLastError();
 }
 
-// One frame step f for all streams.  Each thread produces 8 consecutive HR
-// pixels of one row (inside one 8x8 LR block, since 8s % 8 == 0) on all three
-// planes:  anchor -> skip (SR output already in place); KEY or INTRA block ->
-// up_s(LR[f]); otherwise clamp(warp_{s*mv}(HR[ref]) + up_s(res[f]), 0, 255).
-constexpr int kReconThreads = 128;
-__global__ void __launch_bounds__(kReconThreads)
+// One frame step f for all streams (K9).  A thread owns one LR block column
+// (8s HR pixels wide, the motion vector is uniform there) x 8 HR rows x 3
+// planes:  anchor -> skip (SR output already in place); KEY frame or INTRA
+// block -> up_s(LR[f]); otherwise clamp(warp_{s*mv}(HR[ref]) + up_s(res[f])).
+// The warp (O7) runs two pixels per 32-bit register (16-bit lanes; every
+// intermediate < 2^16): each horizontal pass over a reference row is shared by
+// the two output rows that use it.  up_s (O6) is separable with compile-time
+// taps (the thread's first pixel is a multiple of s).  Reference windows are
+// read with aligned 64-bit loads (edge blocks fall back to clamped byte loads).
+template <int S>
+struct ReconCfg {
+    static constexpr int BW = 8 * S;               // HR pixels per thread row
+    static constexpr int NP = BW / 2;              // 16-bit pairs per row
+    static constexpr int WIN = BW + 1;             // reference bytes per row
+    static constexpr int NQ = (7 + WIN + 7) / 8;   // aligned 64-bit words per row
+    static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
+    static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
+                                                   // or of 8s/.. so that Y0 mod S == 0
+};
+
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+    return r;
+}
+
+// Stage the raw aligned 64-bit words covering reference bytes xs .. xs+BW of
+// one row into shared memory (cp.async for interior windows; edge blocks use
+// clamped byte loads that emulate the same aligned words).  dst[i * stride]
+// is word i (struct-of-arrays across the CTA's threads: conflict-free reads).
+template <int S>
+__device__ __noinline__ void recon_row_stage_edge(const uint8_t *row, int xs, int W, uint2 *dst, int stride) {
+    using Cfg = ReconCfg<S>;
+    const int xb = xs & ~7;
+    for (int i = 0; i < Cfg::NQ; i++) {
+        uint32_t v0 = 0, v1 = 0;
+        for (int b = 0; b < 4; b++) {
+            v0 |= (uint32_t)row[min(max(xb + 8 * i + b, 0), W - 1)] << (8 * b);
+            v1 |= (uint32_t)row[min(max(xb + 8 * i + 4 + b, 0), W - 1)] << (8 * b);
+        }
+        dst[i * stride] = make_uint2(v0, v1);
+    }
+}
+
+template <int S>
+__device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int W, bool interior, uint2 *dst,
+                                                int stride) {
+    using Cfg = ReconCfg<S>;
+    if (interior) {
+        const int xb = xs & ~7;
+#pragma unroll
+        for (int i = 0; i < Cfg::NQ; i++)
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + i * stride)),
+                         "l"(row + xb + 8 * i)
+                         : "memory");
+    } else {
+        recon_row_stage_edge<S>(row, xs, W, dst, stride);
+    }
+}
+
+// Horizontal bilinear pass over one reference row: h[k] = packed pixels
+// (2k, 2k+1) of (R[x](8-fx) + R[x+1]fx + 4) >> 3 for x = xs .. xs+BW-1.
+template <int S>
+__device__ __forceinline__ void recon_hpass(const uint2 (&q)[ReconCfg<S>::NQ], int xs, uint32_t fxc, uint32_t fx,
+                                            uint32_t (&h)[ReconCfg<S>::NP]) {
+    using Cfg = ReconCfg<S>;
+    uint32_t w[2 * Cfg::NQ + 2];
+#pragma unroll
+    for (int i = 0; i < Cfg::NQ; i++) {
+        w[2 * i] = q[i].x;
+        w[2 * i + 1] = q[i].y;
+    }
+    w[2 * Cfg::NQ] = 0;
+    w[2 * Cfg::NQ + 1] = 0;
+    const int m = xs & 7;
+    if (m >= 4) {
+#pragma unroll
+        for (int i = 0; i < 2 * Cfg::NQ + 1; i++) w[i] = w[i + 1];
+    }
+    const uint32_t sh = 8u * (uint32_t)(m & 3);
+    uint32_t A[Cfg::NP + 2];
+#pragma unroll
+    for (int i = 0; i < Cfg::NA32; i++) {
+        const uint32_t a = __funnelshift_r(w[i], w[i + 1], sh);
+        A[2 * i] = prmt(a, 0u, 0x4140u);
+        if (2 * i + 1 < Cfg::NP + 2) A[2 * i + 1] = prmt(a, 0u, 0x4342u);
+    }
+#pragma unroll
+    for (int k = 0; k < Cfg::NP; k++) {
+        const uint32_t B = __funnelshift_r(A[k], A[k + 1], 16);
+        h[k] = ((A[k] * fxc + B * fx + 0x00040004u) >> 3) & 0x1FFF1FFFu;
+    }
+}
+
+// Raw LR-row data for columns 8bx-1 .. 8bx+8: the aligned middle 8 values
+// (16 B of int16 or 8 B of u8, zero-extended) plus the two clamped edges.
+struct LrRaw {
+    uint4 mid;
+    int left, right;
+};
+__device__ __forceinline__ void recon_lr_load(const void *plane, bool is_u8, int row, int bx, int w, LrRaw &r) {
+    if (is_u8) {
+        const uint8_t *p = static_cast<const uint8_t *>(plane) + (size_t)row * w;
+        const uint2 q = __ldg(reinterpret_cast<const uint2 *>(p + 8 * bx));
+        r.mid = make_uint4(q.x, q.y, 0, 0);
+        r.left = p[max(8 * bx - 1, 0)];
+        r.right = p[min(8 * bx + 8, w - 1)];
+    } else {
+        const int16_t *p = static_cast<const int16_t *>(plane) + (size_t)row * w;
+        r.mid = __ldg(reinterpret_cast<const uint4 *>(p + 8 * bx));
+        r.left = p[max(8 * bx - 1, 0)];
+        r.right = p[min(8 * bx + 8, w - 1)];
+    }
+}
+__device__ __forceinline__ void recon_lr_unpack(const LrRaw &r, bool is_u8, int (&v)[10]) {
+    v[0] = r.left;
+    v[9] = r.right;
+    if (is_u8) {
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            v[1 + i] = (r.mid.x >> (8 * i)) & 255;
+            v[5 + i] = (r.mid.y >> (8 * i)) & 255;
+        }
+    } else {
+        const uint32_t qq[4] = {r.mid.x, r.mid.y, r.mid.z, r.mid.w};
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            v[1 + 2 * i] = (int)(int16_t)(qq[i] & 0xFFFFu);
+            v[2 + 2 * i] = (int)(int16_t)(qq[i] >> 16);
+        }
+    }
+}
+
+constexpr int kReconTX = 32, kReconTY = 4;
+
+__device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
+    uint32_t r;
+    asm("max.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+    return r;
+}
+__device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
+    uint32_t r;
+    asm("min.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+    return r;
+}
+
+// Compile-time O6 taps.  For an axis coordinate X = S*m + ph + i:
+//   u = 2X + 1 - S, x0 = m + floor((2(ph+i) + 1 - S) / 2S), w1 = round(128 rem / 2S).
+__host__ __device__ constexpr int fdiv(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+template <int S>
+__host__ __device__ constexpr int tap_d(int k) { return fdiv(2 * k + 1 - S, 2 * S); }
+template <int S>
+__host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S) - 2 * S * tap_d<S>(k)) + S) / (2 * S); }
+
+// All three planes of one thread's 8s x 8 tile; PH = Y0 mod S (compile time).
+template <int S>
+__device__ __forceinline__ void recon_planes(const StreamDesc &d, bool use_lr, const uint8_t *ref, const uint8_t *lr_f,
+                                             const int16_t *res_f, uint8_t *out, size_t lrp, size_t hrp, int H, int W,
+                                             int bx, int X0, int Y0, int Y0m, int xs, int iy0, bool interior,
+                                             uint32_t fxc, uint32_t fxp, uint32_t fyc, uint32_t fyp) {
+    using Cfg = ReconCfg<S>;
+    constexpr int BW = Cfg::BW, NP = Cfg::NP;
+    constexpr int RPT = Cfg::RPT;
+    constexpr int DMIN = tap_d<S>(0), DMAX = tap_d<S>(S - 1) + 1;
+    constexpr int NLR = DMAX - DMIN + 1 + (RPT / S - 1);  // LR rows: one period's window + slides
+    static_assert(RPT % S == 0, "row groups are whole periods");
+    constexpr int NT = kReconTX * kReconTY;
+    extern __shared__ __align__(16) uint2 rsm[];  // [2 planes][9 rows][NQ words][NT threads]
+    const int tid = threadIdx.y * kReconTX + threadIdx.x;
+    auto stage = [&](int c) {
+        if (use_lr) return;
+        const uint8_t *P = ref + c * hrp;
+        uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * Cfg::NQ * NT + tid;
+#pragma unroll
+        for (int j = 0; j <= RPT; j++) {
+            const int r = min(max(iy0 + j, 0), H - 1);
+            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior && !(c == 2 && r == H - 1),
+                               buf + j * Cfg::NQ * NT, NT);
+        }
+    };
+    stage(0);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+#pragma unroll 1
+    for (int c = 0; c < 3; c++) {
+        if (c + 1 < 3) stage(c + 1);
+        asm volatile("cp.async.commit_group;" ::: "memory");
+        const void *src = use_lr ? static_cast<const void *>(lr_f + c * lrp) : static_cast<const void *>(res_f + c * lrp);
+        int lv[NLR][10];
+#pragma unroll
+        for (int t = 0; t < NLR; t++) {
+            LrRaw raw;
+            recon_lr_load(src, use_lr, min(max(Y0m + DMIN + t, 0), d.h - 1), bx, d.w, raw);
+            recon_lr_unpack(raw, use_lr, lv[t]);
+        }
+        asm volatile("cp.async.wait_group 1;" ::: "memory");  // this plane's windows have landed
+        const uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * Cfg::NQ * NT + tid;
+        auto row = [&](int j, uint2 (&q)[Cfg::NQ]) {
+#pragma unroll
+            for (int i = 0; i < Cfg::NQ; i++) q[i] = buf[(j * Cfg::NQ + i) * NT];
+        };
+        uint32_t hprev[NP], hcur[NP];
+        if (!use_lr) {
+            uint2 q[Cfg::NQ];
+            row(0, q);
+            recon_hpass<S>(q, xs, fxc, fxp, hprev);
+        }
+#pragma unroll 1
+        for (int it = 0; it < RPT / S; it++) {
+#pragma unroll
+            for (int jj = 0; jj < S; jj++) {  // one period of the vertical O6 taps
+                const int j = it * S + jj;
+                uint32_t pred[NP];
+                if (!use_lr) {
+                    uint2 q[Cfg::NQ];
+                    row(j + 1, q);
+                    recon_hpass<S>(q, xs, fxc, fxp, hcur);
+#pragma unroll
+                    for (int k = 0; k < NP; k++) {
+                        pred[k] = ((hprev[k] * fyc + hcur[k] * fyp + 0x00040004u) >> 3) & 0x1FFF1FFFu;
+                        hprev[k] = hcur[k];
+                    }
+                } else {
+#pragma unroll
+                    for (int k = 0; k < NP; k++) pred[k] = 0;
+                }
+                // up_s of the residual (or LR) plane at row Y0 + j (O6), compile-time taps;
+                // lv[0] holds LR row Y0/S + DMIN + it (the window slides one LR row per period)
+                const int ta = tap_d<S>(jj) - DMIN;
+                const int wy = tap_w1<S>(jj);
+                // per LR column t: V = (128-wy) a + wy b (vertical, exact); the
+                // horizontal tap of pixel i is 128 V[d] + w1 (V[d+1] - V[d]).  Scaled
+                // by 4 with the rounding constant and the +256 lane bias folded in, the
+                // value r + 256 lands in the high half-word: one IMAD per pixel and one
+                // PRMT per pixel pair.
+                int base[10], dlt[9];
+#pragma unroll
+                for (int t = 0; t < 10; t++) {
+                    const int V = (128 - wy) * lv[ta][t] + wy * lv[ta + 1][t];
+                    base[t] = V * 512 + 4 * (8192 + (256 << 14));
+                }
+#pragma unroll
+                for (int t = 0; t < 9; t++) dlt[t] = base[t + 1] - base[t];
+                uint32_t o[BW / 4];
+#pragma unroll
+                for (int qd = 0; qd < BW / 4; qd++) {
+                    uint32_t pr[2];
+#pragma unroll
+                    for (int hh = 0; hh < 2; hh++) {
+                        const int i0 = 4 * qd + 2 * hh;
+                        const int d0 = tap_d<S>(i0) + 1, d1 = tap_d<S>(i0 + 1) + 1;
+                        const int w0 = tap_w1<S>(i0), w1 = tap_w1<S>(i0 + 1);
+                        // (base + w1 * dlt / 128): dlt is a multiple of 512, so w1*dlt/128 = w1*(dlt/128) exactly
+                        const uint32_t s0 = (uint32_t)(base[d0] + (w0 ? w0 * (dlt[d0] >> 7) : 0));
+                        const uint32_t s1 = (uint32_t)(base[d1] + (w1 ? w1 * (dlt[d1] >> 7) : 0));
+                        uint32_t x = prmt(s0, s1, 0x7632u);  // [r0 + 256, r1 + 256]
+                        x += pred[i0 >> 1];                   // in [1, 766] per lane
+                        pr[hh] = vmin_u16x2(vmax_u16x2(x, 0x01000100u), 0x01FF01FFu);  // clamp to [256, 511]
+                    }
+                    o[qd] = prmt(pr[0], pr[1], 0x6420u);  // low bytes = clamped value (x - 256)
+                }
+                uint2 *dst = reinterpret_cast<uint2 *>(out + c * hrp + (size_t)(Y0 + j) * W + X0);
+#pragma unroll
+                for (int qd = 0; qd < BW / 8; qd++) dst[qd] = make_uint2(o[2 * qd], o[2 * qd + 1]);
+            }
+#pragma unroll
+            for (int t = 0; t + 1 < NLR; t++)
+#pragma unroll
+                for (int e = 0; e < 10; e++) lv[t][e] = lv[t + 1][e];
+        }
+    }
+}
+
+template <int S>
+__global__ void __launch_bounds__(kReconTX *kReconTY, 3)
     k_recon_step(const StreamDesc *sd, int n, int f, const uint8_t *is_anchor, uint8_t *const *hr_tab,
                  const int16_t *gold) {
+    using Cfg = ReconCfg<S>;
+    constexpr int BW = Cfg::BW, NP = Cfg::NP;
     const int sid = blockIdx.z;
     if (is_anchor[(size_t)sid * n + f]) return;
     const StreamDesc d = sd[sid];
-    const int s = d.s, H = d.h * s, W = d.w * s;
-    const int Y = blockIdx.y;
-    const int X0 = (blockIdx.x * kReconThreads + threadIdx.x) * 8;
-    if (Y >= H || X0 >= W) return;
+    if (d.s != S) return;
+    const int H = d.h * S, W = d.w * S;
+    const int bx = blockIdx.x * kReconTX + threadIdx.x;  // LR block column
+    const int rg = blockIdx.y * kReconTY + threadIdx.y;  // group of RPT HR rows
+    const int X0 = bx * BW, Y0 = rg * Cfg::RPT;
+    if (X0 >= W || Y0 >= H) return;
     const int bw = d.w / 8;
-    const ns_block_mv mv = d.mv[(size_t)f * (d.h / 8) * bw + (size_t)(Y / (8 * s)) * bw + X0 / (8 * s)];
-    const uint8_t type = d.type[f];
+    const ns_block_mv mv = d.mv[(size_t)f * (d.h / 8) * bw + (size_t)(Y0 / BW) * bw + bx];
+    const bool key = d.type[f] == NS_KEY;
+    const bool use_lr = key || mv.ref == NS_REF_INTRA;
     uint8_t *out = hr_tab[d.hr_base + f];
     const size_t lrp = (size_t)d.h * d.w, hrp = (size_t)H * W;
-    const bool use_lr = (type == NS_KEY) || (mv.ref == NS_REF_INTRA);
     const uint8_t *ref = nullptr;
     if (!use_lr) {
         if (mv.ref == NS_REF_GOLDEN) {
@@ -66,56 +339,58 @@ __global__ void __launch_bounds__(kReconThreads)
             ref = f > 0 ? hr_tab[d.hr_base + f - 1] : d.hr_last;
         }
     }
-    int ya, yb, wy;
-    up_tap_r(Y, s, d.h, ya, yb, wy);
-    int xa[8], xb[8], wx[8];
-#pragma unroll
-    for (int i = 0; i < 8; i++) up_tap_r(X0 + i, s, d.w, xa[i], xb[i], wx[i]);
     // warp geometry (O7): m = s * mv in 1/8 HR pel
-    const int mx = s * mv.mvx, my = s * mv.mvy;
-    const int ix = X0 + (mx >> 3), fx = mx & 7;
-    const int iy = Y + (my >> 3), fy = my & 7;
-    const int r0 = min(max(iy, 0), H - 1), r1 = min(max(iy + 1, 0), H - 1);
-#pragma unroll
-    for (int c = 0; c < 3; c++) {
-        uint32_t o[2] = {0, 0};
-        if (use_lr) {
-            const uint8_t *L = d.lr + ((size_t)f * 3 + c) * lrp;
-            const uint8_t *La = L + (size_t)ya * d.w, *Lb = L + (size_t)yb * d.w;
-#pragma unroll
-            for (int i = 0; i < 8; i++) {
-                const int v = (128 - wy) * ((128 - wx[i]) * La[xa[i]] + wx[i] * La[xb[i]]) +
-                              wy * ((128 - wx[i]) * Lb[xa[i]] + wx[i] * Lb[xb[i]]);
-                o[i >> 2] |= (uint32_t)((v + 8192) >> 14) << (8 * (i & 3));
-            }
-        } else {
-            const int16_t *Rp = d.res + ((size_t)f * 3 + c) * lrp;
-            const int16_t *Ra = Rp + (size_t)ya * d.w, *Rb = Rp + (size_t)yb * d.w;
-            const uint8_t *P = ref + c * hrp;
-            const uint8_t *P0 = P + (size_t)r0 * W, *P1 = P + (size_t)r1 * W;
-#pragma unroll
-            for (int i = 0; i < 8; i++) {
-                const int xa_ = min(max(ix + i, 0), W - 1), xb_ = min(max(ix + i + 1, 0), W - 1);
-                const int h0 = (P0[xa_] * (8 - fx) + P0[xb_] * fx + 4) >> 3;
-                const int h1 = (P1[xa_] * (8 - fx) + P1[xb_] * fx + 4) >> 3;
-                const int pred = (h0 * (8 - fy) + h1 * fy + 4) >> 3;
-                const int v = (128 - wy) * ((128 - wx[i]) * Ra[xa[i]] + wx[i] * Ra[xb[i]]) +
-                              wy * ((128 - wx[i]) * Rb[xa[i]] + wx[i] * Rb[xb[i]]);
-                const int r = (v + 8192) >> 14;
-                const int val = min(max(pred + r, 0), 255);
-                o[i >> 2] |= (uint32_t)val << (8 * (i & 3));
-            }
-        }
-        *reinterpret_cast<uint2 *>(out + c * hrp + (size_t)Y * W + X0) = make_uint2(o[0], o[1]);
-    }
+    const int mx = S * mv.mvx, my = S * mv.mvy;
+    const int xs = X0 + (mx >> 3);
+    const uint32_t fx = (uint32_t)(mx & 7), fy = (uint32_t)(my & 7);
+    // packed 2 x 16-bit arithmetic multiplies by a SCALAR (no cross-lane terms)
+    const uint32_t fxp = fx, fyp = fy, fxc = 8u - fx, fyc = 8u - fy;
+    const int iy0 = Y0 + (my >> 3);
+    // All used bytes inside the row -> aligned vector loads (they may run up to
+    // 8*NQ - BW - 1 bytes past the row end, which stays inside the plane except
+    // on the very last row of plane 2; recon_planes routes that row to the
+    // clamped path).
+    const bool interior = xs >= 0 && xs + BW <= W - 1;
+    const uint8_t *lr_f = d.lr + (size_t)f * 3 * lrp;
+    const int16_t *res_f = d.res + (size_t)f * 3 * lrp;
+
+    recon_planes<S>(d, use_lr, ref, lr_f, res_f, out, lrp, hrp, H, W, bx, X0, Y0, Y0 / S, xs, iy0, interior, fxc,
+                    fxp, fyc, fyp);
 }
 
-cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, int maxW8, int maxH,
-                              const uint8_t *is_anchor, uint8_t *const *d_hr_table, const int16_t *gold_idx,
-                              cudaStream_t st) {
-    KScope ks(F_RECON, st);
-    dim3 g((maxW8 + kReconThreads - 1) / kReconThreads, maxH, S);
-    k_recon_step<<<g, kReconThreads, 0, st>>>(d_sd, n, f, is_anchor, d_hr_table, gold_idx);
+template <int S>
+static size_t recon_smem() {
+    return (size_t)2 * (ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconTX * kReconTY * sizeof(uint2);
+}
+
+template <int S>
+static void recon_launch(dim3 g, cudaStream_t st, const StreamDesc *d_sd, int n, int f, const uint8_t *is_anchor,
+                         uint8_t *const *hr, const int16_t *gold) {
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)recon_smem<S>());
+        attr = true;
+    }
+    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), recon_smem<S>(), st>>>(d_sd, n, f, is_anchor, hr, gold);
+}
+
+cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const int *max_lr_w,
+                              const int *max_lr_h, const uint8_t *is_anchor, uint8_t *const *d_hr_table,
+                              const int16_t *gold_idx, cudaStream_t st) {
+    int nl = 0;
+    for (int s = 2; s <= 4; s++) nl += max_lr_w[s] > 0;
+    KScope ks(F_RECON, st, nl);
+    for (int s = 2; s <= 4; s++) {
+        if (max_lr_w[s] <= 0) continue;
+        const int nbx = max_lr_w[s] / 8;          // LR block columns
+        const int nrg = max_lr_h[s] * s / (s == 3 ? 6 : 8);  // groups of RPT HR rows
+        dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
+        dim3 b(kReconTX, kReconTY);
+        (void)b;
+        if (s == 2) recon_launch<2>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
+        if (s == 3) recon_launch<3>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
+        if (s == 4) recon_launch<4>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
+    }
     return cudaGetLastError();
 }
 
@@ -216,8 +491,27 @@ cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is
 // bias) -> per-layer UMMA B operand [split][tap][kc][kh][n][8] bf16 + fp32 bias.
 __global__ void k_repack_b(const uint16_t *blob, size_t src_off, LayerShape ls, int C, int s, uint8_t *packed) {
     const size_t NT = ls.ntot / ls.nsplit;
-    const size_t total = (size_t)9 * ls.cin * ls.ntot;
     uint16_t *B = reinterpret_cast<uint16_t *>(packed + ls.b_off);
+    if (ls.rot) {  // [dx 3][kc][kh 2][5 nb][8], strip of kernel rows dy = 2,1,0,2,1
+        const int KC = ls.cin / 16, nb = ls.nb;
+        const size_t total = (size_t)3 * KC * 2 * 5 * nb * 8;
+        const int strip[5] = {2, 1, 0, 2, 1};
+        for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total;
+             e += (size_t)gridDim.x * blockDim.x) {
+            const int k8 = e % 8;
+            const int nn = (e / 8) % (5 * nb);
+            const int kh = (e / (8 * 5 * nb)) % 2;
+            const int kc = (e / (16 * 5 * nb)) % KC;
+            const int dx = (int)(e / ((size_t)16 * 5 * nb * KC));
+            const int dy = strip[nn / nb], co = nn % nb;
+            const int ci = kc * 16 + kh * 8 + k8;
+            uint16_t v = 0;
+            if (ci < ls.cin_real && co < ls.cout_real)
+                v = blob[src_off + (((size_t)co * ls.cin_real + ci) * 3 + dy) * 3 + dx];
+            B[e] = v;
+        }
+    } else {
+    const size_t total = (size_t)9 * ls.cin * ls.ntot;
     for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (size_t)gridDim.x * blockDim.x) {
         const int k8 = e % 8;
         const int nn = (e / 8) % NT;
@@ -233,6 +527,7 @@ __global__ void k_repack_b(const uint16_t *blob, size_t src_off, LayerShape ls, 
             v = blob[src_off + (((size_t)co * ls.cin_real + ci) * 3 + tap / 3) * 3 + tap % 3];
         }
         B[e] = v;
+    }
     }
     float *bias = reinterpret_cast<float *>(packed + ls.bias_off);
     for (int cop = blockIdx.x * blockDim.x + threadIdx.x; cop < ls.ntot; cop += gridDim.x * blockDim.x) {

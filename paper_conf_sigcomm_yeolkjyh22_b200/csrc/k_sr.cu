@@ -167,6 +167,17 @@ __global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtenso
             else if (r + 1 < nrows) issue(r + 1);
         }
         __syncwarp();
+        // residual rows are prefetched before waiting for the MMA (latency overlap)
+        constexpr int RC = (EPI == EPI_RESID) ? NT / 8 : 1;
+        uint4 rres[RC];
+        if constexpr (EPI == EPI_RESID) {
+            if (x < a.W) {
+                const size_t rb = ((size_t)slot_job * a.H + (y0 + r)) * (NT / 8);
+#pragma unroll
+                for (int cg = 0; cg < RC; cg++)
+                    rres[cg] = __ldg(reinterpret_cast<const uint4 *>(a.resid + ((rb + cg) * a.W + x) * 8));
+            }
+        }
         mbar_wait(&bars[7 + (r % ACCB)], (r / ACCB) & 1);
         tc_fence_after();
         const uint32_t acc = tmem + (uint32_t)((r % ACCB) * NTOT) + ((uint32_t)(warp * 32) << 16);
@@ -196,7 +207,7 @@ __global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtenso
                     }
                     const size_t off = ((rowbase + cg) * a.W + x) * 8;
                     if (EPI == EPI_RESID) {
-                        const uint4 rr = *reinterpret_cast<const uint4 *>(a.resid + off);
+                        const uint4 rr = rres[cg];
                         f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
                         f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
                         f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
@@ -278,6 +289,206 @@ __global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtenso
         }
         tc_fence_before();
         __syncthreads();
+    }
+    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
+}
+
+// ------------------------------------------------------------------ rotated-accumulator conv
+// Measured on B200 (tools/ubench.cu): a K=16 tcgen05.mma with A from shared
+// memory costs max(64, N/2) cycles -- the 4 KB A tile is read at ~64 B/clk --
+// so a 32-channel conv (N = 32) can use at most 25% of the tensor cores.
+// Here each input row is read ONCE per 3x3 tap column dx and multiplied by the
+// weights of all three kernel rows at once: N = 3 x Cout.  The three partial
+// products land in three TMEM accumulator blocks that belong to the three
+// output rows the input row contributes to (y+1 via dy=0, y via dy=1, y-1 via
+// dy=2).  Output row r lives in block r mod 3; the B operand is a 5-block
+// strip [W_dy2; W_dy1; W_dy0; W_dy2; W_dy1] and the window start (1 - y mod 3)
+// mod 3 rotates the kernel rows onto the right blocks.  After input row y the
+// block of row y-1 is complete: the epilogue reads it, applies the fused
+// epilogue, and zeroes it for row y+2.  No im2col, no lane shifts, 128-pixel
+// tiles, N = 96 (C = 32) -> up to 3x the MMA efficiency of N = 32.
+template <int CIN, int NB>
+struct RotCfg {
+    static constexpr int KC = CIN / 16;
+    static constexpr uint32_t B_BYTES = 30u * CIN * NB;     // 3 dx x KC x 2 kh x 5NB rows x 16 B
+    static constexpr uint32_t BIAS_BYTES = NB * 4u;
+    static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
+    static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    static constexpr int NSLOT = 3;
+    static constexpr uint32_t TMEM_COLS = tmem_cols_for(3 * NB);
+    static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + 128;
+    static_assert((3 * NB) % 16 == 0 && 3 * NB <= 256, "N = 3 NB");
+    static_assert(SMEM <= 232448, "shared memory");
+};
+
+__device__ __forceinline__ int mod3(int v) { return ((v % 3) + 3) % 3; }
+
+template <int NB>
+__device__ __forceinline__ void tmem_zero(uint32_t taddr) {
+    if constexpr (NB == 32) {
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,"
+            "%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(taddr), "r"(0u) : "memory");
+    } else {
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1,%1};" ::"r"(
+                taddr), "r"(0u) : "memory");
+    }
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+template <int CIN, int NB, int EPI>
+__global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+    using Cfg = RotCfg<CIN, NB>;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *s_w = smem;
+    const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
+    uint8_t *s_ring = smem + Cfg::W_REGION;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + Cfg::NSLOT * Cfg::SLOT);  // [0,3) ring, 3 w, 4 mma
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 6);
+
+    const int slot_job = blockIdx.z;
+    const int job = a.j0 + slot_job;
+    if (a.job_count && job >= *a.job_count) return;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int x0 = blockIdx.x * kTile;
+    const int y0 = blockIdx.y * a.rows_per_cta;
+    const int y1 = min(y0 + a.rows_per_cta, a.H);
+    const int n_loads = y1 - y0 + 2;  // input rows y0-1 .. y1
+
+    if (tid == 0) {
+        for (int i = 0; i < 5; i++) mbar_init(&bars[i], 1);
+        fence_mbar_init();
+    }
+    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *s_tmem;
+    const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);  // this warp's TMEM lanes
+    const SrJob J = a.jobs[job];
+    if (tid == 0) {
+        prefetch_tmap(&tm_in);
+        mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
+        bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
+        bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
+        for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
+            mbar_arrive_expect_tx(&bars[q], Cfg::SLOT_BYTES);
+            tma_load_5d(s_ring + q * Cfg::SLOT, &tm_in, &bars[q], 0, x0 - 1, 0, y0 - 1 + q, slot_job);
+        }
+    }
+    // the three accumulator blocks start at zero
+    tmem_zero<NB>(tl);
+    tmem_zero<NB>(tl + NB);
+    tmem_zero<NB>(tl + 2 * NB);
+    tmem_wait_st();
+    mbar_wait(&bars[3], 0);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+
+    const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
+    const int p = warp * 32 + lane;
+    const int x = x0 + p;
+    for (int q = 0; q < n_loads; q++) {
+        const int yin = y0 - 1 + q;
+        if (tid == 0) {
+            const int sl = q % Cfg::NSLOT;
+            mbar_wait(&bars[sl], (q / Cfg::NSLOT) & 1);
+            tc_fence_after();
+            const uint32_t abase = smem_u32(s_ring + sl * Cfg::SLOT);
+            const uint32_t start = (uint32_t)mod3(1 - yin);  // rotation of the kernel rows
+            const uint32_t wbase = smem_u32(s_w) + start * NB * 16;
+#pragma unroll
+            for (int dx = 0; dx < 3; dx++) {
+#pragma unroll
+                for (int kc = 0; kc < Cfg::KC; kc++) {
+                    const uint64_t ad = smem_desc(abase + (uint32_t)(2 * kc * kHalo * 16 + dx * 16), kHalo * 16, 128);
+                    const uint64_t bd =
+                        smem_desc(wbase + (uint32_t)((dx * Cfg::KC + kc) * 2 * 5 * NB * 16), 5 * NB * 16, 128);
+                    umma_bf16(tmem, ad, bd, idesc, 1u);
+                }
+            }
+            umma_commit(&bars[4]);
+        }
+        __syncwarp();
+        const int r = yin - 1;  // output row completed by this input row
+        const bool valid = r >= y0 && x < a.W;
+        constexpr int RC = (EPI == EPI_RESID) ? NB / 8 : 1;
+        uint4 rres[RC];
+        if constexpr (EPI == EPI_RESID) {
+            if (valid) {
+                const size_t rb = ((size_t)slot_job * a.H + r) * (NB / 8);
+#pragma unroll
+                for (int cg = 0; cg < RC; cg++)
+                    rres[cg] = __ldg(reinterpret_cast<const uint4 *>(a.resid + ((rb + cg) * a.W + x) * 8));
+            }
+        }
+        mbar_wait(&bars[4], q & 1);
+        tc_fence_after();
+        if (tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
+            const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
+            mbar_arrive_expect_tx(&bars[sl], Cfg::SLOT_BYTES);
+            tma_load_5d(s_ring + sl * Cfg::SLOT, &tm_in, &bars[sl], 0, x0 - 1, 0, y0 - 1 + qn, slot_job);
+        }
+        const uint32_t acc = tl + (uint32_t)(mod3(r) * NB);
+        uint32_t v[NB];
+        if constexpr (NB == 32) {
+            uint32_t (&vv)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
+            tmem_ld32(acc, vv);
+        } else {
+            uint32_t (&vv)[16] = *reinterpret_cast<uint32_t(*)[16]>(v);
+            tmem_ld16(acc, vv);
+        }
+        tmem_wait_ld();
+        tmem_zero<NB>(acc);  // row r's block becomes row r+3's
+        if (valid) {
+            if constexpr (EPI == EPI_TAIL) {
+                const int s = a.s, lh = a.lr_h, lw = a.lr_w;
+                int ya, yb, wy, xa, xb, wx;
+                up_tap(r, s, lh, ya, yb, wy);
+                up_tap(x, s, lw, xa, xb, wx);
+                const size_t plane = (size_t)lh * lw, hplane = (size_t)a.H * a.W;
+#pragma unroll
+                for (int c = 0; c < 3; c++) {
+                    const uint8_t *L = J.lr + c * plane;
+                    const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
+                    const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
+                    const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
+                    const int U = (vv + 8192) >> 14;
+                    const float t = __uint_as_float(v[c]) + s_bias[c];
+                    const float o = floorf((float)U + t + 0.5f);
+                    J.hr[c * hplane + (size_t)r * a.W + x] = (uint8_t)fminf(fmaxf(o, 0.f), 255.f);
+                }
+            } else {
+                const size_t rowbase = ((size_t)slot_job * a.H + r) * (NB / 8);
+#pragma unroll
+                for (int cg = 0; cg < NB / 8; cg++) {
+                    float f[8];
+#pragma unroll
+                    for (int i = 0; i < 8; i++) {
+                        f[i] = __uint_as_float(v[cg * 8 + i]) + s_bias[cg * 8 + i];
+                        if (EPI == EPI_RELU) f[i] = fmaxf(f[i], 0.f);
+                    }
+                    if constexpr (EPI == EPI_RESID) {
+                        const uint4 rr = rres[cg];
+                        f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
+                        f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
+                        f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
+                        f[6] += bf_lo(rr.w); f[7] += bf_hi(rr.w);
+                    }
+                    uint4 o;
+                    o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
+                    o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
+                    *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * a.W + x) * 8) = o;
+                }
+            }
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        __syncthreads();
+        tc_fence_after();
     }
     if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
 }
@@ -381,6 +592,25 @@ static cudaError_t conv(int fam, const CUtensorMap &tm, ConvArgs args, int nj, c
     return cudaGetLastError();
 }
 
+constexpr int kRotRows = 64;  // rows per CTA strip of the rotated conv
+template <int CIN, int NB, int EPI>
+static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+    using Cfg = RotCfg<CIN, NB>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_conv_rot<CIN, NB, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    args.n_xtiles = (args.W + kTile - 1) / kTile;
+    args.rows_per_cta = kRotRows;
+    dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
+    KScope ks(fam, st);
+    k_conv_rot<CIN, NB, EPI><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
+    return cudaGetLastError();
+}
+
 template <int C>
 static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                            const int32_t *job_count, cudaStream_t st) {
@@ -398,21 +628,21 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
-        if ((e = conv<16, C, 1, EPI_STORE>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<16, C, EPI_STORE>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     for (int b = 0; b < n_blocks; b++) {
         const CUtensorMap &hin = (b == 0) ? a->tm_h0 : a->tm_hb;
         const uint16_t *hres = (b == 0) ? a->h0 : a->hb;
         ConvArgs g = base; LayerShape l1 = L(1 + 2 * b), l2 = L(2 + 2 * b);
         g.b_off = l1.b_off; g.bias_off = l1.bias_off; g.out = a->tb;
-        if ((e = conv<C, C, 1, EPI_RELU>(F_SR_BODY, hin, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<C, C, EPI_RELU>(F_SR_BODY, hin, g, nj, st)) != cudaSuccess) return e;
         g = base; g.b_off = l2.b_off; g.bias_off = l2.bias_off; g.out = a->hb; g.resid = hres;
-        if ((e = conv<C, C, 1, EPI_RESID>(F_SR_BODY, a->tm_tb, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<C, C, EPI_RESID>(F_SR_BODY, a->tm_tb, g, nj, st)) != cudaSuccess) return e;
     }
     {   // end: h0 + conv(h; W_end) -> tb
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 1);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->tb; g.resid = a->h0;
-        if ((e = conv<C, C, 1, EPI_RESID>(F_SR_END, n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<C, C, EPI_RESID>(F_SR_END, n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
     }
     {   // upsampler conv + pixel shuffle -> u (HR)
         LayerShape ls = L(2 * n_blocks + 2);
@@ -442,7 +672,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 3);
         g.H = h * s; g.W = w * s; g.lr_h = h; g.lr_w = w;
         g.b_off = ls.b_off; g.bias_off = ls.bias_off;
-        if ((e = conv<C, 16, 1, EPI_TAIL>(F_SR_TAIL, a->tm_u, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<C, 16, EPI_TAIL>(F_SR_TAIL, a->tm_u, g, nj, st)) != cudaSuccess) return e;
     }
     return cudaSuccess;
 }

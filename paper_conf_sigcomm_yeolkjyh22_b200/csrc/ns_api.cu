@@ -97,11 +97,14 @@ LayerShape model_layer(int n_blocks, int C, int s, int L) {
         ls.cin = C; ls.cin_real = C; ls.ntot = 16; ls.cout_real = 3;
     }
     ls.nsplit = ls.ntot > 256 ? 2 : 1;
+    ls.rot = ls.perm ? 0 : 1;
+    ls.nb = ls.ntot;
     size_t off = 0;
     for (int l = 0; l < L; l++) off += model_layer(n_blocks, C, s, l).bytes;
+    const size_t bbytes = ls.rot ? (size_t)30 * ls.cin * ls.nb : (size_t)9 * ls.cin * ls.ntot * 2;
     ls.b_off = off;
-    ls.bias_off = off + align128((size_t)9 * ls.cin * ls.ntot * 2);
-    ls.bytes = align128((size_t)9 * ls.cin * ls.ntot * 2) + align128((size_t)ls.ntot * 4);
+    ls.bias_off = off + align128(bbytes);
+    ls.bytes = align128(bbytes) + align128((size_t)ls.ntot * 4);
     return ls;
 }
 
@@ -559,15 +562,15 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
 // ------------------------------------------------------------------ reconstruct
 static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n,
                                  const uint8_t *is_anchor, cudaStream_t st) {
-    int maxW8 = 0, maxH = 0;
+    int mw[5] = {0, 0, 0, 0, 0}, mh[5] = {0, 0, 0, 0, 0};
     size_t maxhr = 0;
     for (int s = 0; s < S; s++) {
-        maxW8 = std::max(maxW8, ch[s].w * ch[s].scale / 8);
-        maxH = std::max(maxH, ch[s].h * ch[s].scale);
+        mw[ch[s].scale] = std::max(mw[ch[s].scale], ch[s].w);
+        mh[ch[s].scale] = std::max(mh[ch[s].scale], ch[s].h);
         maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
     }
     NS_CUDA(launch_golden_index(g.d_sd, S, n, c->gold, st));
-    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(g.d_sd, S, n, f, maxW8, maxH, is_anchor, g.d_hr, c->gold, st));
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(g.d_sd, S, n, f, mw, mh, is_anchor, g.d_hr, c->gold, st));
     NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, maxhr, st));
     return NS_OK;
 }

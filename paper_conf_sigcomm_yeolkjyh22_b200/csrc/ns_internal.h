@@ -42,9 +42,14 @@ struct SrJob {
 // each region 128-B aligned.  Layers: 0 head (CIN 16, 3 real), 1..2B body,
 // 2B+1 end, 2B+2 up (NTOT = s*s*C, rows permuted to (i, j, c) order for the
 // fused pixel shuffle), 2B+3 tail (NTOT = 16, 3 real).
+// Rotated layers (rot = 1: head, body, end, tail) instead hold, per tap column
+// dx and 16-channel K chunk, a 5-block strip [W_dy2; W_dy1; W_dy0; W_dy2;
+// W_dy1] of nb output rows each: [dx 3][kc][kh 2][5 nb][8] bf16, then fp32
+// bias[nb] (see k_conv_rot).
 struct LayerShape {
     int cin, cin_real, ntot, nsplit, cout_real;
     int perm;              // 0 none, 1 pixel-shuffle permutation
+    int rot, nb;           // rotated-accumulator layout and its block width
     size_t b_off, bias_off, bytes;  // offsets from the model base
 };
 
@@ -66,9 +71,10 @@ cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *
                            uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups,
                            int topk, int k, cudaStream_t st);
 cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st);
-cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, int maxW8, int maxH,
-                              const uint8_t *is_anchor, uint8_t *const *d_hr_table, const int16_t *gold_idx,
-                              cudaStream_t st);
+// max_lr_w / max_lr_h: [5] indexed by scale (0 = no stream of that scale)
+cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const int *max_lr_w,
+                              const int *max_lr_h, const uint8_t *is_anchor, uint8_t *const *d_hr_table,
+                              const int16_t *gold_idx, cudaStream_t st);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
