@@ -214,6 +214,7 @@ def main():
     import torch
     import torch.distributed as dist
     import paper_conf_sigcomm_yeolkjyh22_b200 as ns
+    from paper_conf_sigcomm_yeolkjyh22_b200 import shard
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -287,21 +288,12 @@ def main():
     ms = e0.elapsed_time(e1)
     clk = clocks.stop()
     prof = ns.profile_read()
-    if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-        dist.barrier()
+    ms = shard.max_over_ranks(ms)      # job time = the slowest rank (device-timed)
     frames = world * S * n * args.steps
     value = frames / (ms / 1000.0)
 
     # stats gather (the only collective; off the timed region)
-    st = stats.clone()
-    if world > 1:
-        allst = [torch.zeros_like(st) for _ in range(world)]
-        dist.all_gather(allst, st)
-        st = torch.cat(allst)
-    st = st.cpu().numpy()
+    st = shard.gather_stats(stats.clone()).cpu().numpy()
     ia_np = ia.cpu().numpy()
     types = [pool[si % P].type for si in range(S)]
 
@@ -368,11 +360,7 @@ def main():
             e2e_step()
         q1.record(stream)
         torch.cuda.synchronize(dev)
-        ems = q0.elapsed_time(q1)
-        if world > 1:
-            t = torch.tensor([ems], dtype=torch.float64, device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ems = float(t.item())
+        ems = shard.max_over_ranks(q0.elapsed_time(q1))
         e2e = {"value": world * S * n * args.e2e_steps / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
                "note": "H2D of every stream's LR+residual+MV+type from pinned host memory each step; D2H of the "

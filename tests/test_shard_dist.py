@@ -1,0 +1,67 @@
+"""Multi-GPU host logic on CPU: LPT sharding and the gloo (world_size 2)
+stats gather / max-over-ranks used by bench.py after the timed region."""
+import os
+import socket
+
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_sigcomm_yeolkjyh22_b200 import shard
+
+
+def test_flop_model_matches_survey():
+    assert shard.sr_flop_per_lr_px(8, 32, 3) == shard.SR_FLOP_PER_LR_PX[(8, 32, 3)]
+
+
+def test_lpt_balanced_and_complete():
+    # c5-like mix: half 720p->4K, half 360p->1080p
+    costs = [shard.stream_cost(1280, 720, 3, 60, 5) if i % 2 == 0 else shard.stream_cost(640, 360, 3, 60, 5)
+             for i in range(512)]
+    for world in (1, 2, 4, 8):
+        parts = shard.lpt_shard(costs, world)
+        flat = sorted(i for p in parts for i in p)
+        assert flat == list(range(512))
+        loads = [sum(costs[i] for i in p) for p in parts]
+        assert max(loads) - min(loads) <= max(costs) + 1e-12
+        # deterministic
+        assert parts == shard.lpt_shard(costs, world)
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        local = torch.full((3, 8), float(rank), dtype=torch.float64)
+        local[:, 0] = torch.arange(3, dtype=torch.float64) + 10 * rank
+        allst = shard.gather_stats(local)
+        tmax = shard.max_over_ranks(1.5 + rank)
+        q.put((rank, allst.tolist(), tmax))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_gather_and_max():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, allst, tmax in res:
+        assert tmax == 2.5
+        t = torch.tensor(allst)
+        assert t.shape == (6, 8)
+        assert t[:3, 0].tolist() == [0.0, 1.0, 2.0] and t[3:, 0].tolist() == [10.0, 11.0, 12.0]
+        assert (t[3:, 1:] == 1.0).all() and (t[:3, 1:] == 0.0).all()
