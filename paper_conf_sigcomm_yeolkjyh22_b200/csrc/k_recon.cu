@@ -540,14 +540,134 @@ __global__ void k_repack_b(const uint16_t *blob, size_t src_off, LayerShape ls, 
     }
 }
 
+__device__ __forceinline__ float bf2f(uint16_t b) { return __uint_as_float((uint32_t)b << 16); }
+__device__ __forceinline__ uint16_t f2bf(float f) {  // round to nearest even
+    const uint32_t u = __float_as_uint(f);
+    return (uint16_t)((u + 0x7FFFu + ((u >> 16) & 1u)) >> 16);
+}
+
+// Composed weights of tail o pixel-shuffle o upsampler (see CompShape): output
+// n = (i s + j) 3 + co at LR offset (ty-2, tx-2) from input channel ci:
+//   Wc = sum_{dY,dX in -1..1} sum_c Wt[co][c][dY][dX] Wup[c s^2 + i' s + j'][ci][ky][kx]
+// with (i+dY) = s oy + i', (j+dX) = s ox + j', ky = ty - 1 - oy, kx = tx - 1 - ox.
+__global__ void k_repack_comp(const uint16_t *blob, size_t up_off, size_t tail_off, int C, int s, CompShape cs,
+                              uint8_t *packed) {
+    const int nb = cs.nb, KC = C / 16, nout = s * s * 3;
+    const size_t total = (size_t)5 * KC * 2 * 9 * nb * 8;
+    const uint16_t *Wup = blob + up_off, *bup = blob + up_off + (size_t)s * s * C * C * 9;
+    const uint16_t *Wt = blob + tail_off, *bt = blob + tail_off + (size_t)3 * C * 9;
+    const int strip[9] = {4, 3, 2, 1, 0, 4, 3, 2, 1};
+    uint16_t *B = reinterpret_cast<uint16_t *>(packed + cs.b_off);
+    for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (size_t)gridDim.x * blockDim.x) {
+        const int k8 = e % 8;
+        const int nn = (e / 8) % (9 * nb);
+        const int kh = (e / (8 * 9 * nb)) % 2;
+        const int kc = (e / (16 * 9 * nb)) % KC;
+        const int tx = (int)(e / ((size_t)16 * 9 * nb * KC));
+        const int ty = strip[nn / nb], n = nn % nb;
+        const int ci = kc * 16 + kh * 8 + k8;
+        float acc = 0.f;
+        if (n < nout) {
+            const int co = n % 3, ij = n / 3, i = ij / s, j = ij % s;
+            for (int dY = -1; dY <= 1; dY++)
+                for (int dX = -1; dX <= 1; dX++) {
+                    const int oy = (i + dY + s) / s - 1, ip = (i + dY + s) % s;
+                    const int ox = (j + dX + s) / s - 1, jp = (j + dX + s) % s;
+                    const int ky = ty - 1 - oy, kx = tx - 1 - ox;
+                    if (ky < 0 || ky > 2 || kx < 0 || kx > 2) continue;
+                    for (int c = 0; c < C; c++) {
+                        const int uc = c * s * s + ip * s + jp;
+                        acc += bf2f(Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)]) *
+                               bf2f(Wup[((size_t)uc * C + ci) * 9 + ky * 3 + kx]);
+                    }
+                }
+        }
+        B[e] = f2bf(acc);
+    }
+    float *bias = reinterpret_cast<float *>(packed + cs.bias_off);
+    for (int n = blockIdx.x * blockDim.x + threadIdx.x; n < nb; n += gridDim.x * blockDim.x) {
+        float acc = 0.f;
+        if (n < nout) {
+            const int co = n % 3, ij = n / 3, i = ij / s, j = ij % s;
+            acc = bf2f(bt[co]);
+            for (int dY = -1; dY <= 1; dY++)
+                for (int dX = -1; dX <= 1; dX++) {
+                    const int ip = (i + dY + s) % s, jp = (j + dX + s) % s;
+                    for (int c = 0; c < C; c++)
+                        acc += bf2f(Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)]) *
+                               bf2f(bup[c * s * s + ip * s + jp]);
+                }
+        }
+        bias[n] = acc;
+    }
+}
+
+// fp32 composed weights Wc[n][ci][ty*5+tx] and bias (same sums as k_repack_comp)
+__global__ void k_repack_comp32(const uint16_t *blob, size_t up_off, size_t tail_off, int C, int s, float *Wc,
+                                float *bc) {
+    const int nout = s * s * 3;
+    const uint16_t *Wup = blob + up_off, *bup = blob + up_off + (size_t)s * s * C * C * 9;
+    const uint16_t *Wt = blob + tail_off, *bt = blob + tail_off + (size_t)3 * C * 9;
+    const size_t total = (size_t)nout * C * 25;
+    for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total + nout;
+         e += (size_t)gridDim.x * blockDim.x) {
+        if (e < total) {
+            const int tt = e % 25, ci = (e / 25) % C, n = (int)(e / (25 * C));
+            const int ty = tt / 5, tx = tt % 5;
+            const int co = n % 3, ij = n / 3, i = ij / s, j = ij % s;
+            float acc = 0.f;
+            for (int dY = -1; dY <= 1; dY++)
+                for (int dX = -1; dX <= 1; dX++) {
+                    const int oy = (i + dY + s) / s - 1, ip = (i + dY + s) % s;
+                    const int ox = (j + dX + s) / s - 1, jp = (j + dX + s) % s;
+                    const int ky = ty - 1 - oy, kx = tx - 1 - ox;
+                    if (ky < 0 || ky > 2 || kx < 0 || kx > 2) continue;
+                    for (int c = 0; c < C; c++)
+                        acc += bf2f(Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)]) *
+                               bf2f(Wup[((size_t)(c * s * s + ip * s + jp) * C + ci) * 9 + ky * 3 + kx]);
+                }
+            Wc[e] = acc;
+        } else {
+            const int n = (int)(e - total);
+            const int co = n % 3, ij = n / 3, i = ij / s, j = ij % s;
+            float acc = bf2f(bt[co]);
+            for (int dY = -1; dY <= 1; dY++)
+                for (int dX = -1; dX <= 1; dX++) {
+                    const int ip = (i + dY + s) % s, jp = (j + dX + s) % s;
+                    for (int c = 0; c < C; c++)
+                        acc += bf2f(Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)]) *
+                               bf2f(bup[c * s * s + ip * s + jp]);
+                }
+            bc[n] = acc;
+        }
+    }
+}
+
+// fp32 copies of the upsampler and tail (the border fix-up evaluates them exactly)
+__global__ void k_repack_aux(const uint16_t *blob, size_t up_off, size_t n_up, size_t tail_off, size_t n_tail,
+                             float *aux) {
+    for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < n_up + n_tail; e += (size_t)gridDim.x * blockDim.x)
+        aux[e] = bf2f(e < n_up ? blob[up_off + e] : blob[tail_off + (e - n_up)]);
+}
+
 cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint8_t *packed, cudaStream_t st) {
-    KScope ks(F_REPACK, st, model_num_layers(n_blocks));
-    size_t src = 0;
+    KScope ks(F_REPACK, st, model_num_layers(n_blocks) + 3);
+    size_t src = 0, up_off = 0, tail_off = 0;
     for (int l = 0; l < model_num_layers(n_blocks); l++) {
         LayerShape ls = model_layer(n_blocks, C, s, l);
+        if (l == 2 * n_blocks + 2) up_off = src;
+        if (l == 2 * n_blocks + 3) tail_off = src;
         k_repack_b<<<256, 256, 0, st>>>(blob, src, ls, C, s, packed);
         src += (size_t)ls.cout_real * ls.cin_real * 9 + ls.cout_real;
     }
+    const CompShape cs = model_comp(n_blocks, C, s);
+    k_repack_comp<<<256, 256, 0, st>>>(blob, up_off, tail_off, C, s, cs, packed);
+    const size_t n_up = (size_t)s * s * C * C * 9 + (size_t)s * s * C, n_tail = (size_t)3 * C * 9 + 3;
+    float *aux = reinterpret_cast<float *>(packed + cs.aux_off);
+    k_repack_aux<<<256, 256, 0, st>>>(blob, up_off, n_up, tail_off, n_tail, aux);
+    const size_t nout = (size_t)s * s * 3;
+    k_repack_comp32<<<256, 256, 0, st>>>(blob, up_off, tail_off, C, s, aux + n_up + n_tail,
+                                         aux + n_up + n_tail + nout * C * 25);
     return cudaGetLastError();
 }
 

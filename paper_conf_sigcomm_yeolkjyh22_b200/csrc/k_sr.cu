@@ -323,6 +323,13 @@ struct RotCfg {
 };
 
 __device__ __forceinline__ int mod3(int v) { return ((v % 3) + 3) % 3; }
+__host__ __device__ constexpr int fdiv_sr(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+template <int S>
+__host__ __device__ constexpr int tap_d_sr(int k) { return fdiv_sr(2 * k + 1 - S, 2 * S); }
+template <int S>
+__host__ __device__ constexpr int tap_w1_sr(int k) {
+    return (128 * ((2 * k + 1 - S) - 2 * S * tap_d_sr<S>(k)) + S) / (2 * S);
+}
 
 template <int NB>
 __device__ __forceinline__ void tmem_zero(uint32_t taddr) {
@@ -493,6 +500,317 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
 }
 
+// ------------------------------------------------------------------ composed upsampler + tail
+// tail o pixel-shuffle o upsampler is linear (EDSR has no nonlinearity between
+// them), so it equals one 5x5 conv at LR resolution from h (C ch) to s*s*3
+// outputs (CompShape).  This executes 2*25*C*3s^2 FLOP per LR pixel instead of
+// 18 s^2 C^2 + 54 C s^2 and never materialises the HR feature map u (531 MB per
+// 4K anchor).  It equals the definition exactly except on the 1-pixel HR frame
+// border (the tail zero-pads u there); k_uptail_border_* recompute that ring.
+// Same rotated-accumulator scheme as k_conv_rot with 5 kernel rows: output LR
+// row r lives in block r mod 5, the 9-block strip [W4..W0, W4..W1] window start
+// is (2 - y mod 5) mod 5, N = 5 nb.  The epilogue adds the integer bilinear
+// skip up_s(LR) (O6), rounds, clamps and writes the s x s HR pixels of each
+// LR pixel through a shared-memory tile (8-byte stores).
+constexpr int kHalo5 = kTile + 4;
+template <int CIN, int NB, int S>
+struct UpCfg {
+    static constexpr int KC = CIN / 16;
+    static constexpr uint32_t B_BYTES = 5u * KC * 2 * 9 * NB * 16;
+    static constexpr uint32_t BIAS_BYTES = NB * 4u;
+    static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
+    static constexpr uint32_t SLOT_BYTES = kHalo5 * CIN * 2u;
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    static constexpr int NSLOT = 3;
+    static constexpr uint32_t OUT_BYTES = 3u * S * kTile * S;  // HR tile [plane][i][s*128]
+    static constexpr uint32_t TMEM_COLS = tmem_cols_for(5 * NB);
+    static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + round_up(OUT_BYTES, 128) + 128;
+    static_assert((5 * NB) % 16 == 0 && 5 * NB <= 256, "N = 5 nb");
+    static_assert(SMEM <= 232448, "shared memory");
+};
+
+__device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
+
+template <int NB>
+__device__ __forceinline__ void tmem_ldN(uint32_t a, uint32_t (&v)[NB]) {
+    if constexpr (NB == 16) {
+        tmem_ld16(a, v);
+    } else if constexpr (NB == 32) {
+        tmem_ld32(a, v);
+    } else {
+        static_assert(NB == 48, "");
+        uint32_t (&v0)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
+        uint32_t (&v1)[16] = *reinterpret_cast<uint32_t(*)[16]>(v + 32);
+        tmem_ld32(a, v0);
+        tmem_ld16(a + 32, v1);
+    }
+}
+template <int NB>
+__device__ __forceinline__ void tmem_zeroN(uint32_t a) {
+    if constexpr (NB == 48) {
+        tmem_zero<32>(a);
+        tmem_zero<16>(a + 32);
+    } else {
+        tmem_zero<NB>(a);
+    }
+}
+
+template <int CIN, int NB, int S>
+__global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+    using Cfg = UpCfg<CIN, NB, S>;
+    constexpr int NOUT = S * S * 3;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *s_w = smem;
+    const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
+    uint8_t *s_ring = smem + Cfg::W_REGION;
+    uint8_t *s_out = s_ring + Cfg::NSLOT * Cfg::SLOT;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_out + round_up(Cfg::OUT_BYTES, 128));  // [0,3) ring, 3 w, 4 mma
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 6);
+
+    const int slot_job = blockIdx.z;
+    const int job = a.j0 + slot_job;
+    if (a.job_count && job >= *a.job_count) return;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int x0 = blockIdx.x * kTile;
+    const int y0 = blockIdx.y * a.rows_per_cta;
+    const int y1 = min(y0 + a.rows_per_cta, a.H);
+    const int n_loads = y1 - y0 + 4;  // input rows y0-2 .. y1+1
+    const int lh = a.H, lw = a.W;     // LR dims (the conv runs at LR resolution)
+    const int HH = lh * S, WW = lw * S;
+
+    if (tid == 0) {
+        for (int i = 0; i < 5; i++) mbar_init(&bars[i], 1);
+        fence_mbar_init();
+    }
+    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *s_tmem;
+    const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);
+    const SrJob J = a.jobs[job];
+    if (tid == 0) {
+        prefetch_tmap(&tm_in);
+        mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
+        bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
+        bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
+        for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
+            mbar_arrive_expect_tx(&bars[q], Cfg::SLOT_BYTES);
+            tma_load_5d(s_ring + q * Cfg::SLOT, &tm_in, &bars[q], 0, x0 - 2, 0, y0 - 2 + q, slot_job);
+        }
+    }
+#pragma unroll
+    for (int b = 0; b < 5; b++) tmem_zeroN<NB>(tl + b * NB);
+    tmem_wait_st();
+    mbar_wait(&bars[3], 0);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+
+    const uint32_t idesc = idesc_bf16_f32(128, 5 * NB);
+    const int p = warp * 32 + lane;
+    const int x = x0 + p;
+    for (int q = 0; q < n_loads; q++) {
+        const int yin = y0 - 2 + q;
+        if (tid == 0) {
+            const int sl = q % Cfg::NSLOT;
+            mbar_wait(&bars[sl], (q / Cfg::NSLOT) & 1);
+            tc_fence_after();
+            const uint32_t abase = smem_u32(s_ring + sl * Cfg::SLOT);
+            const uint32_t start = (uint32_t)mod5(2 - yin);
+            const uint32_t wbase = smem_u32(s_w) + start * NB * 16;
+#pragma unroll
+            for (int dx = 0; dx < 5; dx++) {
+#pragma unroll
+                for (int kc = 0; kc < Cfg::KC; kc++) {
+                    const uint64_t ad =
+                        smem_desc(abase + (uint32_t)(2 * kc * kHalo5 * 16 + dx * 16), kHalo5 * 16, 128);
+                    const uint64_t bd =
+                        smem_desc(wbase + (uint32_t)((dx * Cfg::KC + kc) * 2 * 9 * NB * 16), 9 * NB * 16, 128);
+                    umma_bf16(tmem, ad, bd, idesc, 1u);
+                }
+            }
+            umma_commit(&bars[4]);
+        }
+        __syncwarp();
+        const int r = yin - 2;  // LR output row completed by this input row
+        const bool valid_row = r >= y0;
+        // bilinear-skip taps for this lane (O6, compile-time sub-pixel weights)
+        int Lv[3][3][3];
+        if (valid_row && x < lw) {
+#pragma unroll
+            for (int c = 0; c < 3; c++) {
+                const uint8_t *L = J.lr + (size_t)c * lh * lw;
+#pragma unroll
+                for (int dy = 0; dy < 3; dy++) {
+                    const uint8_t *Lr = L + (size_t)min(max(r + dy - 1, 0), lh - 1) * lw;
+#pragma unroll
+                    for (int dx = 0; dx < 3; dx++) Lv[c][dy][dx] = Lr[min(max(x + dx - 1, 0), lw - 1)];
+                }
+            }
+        }
+        mbar_wait(&bars[4], q & 1);
+        tc_fence_after();
+        if (tid == 0 && q + Cfg::NSLOT < n_loads) {
+            const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
+            mbar_arrive_expect_tx(&bars[sl], Cfg::SLOT_BYTES);
+            tma_load_5d(s_ring + sl * Cfg::SLOT, &tm_in, &bars[sl], 0, x0 - 2, 0, y0 - 2 + qn, slot_job);
+        }
+        const uint32_t acc = tl + (uint32_t)(mod5(r) * NB);
+        uint32_t v[NB];
+        tmem_ldN<NB>(acc, v);
+        tmem_wait_ld();
+        tmem_zeroN<NB>(acc);
+        if (valid_row) {
+            // HR pixels (S r + i, S x + j): clamp(floor(up_s(LR) + t + 0.5)) -> smem tile
+#pragma unroll
+            for (int i = 0; i < S; i++) {
+                const int dya = tap_d_sr<S>(i) + 1, wy = tap_w1_sr<S>(i);
+#pragma unroll
+                for (int j = 0; j < S; j++) {
+                    const int dxa = tap_d_sr<S>(j) + 1, wx = tap_w1_sr<S>(j);
+#pragma unroll
+                    for (int c = 0; c < 3; c++) {
+                        const int n = (i * S + j) * 3 + c;
+                        const int vv = (128 - wy) * ((128 - wx) * Lv[c][dya][dxa] + wx * Lv[c][dya][dxa + 1]) +
+                                       wy * ((128 - wx) * Lv[c][dya + 1][dxa] + wx * Lv[c][dya + 1][dxa + 1]);
+                        const int U = (vv + 8192) >> 14;
+                        const float t = __uint_as_float(v[n]) + s_bias[n];
+                        const float o = fminf(fmaxf(floorf((float)U + t + 0.5f), 0.f), 255.f);
+                        s_out[(c * S + i) * (kTile * S) + p * S + j] = (uint8_t)o;
+                    }
+                }
+            }
+        }
+        tmem_wait_st();
+        tc_fence_before();
+        __syncthreads();
+        if (valid_row) {  // coalesced 8-byte stores of the HR tile rows
+            const int xs_hr = x0 * S, wv = min(kTile, lw - x0) * S;  // valid HR bytes per row (multiple of 8)
+            constexpr int CH = kTile * S / 8;
+            for (int e = tid; e < 3 * S * CH; e += 128) {
+                const int ch = e % CH, ri = e / CH, c = ri / S, i = ri % S;
+                if (ch * 8 < wv)
+                    *reinterpret_cast<uint2 *>(J.hr + (size_t)c * HH * WW + (size_t)(S * r + i) * WW + xs_hr + ch * 8) =
+                        *reinterpret_cast<const uint2 *>(s_out + ri * (kTile * S) + ch * 8);
+            }
+        }
+        __syncthreads();
+        tc_fence_after();
+    }
+    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
+    (void)NOUT;
+}
+
+// ---- exact frame-border ring.  The composed conv evaluates the tail over
+// u at the out-of-frame HR positions around the frame (rows -1 and H, cols -1
+// and W), where the definition has zeros (tail zero padding).  For every ring
+// pixel:  t = bc + sum Wc h (fp32 composed 5x5)  -  sum_{out-of-frame taps}
+// W_tail u_ext,  with u_ext = the upsampler evaluated at those positions (its
+// own zero padding of h applies).  Out-of-frame index: row -1: X'+1 (X' in
+// -1..W), row H: (W+2) + X'+1, col -1: 2(W+2) + Y', col W: 2(W+2) + H + Y'.
+__device__ __forceinline__ int ext_index(int Y, int X, int H, int W) {
+    if (Y < 0) return X + 1;
+    if (Y >= H) return (W + 2) + X + 1;
+    if (X < 0) return 2 * (W + 2) + Y;
+    return 2 * (W + 2) + H + Y;
+}
+__device__ __forceinline__ void ext_pos(int e, int H, int W, int &Y, int &X) {
+    if (e < W + 2) { Y = -1; X = e - 1; return; }
+    e -= W + 2;
+    if (e < W + 2) { Y = H; X = e - 1; return; }
+    e -= W + 2;
+    if (e < H) { Y = e; X = -1; return; }
+    Y = e - H; X = W;
+}
+__device__ __forceinline__ float act_at(const uint16_t *act, int y, int x, int ci, int h, int w, int C) {
+    if (y < 0 || y >= h || x < 0 || x >= w) return 0.f;
+    return __uint_as_float((uint32_t)act[(((size_t)y * (C / 8) + ci / 8) * w + x) * 8 + ci % 8] << 16);
+}
+
+// one thread per (upsampler channel c, out-of-frame position): consecutive lanes
+// take consecutive positions, so a warp's weight loads broadcast (<= s rows)
+__global__ void k_uptail_ext_u(const SrJob *jobs, int j0, const int32_t *job_count, const uint16_t *hact, int h,
+                               int w, int C, int s, size_t aux_off, float *ext) {
+    const int slot = blockIdx.y, job = j0 + slot;
+    if (job_count && job >= *job_count) return;
+    const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H;
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= next * C) return;
+    const int pos = e % next, c = e / next;
+    int Y, X;
+    ext_pos(pos, H, W, Y, X);
+    const int y = (Y + s) / s - 1, i = Y - s * y, x = (X + s) / s - 1, j = X - s * x;
+    const float *Wup = reinterpret_cast<const float *>(jobs[job].wts + aux_off);
+    const float *bup = Wup + (size_t)s * s * C * C * 9;
+    const int uc = c * s * s + i * s + j;
+    const uint16_t *act = hact + (size_t)slot * h * (C / 8) * w * 8;
+    float acc = bup[uc];
+    for (int ky = 0; ky < 3; ky++)
+        for (int kx = 0; kx < 3; kx++) {
+            const int yy = y + ky - 1, xx = x + kx - 1;
+            if (yy < 0 || yy >= h || xx < 0 || xx >= w) continue;
+            for (int ci = 0; ci < C; ci++) acc += Wup[((size_t)uc * C + ci) * 9 + ky * 3 + kx] * act_at(act, yy, xx, ci, h, w, C);
+        }
+    ext[((size_t)slot * next + pos) * C + c] = acc;
+}
+
+// one thread per ring pixel
+__global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_count, const uint16_t *hact, int h,
+                              int w, int C, int s, size_t aux_off, const float *ext) {
+    const int slot = blockIdx.y, job = j0 + slot;
+    if (job_count && job >= *job_count) return;
+    const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= nring) return;
+    int Y, X;
+    if (e < W) { Y = 0; X = e; }
+    else if (e < 2 * W) { Y = H - 1; X = e - W; }
+    else if (e < 2 * W + (H - 2)) { Y = 1 + (e - 2 * W); X = 0; }
+    else { Y = 1 + (e - 2 * W - (H - 2)); X = W - 1; }
+    const SrJob J = jobs[job];
+    const float *aux = reinterpret_cast<const float *>(J.wts + aux_off);
+    const float *Wt = aux + (size_t)s * s * C * C * 9 + (size_t)s * s * C;
+    const float *Wc = Wt + (size_t)3 * C * 9 + 3;
+    const float *bc = Wc + (size_t)s * s * 3 * C * 25;
+    const uint16_t *act = hact + (size_t)slot * h * (C / 8) * w * 8;
+    const float *E = ext + (size_t)slot * next * C;
+    const int r = Y / s, i = Y % s, x = X / s, j = X % s;
+    float t[3];
+    for (int co = 0; co < 3; co++) {
+        const int n = (i * s + j) * 3 + co;
+        float acc = bc[n];
+        for (int ty = 0; ty < 5; ty++)
+            for (int tx = 0; tx < 5; tx++) {
+                const int yy = r + ty - 2, xx = x + tx - 2;
+                if (yy < 0 || yy >= h || xx < 0 || xx >= w) continue;
+                for (int ci = 0; ci < C; ci++)
+                    acc += Wc[((size_t)n * C + ci) * 25 + ty * 5 + tx] * act_at(act, yy, xx, ci, h, w, C);
+            }
+        t[co] = acc;
+    }
+    for (int dY = -1; dY <= 1; dY++)
+        for (int dX = -1; dX <= 1; dX++) {
+            const int Yn = Y + dY, Xn = X + dX;
+            if (Yn >= 0 && Yn < H && Xn >= 0 && Xn < W) continue;  // in-frame: already right
+            const float *u = E + (size_t)ext_index(Yn, Xn, H, W) * C;
+            for (int c = 0; c < C; c++)
+#pragma unroll
+                for (int co = 0; co < 3; co++) t[co] -= Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)] * u[c];
+        }
+    int ya, yb, wy, xa, xb, wx;
+    up_tap(Y, s, h, ya, yb, wy);
+    up_tap(X, s, w, xa, xb, wx);
+    for (int c = 0; c < 3; c++) {
+        const uint8_t *L = J.lr + (size_t)c * h * w;
+        const int v = (128 - wy) * ((128 - wx) * L[(size_t)ya * w + xa] + wx * L[(size_t)ya * w + xb]) +
+                      wy * ((128 - wx) * L[(size_t)yb * w + xa] + wx * L[(size_t)yb * w + xb]);
+        const int U = (v + 8192) >> 14;
+        const float o = fminf(fmaxf(floorf((float)U + t[c] + 0.5f), 0.f), 255.f);
+        J.hr[(size_t)c * H * W + (size_t)Y * W + X] = (uint8_t)o;
+    }
+}
+
 // LR u8 planar [3][h][w] -> bf16 [h][2][w][8]: channels 0..2 = LR - 128 (Z13), 3..15 = 0.
 __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0) {
     const int slot = blockIdx.y, job = j0 + slot;
@@ -530,13 +848,13 @@ static PFN_encodeTiled get_encode() {
     return fn;
 }
 
-// Activation tensor [nb][H][C/8][W][8] bf16 viewed as 5-D (8, W, C/8, H, nb); box (8, 130, C/8, 1, 1).
-static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int nb) {
+// Activation tensor [nb][H][C/8][W][8] bf16 viewed as 5-D (8, W, C/8, H, nb); box (8, box_w, C/8, 1, 1).
+static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int nb, int box_w) {
     PFN_encodeTiled enc = get_encode();
     if (!enc) return -1;
     cuuint64_t dims[5] = {8, (cuuint64_t)W, (cuuint64_t)(C / 8), (cuuint64_t)H, (cuuint64_t)nb};
     cuuint64_t strides[4] = {16, (cuuint64_t)W * 16, (cuuint64_t)(C / 8) * W * 16, (cuuint64_t)H * (C / 8) * W * 16};
-    cuuint32_t box[5] = {8, kHalo, (cuuint32_t)(C / 8), 1, 1};
+    cuuint32_t box[5] = {8, (cuuint32_t)box_w, (cuuint32_t)(C / 8), 1, 1};
     cuuint32_t estr[5] = {1, 1, 1, 1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 5, base, dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -544,11 +862,16 @@ static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int
     return r == CUDA_SUCCESS ? 0 : -2;
 }
 
+static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u positions x C
+    const size_t H = (size_t)h * s, W = (size_t)w * s;
+    return (2 * (W + 2) + 2 * H) * C;
+}
+
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
     const size_t px = (size_t)h * w * nb;
     size_t b = px * 16 * 2;                  // x0
     b += 3 * px * C * 2;                     // h0, hb, tb
-    b += px * s * s * C * 2;                 // u (HR)
+    b += band_floats(h, w, C, s) * 4 * nb;   // border bands
     return b + 5 * 256;
 }
 
@@ -558,19 +881,19 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     auto take = [&](size_t bytes) {
         uint8_t *p = mem;
         mem += (bytes + 255) / 256 * 256;
-        return reinterpret_cast<uint16_t *>(p);
+        return p;
     };
-    a->x0 = take(px * 16 * 2);
-    a->h0 = take(px * C * 2);
-    a->hb = take(px * C * 2);
-    a->tb = take(px * C * 2);
-    a->u = take(px * s * s * C * 2);
+    a->x0 = reinterpret_cast<uint16_t *>(take(px * 16 * 2));
+    a->h0 = reinterpret_cast<uint16_t *>(take(px * C * 2));
+    a->hb = reinterpret_cast<uint16_t *>(take(px * C * 2));
+    a->tb = reinterpret_cast<uint16_t *>(take(px * C * 2));
+    a->band = reinterpret_cast<float *>(take(band_floats(h, w, C, s) * 4 * nb));
     int rc = 0;
-    rc |= make_act_map(&a->tm_x0, a->x0, h, w, 16, nb);
-    rc |= make_act_map(&a->tm_h0, a->h0, h, w, C, nb);
-    rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb);
-    rc |= make_act_map(&a->tm_tb, a->tb, h, w, C, nb);
-    rc |= make_act_map(&a->tm_u, a->u, h * s, w * s, C, nb);
+    rc |= make_act_map(&a->tm_x0, a->x0, h, w, 16, nb, kHalo);
+    rc |= make_act_map(&a->tm_h0, a->h0, h, w, C, nb, kHalo);
+    rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb, kHalo);
+    rc |= make_act_map(&a->tm_tb, a->tb, h, w, C, nb, kHalo);
+    rc |= make_act_map(&a->tm_tb5, a->tb, h, w, C, nb, kHalo5);
     return rc;
 }
 
@@ -611,6 +934,24 @@ static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int n
     return cudaGetLastError();
 }
 
+template <int CIN, int NB, int S>
+static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+    using Cfg = UpCfg<CIN, NB, S>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_uptail<CIN, NB, S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    args.n_xtiles = (args.W + kTile - 1) / kTile;
+    args.rows_per_cta = kRotRows;
+    dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
+    KScope ks(F_SR_UP, st);
+    k_uptail<CIN, NB, S><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
+    return cudaGetLastError();
+}
+
 template <int C>
 static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                            const int32_t *job_count, cudaStream_t st) {
@@ -644,35 +985,21 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->tb; g.resid = a->h0;
         if ((e = conv_rot<C, C, EPI_RESID>(F_SR_END, n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
     }
-    {   // upsampler conv + pixel shuffle -> u (HR)
-        LayerShape ls = L(2 * n_blocks + 2);
-        ConvArgs g = base; g.out = a->u;
-        const int ntot = s * s * C;
-        if (ntot <= 256) {
-            g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
-            if (C == 16 && s == 2) e = conv<C, 64, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
-            else if (C == 16 && s == 3) e = conv<C, 144, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
-            else if (C == 16 && s == 4) e = conv<C, 256, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
-            else e = conv<C, (C == 32 ? 128 : 64), 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);  // C=32, s=2
-        } else if (ntot == 288) {  // C = 32, s = 3: two N tiles of 144 in one launch
-            g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.sub0 = 0;
-            e = conv<C, 144, 2, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g, nj, st);
-        } else {                   // C = 32, s = 4: two launches of N = 256
-            for (int sp = 0; sp < 2 && e == cudaSuccess; sp++) {
-                ConvArgs g2 = g;
-                g2.b_off = ls.b_off + (size_t)sp * 9 * C * 256 * 2;
-                g2.bias_off = ls.bias_off + (size_t)sp * 256 * 4;
-                g2.sub0 = sp * 8;
-                e = conv<C, 256, 1, EPI_SHUFFLE>(F_SR_UP, a->tm_tb, g2, nj, st);
-            }
-        }
+    {   // tail o shuffle o upsampler as one 5x5 conv at LR (+ bilinear skip, round, clamp) -> u8 HR
+        const CompShape cs = model_comp(n_blocks, C, s);
+        ConvArgs g = base;
+        g.b_off = cs.b_off; g.bias_off = cs.bias_off;
+        if (s == 2) e = uptail<C, 16, 2>(a->tm_tb5, g, nj, st);
+        else if (s == 3) e = uptail<C, 32, 3>(a->tm_tb5, g, nj, st);
+        else e = uptail<C, 48, 4>(a->tm_tb5, g, nj, st);
         if (e != cudaSuccess) return e;
-    }
-    {   // HR tail + integer bilinear skip -> u8 planar
-        ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 3);
-        g.H = h * s; g.W = w * s; g.lr_h = h; g.lr_w = w;
-        g.b_off = ls.b_off; g.bias_off = ls.bias_off;
-        if ((e = conv_rot<C, 16, EPI_TAIL>(F_SR_TAIL, a->tm_u, g, nj, st)) != cudaSuccess) return e;
+        // exact frame-border ring (the tail's zero padding of u)
+        KScope ks(F_SR_TAIL, st, 2);
+        const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
+        dim3 g1((next * C + 127) / 128, nj), g2((nring + 127) / 128, nj);
+        k_uptail_ext_u<<<g1, 128, 0, st>>>(jobs, j0, job_count, a->tb, h, w, C, s, cs.aux_off, a->band);
+        k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, a->tb, h, w, C, s, cs.aux_off, a->band);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     return cudaSuccess;
 }

@@ -108,10 +108,29 @@ LayerShape model_layer(int n_blocks, int C, int s, int L) {
     return ls;
 }
 
-size_t model_packed_bytes(int n_blocks, int C, int s) {
+static size_t blob_layers_bytes(int n_blocks, int C, int s) {
     size_t t = 0;
     for (int l = 0; l < model_num_layers(n_blocks); l++) t += model_layer(n_blocks, C, s, l).bytes;
     return t;
+}
+
+CompShape model_comp(int n_blocks, int C, int s) {
+    CompShape c{};
+    const int nout = s * s * 3;
+    c.nb = (nout + 15) / 16 * 16;
+    const size_t base = blob_layers_bytes(n_blocks, C, s);
+    c.b_off = base;
+    c.bias_off = base + align128((size_t)5 * (C / 16) * 2 * 9 * c.nb * 16);
+    c.aux_off = c.bias_off + align128((size_t)c.nb * 4);
+    return c;
+}
+
+size_t model_packed_bytes(int n_blocks, int C, int s) {
+    const CompShape c = model_comp(n_blocks, C, s);
+    const size_t nout = (size_t)s * s * 3;
+    const size_t aux = ((size_t)s * s * C * C * 9 + (size_t)s * s * C + (size_t)3 * C * 9 + 3 +
+                        nout * C * 25 + nout) * 4;
+    return c.aux_off + align128(aux);
 }
 }  // namespace ns
 

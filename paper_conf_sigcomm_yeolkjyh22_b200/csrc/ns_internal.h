@@ -57,6 +57,20 @@ int model_num_layers(int n_blocks);
 LayerShape model_layer(int n_blocks, int C, int s, int L);
 size_t model_packed_bytes(int n_blocks, int C, int s);
 
+// Derived regions after the blob layers:
+//  * COMP: tail o pixel-shuffle o upsampler composed into one 5x5 conv at LR
+//    resolution, h (C ch) -> s*s*3 outputs (n = (i*s + j)*3 + co), padded to nb;
+//    UMMA B operand of the 5-row rotated conv: [tx 5][kc][kh 2][9 nb][8] bf16
+//    (kernel-row strip ty = 4,3,2,1,0,4,3,2,1), then fp32 bias[nb].
+//  * AUX (fp32, for the exact frame-border fix-up): W_up [s*s*C][C][9], b_up,
+//    W_tail [3][C][9], b_tail, then the composed Wc [s*s*3][C][25], bc [s*s*3].
+struct CompShape {
+    int nb;                  // padded outputs per block (16 | 32 | 48)
+    size_t b_off, bias_off;  // composed operand / bias
+    size_t aux_off;          // fp32 W_up, b_up, W_tail, b_tail (contiguous)
+};
+CompShape model_comp(int n_blocks, int C, int s);
+
 // ------------------------------------------------------------ launch wrappers
 // Every launch goes through these (kernels live in k_*.cu); each returns the
 // cudaError_t of the launch.  `st` is the stream.
@@ -84,8 +98,9 @@ cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint
 // SR (k_sr.cu)
 struct SrArena {
     int h, w, C, s, nb;        // shape and batch capacity (jobs per batch)
-    uint16_t *x0, *h0, *hb, *tb, *u;   // bf16 activations, layout [job][H][C/8][W][8]
-    CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_u;
+    uint16_t *x0, *h0, *hb, *tb;       // bf16 activations, layout [job][H][C/8][W][8]
+    float *band;                       // border fix-up: u on the HR frame-edge bands
+    CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_tb5;   // tm_tb5: 132-px boxes (5x5 conv)
 };
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb);
 int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);  // 0 ok
