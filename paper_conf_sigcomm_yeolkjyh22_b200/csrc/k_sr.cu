@@ -345,6 +345,34 @@ __device__ __forceinline__ void tmem_zero(uint32_t taddr) {
 }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
+__device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
+
+template <int NB>
+__device__ __forceinline__ void tmem_ldN(uint32_t a, uint32_t (&v)[NB]) {
+    if constexpr (NB == 16) {
+        tmem_ld16(a, v);
+    } else if constexpr (NB == 32) {
+        tmem_ld32(a, v);
+    } else {
+        static_assert(NB == 48, "");
+        uint32_t (&v0)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
+        uint32_t (&v1)[16] = *reinterpret_cast<uint32_t(*)[16]>(v + 32);
+        tmem_ld32(a, v0);
+        tmem_ld16(a + 32, v1);
+    }
+}
+template <int NB>
+__device__ __forceinline__ void tmem_zeroN(uint32_t a) {
+    if constexpr (NB == 48) {
+        tmem_zero<32>(a);
+        tmem_zero<16>(a + 32);
+    } else {
+        tmem_zero<NB>(a);
+    }
+}
+
+
+
 template <int CIN, int NB, int EPI>
 __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
     using Cfg = RotCfg<CIN, NB>;
@@ -500,6 +528,248 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
 }
 
+// ------------------------------------------------------------------ fused residual block
+// h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
+// h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
+// written in the UMMA A-operand layout and consumed by conv2's MMAs), and the
+// residual h is read back from the same ring.  Both convs use the rotated
+// accumulators of k_conv_rot.  conv1 computes t for 128 positions x0-1 ..
+// x0+126, so conv2 yields 126 valid outputs: tiles advance by 126 px.  Each CTA
+// ping-pongs two x-tiles so one tile's epilogue overlaps the other's MMAs.
+constexpr int kRbOut = kTile - 2;
+struct RbArgs {
+    int H, W, n_tiles, rows_per_cta, j0;
+    const SrJob *jobs;
+    const int32_t *job_count;
+    size_t b1_off, bias1_off, b2_off, bias2_off;
+    uint16_t *out;
+};
+template <int C>
+struct RbCfg {
+    static constexpr int NB = C, KC = C / 16;
+    static constexpr uint32_t B_BYTES = 30u * C * C;
+    static constexpr uint32_t BIAS_BYTES = C * 4u;
+    static constexpr uint32_t W_CONV = round_up(B_BYTES + BIAS_BYTES, 1024);
+    static constexpr uint32_t SLOT_BYTES = kHalo * C * 2u;
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    static constexpr int NH = 5;                                 // h ring per tile
+    static constexpr int NTS = 2;                                // t slots per tile
+    static constexpr uint32_t TILE_BYTES = (NH + NTS) * SLOT;
+    static constexpr uint32_t TCOLS = 2 * 3 * NB;                // conv1 + conv2 rings per tile
+    static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
+    static constexpr int NBAR = 2 * (2 * NH + 4) + 1;
+    static constexpr uint32_t SMEM = 2 * W_CONV + 2 * TILE_BYTES + NBAR * 8 + 64;
+    static_assert(SMEM <= 232448, "shared memory");
+};
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-5 = epilogue
+// of tile 0, warps 6-9 = epilogue of tile 1 (warp w owns TMEM lanes 32 (w % 4)).
+// Per tile and input step q (h row y0-2+q): M1(q) conv1 -> E1(q) reads t row
+// y0-3+q, writes it (ReLU, bf16) to t slot q%2 -> M2(q) conv2 on it -> E2(q)
+// retires output row y0-4+q (+ b2 + h from the ring).  mbarriers only.
+template <int C>
+__global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
+    using Cfg = RbCfg<C>;
+    constexpr int NB = Cfg::NB, NH = Cfg::NH;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *s_w1 = smem, *s_w2 = smem + Cfg::W_CONV;
+    const float *s_b1 = reinterpret_cast<const float *>(s_w1 + Cfg::B_BYTES);
+    const float *s_b2 = reinterpret_cast<const float *>(s_w2 + Cfg::B_BYTES);
+    uint8_t *s_tile = smem + 2 * Cfg::W_CONV;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_tile + 2 * Cfg::TILE_BYTES);
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + Cfg::NBAR);
+    auto hslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
+    auto tslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + (NH + i) * Cfg::SLOT; };
+    // per tile: hfull[NH], m1, m2, e1, e2, hfree[NH]
+    auto hfull = [&](int k, int i) { return &bars[k * (2 * NH + 4) + i]; };
+    auto hfree = [&](int k, int i) { return &bars[k * (2 * NH + 4) + NH + 4 + i]; };
+    auto m1bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH]; };
+    auto m2bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 1]; };
+    auto e1bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 2]; };
+    auto e2bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 3]; };
+    uint64_t *wbar = &bars[2 * (2 * NH + 4)];
+
+    const int slot_job = blockIdx.z;
+    const int job = a.j0 + slot_job;
+    if (a.job_count && job >= *a.job_count) return;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int y0 = blockIdx.y * a.rows_per_cta;
+    const int y1 = min(y0 + a.rows_per_cta, a.H);
+    const int nq = y1 - y0 + 4;  // h rows y0-2 .. y1+1
+    int x0k[2];
+    bool vk[2];
+    for (int k = 0; k < 2; k++) {
+        const int tix = 2 * blockIdx.x + k;
+        vk[k] = tix < a.n_tiles;
+        x0k[k] = tix * kRbOut;
+    }
+
+    if (tid == 0) {
+        for (int k = 0; k < 2; k++) {
+            for (int i = 0; i < NH; i++) mbar_init(hfull(k, i), 1);
+            for (int i = 0; i < NH; i++) mbar_init(hfree(k, i), 128);
+            mbar_init(m1bar(k), 1);
+            mbar_init(m2bar(k), 1);
+            mbar_init(e1bar(k), 128);
+            mbar_init(e2bar(k), 128);
+        }
+        mbar_init(wbar, 1);
+        fence_mbar_init();
+    }
+    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
+    for (int i = tid; i < (int)(2 * Cfg::NTS * (Cfg::SLOT / 16)); i += blockDim.x) {  // t slots start at zero
+        const int ks = i / (Cfg::SLOT / 16), o = i % (Cfg::SLOT / 16);
+        reinterpret_cast<uint4 *>(tslot(ks / Cfg::NTS, ks % Cfg::NTS))[o] = make_uint4(0, 0, 0, 0);
+    }
+    fence_proxy_async_smem();
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *s_tmem;
+    const SrJob J = a.jobs[job];
+
+    if (warp == 0) {
+        // ---------------------------------------------------------------- TMA producer
+        if (lane == 0) {
+            prefetch_tmap(&tm_in);
+            mbar_arrive_expect_tx(wbar, 2 * (Cfg::B_BYTES + Cfg::BIAS_BYTES));
+            bulk_load(s_w1, J.wts + a.b1_off, Cfg::B_BYTES, wbar);
+            bulk_load(s_w1 + Cfg::B_BYTES, J.wts + a.bias1_off, Cfg::BIAS_BYTES, wbar);
+            bulk_load(s_w2, J.wts + a.b2_off, Cfg::B_BYTES, wbar);
+            bulk_load(s_w2 + Cfg::B_BYTES, J.wts + a.bias2_off, Cfg::BIAS_BYTES, wbar);
+            for (int q = 0; q < nq; q++) {
+                for (int k = 0; k < 2; k++) {
+                    if (!vk[k]) continue;
+                    const int sl = q % NH;
+                    // slot reuse: h row q-NH was last read by E2 at step q-NH+2, which
+                    // arrives on hfree[slot] (one completion per reuse: never runs ahead)
+                    if (q >= NH) mbar_wait(hfree(k, sl), ((q / NH) - 1) & 1);
+                    mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
+                    tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ---------------------------------------------------------------- MMA issuer
+        if (lane == 0) {
+            const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
+            auto mma_rot = [&](uint32_t dcol, const uint8_t *aslot, const uint8_t *wstrip, int yin) {
+                const uint32_t abase = smem_u32(aslot);
+                const uint32_t wbase = smem_u32(wstrip) + (uint32_t)mod3(1 - yin) * NB * 16;
+#pragma unroll
+                for (int dx = 0; dx < 3; dx++)
+#pragma unroll
+                    for (int kc = 0; kc < Cfg::KC; kc++)
+                        umma_bf16(dcol,
+                                  smem_desc(abase + (uint32_t)(2 * kc * kHalo * 16 + dx * 16), kHalo * 16, 128),
+                                  smem_desc(wbase + (uint32_t)((dx * Cfg::KC + kc) * 2 * 5 * NB * 16), 5 * NB * 16,
+                                            128),
+                                  idesc, 1u);
+            };
+            mbar_wait(wbar, 0);
+            for (int q = 0; q < nq; q++) {
+                for (int k = 0; k < 2; k++) {  // conv1 on h row y0-2+q
+                    if (!vk[k]) continue;
+                    mbar_wait(hfull(k, q % NH), (q / NH) & 1);
+                    if (q >= 1) mbar_wait(e1bar(k), (q - 1) & 1);  // E1(q-1) zeroed the block M1(q) first touches
+                    tc_fence_after();
+                    mma_rot(tmem + k * Cfg::TCOLS, hslot(k, q % NH), s_w1, y0 - 2 + q);
+                    umma_commit(m1bar(k));
+                }
+                if (q < 2) continue;
+                for (int k = 0; k < 2; k++) {  // conv2 on t row y0-3+q
+                    if (!vk[k]) continue;
+                    mbar_wait(e1bar(k), q & 1);                     // t row written
+                    if (q >= 3) mbar_wait(e2bar(k), (q - 3) & 1);   // E2(q-1) zeroed the block M2(q) first touches
+                    tc_fence_after();
+                    mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q);
+                    umma_commit(m2bar(k));
+                }
+            }
+        }
+    } else {
+        // ---------------------------------------------------------------- epilogues
+        const int k = (warp - 2) / 4;
+        if (vk[k]) {
+            const int ew = warp % 4;   // TMEM lane quarter
+            const int p = ew * 32 + lane;
+            const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
+            mbar_wait(wbar, 0);
+            for (int q = 0; q < nq; q++) {
+                const int yt = y0 - 3 + q, yo = yt - 1;
+                {   // E1: t = ReLU(conv1 + b1) -> t slot (zero outside the frame: conv2 padding)
+                    mbar_wait(m1bar(k), q & 1);
+                    tc_fence_after();
+                    const uint32_t acc = tl + (uint32_t)(mod3(yt) * NB);
+                    uint32_t v[NB];
+                    tmem_ldN<NB>(acc, v);
+                    tmem_wait_ld();
+                    tmem_zeroN<NB>(acc);
+                    if (q >= 2) {
+                        const int xt = x0k[k] - 1 + p;
+                        const bool inside = yt >= 0 && yt < a.H && xt >= 0 && xt < a.W;
+                        uint8_t *ts = tslot(k, q % Cfg::NTS);
+#pragma unroll
+                        for (int cg = 0; cg < NB / 8; cg++) {
+                            float f[8];
+#pragma unroll
+                            for (int i = 0; i < 8; i++)
+                                f[i] = inside ? fmaxf(__uint_as_float(v[cg * 8 + i]) + s_b1[cg * 8 + i], 0.f) : 0.f;
+                            uint4 o;
+                            o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
+                            o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
+                            *reinterpret_cast<uint4 *>(ts + cg * kHalo * 16 + p * 16) = o;
+                        }
+                    }
+                    tmem_wait_st();
+                    fence_proxy_async_smem();
+                    tc_fence_before();
+                    mbar_arrive(e1bar(k));
+                }
+                if (q >= 2) {  // E2: out = conv2 + b2 + h
+                    mbar_wait(m2bar(k), (q - 2) & 1);
+                    tc_fence_after();
+                    const uint32_t acc = tl + 3 * NB + (uint32_t)(mod3(yo) * NB);
+                    uint32_t v[NB];
+                    tmem_ldN<NB>(acc, v);
+                    tmem_wait_ld();
+                    tmem_zeroN<NB>(acc);
+                    const int x = x0k[k] + p;
+                    if (yo >= y0 && yo < y1 && p < kRbOut && x < a.W) {
+                        const uint8_t *hs = hslot(k, (q - 2) % NH);  // h row yo (step q-2)
+                        const size_t rowbase = ((size_t)slot_job * a.H + yo) * (NB / 8);
+#pragma unroll
+                        for (int cg = 0; cg < NB / 8; cg++) {
+                            const uint4 rr = *reinterpret_cast<const uint4 *>(hs + cg * kHalo * 16 + (p + 2) * 16);
+                            float f[8];
+#pragma unroll
+                            for (int i = 0; i < 8; i++) f[i] = __uint_as_float(v[cg * 8 + i]) + s_b2[cg * 8 + i];
+                            f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
+                            f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
+                            f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
+                            f[6] += bf_lo(rr.w); f[7] += bf_hi(rr.w);
+                            uint4 o;
+                            o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
+                            o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
+                            *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * a.W + x) * 8) = o;
+                        }
+                    }
+                    tmem_wait_st();
+                    tc_fence_before();
+                    mbar_arrive(hfree(k, (q - 2) % NH));
+                    mbar_arrive(e2bar(k));
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
+}
+
 // ------------------------------------------------------------------ composed upsampler + tail
 // tail o pixel-shuffle o upsampler is linear (EDSR has no nonlinearity between
 // them), so it equals one 5x5 conv at LR resolution from h (C ch) to s*s*3
@@ -528,32 +798,6 @@ struct UpCfg {
     static_assert((5 * NB) % 16 == 0 && 5 * NB <= 256, "N = 5 nb");
     static_assert(SMEM <= 232448, "shared memory");
 };
-
-__device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
-
-template <int NB>
-__device__ __forceinline__ void tmem_ldN(uint32_t a, uint32_t (&v)[NB]) {
-    if constexpr (NB == 16) {
-        tmem_ld16(a, v);
-    } else if constexpr (NB == 32) {
-        tmem_ld32(a, v);
-    } else {
-        static_assert(NB == 48, "");
-        uint32_t (&v0)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
-        uint32_t (&v1)[16] = *reinterpret_cast<uint32_t(*)[16]>(v + 32);
-        tmem_ld32(a, v0);
-        tmem_ld16(a + 32, v1);
-    }
-}
-template <int NB>
-__device__ __forceinline__ void tmem_zeroN(uint32_t a) {
-    if constexpr (NB == 48) {
-        tmem_zero<32>(a);
-        tmem_zero<16>(a + 32);
-    } else {
-        tmem_zero<NB>(a);
-    }
-}
 
 template <int CIN, int NB, int S>
 __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
@@ -894,6 +1138,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb, kHalo);
     rc |= make_act_map(&a->tm_tb, a->tb, h, w, C, nb, kHalo);
     rc |= make_act_map(&a->tm_tb5, a->tb, h, w, C, nb, kHalo5);
+    rc |= make_act_map(&a->tm_hb5, a->hb, h, w, C, nb, kHalo5);
     return rc;
 }
 
@@ -952,6 +1197,25 @@ static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStre
     return cudaGetLastError();
 }
 
+constexpr int kRbRows = 120;
+template <int C>
+static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, cudaStream_t st) {
+    using Cfg = RbCfg<C>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_resblock<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    RbArgs args = args0;
+    args.n_tiles = (args.W + kRbOut - 1) / kRbOut;
+    args.rows_per_cta = kRbRows;
+    dim3 grid((args.n_tiles + 1) / 2, (args.H + kRbRows - 1) / kRbRows, nj);
+    KScope ks(F_SR_BODY, st);
+    k_resblock<C><<<grid, 320, Cfg::SMEM, st>>>(tm, args);
+    return cudaGetLastError();
+}
+
 template <int C>
 static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                            const int32_t *job_count, cudaStream_t st) {
@@ -971,34 +1235,42 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
         if ((e = conv_rot<16, C, EPI_STORE>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
+    // residual blocks, fused (conv1 + ReLU + conv2 + skip), ping-pong hb / tb
+    const CUtensorMap *hin = &a->tm_h0;
+    uint16_t *hcur = a->h0;
     for (int b = 0; b < n_blocks; b++) {
-        const CUtensorMap &hin = (b == 0) ? a->tm_h0 : a->tm_hb;
-        const uint16_t *hres = (b == 0) ? a->h0 : a->hb;
-        ConvArgs g = base; LayerShape l1 = L(1 + 2 * b), l2 = L(2 + 2 * b);
-        g.b_off = l1.b_off; g.bias_off = l1.bias_off; g.out = a->tb;
-        if ((e = conv_rot<C, C, EPI_RELU>(F_SR_BODY, hin, g, nj, st)) != cudaSuccess) return e;
-        g = base; g.b_off = l2.b_off; g.bias_off = l2.bias_off; g.out = a->hb; g.resid = hres;
-        if ((e = conv_rot<C, C, EPI_RESID>(F_SR_BODY, a->tm_tb, g, nj, st)) != cudaSuccess) return e;
+        uint16_t *dst = (b % 2 == 0) ? a->hb : a->tb;
+        const LayerShape l1 = L(1 + 2 * b), l2 = L(2 + 2 * b);
+        RbArgs r{};
+        r.H = h; r.W = w; r.j0 = j0; r.jobs = jobs; r.job_count = job_count;
+        r.b1_off = l1.b_off; r.bias1_off = l1.bias_off; r.b2_off = l2.b_off; r.bias2_off = l2.bias_off;
+        r.out = dst;
+        if ((e = resblock<C>(*hin, r, nj, st)) != cudaSuccess) return e;
+        hin = (dst == a->hb) ? &a->tm_hb : &a->tm_tb;
+        hcur = dst;
     }
-    {   // end: h0 + conv(h; W_end) -> tb
+    // end: h0 + conv(h; W_end) -> the other buffer (read next by the 5x5 conv)
+    uint16_t *endout = (hcur == a->hb) ? a->tb : a->hb;
+    const CUtensorMap &tm5 = (endout == a->tb) ? a->tm_tb5 : a->tm_hb5;
+    {
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 1);
-        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->tb; g.resid = a->h0;
-        if ((e = conv_rot<C, C, EPI_RESID>(F_SR_END, n_blocks ? a->tm_hb : a->tm_h0, g, nj, st)) != cudaSuccess) return e;
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = endout; g.resid = a->h0;
+        if ((e = conv_rot<C, C, EPI_RESID>(F_SR_END, *hin, g, nj, st)) != cudaSuccess) return e;
     }
     {   // tail o shuffle o upsampler as one 5x5 conv at LR (+ bilinear skip, round, clamp) -> u8 HR
         const CompShape cs = model_comp(n_blocks, C, s);
         ConvArgs g = base;
         g.b_off = cs.b_off; g.bias_off = cs.bias_off;
-        if (s == 2) e = uptail<C, 16, 2>(a->tm_tb5, g, nj, st);
-        else if (s == 3) e = uptail<C, 32, 3>(a->tm_tb5, g, nj, st);
-        else e = uptail<C, 48, 4>(a->tm_tb5, g, nj, st);
+        if (s == 2) e = uptail<C, 16, 2>(tm5, g, nj, st);
+        else if (s == 3) e = uptail<C, 32, 3>(tm5, g, nj, st);
+        else e = uptail<C, 48, 4>(tm5, g, nj, st);
         if (e != cudaSuccess) return e;
         // exact frame-border ring (the tail's zero padding of u)
         KScope ks(F_SR_TAIL, st, 2);
         const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
         dim3 g1((next * C + 127) / 128, nj), g2((nring + 127) / 128, nj);
-        k_uptail_ext_u<<<g1, 128, 0, st>>>(jobs, j0, job_count, a->tb, h, w, C, s, cs.aux_off, a->band);
-        k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, a->tb, h, w, C, s, cs.aux_off, a->band);
+        k_uptail_ext_u<<<g1, 128, 0, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
+        k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     return cudaSuccess;
