@@ -20,6 +20,26 @@
 
 namespace ns {
 
+#ifdef NS_TRACE
+// debug-only timeline of CTA (0,0,0): per-role regions of {clock64, tag << 32 | step},
+// plain stores (no atomics on the traced threads' critical path)
+__device__ unsigned long long g_trace[8 * 2 * 1024];
+#define NS_TR(tag, q)                                                                            \
+    do {                                                                                         \
+        if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && _trn < 1024) {              \
+            g_trace[2 * (_trr * 1024 + _trn)] = clock64();                                       \
+            g_trace[2 * (_trr * 1024 + _trn) + 1] = ((unsigned long long)(tag) << 32) | (unsigned)(q); \
+            _trn++;                                                                              \
+        }                                                                                        \
+    } while (0)
+#define NS_TR_ROLE(r) int _trr = (r), _trn = 0
+#else
+#define NS_TR(tag, q) \
+    do {              \
+    } while (0)
+#define NS_TR_ROLE(r)
+#endif
+
 enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4 };
 constexpr int kSlots = 6;
 constexpr int kRows = 32;   // rows per CTA strip
@@ -565,13 +585,14 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-// Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-5 = epilogue
-// of tile 0, warps 6-9 = epilogue of tile 1 (warp w owns TMEM lanes 32 (w % 4)).
+// Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-17 = four
+// epilogue groups (tile 0 E1, tile 0 E2, tile 1 E1, tile 1 E2); warp w owns
+// TMEM lanes 32 (w % 4).
 // Per tile and input step q (h row y0-2+q): M1(q) conv1 -> E1(q) reads t row
 // y0-3+q, writes it (ReLU, bf16) to t slot q%2 -> M2(q) conv2 on it -> E2(q)
 // retires output row y0-4+q (+ b2 + h from the ring).  mbarriers only.
 template <int C>
-__global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
+__global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
     using Cfg = RbCfg<C>;
     constexpr int NB = Cfg::NB, NH = Cfg::NH;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -634,6 +655,7 @@ __global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUt
     if (warp == 0) {
         // ---------------------------------------------------------------- TMA producer
         if (lane == 0) {
+            NS_TR_ROLE(0);
             prefetch_tmap(&tm_in);
             mbar_arrive_expect_tx(wbar, 2 * (Cfg::B_BYTES + Cfg::BIAS_BYTES));
             bulk_load(s_w1, J.wts + a.b1_off, Cfg::B_BYTES, wbar);
@@ -649,60 +671,80 @@ __global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUt
                     if (q >= NH) mbar_wait(hfree(k, sl), ((q / NH) - 1) & 1);
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
                     tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                    NS_TR(30 + k, q);
                 }
             }
         }
     } else if (warp == 1) {
         // ---------------------------------------------------------------- MMA issuer
-        if (lane == 0) {
-            const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
-            auto mma_rot = [&](uint32_t dcol, const uint8_t *aslot, const uint8_t *wstrip, int yin) {
-                const uint32_t abase = smem_u32(aslot);
-                const uint32_t wbase = smem_u32(wstrip) + (uint32_t)mod3(1 - yin) * NB * 16;
+        // The whole warp runs the schedule (waits are warp-uniform); one elected
+        // lane issues each group of 6 MMAs + commit.  Order per step q:
+        //   M2(A,q) M1(A,q+1) M2(B,q) M1(B,q+1)
+        // so one tile's MMAs keep the tensor pipe busy while the other tile's
+        // conv1 epilogue runs.
+        NS_TR_ROLE(1);
+        const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
+        auto mma_rot = [&](uint32_t dcol, const uint8_t *aslot, const uint8_t *wstrip, int yin, uint64_t *bar) {
+            const uint32_t abase = smem_u32(aslot);
+            const uint32_t wbase = smem_u32(wstrip) + (uint32_t)mod3(1 - yin) * NB * 16;
+            const uint64_t ad0 = smem_desc(abase, kHalo * 16, 128), bd0 = smem_desc(wbase, 5 * NB * 16, 128);
+            if (elect_one()) {
 #pragma unroll
                 for (int dx = 0; dx < 3; dx++)
 #pragma unroll
-                    for (int kc = 0; kc < Cfg::KC; kc++)
-                        umma_bf16(dcol,
-                                  smem_desc(abase + (uint32_t)(2 * kc * kHalo * 16 + dx * 16), kHalo * 16, 128),
-                                  smem_desc(wbase + (uint32_t)((dx * Cfg::KC + kc) * 2 * 5 * NB * 16), 5 * NB * 16,
-                                            128),
-                                  idesc, 1u);
-            };
-            mbar_wait(wbar, 0);
-            for (int q = 0; q < nq; q++) {
-                for (int k = 0; k < 2; k++) {  // conv1 on h row y0-2+q
-                    if (!vk[k]) continue;
-                    mbar_wait(hfull(k, q % NH), (q / NH) & 1);
-                    if (q >= 1) mbar_wait(e1bar(k), (q - 1) & 1);  // E1(q-1) zeroed the block M1(q) first touches
+                    for (int kc = 0; kc < Cfg::KC; kc++)  // descriptor start address is bits 0-13 (>> 4)
+                        umma_bf16(dcol, ad0 + (uint64_t)((2 * kc * kHalo * 16 + dx * 16) >> 4),
+                                  bd0 + (uint64_t)(((dx * Cfg::KC + kc) * 2 * 5 * NB * 16) >> 4), idesc, 1u);
+                umma_commit(bar);
+            }
+            __syncwarp();
+        };
+        auto issue_m1 = [&](int k, int q) {  // conv1 on h row y0-2+q (E1(q-1) has been waited)
+            mbar_wait(hfull(k, q % NH), (q / NH) & 1);
+            tc_fence_after();
+            mma_rot(tmem + k * Cfg::TCOLS, hslot(k, q % NH), s_w1, y0 - 2 + q, m1bar(k));
+            if (lane == 0) NS_TR(3 + k, q);
+        };
+        mbar_wait(wbar, 0);
+        for (int k = 0; k < 2; k++)
+            if (vk[k]) issue_m1(k, 0);
+        for (int q = 0; q < nq; q++) {
+            for (int k = 0; k < 2; k++) {
+                if (!vk[k]) continue;
+                mbar_wait(e1bar(k), q & 1);  // E1(q): t row written, conv1 block of M1(q+1) zeroed
+                if (lane == 0) NS_TR(5 + k, q);
+                if (q >= 2) {                // conv2 on t row y0-3+q
+                    if (q >= 3) mbar_wait(e2bar(k), (q - 3) & 1);  // E2(q-1) zeroed the block M2(q) first touches
                     tc_fence_after();
-                    mma_rot(tmem + k * Cfg::TCOLS, hslot(k, q % NH), s_w1, y0 - 2 + q);
-                    umma_commit(m1bar(k));
+                    mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q, m2bar(k));
+                    if (lane == 0) NS_TR(7 + k, q);
                 }
-                if (q < 2) continue;
-                for (int k = 0; k < 2; k++) {  // conv2 on t row y0-3+q
-                    if (!vk[k]) continue;
-                    mbar_wait(e1bar(k), q & 1);                     // t row written
-                    if (q >= 3) mbar_wait(e2bar(k), (q - 3) & 1);   // E2(q-1) zeroed the block M2(q) first touches
-                    tc_fence_after();
-                    mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q);
-                    umma_commit(m2bar(k));
-                }
+                if (q + 1 < nq) issue_m1(k, q + 1);
             }
         }
     } else {
         // ---------------------------------------------------------------- epilogues
-        const int k = (warp - 2) / 4;
+        // warps 2..17: group g = (warp-2)/4 -> tile k = g/2, role = g%2 (E1 | E2).
+        // E1 (t -> SMEM, needs the async-proxy fence) and E2 (global stores) run
+        // in different warps so the fence never waits on in-flight global stores.
+        const int g = (warp - 2) / 4, k = g / 2, role = g % 2;
         if (vk[k]) {
             const int ew = warp % 4;   // TMEM lane quarter
             const int p = ew * 32 + lane;
             const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
             mbar_wait(wbar, 0);
-            for (int q = 0; q < nq; q++) {
-                const int yt = y0 - 3 + q, yo = yt - 1;
-                {   // E1: t = ReLU(conv1 + b1) -> t slot (zero outside the frame: conv2 padding)
+            NS_TR_ROLE(2 + g);
+            if (role == 0) {
+                for (int q = 0; q < nq; q++) {  // E1: t = ReLU(conv1 + b1) -> t slot
+                    const int yt = y0 - 3 + q;
                     mbar_wait(m1bar(k), q & 1);
+                    if (warp % 4 == 2 && lane == 0) NS_TR(10 + k, q);
                     tc_fence_after();
+#ifdef NS_TRACE_NOEPI
+                    tc_fence_before();
+                    mbar_arrive(e1bar(k));
+                    continue;
+#endif
                     const uint32_t acc = tl + (uint32_t)(mod3(yt) * NB);
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
@@ -728,10 +770,20 @@ __global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUt
                     fence_proxy_async_smem();
                     tc_fence_before();
                     mbar_arrive(e1bar(k));
+                    if (warp % 4 == 2 && lane == 0) NS_TR(12 + k, q);
                 }
-                if (q >= 2) {  // E2: out = conv2 + b2 + h
+            } else {
+                for (int q = 2; q < nq; q++) {  // E2: out = conv2 + b2 + h
+                    const int yo = y0 - 4 + q;
                     mbar_wait(m2bar(k), (q - 2) & 1);
+                    if (warp % 4 == 2 && lane == 0) NS_TR(20 + k, q);
                     tc_fence_after();
+#ifdef NS_TRACE_NOEPI
+                    tc_fence_before();
+                    mbar_arrive(hfree(k, (q - 2) % NH));
+                    mbar_arrive(e2bar(k));
+                    continue;
+#endif
                     const uint32_t acc = tl + 3 * NB + (uint32_t)(mod3(yo) * NB);
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
@@ -761,6 +813,7 @@ __global__ void __launch_bounds__(320, 1) k_resblock(const __grid_constant__ CUt
                     tc_fence_before();
                     mbar_arrive(hfree(k, (q - 2) % NH));
                     mbar_arrive(e2bar(k));
+                    if (warp % 4 == 2 && lane == 0) NS_TR(22 + k, q);
                 }
             }
         }
@@ -1212,7 +1265,7 @@ static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, 
     args.rows_per_cta = kRbRows;
     dim3 grid((args.n_tiles + 1) / 2, (args.H + kRbRows - 1) / kRbRows, nj);
     KScope ks(F_SR_BODY, st);
-    k_resblock<C><<<grid, 320, Cfg::SMEM, st>>>(tm, args);
+    k_resblock<C><<<grid, 576, Cfg::SMEM, st>>>(tm, args);
     return cudaGetLastError();
 }
 
@@ -1283,3 +1336,15 @@ cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int 
 }
 
 }  // namespace ns
+
+#ifdef NS_TRACE
+extern "C" NS_API int ns_trace_read(unsigned long long *out, int max_pairs) {
+    const int n = max_pairs < 8 * 1024 ? max_pairs : 8 * 1024;
+    cudaMemcpyFromSymbol(out, ns::g_trace, sizeof(unsigned long long) * 2 * n);
+    return n;
+}
+extern "C" NS_API void ns_trace_reset() {
+    static unsigned long long z[8 * 2 * 1024];
+    cudaMemcpyToSymbol(ns::g_trace, z, sizeof(z));
+}
+#endif

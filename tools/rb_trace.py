@@ -1,0 +1,43 @@
+"""Timeline of one CTA of k_resblock (trace build, tools/bin/libneuroscaler_trace.so)."""
+import ctypes, os, sys
+import numpy as np
+import torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_sigcomm_yeolkjyh22_b200 as ns
+import synth
+ns.LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "bin", os.environ.get("NS_TRACE_LIB", "libneuroscaler_trace.so"))
+L = ns.lib()
+L.ns_trace_read.argtypes = [ctypes.c_void_p, ctypes.c_int]
+L.ns_trace_read.restype = ctypes.c_int
+ctx = ns.Context(0, pool_bytes=16 << 30)
+m = ctx.model(8, 32, 3)
+m.set_weights(synth.make_weights(1, 8, 32, 3))
+c = synth.make_chunk(5, 1280, 720, 3, 1)
+lr = torch.from_numpy(c.lr).cuda()
+hr = torch.zeros((16, 3, 2160, 3840), dtype=torch.uint8, device="cuda")
+jobs = [(m, lr[0], hr[i]) for i in range(16)]
+ctx.sr_anchors(jobs); torch.cuda.synchronize()
+L.ns_trace_reset()
+# only the first fused block of one batch is traced: regions are overwritten by later launches,
+# so run exactly one batch and keep the LAST block's timeline (all blocks behave alike)
+ctx.sr_anchors(jobs); torch.cuda.synchronize()
+buf = (ctypes.c_ulonglong * (2 * 8192))()
+n = L.ns_trace_read(buf, 8192)
+a = np.frombuffer(buf, dtype=np.uint64)[:2 * n].reshape(n, 2)
+a = a[a[:, 0] != 0]
+t = a[:, 0].astype(np.int64); tag = (a[:, 1] >> 32).astype(int); q = (a[:, 1] & 0xffffffff).astype(int)
+order = np.argsort(t)
+t, tag, q = t[order], tag[order], q[order]
+t0 = t[0]
+names = {1: "M1 hfull ok A", 2: "M1 hfull ok B", 3: "M1 issued A", 4: "M1 issued B", 5: "M2 e1 ok A", 6: "M2 e1 ok B",
+         7: "M2 issued A", 8: "M2 issued B", 10: "E1 m1 ok A", 11: "E1 m1 ok B", 12: "E1 arrive A", 13: "E1 arrive B",
+         20: "E2 m2 ok A", 21: "E2 m2 ok B", 22: "E2 arrive A", 23: "E2 arrive B", 30: "TMA load A", 31: "TMA load B"}
+for i in range(len(t)):
+    if q[i] < 14 and tag[i] != 30 and tag[i] != 31:
+        print(f"{t[i]-t0:8d}  q={q[i]:3d}  {names.get(tag[i], tag[i])}")
+# steady state period
+for tg in (3, 7, 12, 22):
+    ts = t[tag == tg]
+    if len(ts) > 20:
+        d = np.diff(ts[10:60])
+        print("tag", names[tg], "median period", int(np.median(d)), "cycles")
