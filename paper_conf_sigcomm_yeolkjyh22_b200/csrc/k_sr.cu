@@ -57,6 +57,7 @@ struct ConvArgs {
     int s;                  // scale (shuffle / tail)
     int sub0;               // shuffle: first sub-pixel of this launch
     int lr_h, lr_w;         // tail: LR dims of the bilinear skip
+    float *ring;            // uptail: fp32 t of the HR frame-border ring [job][nring][3]
 };
 
 __host__ __device__ constexpr uint32_t round_up(uint32_t v, uint32_t a) { return (v + a - 1) / a * a; }
@@ -978,6 +979,21 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
                     }
                 }
             }
+            // frame-border ring (rare lanes): keep the fp32 composed t for the exact fix-up
+            if (x < lw && (r == 0 || r == lh - 1 || x == 0 || x == lw - 1)) {
+                for (int i = 0; i < S; i++)
+                    for (int j = 0; j < S; j++) {
+                        const int Y = S * r + i, X = S * x + j;
+                        if (!(Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1)) continue;
+                        const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X
+                                     : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
+                        for (int c = 0; c < 3; c++) {
+                            const int n = (i * S + j) * 3 + c;
+                            a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] =
+                                __uint_as_float(v[n]) + s_bias[n];
+                        }
+                    }
+            }
         }
         tmem_wait_st();
         tc_fence_before();
@@ -1025,36 +1041,75 @@ __device__ __forceinline__ float act_at(const uint16_t *act, int y, int x, int c
     return __uint_as_float((uint32_t)act[(((size_t)y * (C / 8) + ci / 8) * w + x) * 8 + ci % 8] << 16);
 }
 
-// one thread per (upsampler channel c, out-of-frame position): consecutive lanes
-// take consecutive positions, so a warp's weight loads broadcast (<= s rows)
-__global__ void k_uptail_ext_u(const SrJob *jobs, int j0, const int32_t *job_count, const uint16_t *hact, int h,
-                               int w, int C, int s, size_t aux_off, float *ext) {
+// One thread per out-of-frame position, all C channels.  A CTA covers positions
+// of one band (row -1, row H, col -1, col W), whose upsampler taps are the
+// single valid kernel row/column (ky=2 / ky=0 / kx=2 / kx=0): their weights for
+// the s sub-pixels are staged in shared memory ([s][C][C][3] fp32).
+constexpr int kExtThreads = 128;
+__global__ void __launch_bounds__(kExtThreads) k_uptail_ext_u(const SrJob *jobs, int j0, const int32_t *job_count,
+                                                             const uint16_t *hact, int h, int w, int C, int s,
+                                                             size_t aux_off, float *ext) {
+    extern __shared__ float wsm[];  // [s][C out][C in][3]
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
     const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H;
-    const int e = blockIdx.x * blockDim.x + threadIdx.x;
-    if (e >= next * C) return;
-    const int pos = e % next, c = e / next;
-    int Y, X;
-    ext_pos(pos, H, W, Y, X);
-    const int y = (Y + s) / s - 1, i = Y - s * y, x = (X + s) / s - 1, j = X - s * x;
+    // band of this CTA: blocks are laid out band by band
+    const int nbr = (W + 2 + kExtThreads - 1) / kExtThreads, nbc = (H + kExtThreads - 1) / kExtThreads;
+    int band, local_blk = blockIdx.x;
+    if (local_blk < nbr) band = 0;
+    else if ((local_blk -= nbr) < nbr) band = 1;
+    else if ((local_blk -= nbr) < nbc) band = 2;
+    else { local_blk -= nbc; band = 3; }
+    const int bandlen = band < 2 ? W + 2 : H;
+    const int e = local_blk * kExtThreads + threadIdx.x;
     const float *Wup = reinterpret_cast<const float *>(jobs[job].wts + aux_off);
     const float *bup = Wup + (size_t)s * s * C * C * 9;
-    const int uc = c * s * s + i * s + j;
+    // stage weights: sub-pixel index sp in 0..s-1 (j' for row bands, i' for column bands)
+    for (int idx = threadIdx.x; idx < s * C * C * 3; idx += blockDim.x) {
+        const int t = idx % 3, ci = (idx / 3) % C, c = (idx / (3 * C)) % C, sp = idx / (3 * C * C);
+        int ip, jp, ky, kx;
+        if (band == 0) { ip = s - 1; jp = sp; ky = 2; kx = t; }
+        else if (band == 1) { ip = 0; jp = sp; ky = 0; kx = t; }
+        else if (band == 2) { ip = sp; jp = s - 1; ky = t; kx = 2; }
+        else { ip = sp; jp = 0; ky = t; kx = 0; }
+        wsm[idx] = Wup[((size_t)(c * s * s + ip * s + jp) * C + ci) * 9 + ky * 3 + kx];
+    }
+    __syncthreads();
+    if (e >= bandlen) return;
+    int Y, X, pos;
+    if (band == 0) { Y = -1; X = e - 1; pos = e; }
+    else if (band == 1) { Y = H; X = e - 1; pos = (W + 2) + e; }
+    else if (band == 2) { Y = e; X = -1; pos = 2 * (W + 2) + e; }
+    else { Y = e; X = W; pos = 2 * (W + 2) + H + e; }
+    const int y = (Y + s) / s - 1, i = Y - s * y, x = (X + s) / s - 1, j = X - s * x;
+    const int sp = band < 2 ? j : i;
     const uint16_t *act = hact + (size_t)slot * h * (C / 8) * w * 8;
-    float acc = bup[uc];
-    for (int ky = 0; ky < 3; ky++)
-        for (int kx = 0; kx < 3; kx++) {
-            const int yy = y + ky - 1, xx = x + kx - 1;
-            if (yy < 0 || yy >= h || xx < 0 || xx >= w) continue;
-            for (int ci = 0; ci < C; ci++) acc += Wup[((size_t)uc * C + ci) * 9 + ky * 3 + kx] * act_at(act, yy, xx, ci, h, w, C);
-        }
-    ext[((size_t)slot * next + pos) * C + c] = acc;
+    float hv[3][32];
+#pragma unroll
+    for (int t = 0; t < 3; t++) {
+        const int yy = band == 0 ? 0 : band == 1 ? h - 1 : y + t - 1;
+        const int xx = band == 2 ? 0 : band == 3 ? w - 1 : x + t - 1;
+        const bool ok = yy >= 0 && yy < h && xx >= 0 && xx < w;
+#pragma unroll
+        for (int ci = 0; ci < 32; ci++)
+            hv[t][ci] = (ok && ci < C) ? __uint_as_float((uint32_t)act[(((size_t)yy * (C / 8) + ci / 8) * w + xx) * 8 + ci % 8] << 16) : 0.f;
+    }
+    const float *wb = wsm + (size_t)sp * C * C * 3;
+    float *dst = ext + ((size_t)slot * next + pos) * C;
+    for (int c = 0; c < C; c++) {
+        float acc = bup[c * s * s + i * s + j];
+        const float *wr = wb + (size_t)c * C * 3;
+#pragma unroll
+        for (int ci = 0; ci < 32; ci++)
+            if (ci < C) acc += wr[ci * 3 + 0] * hv[0][ci] + wr[ci * 3 + 1] * hv[1][ci] + wr[ci * 3 + 2] * hv[2][ci];
+        dst[c] = acc;
+    }
 }
 
-// one thread per ring pixel
-__global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_count, const uint16_t *hact, int h,
-                              int w, int C, int s, size_t aux_off, const float *ext) {
+// One thread per ring pixel: t = (composed t from the uptail epilogue) minus
+// the out-of-frame tail taps, then the bilinear skip, round, clamp, store.
+__global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, int C, int s,
+                              size_t aux_off, const float *ext, const float *ring) {
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
     const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
@@ -1068,32 +1123,19 @@ __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_coun
     const SrJob J = jobs[job];
     const float *aux = reinterpret_cast<const float *>(J.wts + aux_off);
     const float *Wt = aux + (size_t)s * s * C * C * 9 + (size_t)s * s * C;
-    const float *Wc = Wt + (size_t)3 * C * 9 + 3;
-    const float *bc = Wc + (size_t)s * s * 3 * C * 25;
-    const uint16_t *act = hact + (size_t)slot * h * (C / 8) * w * 8;
     const float *E = ext + (size_t)slot * next * C;
-    const int r = Y / s, i = Y % s, x = X / s, j = X % s;
-    float t[3];
-    for (int co = 0; co < 3; co++) {
-        const int n = (i * s + j) * 3 + co;
-        float acc = bc[n];
-        for (int ty = 0; ty < 5; ty++)
-            for (int tx = 0; tx < 5; tx++) {
-                const int yy = r + ty - 2, xx = x + tx - 2;
-                if (yy < 0 || yy >= h || xx < 0 || xx >= w) continue;
-                for (int ci = 0; ci < C; ci++)
-                    acc += Wc[((size_t)n * C + ci) * 25 + ty * 5 + tx] * act_at(act, yy, xx, ci, h, w, C);
-            }
-        t[co] = acc;
-    }
+    const float *tr = ring + ((size_t)slot * nring + e) * 3;
+    float t[3] = {tr[0], tr[1], tr[2]};
     for (int dY = -1; dY <= 1; dY++)
         for (int dX = -1; dX <= 1; dX++) {
             const int Yn = Y + dY, Xn = X + dX;
-            if (Yn >= 0 && Yn < H && Xn >= 0 && Xn < W) continue;  // in-frame: already right
+            if (Yn >= 0 && Yn < H && Xn >= 0 && Xn < W) continue;  // in-frame: the composed value is right
             const float *u = E + (size_t)ext_index(Yn, Xn, H, W) * C;
-            for (int c = 0; c < C; c++)
+            for (int c = 0; c < C; c++) {
+                const float uc = u[c];
 #pragma unroll
-                for (int co = 0; co < 3; co++) t[co] -= Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)] * u[c];
+                for (int co = 0; co < 3; co++) t[co] -= Wt[((size_t)co * C + c) * 9 + (dY + 1) * 3 + (dX + 1)] * uc;
+            }
         }
     int ya, yb, wy, xa, xb, wx;
     up_tap(Y, s, h, ya, yb, wy);
@@ -1159,9 +1201,9 @@ static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int
     return r == CUDA_SUCCESS ? 0 : -2;
 }
 
-static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u positions x C
+static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u positions x C + ring t x 3
     const size_t H = (size_t)h * s, W = (size_t)w * s;
-    return (2 * (W + 2) + 2 * H) * C;
+    return (2 * (W + 2) + 2 * H) * C + (2 * W + 2 * (H - 2)) * 3;
 }
 
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
@@ -1314,6 +1356,10 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         const CompShape cs = model_comp(n_blocks, C, s);
         ConvArgs g = base;
         g.b_off = cs.b_off; g.bias_off = cs.bias_off;
+        {
+            const size_t H = (size_t)h * s, W = (size_t)w * s;
+            g.ring = a->band + (size_t)a->nb * (2 * (W + 2) + 2 * H) * C;
+        }
         if (s == 2) e = uptail<C, 16, 2>(tm5, g, nj, st);
         else if (s == 3) e = uptail<C, 32, 3>(tm5, g, nj, st);
         else e = uptail<C, 48, 4>(tm5, g, nj, st);
@@ -1321,9 +1367,17 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         // exact frame-border ring (the tail's zero padding of u)
         KScope ks(F_SR_TAIL, st, 2);
         const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
-        dim3 g1((next * C + 127) / 128, nj), g2((nring + 127) / 128, nj);
-        k_uptail_ext_u<<<g1, 128, 0, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
-        k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
+        const int nbr = (W + 2 + kExtThreads - 1) / kExtThreads, nbc = (H + kExtThreads - 1) / kExtThreads;
+        const size_t wsm = (size_t)s * C * C * 3 * sizeof(float);
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_uptail_ext_u, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
+            attr = true;
+        }
+        dim3 g1(2 * nbr + 2 * nbc, nj), g2((nring + 127) / 128, nj);
+        k_uptail_ext_u<<<g1, kExtThreads, wsm, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
+        k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, h, w, C, s, cs.aux_off, a->band,
+                                          a->band + (size_t)a->nb * next * C);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     return cudaSuccess;
