@@ -552,19 +552,21 @@ __device__ __forceinline__ uint16_t f2bf(float f) {  // round to nearest even
 // with (i+dY) = s oy + i', (j+dX) = s ox + j', ky = ty - 1 - oy, kx = tx - 1 - ox.
 __global__ void k_repack_comp(const uint16_t *blob, size_t up_off, size_t tail_off, int C, int s, CompShape cs,
                               uint8_t *packed) {
-    const int nb = cs.nb, KC = C / 16, nout = s * s * 3;
-    const size_t total = (size_t)5 * KC * 2 * 9 * nb * 8;
+    const int nb = cs.nb, KC = C / 16, nout = s * s * 3, ns = cs.nstrip;
+    const size_t total = (size_t)5 * KC * 2 * ns * nb * 8;
     const uint16_t *Wup = blob + up_off, *bup = blob + up_off + (size_t)s * s * C * C * 9;
     const uint16_t *Wt = blob + tail_off, *bt = blob + tail_off + (size_t)3 * C * 9;
-    const int strip[9] = {4, 3, 2, 1, 0, 4, 3, 2, 1};
+    const int strip9[9] = {4, 3, 2, 1, 0, 4, 3, 2, 1};
+    const int strip11[11] = {4, 3, 2, 1, 0, -1, 4, 3, 2, 1, 0};  // -1: zero block (6th ring slot)
     uint16_t *B = reinterpret_cast<uint16_t *>(packed + cs.b_off);
     for (size_t e = (size_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += (size_t)gridDim.x * blockDim.x) {
         const int k8 = e % 8;
-        const int nn = (e / 8) % (9 * nb);
-        const int kh = (e / (8 * 9 * nb)) % 2;
-        const int kc = (e / (16 * 9 * nb)) % KC;
-        const int tx = (int)(e / ((size_t)16 * 9 * nb * KC));
-        const int ty = strip[nn / nb], n = nn % nb;
+        const int nn = (e / 8) % (ns * nb);
+        const int kh = (e / (8 * ns * nb)) % 2;
+        const int kc = (e / (16 * ns * nb)) % KC;
+        const int tx = (int)(e / ((size_t)16 * ns * nb * KC));
+        const int ty = ns == 11 ? strip11[nn / nb] : strip9[nn / nb], n = nn % nb;
+        if (ty < 0) { B[e] = 0; continue; }
         const int ci = kc * 16 + kh * 8 + k8;
         float acc = 0.f;
         if (n < nout) {

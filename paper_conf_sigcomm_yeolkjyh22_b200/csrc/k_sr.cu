@@ -1015,6 +1015,230 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
     (void)NOUT;
 }
 
+// Warp-specialized composed upsampler+tail for s <= 3: warp 0 TMA, warp 1 MMA
+// (elect.sync groups), 2 x-tiles per CTA, and per tile S epilogue groups of 4
+// warps (group g = HR sub-row i) that read the retired row in parallel.  The
+// 5-block accumulator ring (row r -> block r mod 5) is the same as k_uptail;
+// the MMA on input row y waits for the epilogue of row y-3 (previous step),
+// and the other tile's MMAs cover that wait.
+template <int CIN, int NB, int S>
+struct Up2Cfg {
+    static constexpr int KC = CIN / 16, NSTRIP = 9;
+    static constexpr uint32_t B_BYTES = 5u * KC * 2 * NSTRIP * NB * 16;
+    static constexpr uint32_t BIAS_BYTES = NB * 4u;
+    static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
+    static constexpr uint32_t SLOT_BYTES = kHalo5 * CIN * 2u;
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    static constexpr int NS = 3;                                    // input ring per tile
+    static constexpr uint32_t OUTG = round_up(3u * kTile * S, 128);  // per group: [plane][128 s] bytes
+    static constexpr uint32_t TILE_BYTES = NS * SLOT + S * OUTG;
+    static constexpr uint32_t TCOLS = 5 * NB;
+    static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
+    static constexpr int NBAR = 2 * (2 * NS + 3) + 1;
+    static constexpr int NWARPS = 2 + 2 * S * 4;
+    static constexpr uint32_t SMEM = W_REGION + 2 * TILE_BYTES + NBAR * 8 + 64;
+    static_assert(5 * NB <= 256, "N = 5 nb");
+    static_assert(SMEM <= 232448, "shared memory");
+};
+
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+// One HR sub-row I of an LR pixel: the s outputs x 3 planes of the composed
+// conv + the integer bilinear skip, rounded and clamped into the staging row;
+// frame-border ring pixels also keep their fp32 t for the exact fix-up.
+template <int NB, int S, int I>
+__device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[NB], const float *s_bias, const SrJob &J,
+                                              const ConvArgs &a, uint8_t *so, int p, int x, int r, int lh, int lw,
+                                              int slot_job) {
+    const int HH = lh * S, WW = lw * S;
+    int ya, yb, wy;
+    up_tap(S * r + I, S, lh, ya, yb, wy);
+    const size_t plane = (size_t)lh * lw;
+#pragma unroll
+    for (int j = 0; j < S; j++) {
+        int xa, xb, wx;
+        up_tap(S * x + j, S, lw, xa, xb, wx);
+#pragma unroll
+        for (int c = 0; c < 3; c++) {
+            const uint8_t *L = J.lr + c * plane;
+            const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
+            const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
+            const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
+            const int U = (vv + 8192) >> 14;
+            constexpr int dummy = 0;
+            (void)dummy;
+            const int n = (I * S + j) * 3 + c;
+            const float t = __uint_as_float(v[n]) + s_bias[n];
+            so[c * (kTile * S) + p * S + j] = (uint8_t)fminf(fmaxf(floorf((float)U + t + 0.5f), 0.f), 255.f);
+            const int Y = S * r + I, X = S * x + j;
+            if (Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1) {
+                const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
+                a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = t;
+            }
+        }
+    }
+}
+
+template <int CIN, int NB, int S>
+__global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
+    k_uptail2(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+    using Cfg = Up2Cfg<CIN, NB, S>;
+    constexpr int NS = Cfg::NS;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint8_t *s_w = smem;
+    const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
+    uint8_t *s_tile = smem + Cfg::W_REGION;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_tile + 2 * Cfg::TILE_BYTES);
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + Cfg::NBAR);
+    auto islot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
+    auto oslot = [&](int k, int g) { return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + g * Cfg::OUTG; };
+    // per tile: hfull[NS], sfree[NS], mdone[2], edone
+    auto hfull = [&](int k, int i) { return &bars[k * (2 * NS + 3) + i]; };
+    auto sfree = [&](int k, int i) { return &bars[k * (2 * NS + 3) + NS + i]; };
+    auto mdone = [&](int k, int par) { return &bars[k * (2 * NS + 3) + 2 * NS + par]; };
+    auto edone = [&](int k) { return &bars[k * (2 * NS + 3) + 2 * NS + 2]; };
+    uint64_t *wbar = &bars[2 * (2 * NS + 3)];
+
+    const int slot_job = blockIdx.z;
+    const int job = a.j0 + slot_job;
+    if (a.job_count && job >= *a.job_count) return;
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int y0 = blockIdx.y * a.rows_per_cta;
+    const int y1 = min(y0 + a.rows_per_cta, a.H);
+    const int nq = y1 - y0 + 4;  // input rows y0-2 .. y1+1
+    const int lh = a.H, lw = a.W, HH = lh * S, WW = lw * S;
+    int x0k[2];
+    bool vk[2];
+    for (int k = 0; k < 2; k++) {
+        const int tix = 2 * blockIdx.x + k;
+        vk[k] = tix * kTile < lw;
+        x0k[k] = tix * kTile;
+    }
+    if (tid == 0) {
+        for (int k = 0; k < 2; k++) {
+            for (int i = 0; i < NS; i++) { mbar_init(hfull(k, i), 1); mbar_init(sfree(k, i), 1); }
+            mbar_init(mdone(k, 0), 1);
+            mbar_init(mdone(k, 1), 1);
+            mbar_init(edone(k), 128);
+        }
+        mbar_init(wbar, 1);
+        fence_mbar_init();
+    }
+    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *s_tmem;
+    const SrJob J = a.jobs[job];
+    if (warp >= 2 && ((warp - 2) / 4) % S == 0) {
+        // sub-row-0 group of each tile: zero its accumulator ring (the block of
+        // row y0 has no earlier owner whose retirement would have zeroed it)
+        const int k = (warp - 2) / 4 / S;
+        const uint32_t tl = tmem + ((uint32_t)((warp % 4) * 32) << 16) + k * Cfg::TCOLS;
+#pragma unroll 1
+        for (int b = 0; b < 5; b++) tmem_zeroN<NB>(tl + b * NB);
+        tmem_wait_st();
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+
+    if (warp == 0) {
+        if (lane == 0) {  // ---- TMA producer
+            prefetch_tmap(&tm_in);
+            mbar_arrive_expect_tx(wbar, Cfg::B_BYTES + Cfg::BIAS_BYTES);
+            bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, wbar);
+            bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, wbar);
+            for (int q = 0; q < nq; q++)
+                for (int k = 0; k < 2; k++) {
+                    if (!vk[k]) continue;
+                    const int sl = q % NS;
+                    if (q >= NS) mbar_wait(sfree(k, sl), ((q / NS) - 1) & 1);
+                    mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
+                    tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                }
+        }
+    } else if (warp == 1) {  // ---- MMA issuer (whole warp, elected lane issues)
+        const uint32_t idesc = idesc_bf16_f32(128, 5 * NB);
+        mbar_wait(wbar, 0);
+        for (int q = 0; q < nq; q++)
+            for (int k = 0; k < 2; k++) {
+                if (!vk[k]) continue;
+                const int sl = q % NS, yin = y0 - 2 + q;
+                mbar_wait(hfull(k, sl), (q / NS) & 1);
+                if (q >= 1) mbar_wait(edone(k), (q - 1) & 1);  // E(q-1) retired row yin-3 = the block of yin+2
+                tc_fence_after();
+                const uint64_t ad0 = smem_desc(smem_u32(islot(k, sl)), kHalo5 * 16, 128);
+                const uint64_t bd0 = smem_desc(smem_u32(s_w) + (uint32_t)mod5(2 - yin) * NB * 16,
+                                               Cfg::NSTRIP * NB * 16, 128);
+                if (elect_one()) {
+#pragma unroll
+                    for (int dx = 0; dx < 5; dx++)
+#pragma unroll
+                        for (int kc = 0; kc < Cfg::KC; kc++)
+                            umma_bf16(tmem + k * Cfg::TCOLS, ad0 + (uint64_t)((2 * kc * kHalo5 * 16 + dx * 16) >> 4),
+                                      bd0 + (uint64_t)(((dx * Cfg::KC + kc) * 2 * Cfg::NSTRIP * NB * 16) >> 4), idesc,
+                                      1u);
+                    umma_commit(sfree(k, sl));
+                    umma_commit(mdone(k, q & 1));
+                }
+                __syncwarp();
+            }
+    } else {  // ---- epilogue groups: tile k, HR sub-row g
+        const int grp = (warp - 2) / 4, k = grp / S, g = grp % S;
+        const int ew = warp % 4;
+        const int p = ew * 32 + lane;
+        const int x = x0k[k] + p;
+        const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
+        uint8_t *so = oslot(k, g);
+        if (vk[k]) {
+            mbar_wait(wbar, 0);
+            for (int q = 0; q < nq; q++) {
+                const int r = y0 - 4 + q;  // LR output row completed at this step
+                const bool valid = r >= y0;
+                // skip taps for sub-row g (compile-time per g via switch below)
+                mbar_wait(mdone(k, q & 1), (q >> 1) & 1);
+                tc_fence_after();
+                const uint32_t acc = tl + (uint32_t)(mod5(r) * NB);
+                uint32_t v[NB];
+                tmem_ldN<NB>(acc, v);
+                tmem_wait_ld();
+                tc_fence_before();
+                named_bar(1 + k, 128 * S);  // every group of this tile has read the block
+                if (g == 0) {
+                    tc_fence_after();
+                    tmem_zeroN<NB>(acc);
+                    tmem_wait_st();
+                    tc_fence_before();
+                    mbar_arrive(edone(k));
+                }
+                if (valid) {
+                    if (x < lw) {
+                        if (g == 0) uptail_subrow<NB, S, 0>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 1 && g == 1) uptail_subrow<NB, S, (S > 1 ? 1 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 2 && g == 2) uptail_subrow<NB, S, (S > 2 ? 2 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 3 && g == 3) uptail_subrow<NB, S, (S > 3 ? 3 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
+                    }
+                    const int i = g;
+                    named_bar(3 + grp, 128);  // this group's staging row is complete
+                    const int xs_hr = x0k[k] * S, wv = min(kTile, lw - x0k[k]) * S;
+                    constexpr int CH = kTile * S / 8;
+                    for (int e = ew * 32 + lane; e < 3 * CH; e += 128) {
+                        const int ch = e % CH, c = e / CH;
+                        if (ch * 8 < wv)
+                            *reinterpret_cast<uint2 *>(J.hr + (size_t)c * HH * WW + (size_t)(S * r + i) * WW + xs_hr + ch * 8) =
+                                *reinterpret_cast<const uint2 *>(so + c * (kTile * S) + ch * 8);
+                    }
+                    named_bar(3 + grp, 128);  // staging can be overwritten
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
+}
+
 // ---- exact frame-border ring.  The composed conv evaluates the tail over
 // u at the out-of-frame HR positions around the frame (rows -1 and H, cols -1
 // and W), where the definition has zeros (tail zero padding).  For every ring
@@ -1311,6 +1535,24 @@ static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, 
     return cudaGetLastError();
 }
 
+template <int CIN, int NB, int S>
+static cudaError_t uptail2(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+    using Cfg = Up2Cfg<CIN, NB, S>;
+    static bool attr = false;
+    if (!attr) {
+        cudaError_t e = cudaFuncSetAttribute(k_uptail2<CIN, NB, S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             Cfg::SMEM);
+        if (e != cudaSuccess) return e;
+        attr = true;
+    }
+    const int ntiles = (args.W + kTile - 1) / kTile;
+    args.rows_per_cta = kRotRows;
+    dim3 grid((ntiles + 1) / 2, (args.H + kRotRows - 1) / kRotRows, nj);
+    KScope ks(F_SR_UP, st);
+    k_uptail2<CIN, NB, S><<<grid, Cfg::NWARPS * 32, Cfg::SMEM, st>>>(tm, args);
+    return cudaGetLastError();
+}
+
 template <int C>
 static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                            const int32_t *job_count, cudaStream_t st) {
@@ -1360,8 +1602,8 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
             const size_t H = (size_t)h * s, W = (size_t)w * s;
             g.ring = a->band + (size_t)a->nb * (2 * (W + 2) + 2 * H) * C;
         }
-        if (s == 2) e = uptail<C, 16, 2>(tm5, g, nj, st);
-        else if (s == 3) e = uptail<C, 32, 3>(tm5, g, nj, st);
+        if (s == 2) e = uptail2<C, 16, 2>(tm5, g, nj, st);
+        else if (s == 3) e = uptail2<C, 32, 3>(tm5, g, nj, st);
         else e = uptail<C, 48, 4>(tm5, g, nj, st);
         if (e != cudaSuccess) return e;
         // exact frame-border ring (the tail's zero padding of u)

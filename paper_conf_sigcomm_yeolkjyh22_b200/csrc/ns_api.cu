@@ -118,9 +118,10 @@ CompShape model_comp(int n_blocks, int C, int s) {
     CompShape c{};
     const int nout = s * s * 3;
     c.nb = (nout + 15) / 16 * 16;
+    c.nstrip = 9;
     const size_t base = blob_layers_bytes(n_blocks, C, s);
     c.b_off = base;
-    c.bias_off = base + align128((size_t)5 * (C / 16) * 2 * 9 * c.nb * 16);
+    c.bias_off = base + align128((size_t)5 * (C / 16) * 2 * c.nstrip * c.nb * 16);
     c.aux_off = c.bias_off + align128((size_t)c.nb * 4);
     return c;
 }

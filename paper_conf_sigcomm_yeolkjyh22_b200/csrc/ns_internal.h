@@ -60,12 +60,13 @@ size_t model_packed_bytes(int n_blocks, int C, int s);
 // Derived regions after the blob layers:
 //  * COMP: tail o pixel-shuffle o upsampler composed into one 5x5 conv at LR
 //    resolution, h (C ch) -> s*s*3 outputs (n = (i*s + j)*3 + co), padded to nb;
-//    UMMA B operand of the 5-row rotated conv: [tx 5][kc][kh 2][9 nb][8] bf16
-//    (kernel-row strip ty = 4,3,2,1,0,4,3,2,1), then fp32 bias[nb].
+//    UMMA B operand of the rotated 5x5 conv: [tx 5][kc][kh 2][nstrip nb][8] bf16,
+//    then fp32 bias[nb].
 //  * AUX (fp32, for the exact frame-border fix-up): W_up [s*s*C][C][9], b_up,
 //    W_tail [3][C][9], b_tail, then the composed Wc [s*s*3][C][25], bc [s*s*3].
 struct CompShape {
     int nb;                  // padded outputs per block (16 | 32 | 48)
+    int nstrip;              // strip blocks: 9 = [4,3,2,1,0,4,3,2,1] (5-block window)
     size_t b_off, bias_off;  // composed operand / bias
     size_t aux_off;          // fp32 W_up, b_up, W_tail, b_tail (contiguous)
 };

@@ -284,3 +284,45 @@ def test_c2_full_size(ctx):
     # reuse: bit-exact against the oracle given the GPU's own SR anchor bytes
     exp, _, _ = oracle.reconstruct(c, ea, got, np.zeros_like(got[0]), np.zeros_like(got[0]))
     assert np.array_equal(got, exp)
+
+
+# ---------------------------------------------------------------- c3 / c4 full size (bench config)
+@pytest.mark.slow
+def test_c3_full_size_batched(ctx):
+    """BASELINE configs[2]/[3] at full size through the bench's call
+    (ns_enhance_streams, several streams with distinct content-aware models,
+    SR jobs batched across streams): selection bit-exact for every stream; SR
+    on sampled windows incl. the four frame corners (exercises the exact
+    frame-border fix-up of the composed upsampler+tail); reconstruction of a
+    whole 60-frame 4K chunk bit-exact given the GPU's SR anchor bytes."""
+    cfg = synth.CONFIGS[3]
+    B, C, s, n, k = cfg["n_blocks"], cfg["n_ch"], cfg["scale"], cfg["n"], cfg["k"]
+    w, h = cfg["w"], cfg["h"]
+    S = 3
+    cs = [synth.make_chunk(3001 + i, w, h, s, n, types=synth.default_types(n, 16)) for i in range(S)]
+    blobs, dcs, hrs = [], [], []
+    for i, c in enumerate(cs):
+        m, blob = _model(ctx, B, C, s, seed=3001 + i)
+        blobs.append(blob)
+        dcs.append(dev_chunk(ns, c, DEV, model=m, state=True))
+        hrs.append(alloc_hr(n, c, DEV))
+    ia = torch.zeros((S, n), dtype=torch.uint8, device=DEV)
+    ctx.enhance_streams(dcs, hrs, is_anchor_out=ia, k=k)
+    torch.cuda.synchronize()
+    ia = ia.cpu().numpy()
+    for i, c in enumerate(cs):
+        sc = [int(v) for v in oracle.score(c.res)]
+        _, _, ea = oracle.select_topk(list(c.type), sc, k)
+        assert list(ia[i]) == ea, i
+    c, blob = cs[0], blobs[0]
+    got = np.stack([t.cpu().numpy() for t in hrs[0]])
+    wins = [(0, 0, 16, 24), (0, w - 24, 16, 24), (h - 16, 0, 16, 24), (h - 16, w - 24, 16, 24), (352, 640, 16, 24)]
+    anchors = [f for f in range(n) if ia[0, f]]
+    worst = 0
+    for f in anchors[:3]:
+        for (Y0, X0, HH, WW), patch in oracle_sr_crops(c.lr[f], blob, B, C, s, wins):
+            d = np.abs(got[f][:, Y0:Y0 + HH, X0:X0 + WW].astype(int) - patch.astype(int))
+            worst = max(worst, int(d.max()))
+    assert worst <= SR_MAX_ABS, worst
+    exp, _, _ = oracle.reconstruct(c, list(ia[0]), got, np.zeros_like(got[0]), np.zeros_like(got[0]))
+    assert np.array_equal(got, exp)
