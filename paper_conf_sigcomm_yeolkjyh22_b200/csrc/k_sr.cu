@@ -1043,37 +1043,76 @@ struct Up2Cfg {
 
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
+// Compile-time bilinear tap of HR index S*x + I (same formula as up_tap with
+// the x-dependent part split off): source index x + off, weight w1 / 128.
+template <int S, int I>
+struct UpTapC {
+    static constexpr int u = 2 * I + 1 - S;  // |u| < 2S
+    static constexpr int off = u < 0 ? -1 : 0;
+    static constexpr int w1 = (128 * (u - 2 * S * off) + S) / (2 * S);
+};
+
+// The 2 x 3 LR window (rows of sub-row g's taps, columns x-1..x+1, clamped
+// like up_tap) of all 3 planes, 3 bytes per word; loaded before the step's MMA
+// wait so the latency hides under it.
+__device__ __forceinline__ void lr_window(const uint8_t *lr, int lh, int lw, int r, int x, int oy,
+                                          uint32_t (&lv)[3][2]) {
+    const int ya = min(max(r + oy, 0), lh - 1), yb = min(max(r + oy + 1, 0), lh - 1);
+    const int xm = max(x - 1, 0), xp = min(x + 1, lw - 1);
+    const size_t plane = (size_t)lh * lw;
+#pragma unroll
+    for (int c = 0; c < 3; c++)
+#pragma unroll
+        for (int rr = 0; rr < 2; rr++) {
+            const uint8_t *row = lr + c * plane + (size_t)(rr ? yb : ya) * lw;
+            lv[c][rr] = (uint32_t)__ldg(row + xm) | ((uint32_t)__ldg(row + x) << 8) | ((uint32_t)__ldg(row + xp) << 16);
+        }
+}
+
+// Accumulator columns one epilogue group reads: sub-row I uses n in
+// [3 S I, 3 S (I+1)); a 16-column window from the 8-aligned base covers it.
+template <int NB, int S>
+struct UpCols {
+    static constexpr int LW = NB < 16 ? NB : 16;
+    __host__ __device__ static constexpr int base(int I) { return NB <= 16 ? 0 : 8 * ((3 * S * I) / 8); }
+    __host__ __device__ static constexpr bool fits() {
+        for (int I = 0; I < S; I++)
+            if (3 * S * (I + 1) - base(I) > LW) return false;
+        return true;
+    }
+    static_assert(fits(), "sub-row column window");
+};
+
 // One HR sub-row I of an LR pixel: the s outputs x 3 planes of the composed
 // conv + the integer bilinear skip, rounded and clamped into the staging row;
 // frame-border ring pixels also keep their fp32 t for the exact fix-up.
 template <int NB, int S, int I>
-__device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[NB], const float *s_bias, const SrJob &J,
-                                              const ConvArgs &a, uint8_t *so, int p, int x, int r, int lh, int lw,
-                                              int slot_job) {
+__device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
+                                              const uint32_t (&lv)[3][2], const ConvArgs &a, uint8_t *so, int p,
+                                              int x, int r, int lh, int lw, int slot_job) {
+    constexpr int wy = UpTapC<S, I>::w1;
+    constexpr int base = UpCols<NB, S>::base(I);
     const int HH = lh * S, WW = lw * S;
-    int ya, yb, wy;
-    up_tap(S * r + I, S, lh, ya, yb, wy);
-    const size_t plane = (size_t)lh * lw;
+    const bool edge = r == 0 || r == lh - 1 || x == 0 || x == lw - 1;
 #pragma unroll
     for (int j = 0; j < S; j++) {
-        int xa, xb, wx;
-        up_tap(S * x + j, S, lw, xa, xb, wx);
+        const int ox = 1 + (2 * j + 1 - S < 0 ? -1 : 0);
+        const int wx = (128 * ((2 * j + 1 - S) - 2 * S * (ox - 1)) + S) / (2 * S);
 #pragma unroll
         for (int c = 0; c < 3; c++) {
-            const uint8_t *L = J.lr + c * plane;
-            const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
-            const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
+            const int p00 = (lv[c][0] >> (8 * ox)) & 0xFF, p01 = (lv[c][0] >> (8 * ox + 8)) & 0xFF;
+            const int p10 = (lv[c][1] >> (8 * ox)) & 0xFF, p11 = (lv[c][1] >> (8 * ox + 8)) & 0xFF;
             const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
             const int U = (vv + 8192) >> 14;
-            constexpr int dummy = 0;
-            (void)dummy;
             const int n = (I * S + j) * 3 + c;
-            const float t = __uint_as_float(v[n]) + s_bias[n];
+            const float t = __uint_as_float(v[n - base]) + s_bias[n];
             so[c * (kTile * S) + p * S + j] = (uint8_t)fminf(fmaxf(floorf((float)U + t + 0.5f), 0.f), 255.f);
-            const int Y = S * r + I, X = S * x + j;
-            if (Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1) {
-                const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
-                a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = t;
+            if (edge) {
+                const int Y = S * r + I, X = S * x + j;
+                if (Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1) {
+                    const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
+                    a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = t;
+                }
             }
         }
     }
@@ -1193,15 +1232,17 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
         uint8_t *so = oslot(k, g);
         if (vk[k]) {
             mbar_wait(wbar, 0);
+            const int oy = (2 * g + 1 - S < 0) ? -1 : 0;
             for (int q = 0; q < nq; q++) {
                 const int r = y0 - 4 + q;  // LR output row completed at this step
                 const bool valid = r >= y0;
-                // skip taps for sub-row g (compile-time per g via switch below)
+                uint32_t lv[3][2];
+                if (valid && x < lw) lr_window(J.lr, lh, lw, r, x, oy, lv);  // latency hides under the MMA wait
                 mbar_wait(mdone(k, q & 1), (q >> 1) & 1);
                 tc_fence_after();
                 const uint32_t acc = tl + (uint32_t)(mod5(r) * NB);
-                uint32_t v[NB];
-                tmem_ldN<NB>(acc, v);
+                uint32_t v[UpCols<NB, S>::LW];
+                tmem_ldN<UpCols<NB, S>::LW>(acc + (uint32_t)(NB <= 16 ? 0 : 8 * ((3 * S * g) / 8)), v);
                 tmem_wait_ld();
                 tc_fence_before();
                 named_bar(1 + k, 128 * S);  // every group of this tile has read the block
@@ -1214,10 +1255,10 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                 }
                 if (valid) {
                     if (x < lw) {
-                        if (g == 0) uptail_subrow<NB, S, 0>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 1 && g == 1) uptail_subrow<NB, S, (S > 1 ? 1 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 2 && g == 2) uptail_subrow<NB, S, (S > 2 ? 2 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 3 && g == 3) uptail_subrow<NB, S, (S > 3 ? 3 : 0)>(v, s_bias, J, a, so, p, x, r, lh, lw, slot_job);
+                        if (g == 0) uptail_subrow<NB, S, 0>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 1 && g == 1) uptail_subrow<NB, S, (S > 1 ? 1 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 2 && g == 2) uptail_subrow<NB, S, (S > 2 ? 2 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
+                        else if (S > 3 && g == 3) uptail_subrow<NB, S, (S > 3 ? 3 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
                     }
                     const int i = g;
                     named_bar(3 + grp, 128);  // this group's staging row is complete
