@@ -837,6 +837,8 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
 // skip up_s(LR) (O6), rounds, clamps and writes the s x s HR pixels of each
 // LR pixel through a shared-memory tile (8-byte stores).
 constexpr int kHalo5 = kTile + 4;
+constexpr int kLrBoxW = kTile + 32;  // u8 LR box x0-16 .. x0+143: the innermost TMA start must be 16-B aligned
+constexpr int kLrBoxX = 16;          // box origin = x0 - kLrBoxX
 template <int CIN, int NB, int S>
 struct UpCfg {
     static constexpr int KC = CIN / 16;
@@ -1020,7 +1022,9 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
 // warps (group g = HR sub-row i) that read the retired row in parallel.  The
 // 5-block accumulator ring (row r -> block r mod 5) is the same as k_uptail;
 // the MMA on input row y waits for the epilogue of row y-3 (previous step),
-// and the other tile's MMAs cover that wait.
+// and the other tile's MMAs cover that wait.  The TMA warp also stages the
+// three u8 LR rows r-1..r+1 of each output row r (bilinear skip taps) in a
+// separate ring that the epilogue groups release.
 template <int CIN, int NB, int S>
 struct Up2Cfg {
     static constexpr int KC = CIN / 16, NSTRIP = 9;
@@ -1030,11 +1034,15 @@ struct Up2Cfg {
     static constexpr uint32_t SLOT_BYTES = kHalo5 * CIN * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
     static constexpr int NS = 3;                                    // input ring per tile
+    static constexpr int NL = 3;                                    // LR ring per tile
+    static constexpr uint32_t LR_BYTES = 9u * kLrBoxW;              // [row 3][plane 3][kLrBoxW]
+    static constexpr uint32_t LSLOT = round_up(LR_BYTES, 128);
     static constexpr uint32_t OUTG = round_up(3u * kTile * S, 128);  // per group: [plane][128 s] bytes
-    static constexpr uint32_t TILE_BYTES = NS * SLOT + S * OUTG;
+    static constexpr uint32_t TILE_BYTES = NS * SLOT + NL * LSLOT + S * OUTG;
     static constexpr uint32_t TCOLS = 5 * NB;
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
-    static constexpr int NBAR = 2 * (2 * NS + 3) + 1;
+    static constexpr int BPT = 2 * NS + 3 + 2 * NL;                // barriers per tile
+    static constexpr int NBAR = 2 * BPT + 1;
     static constexpr int NWARPS = 2 + 2 * S * 4;
     static constexpr uint32_t SMEM = W_REGION + 2 * TILE_BYTES + NBAR * 8 + 64;
     static_assert(5 * NB <= 256, "N = 5 nb");
@@ -1052,23 +1060,6 @@ struct UpTapC {
     static constexpr int w1 = (128 * (u - 2 * S * off) + S) / (2 * S);
 };
 
-// The 2 x 3 LR window (rows of sub-row g's taps, columns x-1..x+1, clamped
-// like up_tap) of all 3 planes, 3 bytes per word; loaded before the step's MMA
-// wait so the latency hides under it.
-__device__ __forceinline__ void lr_window(const uint8_t *lr, int lh, int lw, int r, int x, int oy,
-                                          uint32_t (&lv)[3][2]) {
-    const int ya = min(max(r + oy, 0), lh - 1), yb = min(max(r + oy + 1, 0), lh - 1);
-    const int xm = max(x - 1, 0), xp = min(x + 1, lw - 1);
-    const size_t plane = (size_t)lh * lw;
-#pragma unroll
-    for (int c = 0; c < 3; c++)
-#pragma unroll
-        for (int rr = 0; rr < 2; rr++) {
-            const uint8_t *row = lr + c * plane + (size_t)(rr ? yb : ya) * lw;
-            lv[c][rr] = (uint32_t)__ldg(row + xm) | ((uint32_t)__ldg(row + x) << 8) | ((uint32_t)__ldg(row + xp) << 16);
-        }
-}
-
 // Accumulator columns one epilogue group reads: sub-row I uses n in
 // [3 S I, 3 S (I+1)); a 16-column window from the 8-aligned base covers it.
 template <int NB, int S>
@@ -1083,46 +1074,85 @@ struct UpCols {
     static_assert(fits(), "sub-row column window");
 };
 
+// floor + clamp to [0, 255] in one conversion
+__device__ __forceinline__ uint32_t f2u8_floor_sat(float v) {
+    uint32_t o;
+    asm("cvt.rmi.sat.u8.f32 %0, %1;" : "=r"(o) : "f"(v));
+    return o;
+}
+
 // One HR sub-row I of an LR pixel: the s outputs x 3 planes of the composed
-// conv + the integer bilinear skip, rounded and clamped into the staging row;
-// frame-border ring pixels also keep their fp32 t for the exact fix-up.
+// conv + the integer bilinear skip, rounded and clamped into the staging row.
+// lr: this step's staged LR rows [3][3][kLrBoxW] (row r-1+i, column x0-kLrBoxX+j);
+// ra/rb: staged rows of the vertical taps; cm/c0/cp: staged columns of x-1,
+// x, x+1 (clamped as up_tap clamps); bh: bias + 0.5 of this sub-row's outputs.
 template <int NB, int S, int I>
-__device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
-                                              const uint32_t (&lv)[3][2], const ConvArgs &a, uint8_t *so, int p,
-                                              int x, int r, int lh, int lw, int slot_job) {
+__device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>::LW], const float (&bh)[3 * S],
+                                              const uint8_t *lr, int ra, int rb, int cm, int c0, int cp,
+                                              uint8_t *so, int p) {
     constexpr int wy = UpTapC<S, I>::w1;
     constexpr int base = UpCols<NB, S>::base(I);
-    const int HH = lh * S, WW = lw * S;
-    const bool edge = r == 0 || r == lh - 1 || x == 0 || x == lw - 1;
+    int pa[3][3], pb[3][3];
+#pragma unroll
+    for (int c = 0; c < 3; c++) {
+        const uint8_t *La = lr + (ra * 3 + c) * kLrBoxW, *Lb = lr + (rb * 3 + c) * kLrBoxW;
+        pa[c][0] = La[cm]; pa[c][1] = La[c0]; pa[c][2] = La[cp];
+        pb[c][0] = Lb[cm]; pb[c][1] = Lb[c0]; pb[c][2] = Lb[cp];
+    }
 #pragma unroll
     for (int j = 0; j < S; j++) {
         const int ox = 1 + (2 * j + 1 - S < 0 ? -1 : 0);
         const int wx = (128 * ((2 * j + 1 - S) - 2 * S * (ox - 1)) + S) / (2 * S);
 #pragma unroll
         for (int c = 0; c < 3; c++) {
-            const int p00 = (lv[c][0] >> (8 * ox)) & 0xFF, p01 = (lv[c][0] >> (8 * ox + 8)) & 0xFF;
-            const int p10 = (lv[c][1] >> (8 * ox)) & 0xFF, p11 = (lv[c][1] >> (8 * ox + 8)) & 0xFF;
-            const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
-            const int U = (vv + 8192) >> 14;
+            const int ha = (128 - wx) * pa[c][ox] + wx * pa[c][ox + 1];
+            const int hb = (128 - wx) * pb[c][ox] + wx * pb[c][ox + 1];
+            const int U = ((128 - wy) * ha + wy * hb + 8192) >> 14;
             const int n = (I * S + j) * 3 + c;
-            const float t = __uint_as_float(v[n - base]) + s_bias[n];
-            so[c * (kTile * S) + p * S + j] = (uint8_t)fminf(fmaxf(floorf((float)U + t + 0.5f), 0.f), 255.f);
-            if (edge) {
-                const int Y = S * r + I, X = S * x + j;
-                if (Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1) {
-                    const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
-                    a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = t;
-                }
+            so[c * (kTile * S) + p * S + j] = (uint8_t)f2u8_floor_sat((float)U + (__uint_as_float(v[n - base]) + bh[n - 3 * S * I]));
+        }
+    }
+}
+
+// frame-border ring pixels of sub-row I keep their fp32 t = acc + bias for the
+// exact fix-up (k_uptail_ring)
+template <int NB, int S, int I>
+__device__ __noinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
+                                               const ConvArgs &a, int x, int r, int lh, int lw, int slot_job) {
+    constexpr int base = UpCols<NB, S>::base(I);
+    const int HH = lh * S, WW = lw * S;
+    const int Y = S * r + I;
+#pragma unroll
+    for (int j = 0; j < S; j++) {
+        const int X = S * x + j;
+        if (Y == 0 || Y == HH - 1 || X == 0 || X == WW - 1) {
+            const int ri = Y == 0 ? X : Y == HH - 1 ? WW + X : X == 0 ? 2 * WW + (Y - 1) : 2 * WW + (HH - 2) + (Y - 1);
+#pragma unroll
+            for (int c = 0; c < 3; c++) {
+                const int n = (I * S + j) * 3 + c;
+                a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = __uint_as_float(v[n - base]) + s_bias[n];
             }
         }
     }
 }
 
+template <int NB, int S, int I>
+__device__ __forceinline__ void uptail_group_step(const uint32_t (&v)[UpCols<NB, S>::LW], const float (&bh)[3 * S],
+                                                  const float *s_bias, const uint8_t *lr, int r, int x, int x0,
+                                                  int lh, int lw, const ConvArgs &a, uint8_t *so, int p,
+                                                  int slot_job) {
+    constexpr int oy = UpTapC<S, I>::off;
+    const int ra = min(max(r + oy, 0), lh - 1) - (r - 1), rb = min(max(r + oy + 1, 0), lh - 1) - (r - 1);
+    const int cm = max(x - 1, 0) - (x0 - kLrBoxX), c0 = x - (x0 - kLrBoxX), cp = min(x + 1, lw - 1) - (x0 - kLrBoxX);
+    uptail_subrow<NB, S, I>(v, bh, lr, ra, rb, cm, c0, cp, so, p);
+    if (r == 0 || r == lh - 1 || x == 0 || x == lw - 1) uptail_ring_store<NB, S, I>(v, s_bias, a, x, r, lh, lw, slot_job);
+}
+
 template <int CIN, int NB, int S>
 __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
-    k_uptail2(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+    k_uptail2(const __grid_constant__ CUtensorMap tm_in, const __grid_constant__ CUtensorMap tm_lr, const ConvArgs a) {
     using Cfg = Up2Cfg<CIN, NB, S>;
-    constexpr int NS = Cfg::NS;
+    constexpr int NS = Cfg::NS, NL = Cfg::NL, BPT = Cfg::BPT;
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *s_w = smem;
     const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
@@ -1130,13 +1160,18 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     uint64_t *bars = reinterpret_cast<uint64_t *>(s_tile + 2 * Cfg::TILE_BYTES);
     uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + Cfg::NBAR);
     auto islot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
-    auto oslot = [&](int k, int g) { return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + g * Cfg::OUTG; };
-    // per tile: hfull[NS], sfree[NS], mdone[2], edone
-    auto hfull = [&](int k, int i) { return &bars[k * (2 * NS + 3) + i]; };
-    auto sfree = [&](int k, int i) { return &bars[k * (2 * NS + 3) + NS + i]; };
-    auto mdone = [&](int k, int par) { return &bars[k * (2 * NS + 3) + 2 * NS + par]; };
-    auto edone = [&](int k) { return &bars[k * (2 * NS + 3) + 2 * NS + 2]; };
-    uint64_t *wbar = &bars[2 * (2 * NS + 3)];
+    auto lslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + i * Cfg::LSLOT; };
+    auto oslot = [&](int k, int g) {
+        return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + NL * Cfg::LSLOT + g * Cfg::OUTG;
+    };
+    // per tile: hfull[NS], sfree[NS], mdone[2], edone, lfull[NL], lfree[NL]
+    auto hfull = [&](int k, int i) { return &bars[k * BPT + i]; };
+    auto sfree = [&](int k, int i) { return &bars[k * BPT + NS + i]; };
+    auto mdone = [&](int k, int par) { return &bars[k * BPT + 2 * NS + par]; };
+    auto edone = [&](int k) { return &bars[k * BPT + 2 * NS + 2]; };
+    auto lfull = [&](int k, int i) { return &bars[k * BPT + 2 * NS + 3 + i]; };
+    auto lfree = [&](int k, int i) { return &bars[k * BPT + 2 * NS + 3 + NL + i]; };
+    uint64_t *wbar = &bars[2 * BPT];
 
     const int slot_job = blockIdx.z;
     const int job = a.j0 + slot_job;
@@ -1145,7 +1180,8 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     const int y0 = blockIdx.y * a.rows_per_cta;
     const int y1 = min(y0 + a.rows_per_cta, a.H);
     const int nq = y1 - y0 + 4;  // input rows y0-2 .. y1+1
-    const int lh = a.H, lw = a.W, HH = lh * S, WW = lw * S;
+    const int lh = a.H, lw = a.W;
+    const int HH = lh * S, WW = lw * S;
     int x0k[2];
     bool vk[2];
     for (int k = 0; k < 2; k++) {
@@ -1156,6 +1192,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     if (tid == 0) {
         for (int k = 0; k < 2; k++) {
             for (int i = 0; i < NS; i++) { mbar_init(hfull(k, i), 1); mbar_init(sfree(k, i), 1); }
+            for (int i = 0; i < NL; i++) { mbar_init(lfull(k, i), 1); mbar_init(lfree(k, i), S); }
             mbar_init(mdone(k, 0), 1);
             mbar_init(mdone(k, 1), 1);
             mbar_init(edone(k), 128);
@@ -1168,7 +1205,6 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *s_tmem;
-    const SrJob J = a.jobs[job];
     if (warp >= 2 && ((warp - 2) / 4) % S == 0) {
         // sub-row-0 group of each tile: zero its accumulator ring (the block of
         // row y0 has no earlier owner whose retirement would have zeroed it)
@@ -1184,7 +1220,9 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
 
     if (warp == 0) {
         if (lane == 0) {  // ---- TMA producer
+            const SrJob J = a.jobs[job];
             prefetch_tmap(&tm_in);
+            prefetch_tmap(&tm_lr);
             mbar_arrive_expect_tx(wbar, Cfg::B_BYTES + Cfg::BIAS_BYTES);
             bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, wbar);
             bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, wbar);
@@ -1195,6 +1233,13 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     if (q >= NS) mbar_wait(sfree(k, sl), ((q / NS) - 1) & 1);
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
                     tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                    const int qv = q - 4;  // output row y0 + qv retires at this step
+                    if (qv >= 0) {
+                        const int ls = qv % NL;
+                        if (qv >= NL) mbar_wait(lfree(k, ls), ((qv / NL) - 1) & 1);
+                        mbar_arrive_expect_tx(lfull(k, ls), Cfg::LR_BYTES);
+                        tma_load_4d(lslot(k, ls), &tm_lr, lfull(k, ls), x0k[k] - kLrBoxX, 0, y0 + qv - 1, slot_job);
+                    }
                 }
         }
     } else if (warp == 1) {  // ---- MMA issuer (whole warp, elected lane issues)
@@ -1232,17 +1277,19 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
         uint8_t *so = oslot(k, g);
         if (vk[k]) {
             mbar_wait(wbar, 0);
-            const int oy = (2 * g + 1 - S < 0) ? -1 : 0;
+            float bh[3 * S];
+#pragma unroll
+            for (int i = 0; i < 3 * S; i++) bh[i] = s_bias[3 * S * g + i] + 0.5f;
+            const uint32_t cbase = (uint32_t)(NB <= 16 ? 0 : 8 * ((3 * S * g) / 8));
+            const int xs_hr = x0k[k] * S, wv = min(kTile, lw - x0k[k]) * S;
+            uint8_t *const hr = a.jobs[job].hr + xs_hr;
             for (int q = 0; q < nq; q++) {
                 const int r = y0 - 4 + q;  // LR output row completed at this step
-                const bool valid = r >= y0;
-                uint32_t lv[3][2];
-                if (valid && x < lw) lr_window(J.lr, lh, lw, r, x, oy, lv);  // latency hides under the MMA wait
                 mbar_wait(mdone(k, q & 1), (q >> 1) & 1);
                 tc_fence_after();
                 const uint32_t acc = tl + (uint32_t)(mod5(r) * NB);
                 uint32_t v[UpCols<NB, S>::LW];
-                tmem_ldN<UpCols<NB, S>::LW>(acc + (uint32_t)(NB <= 16 ? 0 : 8 * ((3 * S * g) / 8)), v);
+                tmem_ldN<UpCols<NB, S>::LW>(acc + cbase, v);
                 tmem_wait_ld();
                 tc_fence_before();
                 named_bar(1 + k, 128 * S);  // every group of this tile has read the block
@@ -1253,21 +1300,24 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     tc_fence_before();
                     mbar_arrive(edone(k));
                 }
-                if (valid) {
+                if (r >= y0) {
+                    const int qv = r - y0, ls = qv % NL;
+                    mbar_wait(lfull(k, ls), (qv / NL) & 1);
+                    const uint8_t *lr = lslot(k, ls);
                     if (x < lw) {
-                        if (g == 0) uptail_subrow<NB, S, 0>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 1 && g == 1) uptail_subrow<NB, S, (S > 1 ? 1 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 2 && g == 2) uptail_subrow<NB, S, (S > 2 ? 2 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
-                        else if (S > 3 && g == 3) uptail_subrow<NB, S, (S > 3 ? 3 : 0)>(v, s_bias, lv, a, so, p, x, r, lh, lw, slot_job);
+                        if (g == 0) uptail_group_step<NB, S, 0>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
+                        else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
+                        else if (S > 2 && g == 2) uptail_group_step<NB, S, (S > 2 ? 2 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
+                        else if (S > 3 && g == 3) uptail_group_step<NB, S, (S > 3 ? 3 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
                     }
-                    const int i = g;
-                    named_bar(3 + grp, 128);  // this group's staging row is complete
-                    const int xs_hr = x0k[k] * S, wv = min(kTile, lw - x0k[k]) * S;
+                    named_bar(3 + grp, 128);  // this group's staging row is complete, its LR reads done
+                    if (p == 0) mbar_arrive(lfree(k, ls));
                     constexpr int CH = kTile * S / 8;
-                    for (int e = ew * 32 + lane; e < 3 * CH; e += 128) {
+                    uint8_t *dst = hr + (size_t)(S * r + g) * WW;
+                    for (int e = p; e < 3 * CH; e += 128) {
                         const int ch = e % CH, c = e / CH;
                         if (ch * 8 < wv)
-                            *reinterpret_cast<uint2 *>(J.hr + (size_t)c * HH * WW + (size_t)(S * r + i) * WW + xs_hr + ch * 8) =
+                            *reinterpret_cast<uint2 *>(dst + (size_t)c * HH * WW + ch * 8) =
                                 *reinterpret_cast<const uint2 *>(so + c * (kTile * S) + ch * 8);
                     }
                     named_bar(3 + grp, 128);  // staging can be overwritten
@@ -1416,7 +1466,8 @@ __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_coun
 }
 
 // LR u8 planar [3][h][w] -> bf16 [h][2][w][8]: channels 0..2 = LR - 128 (Z13), 3..15 = 0.
-__global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0) {
+__global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0,
+                          uint8_t *lr8, int wp) {
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
     const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1433,6 +1484,10 @@ __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, i
     uint16_t *base = x0 + (((size_t)slot * h + y) * 2) * (size_t)w * 8;
     *reinterpret_cast<uint4 *>(base + (size_t)x * 8) = o0;
     *reinterpret_cast<uint4 *>(base + ((size_t)w + x) * 8) = z;
+    uint8_t *l8 = lr8 + ((size_t)slot * h + y) * 3 * wp + x;
+    l8[0] = L[idx];
+    l8[wp] = L[plane + idx];
+    l8[2 * wp] = L[2 * plane + idx];
 }
 
 // ------------------------------------------------------------------ host side
@@ -1466,6 +1521,19 @@ static int make_act_map(CUtensorMap *m, uint16_t *base, int H, int W, int C, int
     return r == CUDA_SUCCESS ? 0 : -2;
 }
 
+// u8 LR copy [job][H][3][wp]: box of kLrBoxW px x 3 planes x 3 rows of one job
+static int make_lr8_map(CUtensorMap *m, uint8_t *base, int H, int wp, int nb) {
+    PFN_encodeTiled enc = get_encode();
+    if (!enc) return -1;
+    cuuint64_t dims[4] = {(cuuint64_t)wp, 3, (cuuint64_t)H, (cuuint64_t)nb};
+    cuuint64_t strides[3] = {(cuuint64_t)wp, (cuuint64_t)wp * 3, (cuuint64_t)wp * 3 * H};
+    cuuint32_t box[4] = {kLrBoxW, 3, 3, 1};
+    cuuint32_t estr[4] = {1, 1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? 0 : -2;
+}
+
 static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u positions x C + ring t x 3
     const size_t H = (size_t)h * s, W = (size_t)w * s;
     return (2 * (W + 2) + 2 * H) * C + (2 * W + 2 * (H - 2)) * 3;
@@ -1476,7 +1544,8 @@ size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
     size_t b = px * 16 * 2;                  // x0
     b += 3 * px * C * 2;                     // h0, hb, tb
     b += band_floats(h, w, C, s) * 4 * nb;   // border bands
-    return b + 5 * 256;
+    b += (size_t)h * 3 * ((w + 15) / 16 * 16) * nb;  // lr8
+    return b + 6 * 256;
 }
 
 int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) {
@@ -1492,7 +1561,10 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     a->hb = reinterpret_cast<uint16_t *>(take(px * C * 2));
     a->tb = reinterpret_cast<uint16_t *>(take(px * C * 2));
     a->band = reinterpret_cast<float *>(take(band_floats(h, w, C, s) * 4 * nb));
+    a->wp = (w + 15) / 16 * 16;
+    a->lr8 = take((size_t)h * 3 * a->wp * nb);
     int rc = 0;
+    rc |= make_lr8_map(&a->tm_lr8, a->lr8, h, a->wp, nb);
     rc |= make_act_map(&a->tm_x0, a->x0, h, w, 16, nb, kHalo);
     rc |= make_act_map(&a->tm_h0, a->h0, h, w, C, nb, kHalo);
     rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb, kHalo);
@@ -1577,7 +1649,7 @@ static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, 
 }
 
 template <int CIN, int NB, int S>
-static cudaError_t uptail2(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
+static cudaError_t uptail2(const CUtensorMap &tm, const CUtensorMap &tm_lr, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = Up2Cfg<CIN, NB, S>;
     static bool attr = false;
     if (!attr) {
@@ -1590,7 +1662,7 @@ static cudaError_t uptail2(const CUtensorMap &tm, ConvArgs args, int nj, cudaStr
     args.rows_per_cta = kRotRows;
     dim3 grid((ntiles + 1) / 2, (args.H + kRotRows - 1) / kRotRows, nj);
     KScope ks(F_SR_UP, st);
-    k_uptail2<CIN, NB, S><<<grid, Cfg::NWARPS * 32, Cfg::SMEM, st>>>(tm, args);
+    k_uptail2<CIN, NB, S><<<grid, Cfg::NWARPS * 32, Cfg::SMEM, st>>>(tm, tm_lr, args);
     return cudaGetLastError();
 }
 
@@ -1602,7 +1674,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     {
         dim3 g((h * w + 255) / 256, nj);
         KScope ks(F_SR_PREP, st);
-        k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0);
+        k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     ConvArgs base{};
@@ -1643,8 +1715,8 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
             const size_t H = (size_t)h * s, W = (size_t)w * s;
             g.ring = a->band + (size_t)a->nb * (2 * (W + 2) + 2 * H) * C;
         }
-        if (s == 2) e = uptail2<C, 16, 2>(tm5, g, nj, st);
-        else if (s == 3) e = uptail2<C, 32, 3>(tm5, g, nj, st);
+        if (s == 2) e = uptail2<C, 16, 2>(tm5, a->tm_lr8, g, nj, st);
+        else if (s == 3) e = uptail2<C, 32, 3>(tm5, a->tm_lr8, g, nj, st);
         else e = uptail<C, 48, 4>(tm5, g, nj, st);
         if (e != cudaSuccess) return e;
         // exact frame-border ring (the tail's zero padding of u)

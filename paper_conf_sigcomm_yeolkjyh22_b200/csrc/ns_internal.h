@@ -101,7 +101,10 @@ struct SrArena {
     int h, w, C, s, nb;        // shape and batch capacity (jobs per batch)
     uint16_t *x0, *h0, *hb, *tb;       // bf16 activations, layout [job][H][C/8][W][8]
     float *band;                       // border fix-up: u on the HR frame-edge bands
+    uint8_t *lr8;                      // u8 LR copy [job][H][3][wp] (upsampler skip taps), wp = W rounded to 16
+    int wp;
     CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_tb5, tm_hb5;   // *5: 132-px boxes (5x5 conv)
+    CUtensorMap tm_lr8;                // box: kLrBoxW px x 3 planes x 3 rows
 };
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb);
 int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);  // 0 ok
