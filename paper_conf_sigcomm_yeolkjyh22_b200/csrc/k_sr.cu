@@ -621,13 +621,9 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
     const int y0 = blockIdx.y * a.rows_per_cta;
     const int y1 = min(y0 + a.rows_per_cta, a.H);
     const int nq = y1 - y0 + 4;  // h rows y0-2 .. y1+1
-    int x0k[2];
-    bool vk[2];
-    for (int k = 0; k < 2; k++) {
-        const int tix = 2 * blockIdx.x + k;
-        vk[k] = tix < a.n_tiles;
-        x0k[k] = tix * kRbOut;
-    }
+    // tile k of this CTA: x0 = (2 blockIdx.x + k) kRbOut (computed, not indexed: no local memory)
+    auto x0k = [&](int k) { return (2 * (int)blockIdx.x + k) * kRbOut; };
+    auto vk = [&](int k) { return 2 * (int)blockIdx.x + k < a.n_tiles; };
 
     if (tid == 0) {
         for (int k = 0; k < 2; k++) {
@@ -665,13 +661,13 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
             bulk_load(s_w2 + Cfg::B_BYTES, J.wts + a.bias2_off, Cfg::BIAS_BYTES, wbar);
             for (int q = 0; q < nq; q++) {
                 for (int k = 0; k < 2; k++) {
-                    if (!vk[k]) continue;
+                    if (!vk(k)) continue;
                     const int sl = q % NH;
                     // slot reuse: h row q-NH was last read by E2 at step q-NH+2, which
                     // arrives on hfree[slot] (one completion per reuse: never runs ahead)
                     if (q >= NH) mbar_wait(hfree(k, sl), ((q / NH) - 1) & 1);
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
-                    tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                    tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
                     NS_TR(30 + k, q);
                 }
             }
@@ -708,10 +704,10 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
         };
         mbar_wait(wbar, 0);
         for (int k = 0; k < 2; k++)
-            if (vk[k]) issue_m1(k, 0);
+            if (vk(k)) issue_m1(k, 0);
         for (int q = 0; q < nq; q++) {
             for (int k = 0; k < 2; k++) {
-                if (!vk[k]) continue;
+                if (!vk(k)) continue;
                 mbar_wait(e1bar(k), q & 1);  // E1(q): t row written, conv1 block of M1(q+1) zeroed
                 if (lane == 0) NS_TR(5 + k, q);
                 if (q >= 2) {                // conv2 on t row y0-3+q
@@ -729,12 +725,18 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
         // E1 (t -> SMEM, needs the async-proxy fence) and E2 (global stores) run
         // in different warps so the fence never waits on in-flight global stores.
         const int g = (warp - 2) / 4, k = g / 2, role = g % 2;
-        if (vk[k]) {
+        if (vk(k)) {
             const int ew = warp % 4;   // TMEM lane quarter
             const int p = ew * 32 + lane;
             const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
             mbar_wait(wbar, 0);
             NS_TR_ROLE(2 + g);
+            float bias[NB];  // b1 (E1) or b2 (E2), kept in registers: no shared loads on the critical chain
+#pragma unroll
+            for (int i = 0; i < NB; i += 4) {
+                const float4 b4 = *reinterpret_cast<const float4 *>((role == 0 ? s_b1 : s_b2) + i);
+                bias[i] = b4.x; bias[i + 1] = b4.y; bias[i + 2] = b4.z; bias[i + 3] = b4.w;
+            }
             if (role == 0) {
                 for (int q = 0; q < nq; q++) {  // E1: t = ReLU(conv1 + b1) -> t slot
                     const int yt = y0 - 3 + q;
@@ -750,9 +752,10 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
+                    if (warp % 4 == 2 && lane == 0) NS_TR(40 + k, q);
                     tmem_zeroN<NB>(acc);
                     if (q >= 2) {
-                        const int xt = x0k[k] - 1 + p;
+                        const int xt = x0k(k) - 1 + p;
                         const bool inside = yt >= 0 && yt < a.H && xt >= 0 && xt < a.W;
                         uint8_t *ts = tslot(k, q % Cfg::NTS);
 #pragma unroll
@@ -760,15 +763,18 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                             float f[8];
 #pragma unroll
                             for (int i = 0; i < 8; i++)
-                                f[i] = inside ? fmaxf(__uint_as_float(v[cg * 8 + i]) + s_b1[cg * 8 + i], 0.f) : 0.f;
+                                f[i] = inside ? fmaxf(__uint_as_float(v[cg * 8 + i]) + bias[cg * 8 + i], 0.f) : 0.f;
                             uint4 o;
                             o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
                             o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
                             *reinterpret_cast<uint4 *>(ts + cg * kHalo * 16 + p * 16) = o;
                         }
                     }
+                    if (warp % 4 == 2 && lane == 0) NS_TR(42 + k, q);
                     tmem_wait_st();
+                    if (warp % 4 == 2 && lane == 0) NS_TR(44 + k, q);
                     fence_proxy_async_smem();
+                    if (warp % 4 == 2 && lane == 0) NS_TR(46 + k, q);
                     tc_fence_before();
                     mbar_arrive(e1bar(k));
                     if (warp % 4 == 2 && lane == 0) NS_TR(12 + k, q);
@@ -790,7 +796,7 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
                     tmem_zeroN<NB>(acc);
-                    const int x = x0k[k] + p;
+                    const int x = x0k(k) + p;
                     if (yo >= y0 && yo < y1 && p < kRbOut && x < a.W) {
                         const uint8_t *hs = hslot(k, (q - 2) % NH);  // h row yo (step q-2)
                         const size_t rowbase = ((size_t)slot_job * a.H + yo) * (NB / 8);
@@ -799,7 +805,7 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                             const uint4 rr = *reinterpret_cast<const uint4 *>(hs + cg * kHalo * 16 + (p + 2) * 16);
                             float f[8];
 #pragma unroll
-                            for (int i = 0; i < 8; i++) f[i] = __uint_as_float(v[cg * 8 + i]) + s_b2[cg * 8 + i];
+                            for (int i = 0; i < 8; i++) f[i] = __uint_as_float(v[cg * 8 + i]) + bias[cg * 8 + i];
                             f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
                             f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
                             f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);

@@ -31,11 +31,23 @@ t, tag, q = t[order], tag[order], q[order]
 t0 = t[0]
 names = {1: "M1 hfull ok A", 2: "M1 hfull ok B", 3: "M1 issued A", 4: "M1 issued B", 5: "M2 e1 ok A", 6: "M2 e1 ok B",
          7: "M2 issued A", 8: "M2 issued B", 10: "E1 m1 ok A", 11: "E1 m1 ok B", 12: "E1 arrive A", 13: "E1 arrive B",
-         20: "E2 m2 ok A", 21: "E2 m2 ok B", 22: "E2 arrive A", 23: "E2 arrive B", 30: "TMA load A", 31: "TMA load B"}
+         20: "E2 m2 ok A", 21: "E2 m2 ok B", 22: "E2 arrive A", 23: "E2 arrive B", 30: "TMA load A", 31: "TMA load B",
+         40: "E1 ld done A", 41: "E1 ld done B", 42: "E1 sts done A", 43: "E1 sts done B", 44: "E1 wait_st A",
+         45: "E1 wait_st B", 46: "E1 fence A", 47: "E1 fence B"}
 for i in range(len(t)):
     if q[i] < 14 and tag[i] != 30 and tag[i] != 31:
         print(f"{t[i]-t0:8d}  q={q[i]:3d}  {names.get(tag[i], tag[i])}")
 # steady state period
+# E1 phase durations (tile A), steady state
+def col(tg):
+    return t[tag == tg][10:60].astype(np.int64)
+try:
+    m1, ld, sts, wst, fen, arr = col(10), col(40), col(42), col(44), col(46), col(12)
+    n = min(map(len, (m1, ld, sts, wst, fen, arr)))
+    print("E1 A phases (median cycles): ld", int(np.median(ld[:n] - m1[:n])), "zero+compute+sts", int(np.median(sts[:n] - ld[:n])),
+          "wait_st", int(np.median(wst[:n] - sts[:n])), "fence.proxy", int(np.median(fen[:n] - wst[:n])), "arrive", int(np.median(arr[:n] - fen[:n])))
+except Exception as e:
+    print("phase summary failed", e)
 for tg in (3, 7, 12, 22):
     ts = t[tag == tg]
     if len(ts) > 20:
