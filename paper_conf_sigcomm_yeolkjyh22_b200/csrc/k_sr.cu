@@ -23,7 +23,7 @@ namespace ns {
 #ifdef NS_TRACE
 // debug-only timeline of CTA (0,0,0): per-role regions of {clock64, tag << 32 | step},
 // plain stores (no atomics on the traced threads' critical path)
-__device__ unsigned long long g_trace[8 * 2 * 1024];
+__device__ unsigned long long g_trace[16 * 2 * 1024];
 #define NS_TR(tag, q)                                                                            \
     do {                                                                                         \
         if (blockIdx.x == 0 && blockIdx.y == 0 && blockIdx.z == 0 && _trn < 1024) {              \
@@ -550,6 +550,8 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
 }
 
 // ------------------------------------------------------------------ fused residual block
+constexpr int kRbMmaWarps = 4;
+constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 // h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
 // h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
 // written in the UMMA A-operand layout and consumed by conv2's MMAs), and the
@@ -578,7 +580,8 @@ struct RbCfg {
     static constexpr uint32_t TILE_BYTES = (NH + NTS) * SLOT;
     static constexpr uint32_t TCOLS = 2 * 3 * NB;                // conv1 + conv2 rings per tile
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
-    static constexpr int NBAR = 2 * (2 * NH + 4) + 1;
+    static constexpr int BPT = 2 * NH + 10;                      // barriers per tile
+    static constexpr int NBAR = 2 * BPT + 1;
     static constexpr uint32_t SMEM = 2 * W_CONV + 2 * TILE_BYTES + NBAR * 8 + 64;
     static_assert(SMEM <= 232448, "shared memory");
 };
@@ -592,8 +595,14 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 // Per tile and input step q (h row y0-2+q): M1(q) conv1 -> E1(q) reads t row
 // y0-3+q, writes it (ReLU, bf16) to t slot q%2 -> M2(q) conv2 on it -> E2(q)
 // retires output row y0-4+q (+ b2 + h from the ring).  mbarriers only.
+// Each epilogue signals twice: as soon as its accumulator block is read and
+// zeroed (e1z / e2z: the next MMA group of that conv may start) and when its
+// output is written (e1t: conv2 may read the t row).  So the next conv1 group
+// never waits for the t row's conversion and stores: the tensor queue keeps
+// both tiles' groups while the epilogues run (a drained queue costs the ~300-
+// cycle commit round trip, tools/ubench.cu).
 template <int C>
-__global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
+__global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
     using Cfg = RbCfg<C>;
     constexpr int NB = Cfg::NB, NH = Cfg::NH;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -605,14 +614,17 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
     uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + Cfg::NBAR);
     auto hslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
     auto tslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + (NH + i) * Cfg::SLOT; };
-    // per tile: hfull[NH], m1, m2, e1, e2, hfree[NH]
-    auto hfull = [&](int k, int i) { return &bars[k * (2 * NH + 4) + i]; };
-    auto hfree = [&](int k, int i) { return &bars[k * (2 * NH + 4) + NH + 4 + i]; };
-    auto m1bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH]; };
-    auto m2bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 1]; };
-    auto e1bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 2]; };
-    auto e2bar = [&](int k) { return &bars[k * (2 * NH + 4) + NH + 3]; };
-    uint64_t *wbar = &bars[2 * (2 * NH + 4)];
+    // per tile: hfull[NH], m1, m2, e1z, e2z, e1t[4], tfree[2], hfree[NH]
+    constexpr int BPT = Cfg::BPT;
+    auto hfull = [&](int k, int i) { return &bars[k * BPT + i]; };
+    auto m1bar = [&](int k) { return &bars[k * BPT + NH]; };
+    auto m2bar = [&](int k) { return &bars[k * BPT + NH + 1]; };
+    auto e1z = [&](int k) { return &bars[k * BPT + NH + 2]; };
+    auto e2z = [&](int k) { return &bars[k * BPT + NH + 3]; };
+    auto e1t = [&](int k, int i) { return &bars[k * BPT + NH + 4 + i]; };
+    auto tfree = [&](int k, int i) { return &bars[k * BPT + NH + 8 + i]; };
+    auto hfree = [&](int k, int i) { return &bars[k * BPT + NH + 10 + i]; };
+    uint64_t *wbar = &bars[2 * BPT];
 
     const int slot_job = blockIdx.z;
     const int job = a.j0 + slot_job;
@@ -631,8 +643,11 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
             for (int i = 0; i < NH; i++) mbar_init(hfree(k, i), 128);
             mbar_init(m1bar(k), 1);
             mbar_init(m2bar(k), 1);
-            mbar_init(e1bar(k), 128);
-            mbar_init(e2bar(k), 128);
+            mbar_init(e1z(k), 128);
+            mbar_init(e2z(k), 128);
+            for (int i = 0; i < 4; i++) mbar_init(e1t(k, i), 128);
+            mbar_init(tfree(k, 0), 1);
+            mbar_init(tfree(k, 1), 1);
         }
         mbar_init(wbar, 1);
         fence_mbar_init();
@@ -672,65 +687,75 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                 }
             }
         }
-    } else if (warp == 1) {
-        // ---------------------------------------------------------------- MMA issuer
-        // The whole warp runs the schedule (waits are warp-uniform); one elected
-        // lane issues each group of 6 MMAs + commit.  Order per step q:
-        //   M2(A,q) M1(A,q+1) M2(B,q) M1(B,q+1)
-        // so one tile's MMAs keep the tensor pipe busy while the other tile's
-        // conv1 epilogue runs.
-        NS_TR_ROLE(1);
-        const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
-        auto mma_rot = [&](uint32_t dcol, const uint8_t *aslot, const uint8_t *wstrip, int yin, uint64_t *bar) {
-            const uint32_t abase = smem_u32(aslot);
-            const uint32_t wbase = smem_u32(wstrip) + (uint32_t)mod3(1 - yin) * NB * 16;
-            const uint64_t ad0 = smem_desc(abase, kHalo * 16, 128), bd0 = smem_desc(wbase, 5 * NB * 16, 128);
-            if (elect_one()) {
+    } else if (warp <= kRbMmaWarps) {
+        // ---------------------------------------------------------------- MMA issuers
+        // Four independent issuer warps, one per (conv, tile): warp 1 M1(A),
+        // 2 M1(B), 3 M2(A), 4 M2(B).  A waiting issuer (each mbarrier hop is
+        // ~130 cycles, tools/ubench.cu) no longer stalls the other streams, so
+        // the tensor queue is fed while any one of them waits.  Each warp runs
+        // its schedule uniformly; one elected lane issues the 6 MMAs + commit.
+        //   M1(k,q) needs hfull(k,q) and e1z(k,q-1) (block of row y0-3+q+1 zeroed);
+        //   M2(k,q) needs e1t(k,q) (t row written) and e2z(k,q-1), and releases t
+        //   slot q%2 through tfree.
+        // Bound on how far conv1 runs ahead: M1(q) needs h row q, whose ring slot
+        // E2(q-3) frees, so M2(q-3) is complete whenever E1(q) runs; E1 therefore
+        // leads conv2's wait by <= 2 steps and e1t rotates over 4 barriers.
+        const int mw = warp - 1, conv = mw >> 1, k = mw & 1;
+        NS_TR_ROLE(1 + mw);
+        if (vk(k)) {
+            const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
+            auto mma_rot = [&](uint32_t dcol, const uint8_t *aslot, const uint8_t *wstrip, int yin, uint64_t *bar,
+                               uint64_t *bar0) {
+                const uint32_t abase = smem_u32(aslot);
+                const uint32_t wbase = smem_u32(wstrip) + (uint32_t)mod3(1 - yin) * NB * 16;
+                const uint64_t ad0 = smem_desc(abase, kHalo * 16, 128), bd0 = smem_desc(wbase, 5 * NB * 16, 128);
+                if (elect_one()) {
 #pragma unroll
-                for (int dx = 0; dx < 3; dx++)
+                    for (int dx = 0; dx < 3; dx++)
 #pragma unroll
-                    for (int kc = 0; kc < Cfg::KC; kc++)  // descriptor start address is bits 0-13 (>> 4)
-                        umma_bf16(dcol, ad0 + (uint64_t)((2 * kc * kHalo * 16 + dx * 16) >> 4),
-                                  bd0 + (uint64_t)(((dx * Cfg::KC + kc) * 2 * 5 * NB * 16) >> 4), idesc, 1u);
-                umma_commit(bar);
-            }
-            __syncwarp();
-        };
-        auto issue_m1 = [&](int k, int q) {  // conv1 on h row y0-2+q (E1(q-1) has been waited)
-            mbar_wait(hfull(k, q % NH), (q / NH) & 1);
-            tc_fence_after();
-            mma_rot(tmem + k * Cfg::TCOLS, hslot(k, q % NH), s_w1, y0 - 2 + q, m1bar(k));
-            if (lane == 0) NS_TR(3 + k, q);
-        };
-        mbar_wait(wbar, 0);
-        for (int k = 0; k < 2; k++)
-            if (vk(k)) issue_m1(k, 0);
-        for (int q = 0; q < nq; q++) {
-            for (int k = 0; k < 2; k++) {
-                if (!vk(k)) continue;
-                mbar_wait(e1bar(k), q & 1);  // E1(q): t row written, conv1 block of M1(q+1) zeroed
-                if (lane == 0) NS_TR(5 + k, q);
-                if (q >= 2) {                // conv2 on t row y0-3+q
-                    if (q >= 3) mbar_wait(e2bar(k), (q - 3) & 1);  // E2(q-1) zeroed the block M2(q) first touches
+                        for (int kc = 0; kc < Cfg::KC; kc++)  // descriptor start address is bits 0-13 (>> 4)
+                            umma_bf16(dcol, ad0 + (uint64_t)((2 * kc * kHalo * 16 + dx * 16) >> 4),
+                                      bd0 + (uint64_t)(((dx * Cfg::KC + kc) * 2 * 5 * NB * 16) >> 4), idesc, 1u);
+                    if (bar0) umma_commit(bar0);  // (the issuing thread's commits track its own MMAs)
+                    umma_commit(bar);
+                }
+                __syncwarp();
+            };
+            mbar_wait(wbar, 0);
+            if (conv == 0) {
+                for (int q = 0; q < nq; q++) {  // conv1 on h row y0-2+q
+                    if (q >= 1) mbar_wait(e1z(k), (q - 1) & 1);
+                    mbar_wait(hfull(k, q % NH), (q / NH) & 1);
+                    if (lane == 0) NS_TR(1 + k, q);
                     tc_fence_after();
-                    mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q, m2bar(k));
+                    mma_rot(tmem + k * Cfg::TCOLS, hslot(k, q % NH), s_w1, y0 - 2 + q, m1bar(k), nullptr);
+                    if (lane == 0) NS_TR(3 + k, q);
+                }
+            } else {
+                for (int q = 2; q < nq; q++) {  // conv2 on t row y0-3+q
+                    mbar_wait(e1t(k, q & 3), (q >> 2) & 1);
+                    if (q >= 3) mbar_wait(e2z(k), (q - 3) & 1);
+                    if (lane == 0) NS_TR(5 + k, q);
+                    tc_fence_after();
+                    // tfree: t slot q%2 may be overwritten once these MMAs complete
+                    mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q, m2bar(k),
+                            tfree(k, q & 1));
                     if (lane == 0) NS_TR(7 + k, q);
                 }
-                if (q + 1 < nq) issue_m1(k, q + 1);
             }
         }
     } else {
         // ---------------------------------------------------------------- epilogues
-        // warps 2..17: group g = (warp-2)/4 -> tile k = g/2, role = g%2 (E1 | E2).
+        // warps 5..20: group g -> tile k = g/2, role = g%2 (E1 | E2).
         // E1 (t -> SMEM, needs the async-proxy fence) and E2 (global stores) run
         // in different warps so the fence never waits on in-flight global stores.
-        const int g = (warp - 2) / 4, k = g / 2, role = g % 2;
+        const int g = (warp - 1 - kRbMmaWarps) / 4, k = g / 2, role = g % 2;
         if (vk(k)) {
             const int ew = warp % 4;   // TMEM lane quarter
             const int p = ew * 32 + lane;
             const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
             mbar_wait(wbar, 0);
-            NS_TR_ROLE(2 + g);
+            NS_TR_ROLE(5 + g);
             float bias[NB];  // b1 (E1) or b2 (E2), kept in registers: no shared loads on the critical chain
 #pragma unroll
             for (int i = 0; i < NB; i += 4) {
@@ -745,7 +770,8 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                     tc_fence_after();
 #ifdef NS_TRACE_NOEPI
                     tc_fence_before();
-                    mbar_arrive(e1bar(k));
+                    mbar_arrive(e1z(k));
+                    mbar_arrive(e1t(k, q & 3));
                     continue;
 #endif
                     const uint32_t acc = tl + (uint32_t)(mod3(yt) * NB);
@@ -754,6 +780,12 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                     tmem_wait_ld();
                     if (warp % 4 == 2 && lane == 0) NS_TR(40 + k, q);
                     tmem_zeroN<NB>(acc);
+                    tmem_wait_st();
+                    tc_fence_before();
+                    mbar_arrive(e1z(k));  // the next conv1 group may start
+                    // t slot q%2 was last read by M2(q-2) (another warp's MMAs): completion
+                    // #((q-4)/2) of tfree[q%2]; M2(q-4) is done, M2(q) cannot be -> exact
+                    if (q >= 4) mbar_wait(tfree(k, q & 1), ((q - 4) >> 1) & 1);
                     if (q >= 2) {
                         const int xt = x0k(k) - 1 + p;
                         const bool inside = yt >= 0 && yt < a.H && xt >= 0 && xt < a.W;
@@ -771,12 +803,9 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                         }
                     }
                     if (warp % 4 == 2 && lane == 0) NS_TR(42 + k, q);
-                    tmem_wait_st();
-                    if (warp % 4 == 2 && lane == 0) NS_TR(44 + k, q);
                     fence_proxy_async_smem();
                     if (warp % 4 == 2 && lane == 0) NS_TR(46 + k, q);
-                    tc_fence_before();
-                    mbar_arrive(e1bar(k));
+                    mbar_arrive(e1t(k, q & 3));
                     if (warp % 4 == 2 && lane == 0) NS_TR(12 + k, q);
                 }
             } else {
@@ -788,7 +817,7 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
 #ifdef NS_TRACE_NOEPI
                     tc_fence_before();
                     mbar_arrive(hfree(k, (q - 2) % NH));
-                    mbar_arrive(e2bar(k));
+                    mbar_arrive(e2z(k));
                     continue;
 #endif
                     const uint32_t acc = tl + 3 * NB + (uint32_t)(mod3(yo) * NB);
@@ -796,6 +825,9 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
                     tmem_zeroN<NB>(acc);
+                    tmem_wait_st();
+                    tc_fence_before();
+                    mbar_arrive(e2z(k));  // the next conv2 group may start
                     const int x = x0k(k) + p;
                     if (yo >= y0 && yo < y1 && p < kRbOut && x < a.W) {
                         const uint8_t *hs = hslot(k, (q - 2) % NH);  // h row yo (step q-2)
@@ -816,10 +848,7 @@ __global__ void __launch_bounds__(576, 1) k_resblock(const __grid_constant__ CUt
                             *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * a.W + x) * 8) = o;
                         }
                     }
-                    tmem_wait_st();
-                    tc_fence_before();
                     mbar_arrive(hfree(k, (q - 2) % NH));
-                    mbar_arrive(e2bar(k));
                     if (warp % 4 == 2 && lane == 0) NS_TR(22 + k, q);
                 }
             }
@@ -1650,7 +1679,7 @@ static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, 
     args.rows_per_cta = kRbRows;
     dim3 grid((args.n_tiles + 1) / 2, (args.H + kRbRows - 1) / kRbRows, nj);
     KScope ks(F_SR_BODY, st);
-    k_resblock<C><<<grid, 576, Cfg::SMEM, st>>>(tm, args);
+    k_resblock<C><<<grid, kRbThreads, Cfg::SMEM, st>>>(tm, args);
     return cudaGetLastError();
 }
 
@@ -1754,12 +1783,12 @@ cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int 
 
 #ifdef NS_TRACE
 extern "C" NS_API int ns_trace_read(unsigned long long *out, int max_pairs) {
-    const int n = max_pairs < 8 * 1024 ? max_pairs : 8 * 1024;
+    const int n = max_pairs < 16 * 1024 ? max_pairs : 16 * 1024;
     cudaMemcpyFromSymbol(out, ns::g_trace, sizeof(unsigned long long) * 2 * n);
     return n;
 }
 extern "C" NS_API void ns_trace_reset() {
-    static unsigned long long z[8 * 2 * 1024];
+    static unsigned long long z[16 * 2 * 1024];
     cudaMemcpyToSymbol(ns::g_trace, z, sizeof(z));
 }
 #endif

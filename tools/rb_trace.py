@@ -21,15 +21,15 @@ L.ns_trace_reset()
 # only the first fused block of one batch is traced: regions are overwritten by later launches,
 # so run exactly one batch and keep the LAST block's timeline (all blocks behave alike)
 ctx.sr_anchors(jobs); torch.cuda.synchronize()
-buf = (ctypes.c_ulonglong * (2 * 8192))()
-n = L.ns_trace_read(buf, 8192)
+buf = (ctypes.c_ulonglong * (2 * 16384))()
+n = L.ns_trace_read(buf, 16384)
 a = np.frombuffer(buf, dtype=np.uint64)[:2 * n].reshape(n, 2)
 a = a[a[:, 0] != 0]
 t = a[:, 0].astype(np.int64); tag = (a[:, 1] >> 32).astype(int); q = (a[:, 1] & 0xffffffff).astype(int)
 order = np.argsort(t)
 t, tag, q = t[order], tag[order], q[order]
 t0 = t[0]
-names = {1: "M1 hfull ok A", 2: "M1 hfull ok B", 3: "M1 issued A", 4: "M1 issued B", 5: "M2 e1 ok A", 6: "M2 e1 ok B",
+names = {1: "M1 e1z ok A", 2: "M1 e1z ok B", 48: "M2 e2z ok A", 49: "M2 e2z ok B", 50: "M1 hfull ok A", 51: "M1 hfull ok B", 3: "M1 issued A", 4: "M1 issued B", 5: "M2 e1t ok A", 6: "M2 e1t ok B",
          7: "M2 issued A", 8: "M2 issued B", 10: "E1 m1 ok A", 11: "E1 m1 ok B", 12: "E1 arrive A", 13: "E1 arrive B",
          20: "E2 m2 ok A", 21: "E2 m2 ok B", 22: "E2 arrive A", 23: "E2 arrive B", 30: "TMA load A", 31: "TMA load B",
          40: "E1 ld done A", 41: "E1 ld done B", 42: "E1 sts done A", 43: "E1 sts done B", 44: "E1 wait_st A",
@@ -42,10 +42,10 @@ for i in range(len(t)):
 def col(tg):
     return t[tag == tg][10:60].astype(np.int64)
 try:
-    m1, ld, sts, wst, fen, arr = col(10), col(40), col(42), col(44), col(46), col(12)
-    n = min(map(len, (m1, ld, sts, wst, fen, arr)))
-    print("E1 A phases (median cycles): ld", int(np.median(ld[:n] - m1[:n])), "zero+compute+sts", int(np.median(sts[:n] - ld[:n])),
-          "wait_st", int(np.median(wst[:n] - sts[:n])), "fence.proxy", int(np.median(fen[:n] - wst[:n])), "arrive", int(np.median(arr[:n] - fen[:n])))
+    m1, ld, sts, fen, arr = col(10), col(40), col(42), col(46), col(12)
+    n = min(map(len, (m1, ld, sts, fen, arr)))
+    print("E1 A phases (median cycles): ld", int(np.median(ld[:n] - m1[:n])), "zero+arrive+compute+sts", int(np.median(sts[:n] - ld[:n])),
+          "fence.proxy", int(np.median(fen[:n] - sts[:n])), "arrive", int(np.median(arr[:n] - fen[:n])))
 except Exception as e:
     print("phase summary failed", e)
 for tg in (3, 7, 12, 22):
