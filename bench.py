@@ -16,6 +16,7 @@ timing).
 from __future__ import annotations
 
 import argparse
+import dataclasses
 import json
 import os
 import subprocess
@@ -236,7 +237,8 @@ def main():
     pool = gen_pool(cfg, P, rank)
     t_gen = time.time() - t_gen
 
-    ctx = ns.Context(local, pool_bytes=int((1.2 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)))
+    host_pool = ns.Context.host_pool_bytes(w, h, n, k, S) if args.e2e_steps > 0 else 0
+    ctx = ns.Context(local, pool_bytes=int((1.2 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)) + host_pool)
     # per-stream content-aware models: distinct weights per stream
     models = []
     for si in range(S):
@@ -335,25 +337,24 @@ def main():
                 "per_launch_algorithmic": per_launch,
                 "peak_source": f"{pk['src']} ({'bf16 sustained' if d['bound'] == 'tensor' else 'HBM copy'})"}
 
-    # e2e: host (pinned) -> device copy of every stream's inputs + the whole
-    # path + device -> host read of the step's result (stats, anchor map)
+    # e2e: the public host-input call (ns_enhance_streams_host): every step the
+    # library uploads each stream's res/mv/type from pinned host memory (stream
+    # groups overlapped with compute on its copy stream) and gathers the
+    # anchors' LR frames; then the step's result (stats, anchor map) is read back.
     e2e = None
     if args.e2e_steps > 0:
-        pin = [dict(lr=torch.from_numpy(c.lr).pin_memory(), res=torch.from_numpy(c.res).pin_memory(),
-                    mv=torch.from_numpy(np.ascontiguousarray(c.mv).view(np.uint8).reshape(n, h // 8, w // 8, 8))
-                    .pin_memory(), ty=torch.from_numpy(c.type).pin_memory()) for c in pool]
+        hpool = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, w, h, s) for c in pool]
+        hchunks = []
+        for si in range(S):
+            hc = dataclasses.replace(hpool[si % P], model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1])
+            hchunks.append(hc)
         st_h = torch.empty((S, 8), dtype=torch.float64).pin_memory()
         ia_h = torch.empty((S, n), dtype=torch.uint8).pin_memory()
-        h2d = sum(int(pin[si % P][kk].numel() * pin[si % P][kk].element_size()) for si in range(S)
-                  for kk in ("lr", "res", "mv", "ty"))
         d2h = st_h.numel() * 8 + ia_h.numel()
+        moved = [0]
 
         def e2e_step():
-            for si in range(S):
-                p = pin[si % P]
-                lr_d[si].copy_(p["lr"], non_blocking=True); res_d[si].copy_(p["res"], non_blocking=True)
-                mv_d[si].copy_(p["mv"], non_blocking=True); ty_d[si].copy_(p["ty"], non_blocking=True)
-            step()
+            moved[0] = ctx.enhance_streams_host(hchunks, hr_out, is_anchor_out=ia, stats=stats, k=k, stream=stream)
             st_h.copy_(stats, non_blocking=True)
             ia_h.copy_(ia, non_blocking=True)
 
@@ -368,10 +369,13 @@ def main():
         q1.record(stream)
         torch.cuda.synchronize(dev)
         ems = shard.max_over_ranks(q0.elapsed_time(q1))
-        e2e = {"value": world * S * n * args.e2e_steps / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": h2d,
+        e2e = {"value": world * S * n * args.e2e_steps / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": moved[0],
                "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
-               "note": "H2D of every stream's LR+residual+MV+type from pinned host memory each step; D2H of the "
-                       "per-stream stats and anchor map; HR frames stay in HBM for the downstream encoder"}
+               "api": "ns_enhance_streams_host (C ABI, pinned host inputs)",
+               "note": "per step: H2D of every stream's residual+MV+type (uploaded in stream groups on the library's "
+                       "copy stream, overlapped with compute) and of the anchors' LR frames (gathered after "
+                       "selection; non-anchor LR is read only for intra blocks, in place); D2H of the per-stream "
+                       "stats and anchor map; HR frames stay in HBM for the downstream encoder"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -401,9 +405,11 @@ def main():
 
 
 def ns_arena_gb(cfg, nb):
+    """SR arena of one shape (csrc/k_sr.cu sr_arena_bytes): x0 (16 ch) + h0/hb/tb
+    (C ch) bf16 + the u8 LR copy + border bands (small)."""
     h, w, C, s = cfg["h"], cfg["w"], cfg["n_ch"], cfg["scale"]
     px = h * w * nb
-    return (px * 16 * 2 + 3 * px * C * 2 + px * s * s * C * 2) / (1 << 30)
+    return (px * 16 * 2 + 3 * px * C * 2 + px * 3 + nb * (8 * (w + h) * s * (C + 3) * 4)) / (1 << 30)
 
 
 if __name__ == "__main__":

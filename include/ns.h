@@ -167,6 +167,28 @@ NS_API ns_status ns_reconstruct_chunk(ns_ctx *ctx, const ns_chunk *chunks, int S
 NS_API ns_status ns_enhance_streams(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
                              uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream);
 
+/* The whole hot path with the decoder's outputs in HOST memory -- the ingest
+   case, where decoded chunks arrive on the host -- and the outputs
+   in HBM.  Same arguments and results as ns_enhance_streams, except:
+     - chunks[s].lr, .res, .mv, .type, .res_size are HOST pointers to
+       page-locked, device-mapped memory (cudaHostAlloc / cudaHostRegister;
+       checked: NS_EINVAL otherwise); hr_last, hr_golden, gt stay DEVICE.
+     - The library uploads the streams in groups on an internal copy stream:
+       res/mv/type/res_size of group g+1 are copied while group g runs on
+       `stream` (two staging buffers carved from the context pool on first use;
+       NS_ENOMEM if the pool is too small).  LR is never copied wholesale: only
+       the anchors' LR frames (the SR input) are gathered from host memory after
+       selection, and KEY-frame / intra blocks read their LR in place.
+     - NS_GLOBAL_BUDGET needs every stream's scores before selecting, so it
+       runs as one group (no overlap).
+   *h2d_bytes (HOST, may be NULL) receives the bytes this call moves from host
+   to device: the uploads plus the gathered anchor LR frames (intra-block LR
+   reads, a few percent of blocks, are not counted).  The call returns once
+   everything is enqueued; results are ready when `stream` reaches them. */
+NS_API ns_status ns_enhance_streams_host(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
+                                         uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats,
+                                         uint64_t *h2d_bytes, void *stream);
+
 /* Number of this library's kernel launches enqueued by the calling thread
    since the last reset (for the bench's gpu_launches claim). */
 NS_API uint64_t ns_launch_count(int reset);

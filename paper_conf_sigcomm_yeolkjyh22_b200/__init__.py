@@ -49,7 +49,7 @@ class NsSrJob(ctypes.Structure):
 
 EXPORTS = ["ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_blob_len",
            "ns_model_destroy", "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
-           "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read"]
+           "ns_enhance_streams_host", "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read"]
 
 _lib = None
 
@@ -79,6 +79,8 @@ def lib() -> ctypes.CDLL:
         L.ns_sr_anchors.argtypes = [P, P, i32, P]
         L.ns_reconstruct_chunk.argtypes = [P, P, i32, P, P, P]
         L.ns_enhance_streams.argtypes = [P, P, i32, ctypes.POINTER(NsSelectParams), P, P, P, P]
+        L.ns_enhance_streams_host.argtypes = [P, P, i32, ctypes.POINTER(NsSelectParams), P, P, P,
+                                              ctypes.POINTER(ctypes.c_uint64), P]
         L.ns_launch_count.argtypes = [i32]
         L.ns_launch_count.restype = ctypes.c_uint64
         L.ns_last_error.restype = ctypes.c_char_p
@@ -87,7 +89,8 @@ def lib() -> ctypes.CDLL:
         L.ns_profile_read.argtypes = [P, i32]
         L.ns_profile_read.restype = i32
         for f in ("ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_destroy",
-                  "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams"):
+                  "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
+                  "ns_enhance_streams_host"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -170,6 +173,19 @@ class DeviceChunk:
         return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
                            model=model, res_size=rs, gt=None if gt is None else t(gt),
                            hr_last=hr_last, hr_golden=hr_golden)
+
+
+    @staticmethod
+    def pinned_from_numpy(lr, res, mv, types, w, h, scale, res_size=None, model=None,
+                          hr_last=None, hr_golden=None) -> "DeviceChunk":
+        """Host chunk for ns_enhance_streams_host: inputs in page-locked host
+        memory (torch pinned tensors); hr_last / hr_golden stay on the device."""
+        import torch
+        mvb = np.ascontiguousarray(mv).view(np.uint8).reshape(mv.shape[0], h // 8, w // 8, 8)
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+        rs = None if res_size is None else t(np.asarray(res_size).astype(np.int32))
+        return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
+                           model=model, res_size=rs, hr_last=hr_last, hr_golden=hr_golden)
 
 
 class Model:
@@ -267,3 +283,26 @@ class Context:
         _check(lib().ns_enhance_streams(self.handle, arr, len(chunks), ctypes.byref(p), tab, _ptr(is_anchor_out),
                                         _ptr(stats), _stream(stream)), "ns_enhance_streams")
         del keep
+
+    def enhance_streams_host(self, chunks, hr_out, is_anchor_out=None, stats=None, stream=None, **kw) -> int:
+        """ns_enhance_streams_host: chunks' inputs in pinned host memory
+        (DeviceChunk.pinned_from_numpy); returns the host->device bytes moved."""
+        arr = self._chunks(chunks)
+        tab = self._hr_table(hr_out)
+        p, keep = _params(**kw)
+        moved = ctypes.c_uint64(0)
+        _check(lib().ns_enhance_streams_host(self.handle, arr, len(chunks), ctypes.byref(p), tab,
+                                             _ptr(is_anchor_out), _ptr(stats), ctypes.byref(moved), _stream(stream)),
+               "ns_enhance_streams_host")
+        del keep
+        return int(moved.value)
+
+    @staticmethod
+    def host_pool_bytes(w: int, h: int, n: int, k: int, streams: int) -> int:
+        """Pool bytes ns_enhance_streams_host carves on first use (two input
+        staging buffers of one ~S/8-stream group + the anchors' LR staging)."""
+        a = lambda v: (v + 255) // 256 * 256
+        gs = max(1, (streams + 7) // 8)
+        px = h * w
+        per = a(n * 3 * px * 2) + a(n * (px // 64) * 8) + a(n) + a(n * 4)
+        return 2 * gs * per + gs * k * a(3 * px) + (1 << 20)

@@ -3,6 +3,7 @@
 // SR job compaction (K3).
 #include <cstdint>
 #include "ns_internal.h"
+#include <algorithm>
 
 namespace ns {
 
@@ -253,7 +254,8 @@ cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *g
 // Top-k mode: stream s owns slots [job_base, job_base + k) in frame order
 // (deterministic); global mode: slots are claimed with an atomic per group.
 __global__ void k_compact(const StreamDesc *sd, int S, int n, const uint8_t *is_anchor,
-                          uint8_t *const *hr_tab, SrJob *jobs, int32_t *job_count, int topk) {
+                          uint8_t *const *hr_tab, SrJob *jobs, int32_t *job_count, int topk, uint8_t *lr_stage,
+                          size_t lr_stride, const uint8_t **lr_src, uint32_t *lr_len) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
     const StreamDesc d = sd[s];
@@ -267,20 +269,47 @@ __global__ void k_compact(const StreamDesc *sd, int S, int n, const uint8_t *is_
         j.lr = d.lr + f * lr_frame;
         j.hr = hr_tab[d.hr_base + f];
         j.wts = d.wts;
+        if (lr_stage) {  // host-resident LR: gather into device staging, SR reads the copy
+            lr_src[slot] = j.lr;
+            lr_len[slot] = (uint32_t)lr_frame;
+            j.lr = lr_stage + (size_t)slot * lr_stride;
+        }
         jobs[slot] = j;
     }
 }
 
+// One CTA row per job, CTAs stride over the frame in 16-B words: wide,
+// coalesced reads of page-locked host memory over PCIe.
+__global__ void k_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len) {
+    const int j = blockIdx.y;
+    const uint32_t len = lr_len[j];
+    if (len == 0) return;
+    const uint4 *src = reinterpret_cast<const uint4 *>(lr_src[j]);
+    uint4 *dst = reinterpret_cast<uint4 *>(const_cast<uint8_t *>(jobs[j].lr));
+    const uint32_t nw = len / 16;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += gridDim.x * blockDim.x) dst[i] = src[i];
+}
+
+cudaError_t launch_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len, int max_jobs,
+                             size_t max_len, cudaStream_t st) {
+    KScope ks(F_COMPACT, st);
+    const int bx = (int)std::min<size_t>((max_len / 16 + 1023) / 1024, 256);
+    k_lr_gather<<<dim3(std::max(bx, 1), max_jobs), 256, 0, st>>>(jobs, lr_src, lr_len);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
                            uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups, int topk,
-                           int k, cudaStream_t st) {
+                           int k, cudaStream_t st, uint8_t *lr_stage, size_t lr_stride, const uint8_t **lr_src,
+                           uint32_t *lr_len) {
     (void)k;
     KScope ks(F_COMPACT, st);
     if (!topk) {
         cudaError_t e = cudaMemsetAsync(job_count, 0, sizeof(int32_t) * n_groups, st);
         if (e != cudaSuccess) return e;
     }
-    k_compact<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, jobs, job_count, topk);
+    k_compact<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, jobs, job_count, topk, lr_stage,
+                                               lr_stride, lr_src, lr_len);
     return cudaGetLastError();
 }
 

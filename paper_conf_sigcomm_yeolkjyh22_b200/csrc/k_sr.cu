@@ -663,6 +663,19 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
     tc_fence_after();
     const uint32_t tmem = *s_tmem;
     const SrJob J = a.jobs[job];
+    if (warp > kRbMmaWarps) {
+        // both accumulator rings start at zero: the blocks of t row y0-1 and of
+        // output row y0 are first touched before any retirement could zero them
+        // (TMEM keeps whatever an earlier CTA on this SM left unretired)
+        const int g = (warp - 1 - kRbMmaWarps) / 4, k = g / 2, role = g % 2;
+        const uint32_t tl = tmem + ((uint32_t)((warp % 4) * 32) << 16) + k * Cfg::TCOLS + role * 3 * NB;
+#pragma unroll 1
+        for (int b = 0; b < 3; b++) tmem_zeroN<NB>(tl + b * NB);
+        tmem_wait_st();
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
 
     if (warp == 0) {
         // ---------------------------------------------------------------- TMA producer

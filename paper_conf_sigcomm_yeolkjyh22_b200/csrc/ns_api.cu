@@ -175,6 +175,18 @@ struct ns_ctx {
     size_t blob_stage_elems;
     int sr_batch = 16;
     std::vector<ArenaEntry> arenas;
+    // host-input path (ns_enhance_streams_host): copy stream, two input staging
+    // buffers (group ping-pong) and the anchor-LR gather staging, carved from
+    // the pool on first use and grown (bump) if a later call needs more
+    cudaStream_t cst = nullptr;
+    cudaEvent_t ev_copied[2] = {}, ev_free[2] = {};
+    bool hin_used[2] = {};
+    uint8_t *hin[2] = {};
+    size_t hin_cap = 0;
+    uint8_t *lr_stage = nullptr;
+    size_t lr_stage_cap = 0;
+    const uint8_t **lr_src = nullptr;
+    uint32_t *lr_len = nullptr;
 };
 
 static uint8_t *pool_take(ns_ctx *c, size_t bytes) {
@@ -218,7 +230,8 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     NS_CUDA(cudaSetDevice(device));
     ns_ctx *c = new ns_ctx();
     c->device = device;
-    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2) + (size_t)kMaxJobs * sizeof(SrJob) +
+    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2) +
+                         (size_t)kMaxJobs * (sizeof(SrJob) + sizeof(uint8_t *) + sizeof(uint32_t)) +
                          kStageSlots * kStageBytes + (64u << 20) + 64 * 1024;
     if (pool_bytes < fixed + (64u << 20)) {
         delete c;
@@ -252,6 +265,18 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
             return cuda_fail(e, "staging");
         }
     }
+    c->lr_src = (const uint8_t **)pool_take(c, sizeof(uint8_t *) * kMaxJobs);
+    c->lr_len = (uint32_t *)pool_take(c, sizeof(uint32_t) * kMaxJobs);
+    if ((e = cudaStreamCreateWithFlags(&c->cst, cudaStreamNonBlocking)) != cudaSuccess) {
+        ns_ctx_destroy(c);
+        return cuda_fail(e, "copy stream");
+    }
+    for (int i = 0; i < 2; i++)
+        if ((e = cudaEventCreateWithFlags(&c->ev_copied[i], cudaEventDisableTiming)) != cudaSuccess ||
+            (e = cudaEventCreateWithFlags(&c->ev_free[i], cudaEventDisableTiming)) != cudaSuccess) {
+            ns_ctx_destroy(c);
+            return cuda_fail(e, "events");
+        }
     *out = c;
     return NS_OK;
 }
@@ -264,6 +289,11 @@ extern "C" ns_status ns_ctx_destroy(ns_ctx *c) {
         if (c->stage_host[i]) cudaFreeHost(c->stage_host[i]);
         if (c->stage_ev[i]) cudaEventDestroy(c->stage_ev[i]);
     }
+    for (int i = 0; i < 2; i++) {
+        if (c->ev_copied[i]) cudaEventDestroy(c->ev_copied[i]);
+        if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
+    }
+    if (c->cst) cudaStreamDestroy(c->cst);
     if (c->pool) cudaFree(c->pool);
     delete c;
     return NS_OK;
@@ -614,16 +644,16 @@ extern "C" ns_status ns_reconstruct_chunk(ns_ctx *c, const ns_chunk *ch, int S, 
 }
 
 // ------------------------------------------------------------------ the whole path
-extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
-                                        uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream) {
-    if (!c) return fail(NS_EINVAL, "ns_enhance_streams: ctx is NULL");
-    int n = 0;
-    ns_status r = check_chunks(ch, S, true, &n);
-    if (r != NS_OK) return r;
-    if ((r = check_params(p, S, n)) != NS_OK) return r;
-    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
-    cudaStream_t st = (cudaStream_t)stream;
-    NS_CUDA(cudaSetDevice(c->device));
+// Optional host-input mode of enhance_impl: SR jobs read LR from a device copy
+// gathered after selection (lr_stage, one frame of lr_stride bytes per job slot).
+struct LrGather {
+    uint8_t *stage;
+    size_t stride;
+};
+
+static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const ns_select_params *p,
+                              uint8_t *const *hr_out, uint8_t *anchor, double *stats, cudaStream_t st,
+                              const LrGather *lg, uint64_t *gathered) {
     const bool topk = p->mode == NS_TOPK_PER_STREAM;
     // SR shape groups and job slots (multi-stream batcher)
     std::map<std::tuple<int, int, int, int, int>, int> gid;
@@ -656,6 +686,8 @@ extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, co
         total += (int)mx;
     }
     if (total > kMaxJobs) return fail(NS_EINVAL, "too many SR jobs (%d)", total);
+    if (lg && (size_t)total * lg->stride > c->lr_stage_cap)
+        return fail(NS_EINVAL, "anchor LR staging too small (%d jobs)", total);
     {
         std::vector<int> local(G, 0);
         for (int s = 0; s < S; s++) {
@@ -663,16 +695,27 @@ extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, co
             job_base[s] = topk ? goff[gi] + local[gi]++ * p->k : goff[gi];
         }
     }
+    if (gathered && lg) {  // exact in top-k mode (k frames per stream); upper bound otherwise
+        uint64_t b = 0;
+        for (int s = 0; s < S; s++) b += (uint64_t)3 * ch[s].h * ch[s].w * (topk ? p->k : 0);
+        if (!topk) b = (uint64_t)total * lg->stride;
+        *gathered += b;
+    }
     Staged g;
+    ns_status r;
     if ((r = stage_streams(c, ch, S, n, hr_out, topk ? nullptr : p->cost, group.data(), job_base.data(),
                            p->use_res_size != 0, &g)) != NS_OK)
         return r;
     if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
-    uint8_t *anchor = is_anchor_out ? is_anchor_out : c->anchor;
     do {
         if ((r = run_select(c, g, ch, S, n, p, c->gain, c->rank, anchor, st)) != NS_OK) break;
         if (total > 0) {
-            cudaError_t e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, topk, p->k, st);
+            cudaError_t e = cudaSuccess;
+            if (lg) e = cudaMemsetAsync(c->lr_len, 0, sizeof(uint32_t) * total, st);
+            if (e == cudaSuccess)
+                e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, topk, p->k, st,
+                                   lg ? lg->stage : nullptr, lg ? lg->stride : 0, c->lr_src, c->lr_len);
+            if (e == cudaSuccess && lg) e = launch_lr_gather(c->jobs, c->lr_src, c->lr_len, total, lg->stride, st);
             if (e != cudaSuccess) { r = cuda_fail(e, "compact"); break; }
             for (int gi = 0; gi < G && r == NS_OK; gi++) {
                 int h, w, C, s, B;
@@ -691,4 +734,135 @@ extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, co
     } while (0);
     stage_release(c, g.slot, st);
     return r;
+}
+
+extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
+                                        uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_enhance_streams: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, true, &n);
+    if (r != NS_OK) return r;
+    if ((r = check_params(p, S, n)) != NS_OK) return r;
+    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    NS_CUDA(cudaSetDevice(c->device));
+    return enhance_impl(c, ch, S, n, p, hr_out, is_anchor_out ? is_anchor_out : c->anchor, stats,
+                        (cudaStream_t)stream, nullptr, nullptr);
+}
+
+// ------------------------------------------------------------------ host-input path
+static bool host_mapped(const void *p) {
+    if (!p) return true;
+    cudaPointerAttributes at;
+    if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return at.type == cudaMemoryTypeHost && at.devicePointer == p;  // UVA: same address on the device
+}
+
+// bytes of one stream's uploaded inputs in a staging buffer (256-B aligned pieces)
+static size_t host_stream_bytes(const ns_chunk &k) {
+    const size_t n = (size_t)k.n_frames, px = (size_t)k.h * k.w;
+    return a256(n * 3 * px * 2) + a256(n * (px / 64) * sizeof(ns_block_mv)) + a256(n) + (k.res_size ? a256(n * 4) : 0);
+}
+
+extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
+                                             uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats,
+                                             uint64_t *h2d_bytes, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_enhance_streams_host: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, true, &n);
+    if (r != NS_OK) return r;
+    if ((r = check_params(p, S, n)) != NS_OK) return r;
+    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    for (int s = 0; s < S; s++)
+        if (!host_mapped(ch[s].lr) || !host_mapped(ch[s].res) || !host_mapped(ch[s].mv) || !host_mapped(ch[s].type) ||
+            !host_mapped(ch[s].res_size))
+            return fail(NS_EINVAL, "chunk %d: lr/res/mv/type/res_size must be page-locked, device-mapped host memory", s);
+    NS_CUDA(cudaSetDevice(c->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    const bool topk = p->mode == NS_TOPK_PER_STREAM;
+    // groups of consecutive streams: ~8 per call so the first group's upload is
+    // short; global budget mode needs all scores before selecting -> one group
+    const int gs = topk ? std::max(1, (S + 7) / 8) : S;
+    size_t cap = 0, lr_stride = 0;
+    int max_jobs = 0;
+    for (int g0 = 0; g0 < S; g0 += gs) {
+        size_t b = 0;
+        int jobs = 0;
+        for (int s = g0; s < std::min(S, g0 + gs); s++) {
+            b += host_stream_bytes(ch[s]);
+            jobs += topk ? p->k : n;
+        }
+        cap = std::max(cap, b);
+        max_jobs = std::max(max_jobs, jobs);
+    }
+    for (int s = 0; s < S; s++) lr_stride = std::max(lr_stride, a256((size_t)3 * ch[s].h * ch[s].w));
+    if (!topk) {  // one group; job slots as enhance_impl lays them out: per SR shape, min(streams * n, budget / min cost)
+        int64_t min_cost = INT64_MAX;
+        for (int s = 0; s < S; s++) min_cost = std::min(min_cost, p->cost[s]);
+        std::map<std::tuple<int, int, int, int, int>, int> cnt;
+        for (int s = 0; s < S; s++)
+            cnt[std::make_tuple(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks)]++;
+        int64_t t = 0;
+        for (auto &kv : cnt) t += std::min<int64_t>((int64_t)kv.second * n, p->budget / std::max<int64_t>(min_cost, 1));
+        max_jobs = (int)std::min<int64_t>(t, kMaxJobs);
+    }
+    if (cap > c->hin_cap) {
+        for (int i = 0; i < 2; i++) {
+            if (c->hin_used[i]) NS_CUDA(cudaEventSynchronize(c->ev_free[i]));
+            c->hin_used[i] = false;
+            if (!(c->hin[i] = pool_take(c, cap)))
+                return fail(NS_ENOMEM, "ns_enhance_streams_host: pool too small for input staging (%zu bytes x 2)", cap);
+        }
+        c->hin_cap = cap;
+    }
+    if ((size_t)max_jobs * lr_stride > c->lr_stage_cap) {
+        const size_t need = (size_t)max_jobs * lr_stride;
+        NS_CUDA(cudaStreamSynchronize(st));  // the old staging may still be read (not the steady state)
+        if (!(c->lr_stage = pool_take(c, need)))
+            return fail(NS_ENOMEM, "ns_enhance_streams_host: pool too small for anchor LR staging (%zu bytes)", need);
+        c->lr_stage_cap = need;
+    }
+    uint8_t *anchor = is_anchor_out ? is_anchor_out : c->anchor;
+    uint64_t moved = 0;
+    std::vector<ns_chunk> dch(gs);
+    for (int g0 = 0, gi = 0; g0 < S; g0 += gs, gi++) {
+        const int b = gi & 1, cnt = std::min(gs, S - g0);
+        // upload group gi into buffer b once the compute that last used b is done
+        if (c->hin_used[b]) NS_CUDA(cudaStreamWaitEvent(c->cst, c->ev_free[b], 0));
+        uint8_t *dst = c->hin[b];
+        for (int i = 0; i < cnt; i++) {
+            const ns_chunk &k = ch[g0 + i];
+            const size_t nf = (size_t)k.n_frames, px = (size_t)k.h * k.w;
+            dch[i] = k;
+            const size_t rb = nf * 3 * px * 2, mb = nf * (px / 64) * sizeof(ns_block_mv);
+            NS_CUDA(cudaMemcpyAsync(dst, k.res, rb, cudaMemcpyHostToDevice, c->cst));
+            dch[i].res = reinterpret_cast<const int16_t *>(dst);
+            dst += a256(rb);
+            NS_CUDA(cudaMemcpyAsync(dst, k.mv, mb, cudaMemcpyHostToDevice, c->cst));
+            dch[i].mv = reinterpret_cast<const ns_block_mv *>(dst);
+            dst += a256(mb);
+            NS_CUDA(cudaMemcpyAsync(dst, k.type, nf, cudaMemcpyHostToDevice, c->cst));
+            dch[i].type = dst;
+            dst += a256(nf);
+            if (k.res_size) {
+                NS_CUDA(cudaMemcpyAsync(dst, k.res_size, nf * 4, cudaMemcpyHostToDevice, c->cst));
+                dch[i].res_size = reinterpret_cast<const uint32_t *>(dst);
+                dst += a256(nf * 4);
+                moved += nf * 4;
+            }
+            moved += rb + mb + nf;
+        }
+        NS_CUDA(cudaEventRecord(c->ev_copied[b], c->cst));
+        NS_CUDA(cudaStreamWaitEvent(st, c->ev_copied[b], 0));
+        LrGather lg{c->lr_stage, lr_stride};
+        r = enhance_impl(c, dch.data(), cnt, n, p, hr_out + (size_t)g0 * n, anchor + (size_t)g0 * n,
+                         stats ? stats + (size_t)8 * g0 : nullptr, st, &lg, &moved);
+        if (r != NS_OK) return r;
+        NS_CUDA(cudaEventRecord(c->ev_free[b], st));
+        c->hin_used[b] = true;
+    }
+    if (h2d_bytes) *h2d_bytes = moved;
+    return NS_OK;
 }

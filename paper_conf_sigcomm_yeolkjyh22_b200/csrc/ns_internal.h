@@ -83,8 +83,13 @@ cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *g
                           const int64_t *cost, int64_t budget, int32_t *grank, int32_t *pos_stream,
                           int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st);
 cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
-                           uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups,
-                           int topk, int k, cudaStream_t st);
+                           uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups, int topk,
+                           int k, cudaStream_t st, uint8_t *lr_stage = nullptr, size_t lr_stride = 0,
+                           const uint8_t **lr_src = nullptr, uint32_t *lr_len = nullptr);
+// Copies every filled job's LR frame (lr_len[j] > 0) from lr_src[j] (host-mapped
+// memory) to jobs[j].lr (device staging set by launch_compact).
+cudaError_t launch_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len, int max_jobs,
+                             size_t max_len, cudaStream_t st);
 cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st);
 // max_lr_w / max_lr_h: [5] indexed by scale (0 = no stream of that scale)
 cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const int *max_lr_w,

@@ -326,3 +326,28 @@ def test_c3_full_size_batched(ctx):
     assert worst <= SR_MAX_ABS, worst
     exp, _, _ = oracle.reconstruct(c, list(ia[0]), got, np.zeros_like(got[0]), np.zeros_like(got[0]))
     assert np.array_equal(got, exp)
+
+
+# ---------------------------------------------------------------- SR is a pure function
+@pytest.mark.parametrize("C,s", [(16, 2), (32, 3)])
+def test_sr_deterministic_across_batches(ctx, C, s):
+    """SR(weights, LR) must not depend on what ran before or on the batch it is
+    in: tensor-memory accumulators start at zero in every CTA (TMEM keeps what
+    an earlier CTA on the SM left unretired).  256 LR rows span three res-block
+    strips (y0 = 0, 120, 240) and several uptail / head strips."""
+    m, _ = _model(ctx, 2, C, s, seed=91)
+    w, h = 136, 256
+    lrs = [torch.from_numpy(synth.make_chunk(9100 + i, w, h, s, 1).lr[0]).to(DEV) for i in range(5)]
+    outs = []
+    for order in ([0, 1, 2, 3, 4], [4, 3, 2, 1, 0], [2], [0, 2, 4]):
+        hr = {i: torch.zeros((3, s * h, s * w), dtype=torch.uint8, device=DEV) for i in order}
+        # unrelated work in between leaves different TMEM contents behind
+        other, _ = _model(ctx, 1, C, s, seed=92 + len(outs))
+        junk = torch.zeros((3, s * 64, s * 64), dtype=torch.uint8, device=DEV)
+        ctx.sr_anchors([(other, torch.randint(0, 256, (3, 64, 64), dtype=torch.uint8, device=DEV), junk)])
+        ctx.sr_anchors([(m, lrs[i], hr[i]) for i in order])
+        torch.cuda.synchronize()
+        outs.append({i: t.cpu().numpy() for i, t in hr.items()})
+    for o in outs[1:]:
+        for i, a in o.items():
+            assert np.array_equal(a, outs[0][i]), i
