@@ -141,6 +141,7 @@ constexpr int kStageSlots = 4;
 constexpr size_t kStageBytes = 8u << 20;
 constexpr int kMaxSN = 1 << 20;           // max streams x frames per call
 constexpr int kMaxJobs = 1 << 20;
+constexpr int kHostGroups = 8;            // stream groups per ns_enhance_streams_host call
 
 struct ArenaEntry {
     int h, w, C, s;
@@ -782,9 +783,10 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
     NS_CUDA(cudaSetDevice(c->device));
     cudaStream_t st = (cudaStream_t)stream;
     const bool topk = p->mode == NS_TOPK_PER_STREAM;
-    // groups of consecutive streams: ~8 per call so the first group's upload is
-    // short; global budget mode needs all scores before selecting -> one group
-    const int gs = topk ? std::max(1, (S + 7) / 8) : S;
+    // groups of consecutive streams, ~kHostGroups per call: the first group's
+    // upload and the last group's compute are the unhidden fill and drain; global
+    // budget mode needs all scores before selecting -> one group
+    const int gs = topk ? std::max(1, (S + kHostGroups - 1) / kHostGroups) : S;
     size_t cap = 0, lr_stride = 0;
     int max_jobs = 0;
     for (int g0 = 0; g0 < S; g0 += gs) {
