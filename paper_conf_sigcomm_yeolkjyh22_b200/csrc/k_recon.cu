@@ -64,36 +64,35 @@ __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
 }
 
 // Stage the raw aligned 64-bit words covering reference bytes xs .. xs+BW of
-// one row into shared memory (cp.async for interior windows; edge blocks use
-// clamped byte loads that emulate the same aligned words).  dst[i * stride]
-// is word i (struct-of-arrays across the CTA's threads: conflict-free reads).
-template <int S>
-__device__ __noinline__ void recon_row_stage_edge(const uint8_t *row, int xs, int W, uint2 *dst, int stride) {
-    using Cfg = ReconCfg<S>;
-    const int xb = xs & ~7;
-    for (int i = 0; i < Cfg::NQ; i++) {
-        uint32_t v0 = 0, v1 = 0;
-        for (int b = 0; b < 4; b++) {
-            v0 |= (uint32_t)row[min(max(xb + 8 * i + b, 0), W - 1)] << (8 * b);
-            v1 |= (uint32_t)row[min(max(xb + 8 * i + 4 + b, 0), W - 1)] << (8 * b);
-        }
-        dst[i * stride] = make_uint2(v0, v1);
-    }
-}
-
+// one row into shared memory: dst[i * stride] is word i (struct-of-arrays
+// across the CTA's threads: conflict-free reads).  W and the word base are
+// multiples of 8, so every word lies wholly inside the row (cp.async) or wholly
+// outside it, where edge replication (Z16) makes it 8 copies of the first or
+// last pixel: no byte-wise clamped loads, and no read past the row end.
 template <int S>
 __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int W, bool interior, uint2 *dst,
                                                 int stride) {
     using Cfg = ReconCfg<S>;
+    const int xb = xs & ~7;
     if (interior) {
-        const int xb = xs & ~7;
 #pragma unroll
         for (int i = 0; i < Cfg::NQ; i++)
             asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + i * stride)),
                          "l"(row + xb + 8 * i)
                          : "memory");
     } else {
-        recon_row_stage_edge<S>(row, xs, W, dst, stride);
+#pragma unroll
+        for (int i = 0; i < Cfg::NQ; i++) {
+            const int st = xb + 8 * i;
+            if (st >= 0 && st < W) {
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + i * stride)),
+                             "l"(row + st)
+                             : "memory");
+            } else {
+                const uint32_t v = 0x01010101u * row[st < 0 ? 0 : W - 1];
+                dst[i * stride] = make_uint2(v, v);
+            }
+        }
     }
 }
 
@@ -213,8 +212,7 @@ __device__ __forceinline__ void recon_planes(const StreamDesc &d, bool use_lr, c
 #pragma unroll
         for (int j = 0; j <= RPT; j++) {
             const int r = min(max(iy0 + j, 0), H - 1);
-            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior && !(c == 2 && r == H - 1),
-                               buf + j * Cfg::NQ * NT, NT);
+            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior, buf + j * Cfg::NQ * NT, NT);
         }
     };
     stage(0);
@@ -346,11 +344,8 @@ __global__ void __launch_bounds__(kReconTX *kReconTY, 3)
     // packed 2 x 16-bit arithmetic multiplies by a SCALAR (no cross-lane terms)
     const uint32_t fxp = fx, fyp = fy, fxc = 8u - fx, fyc = 8u - fy;
     const int iy0 = Y0 + (my >> 3);
-    // All used bytes inside the row -> aligned vector loads (they may run up to
-    // 8*NQ - BW - 1 bytes past the row end, which stays inside the plane except
-    // on the very last row of plane 2; recon_planes routes that row to the
-    // clamped path).
-    const bool interior = xs >= 0 && xs + BW <= W - 1;
+    // every aligned word of the window inside the row -> unconditional cp.async
+    const bool interior = xs >= 0 && (xs & ~7) + 8 * Cfg::NQ <= W;
     const uint8_t *lr_f = d.lr + (size_t)f * 3 * lrp;
     const int16_t *res_f = d.res + (size_t)f * 3 * lrp;
 
