@@ -52,6 +52,14 @@ def cfg_of(args):
     return c
 
 
+def workload_config(cfg, world):
+    """The `config` object both arms print (same workload, same keys)."""
+    S, s, w, h = cfg["streams"], cfg["scale"], cfg["w"], cfg["h"]
+    return {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{s * w}x{s * h} x{s} streams per GPU, "
+                        f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} (top-k per stream)",
+            "streams_per_gpu": S, "frames_per_step_per_gpu": S * cfg["n"], "parallelism": f"streams x{world}"}
+
+
 def _gen(a):
     seed, w, h, s, n, alt = a
     return synth.make_chunk(seed, w, h, s, n, types=synth.default_types(n, alt))
@@ -150,6 +158,9 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
+    # rank 0 alone runs the oracle, on all host cores (torchrun sets OMP_NUM_THREADS=1
+    # per rank; nothing has initialised OpenMP in this process yet)
+    os.environ["OMP_NUM_THREADS"] = str(os.cpu_count() or 1)
     cfg = cfg_of(args)
     chunk = _gen((4000, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"]))
     blob = synth.make_weights(4000, cfg["n_blocks"], cfg["n_ch"], cfg["scale"])
@@ -163,7 +174,8 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{cfg['name']} (one stream-chunk sample per step)"},
+            "config": dict(workload_config(cfg, args.gpus), sample="one stream-chunk of the workload per step "
+                                                                    "(see cpu_baseline.sample), scaled to frames/s"),
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["cores"], "kind": "oracle", "sample": r["sample"]},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -388,11 +400,9 @@ def main():
                 "vs_baseline": None, "dtype": "bf16",
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
-                "config": {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{W}x{H} x{s} streams per GPU, "
-                                       f"B{B}/C{C}, n={n}, k={k} (top-k per stream)",
-                           "streams_per_gpu": S, "frames_per_step_per_gpu": S * n, "parallelism": f"streams x{world}",
-                           "l2": "inputs larger than L2 (~130 GB touched per step)", "sr_batch": args.sr_batch,
-                           "gen_s": round(t_gen, 1)},
+                "config": dict(workload_config(cfg, world),
+                               l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
+                               gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
                              "anchors_per_step": int(ia_np.sum())},
