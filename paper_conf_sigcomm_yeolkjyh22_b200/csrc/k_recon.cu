@@ -55,6 +55,10 @@ struct ReconCfg {
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
     static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
                                                    // or of 8s/.. so that Y0 mod S == 0
+    // resident CTAs per SM: s = 3 fits 128 registers without spills and its
+    // 56 KB of staging exactly fills 4 CTAs' worth of shared memory (latency-
+    // bound kernel: occupancy 3 -> 4 CTAs); s = 2, 4 would spill at 128
+    static constexpr int MINB = (S == 3) ? 4 : 3;
 };
 
 __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
@@ -308,7 +312,7 @@ __device__ __forceinline__ void recon_planes(const StreamDesc &d, bool use_lr, c
 }
 
 template <int S>
-__global__ void __launch_bounds__(kReconTX *kReconTY, 3)
+__global__ void __launch_bounds__(kReconTX *kReconTY, ReconCfg<S>::MINB)
     k_recon_step(const StreamDesc *sd, int n, int f, const uint8_t *is_anchor, uint8_t *const *hr_tab,
                  const int16_t *gold) {
     using Cfg = ReconCfg<S>;
@@ -364,6 +368,9 @@ static void recon_launch(dim3 g, cudaStream_t st, const StreamDesc *d_sd, int n,
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)recon_smem<S>());
+        // all of the unified L1/shared array as shared memory, so MINB CTAs fit
+        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             (int)cudaSharedmemCarveoutMaxShared);
         attr = true;
     }
     k_recon_step<S><<<g, dim3(kReconTX, kReconTY), recon_smem<S>(), st>>>(d_sd, n, f, is_anchor, hr, gold);
