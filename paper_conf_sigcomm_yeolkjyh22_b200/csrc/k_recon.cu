@@ -2,6 +2,7 @@
 // §2 P:89-91 and §6.1), chunk-end reference state, per-stream stats
 // (K10) and the model weight repack (model pre-optimisation, §6.2).
 #include <cstdint>
+#include <type_traits>
 #include "ns_internal.h"
 #include "ptx.cuh"
 
@@ -38,14 +39,36 @@ cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *g
 }
 
 // One frame step f for all streams (K9).  A thread owns one LR block column
-// (8s HR pixels wide, the motion vector is uniform there) x 8 HR rows x 3
+// (8s HR pixels wide, the motion vector is uniform there) x RPT HR rows x 3
 // planes:  anchor -> skip (SR output already in place); KEY frame or INTRA
 // block -> up_s(LR[f]); otherwise clamp(warp_{s*mv}(HR[ref]) + up_s(res[f])).
-// The warp (O7) runs two pixels per 32-bit register (16-bit lanes; every
-// intermediate < 2^16): each horizontal pass over a reference row is shared by
-// the two output rows that use it.  up_s (O6) is separable with compile-time
-// taps (the thread's first pixel is a multiple of s).  Reference windows are
-// read with aligned 64-bit loads (edge blocks fall back to clamped byte loads).
+//
+// Memory: every global read is asynchronous.  The CTA's residual tile (all
+// three planes: 4*RPT/s + 2 LR rows x 256 + 16 columns of i16) is staged
+// cooperatively with 16-B cp.async at entry; each thread's warp windows (the
+// MV-displaced reference rows, as aligned 8-B words) are staged per plane with
+// cp.async, double-buffered so plane c+1 is in flight while plane c computes.
+//
+// Arithmetic (two pixels per 32-bit register, 16-bit lanes, every lane value
+// < 2^16 so lanes never carry into each other):
+//  * warp, horizontal pass (O7): v = R[x](8-fx) + R[x+1]fx + 4 in [4, 2044];
+//    the pass result floor(v/8) is kept scaled by 8, h8 = v & ~7 (no shift);
+//  * vertical pass: 8 (h0(8-fy) + h1 fy + 4) = h8_0(8-fy) + h8_1 fy + 32, so
+//    pred = floor(that / 64);
+//  * up_s (O6) per pixel r = floor((v + 8192) / 2^14) lands in the high half of
+//    a 32-bit value with a +256 bias; one PRMT packs a pixel pair;
+//  * X = 64 (r + 256) + h8_0(8-fy) + h8_1 fy + 32 <= 49056 per lane, and
+//    floor(X / 64) = pred + r + 256 (64 (r + 256) is a multiple of 64), so the
+//    clamp of pred + r to [0, 255] is a clamp of X to [2^14, 2^15 - 1]; X >> 6
+//    then holds 256 + out in each lane and one PRMT packs 4 output bytes.
+template <int N, int I = 0, class F>
+__device__ __forceinline__ void static_for(F &&f) {
+    if constexpr (I < N) {
+        f(std::integral_constant<int, I>{});
+        static_for<N, I + 1>(f);
+    }
+}
+
 template <int S>
 struct ReconCfg {
     static constexpr int BW = 8 * S;               // HR pixels per thread row
@@ -54,11 +77,19 @@ struct ReconCfg {
     static constexpr int NQ = (7 + WIN + 7) / 8;   // aligned 64-bit words per row
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
     static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
-                                                   // or of 8s/.. so that Y0 mod S == 0
-    // resident CTAs per SM: s = 3 fits 128 registers without spills and its
-    // 56 KB of staging exactly fills 4 CTAs' worth of shared memory (latency-
-    // bound kernel: occupancy 3 -> 4 CTAs); s = 2, 4 would spill at 128
-    static constexpr int MINB = (S == 3) ? 4 : 3;
+    static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
+    static constexpr int MINB = (S == 3) ? 3 : 2;  // resident CTAs per SM (shared memory)
+};
+constexpr int kReconTX = 32, kReconTY = 4;
+constexpr int kReconNT = kReconTX * kReconTY;
+constexpr int kResCols = 8 * kReconTX + 16;        // residual tile columns (one 16-B chunk of halo per side)
+
+template <int S>
+struct ReconSmem {
+    static constexpr int RROWS = kReconTY * ReconCfg<S>::PER + 2;      // residual tile LR rows
+    static constexpr size_t REF = (size_t)2 * (ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconNT * 8;
+    static constexpr size_t RES = (size_t)3 * RROWS * kResCols * 2;
+    static constexpr size_t BYTES = REF + RES;
 };
 
 __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
@@ -66,55 +97,64 @@ __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
     return r;
 }
+__device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
 
 // Stage the raw aligned 64-bit words covering reference bytes xs .. xs+BW of
 // one row into shared memory: dst[i * stride] is word i (struct-of-arrays
 // across the CTA's threads: conflict-free reads).  W and the word base are
-// multiples of 8, so every word lies wholly inside the row (cp.async) or wholly
-// outside it, where edge replication (Z16) makes it 8 copies of the first or
-// last pixel: no byte-wise clamped loads, and no read past the row end.
+// multiples of 8, so every word lies wholly inside the row or wholly outside
+// it; an outside word stages the row's first / last word instead, and
+// recon_fix_edges replicates its edge pixel (Z16) after the copy lands: every
+// global read stays an asynchronous copy, and none reads past the row.
 template <int S>
 __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int W, bool interior, uint2 *dst,
                                                 int stride) {
     using Cfg = ReconCfg<S>;
     const int xb = xs & ~7;
-    if (interior) {
 #pragma unroll
-        for (int i = 0; i < Cfg::NQ; i++)
-            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + i * stride)),
-                         "l"(row + xb + 8 * i)
-                         : "memory");
-    } else {
-#pragma unroll
-        for (int i = 0; i < Cfg::NQ; i++) {
-            const int st = xb + 8 * i;
-            if (st >= 0 && st < W) {
-                asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst + i * stride)),
-                             "l"(row + st)
-                             : "memory");
-            } else {
-                const uint32_t v = 0x01010101u * row[st < 0 ? 0 : W - 1];
-                dst[i * stride] = make_uint2(v, v);
-            }
+    for (int i = 0; i < Cfg::NQ; i++) {
+        const int st = interior ? xb + 8 * i : min(max(xb + 8 * i, 0), W - 8);
+        cp_async8(dst + i * stride, row + st);
+    }
+}
+// After the copies of a non-interior window have landed: replicate the edge
+// pixel into the staged words that lie outside the row (first word at xb).
+template <int S>
+__device__ __noinline__ void recon_fix_edges(uint2 *buf, int xb, int W) {
+    using Cfg = ReconCfg<S>;
+#pragma unroll 1
+    for (int i = 0; i < Cfg::NQ; i++) {
+        const int st = xb + 8 * i;
+        if (st >= 0 && st < W) continue;
+#pragma unroll 1
+        for (int j = 0; j <= Cfg::RPT; j++) {
+            uint2 *q = buf + (j * Cfg::NQ + i) * kReconNT;
+            const uint32_t v = st < 0 ? prmt(q->x, 0u, 0x0000u) : prmt(q->y, 0u, 0x3333u);
+            *q = make_uint2(v, v);
         }
     }
 }
 
-// Horizontal bilinear pass over one reference row: h[k] = packed pixels
-// (2k, 2k+1) of (R[x](8-fx) + R[x+1]fx + 4) >> 3 for x = xs .. xs+BW-1.
+// Horizontal bilinear pass over one staged reference row, scaled by 8:
+// h8[k] = packed pixels (2k, 2k+1) of (R[x](8-fx) + R[x+1]fx + 4) & ~7.
 template <int S>
-__device__ __forceinline__ void recon_hpass(const uint2 (&q)[ReconCfg<S>::NQ], int xs, uint32_t fxc, uint32_t fx,
-                                            uint32_t (&h)[ReconCfg<S>::NP]) {
+__device__ __forceinline__ void recon_hpass8(const uint2 *buf, int m, uint32_t fxc, uint32_t fx,
+                                             uint32_t (&h)[ReconCfg<S>::NP]) {
     using Cfg = ReconCfg<S>;
     uint32_t w[2 * Cfg::NQ + 2];
 #pragma unroll
     for (int i = 0; i < Cfg::NQ; i++) {
-        w[2 * i] = q[i].x;
-        w[2 * i + 1] = q[i].y;
+        const uint2 q = buf[i * kReconNT];
+        w[2 * i] = q.x;
+        w[2 * i + 1] = q.y;
     }
     w[2 * Cfg::NQ] = 0;
     w[2 * Cfg::NQ + 1] = 0;
-    const int m = xs & 7;
     if (m >= 4) {
 #pragma unroll
         for (int i = 0; i < 2 * Cfg::NQ + 1; i++) w[i] = w[i + 1];
@@ -130,50 +170,88 @@ __device__ __forceinline__ void recon_hpass(const uint2 (&q)[ReconCfg<S>::NQ], i
 #pragma unroll
     for (int k = 0; k < Cfg::NP; k++) {
         const uint32_t B = __funnelshift_r(A[k], A[k + 1], 16);
-        h[k] = ((A[k] * fxc + B * fx + 0x00040004u) >> 3) & 0x1FFF1FFFu;
+        h[k] = (A[k] * fxc + B * fx + 0x00040004u) & 0xFFF8FFF8u;
     }
 }
 
-// Raw LR-row data for columns 8bx-1 .. 8bx+8: the aligned middle 8 values
-// (16 B of int16 or 8 B of u8, zero-extended) plus the two clamped edges.
-struct LrRaw {
-    uint4 mid;
-    int left, right;
-};
-__device__ __forceinline__ void recon_lr_load(const void *plane, bool is_u8, int row, int bx, int w, LrRaw &r) {
-    if (is_u8) {
-        const uint8_t *p = static_cast<const uint8_t *>(plane) + (size_t)row * w;
-        const uint2 q = __ldg(reinterpret_cast<const uint2 *>(p + 8 * bx));
-        r.mid = make_uint4(q.x, q.y, 0, 0);
-        r.left = p[max(8 * bx - 1, 0)];
-        r.right = p[min(8 * bx + 8, w - 1)];
-    } else {
-        const int16_t *p = static_cast<const int16_t *>(plane) + (size_t)row * w;
-        r.mid = __ldg(reinterpret_cast<const uint4 *>(p + 8 * bx));
-        r.left = p[max(8 * bx - 1, 0)];
-        r.right = p[min(8 * bx + 8, w - 1)];
-    }
+// LR rows of KEY frames / INTRA blocks (Z17) are staged per thread in the
+// thread's (otherwise unused) warp-window slots: LR row t as the three aligned
+// words of columns 8bx-8 .. 8bx+15 (clamped to the row; edges fixed on use).
+__device__ __forceinline__ void recon_lr_row_stage(const uint8_t *plane, int row, int bx, int w, uint2 *dst) {
+    const uint8_t *p = plane + (size_t)row * w;
+#pragma unroll
+    for (int k = 0; k < 3; k++) cp_async8(dst + k * kReconNT, p + min(max(8 * (bx - 1 + k), 0), w - 8));
 }
-__device__ __forceinline__ void recon_lr_unpack(const LrRaw &r, bool is_u8, int (&v)[10]) {
-    v[0] = r.left;
-    v[9] = r.right;
-    if (is_u8) {
+__device__ __forceinline__ void recon_lr_row_smem(const uint2 *src, bool left_in, bool right_in, int (&v)[10]) {
+    const uint2 l = src[0], q = src[kReconNT], r = src[2 * kReconNT];
 #pragma unroll
-        for (int i = 0; i < 4; i++) {
-            v[1 + i] = (r.mid.x >> (8 * i)) & 255;
-            v[5 + i] = (r.mid.y >> (8 * i)) & 255;
-        }
-    } else {
-        const uint32_t qq[4] = {r.mid.x, r.mid.y, r.mid.z, r.mid.w};
+    for (int i = 0; i < 4; i++) {
+        v[1 + i] = (q.x >> (8 * i)) & 255;
+        v[5 + i] = (q.y >> (8 * i)) & 255;
+    }
+    v[0] = left_in ? (int)(l.y >> 24) : v[1];
+    v[9] = right_in ? (int)(r.x & 255) : v[8];
+}
+
+// Residual-row values for columns 8bx-1 .. 8bx+8 from the staged tile row `p`
+// (p points at tile column 8 tx, i.e. LR column 8bx - 8).
+__device__ __forceinline__ void recon_res_row_smem(const int16_t *p, bool left_in, bool right_in, int (&v)[10]) {
+    const uint4 m = *reinterpret_cast<const uint4 *>(p + 8);
+    const uint32_t qq[4] = {m.x, m.y, m.z, m.w};
 #pragma unroll
-        for (int i = 0; i < 4; i++) {
-            v[1 + 2 * i] = (int)(int16_t)(qq[i] & 0xFFFFu);
-            v[2 + 2 * i] = (int)(int16_t)(qq[i] >> 16);
+    for (int i = 0; i < 4; i++) {
+        v[1 + 2 * i] = (int)(int16_t)(qq[i] & 0xFFFFu);
+        v[2 + 2 * i] = (int)qq[i] >> 16;
+    }
+    const int l = p[7], r = p[16];
+    v[0] = left_in ? l : v[1];
+    v[9] = right_in ? r : v[8];
+}
+
+// Compile-time O6 taps.  For an axis coordinate X = S*m + ph + i:
+//   u = 2X + 1 - S, x0 = m + floor((2(ph+i) + 1 - S) / 2S), w1 = round(128 rem / 2S).
+__host__ __device__ constexpr int fdiv(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+template <int S>
+__host__ __device__ constexpr int tap_d(int k) { return fdiv(2 * k + 1 - S, 2 * S); }
+template <int S>
+__host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S) - 2 * S * tap_d<S>(k)) + S) / (2 * S); }
+
+// up_s (O6) of one output row from the two LR rows a (top) and b (bottom) with
+// vertical weight WY: u[k] = pixel pair k as [r + 256 | r' + 256] (16-bit lanes).
+//   V[t] = (128 - WY) a[t] + WY b[t]            (exact, per LR column t)
+//   v    = 128 V[d] + w1 (V[d+1] - V[d])          (exact 2-D O6 sum, d = tap)
+//   s    = 4 (v + 8192 + 2^22) = 512 V[d] + 4 w1 (V[d+1] - V[d]) + KB
+// and r + 256 = s >> 16 (high half-word).
+template <int S, int WY>
+__device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[10], uint32_t (&u)[ReconCfg<S>::NP]) {
+    constexpr int BW = ReconCfg<S>::BW;
+    constexpr int KB = 4 * 8192 + 4 * (256 << 14);
+    int V[10], base[10];
+#pragma unroll
+    for (int t = 0; t < 10; t++) {
+        V[t] = WY ? (128 - WY) * a[t] + WY * b[t] : 128 * a[t];
+        base[t] = V[t] * 512 + KB;
+    }
+#pragma unroll
+    for (int k = 0; k < BW / 2; k++) {
+        uint32_t sv[2];
+#pragma unroll
+        for (int e = 0; e < 2; e++) {
+            const int i = 2 * k + e;
+            const int d = tap_d<S>(i) + 1, w1 = tap_w1<S>(i);
+            sv[e] = (uint32_t)(w1 ? base[d] + (4 * w1) * (V[d + 1] - V[d]) : base[d]);
         }
+        u[k] = prmt(sv[0], sv[1], 0x7632u);
     }
 }
 
-constexpr int kReconTX = 32, kReconTY = 4;
+template <int S>
+__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4]) {
+#pragma unroll
+    for (int q = 0; q < ReconCfg<S>::BW / 8; q++)
+        asm volatile("st.global.v2.b32 [%0], {%1, %2};" ::"l"(dst + 8 * q), "r"(o[2 * q]), "r"(o[2 * q + 1])
+                     : "memory");
+}
 
 __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
     uint32_t r;
@@ -186,199 +264,174 @@ __device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
     return r;
 }
 
-// Compile-time O6 taps.  For an axis coordinate X = S*m + ph + i:
-//   u = 2X + 1 - S, x0 = m + floor((2(ph+i) + 1 - S) / 2S), w1 = round(128 rem / 2S).
-__host__ __device__ constexpr int fdiv(int a, int b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
-template <int S>
-__host__ __device__ constexpr int tap_d(int k) { return fdiv(2 * k + 1 - S, 2 * S); }
-template <int S>
-__host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S) - 2 * S * tap_d<S>(k)) + S) / (2 * S); }
+// fd[s][f]: the frame step's pointers resolved once per chunk.
+__global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *is_anchor, uint8_t *const *hr_tab,
+                             const int16_t *gold, FrameDesc *fd) {
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= S * n) return;
+    const int sid = e / n, f = e % n;
+    const StreamDesc d = sd[sid];
+    const size_t lrp = (size_t)d.h * d.w;
+    FrameDesc o;
+    o.lr_f = d.lr + (size_t)f * 3 * lrp;
+    o.res_f = d.res + (size_t)f * 3 * lrp;
+    o.mv_f = d.mv + (size_t)f * (d.h / 8) * (d.w / 8);
+    o.out = hr_tab[d.hr_base + f];
+    o.ref_last = f > 0 ? hr_tab[d.hr_base + f - 1] : d.hr_last;
+    const int g = gold[(size_t)sid * (n + 1) + f];
+    o.ref_gold = g >= 0 ? hr_tab[d.hr_base + g] : d.hr_golden;
+    o.w = d.w;
+    o.h = d.h;
+    o.s = (int16_t)d.s;
+    o.anchor = is_anchor[e] ? 1 : 0;
+    o.key = d.type[f] == NS_KEY;
+    o.pad = 0;
+    fd[e] = o;
+}
 
-// All three planes of one thread's 8s x 8 tile; PH = Y0 mod S (compile time).
+cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
+                              uint8_t *const *d_hr_table, const int16_t *gold_idx, FrameDesc *fd, cudaStream_t st) {
+    KScope ks(F_RECON, st);
+    k_frame_desc<<<(S * n + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, gold_idx, fd);
+    return cudaGetLastError();
+}
+
 template <int S>
-__device__ __forceinline__ void recon_planes(const StreamDesc &d, bool use_lr, const uint8_t *ref, const uint8_t *lr_f,
-                                             const int16_t *res_f, uint8_t *out, size_t lrp, size_t hrp, int H, int W,
-                                             int bx, int X0, int Y0, int Y0m, int xs, int iy0, bool interior,
-                                             uint32_t fxc, uint32_t fxp, uint32_t fyc, uint32_t fyp) {
+__global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
+    k_recon_step(const FrameDesc *fdesc, int n, int f) {
     using Cfg = ReconCfg<S>;
-    constexpr int BW = Cfg::BW, NP = Cfg::NP;
-    constexpr int RPT = Cfg::RPT;
-    constexpr int DMIN = tap_d<S>(0), DMAX = tap_d<S>(S - 1) + 1;
-    constexpr int NLR = DMAX - DMIN + 1 + (RPT / S - 1);  // LR rows: one period's window + slides
-    static_assert(RPT % S == 0, "row groups are whole periods");
-    constexpr int NT = kReconTX * kReconTY;
-    extern __shared__ __align__(16) uint2 rsm[];  // [2 planes][9 rows][NQ words][NT threads]
+    using Sm = ReconSmem<S>;
+    constexpr int NP = Cfg::NP, RPT = Cfg::RPT, NQ = Cfg::NQ;
+    const int sid = blockIdx.z;
+    const FrameDesc fd = fdesc[(size_t)sid * n + f];
+    if (fd.anchor || fd.s != S) return;                 // CTA-uniform: anchors already hold SR bytes
+    const int w = fd.w, h = fd.h, H = h * S, W = w * S;
+    const int bx0 = blockIdx.x * kReconTX;              // first LR block column of the CTA
+    const int Y0c = blockIdx.y * kReconTY * RPT;        // first HR row of the CTA
+    if (8 * bx0 >= w || Y0c >= H) return;               // CTA-uniform
     const int tid = threadIdx.y * kReconTX + threadIdx.x;
+    const size_t lrp = (size_t)h * w, hrp = (size_t)H * W;
+
+    extern __shared__ __align__(16) uint8_t recon_sm[];
+    uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [2][RPT+1][NQ][NT] warp windows
+    int16_t *tres = reinterpret_cast<int16_t *>(recon_sm + Sm::REF);   // [3][RROWS][kResCols] residual tile
+
+    // cooperative residual tile: tile row r <-> LR row Y0c/S - 1 + r (clamped, Z16),
+    // tile column 8q+e <-> LR column 8 bx0 - 8 + 8q + e (chunks outside the row are
+    // never read: the edge columns are clamped on use)
+    if (!fd.key) {
+        constexpr int CH = kResCols / 8;
+        for (int e = tid; e < 3 * Sm::RROWS * CH; e += kReconNT) {
+            const int c = e / (Sm::RROWS * CH), rr = (e / CH) % Sm::RROWS, q = e % CH;
+            const int col = 8 * bx0 - 8 + 8 * q;
+            if (col < 0 || col >= w) continue;
+            const int row = min(max(Y0c / S - 1 + rr, 0), h - 1);
+            cp_async16(tres + ((size_t)c * Sm::RROWS + rr) * kResCols + 8 * q,
+                       fd.res_f + c * lrp + (size_t)row * w + col);
+        }
+    }
+
+    const int bx = bx0 + threadIdx.x;
+    const int Y0 = Y0c + threadIdx.y * RPT;
+    const bool valid = 8 * bx < w && Y0 < H;
+    const int X0 = bx * Cfg::BW;
+    ns_block_mv mv{};
+    if (valid) mv = fd.mv_f[(size_t)(Y0 / Cfg::BW) * (w / 8) + bx];
+    // KEY frames and INTRA blocks: up_s(LR[f]) (Z17) through the same arithmetic,
+    // with a zero prediction (all warp weights 0) and LR rows instead of residual rows
+    const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;
+    const uint8_t *ref = mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last;
+    // warp geometry (O7): m = s * mv in 1/8 HR pel
+    const int mx = S * mv.mvx, my = S * mv.mvy;
+    const int xs = X0 + (mx >> 3);
+    const uint32_t fx = use_lr ? 0u : (uint32_t)(mx & 7), fy = use_lr ? 0u : (uint32_t)(my & 7);
+    const uint32_t fxc = use_lr ? 0u : 8u - fx, fyc = use_lr ? 0u : 8u - fy;  // lanes x SCALAR: no cross-lane terms
+    const int iy0 = Y0 + (my >> 3);
+    const bool interior = xs >= 0 && (xs & ~7) + 8 * NQ <= W;
     auto stage = [&](int c) {
-        if (use_lr) return;
+        if (!valid) return;
+        if (use_lr) {
+            uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
+#pragma unroll
+            for (int t = 0; t < Cfg::PER + 2; t++)
+                recon_lr_row_stage(fd.lr_f + c * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
+                                   buf + 3 * t * kReconNT);
+            return;
+        }
         const uint8_t *P = ref + c * hrp;
-        uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * Cfg::NQ * NT + tid;
+        uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
 #pragma unroll
         for (int j = 0; j <= RPT; j++) {
             const int r = min(max(iy0 + j, 0), H - 1);
-            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior, buf + j * Cfg::NQ * NT, NT);
+            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior, buf + j * NQ * kReconNT, kReconNT);
         }
     };
     stage(0);
     asm volatile("cp.async.commit_group;" ::: "memory");
+    const bool left_in = bx > 0, right_in = 8 * bx + 8 < w;
+    const int m = xs & 7;
+    uint8_t *outp = fd.out + (size_t)Y0 * W + X0;
+
 #pragma unroll 1
     for (int c = 0; c < 3; c++) {
         if (c + 1 < 3) stage(c + 1);
         asm volatile("cp.async.commit_group;" ::: "memory");
-        const void *src = use_lr ? static_cast<const void *>(lr_f + c * lrp) : static_cast<const void *>(res_f + c * lrp);
-        int lv[NLR][10];
-#pragma unroll
-        for (int t = 0; t < NLR; t++) {
-            LrRaw raw;
-            recon_lr_load(src, use_lr, min(max(Y0m + DMIN + t, 0), d.h - 1), bx, d.w, raw);
-            recon_lr_unpack(raw, use_lr, lv[t]);
-        }
-        asm volatile("cp.async.wait_group 1;" ::: "memory");  // this plane's windows have landed
-        const uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * Cfg::NQ * NT + tid;
-        auto row = [&](int j, uint2 (&q)[Cfg::NQ]) {
-#pragma unroll
-            for (int i = 0; i < Cfg::NQ; i++) q[i] = buf[(j * Cfg::NQ + i) * NT];
-        };
-        uint32_t hprev[NP], hcur[NP];
-        if (!use_lr) {
-            uint2 q[Cfg::NQ];
-            row(0, q);
-            recon_hpass<S>(q, xs, fxc, fxp, hprev);
-        }
-#pragma unroll 1
-        for (int it = 0; it < RPT / S; it++) {
-#pragma unroll
-            for (int jj = 0; jj < S; jj++) {  // one period of the vertical O6 taps
-                const int j = it * S + jj;
-                uint32_t pred[NP];
+        asm volatile("cp.async.wait_group 1;" ::: "memory");  // plane c's windows (and at c = 0 the tile) landed
+        if (c == 0) __syncthreads();                            // the residual tile is cooperative
+        if (!valid) continue;
+        const uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
+        if (!interior && !use_lr) recon_fix_edges<S>(const_cast<uint2 *>(buf), xs & ~7, W);
+        // (use_lr threads run the warp pass over their LR words: every weight is 0, so pred = 0)
+        const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
+        uint8_t *outc = outp + c * hrp;
+        uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
+        recon_hpass8<S>(buf, m, fxc, fx, hA);
+        int rv[3][10];
+        auto one = [&](auto jc) {
+            constexpr int j = decltype(jc)::value, it = j / S, jj = j % S;
+            constexpr int ta = tap_d<S>(jj) + 1;
+            if constexpr (jj == 0) {  // a new period: LR rows it .. it + 2 of this thread
                 if (!use_lr) {
-                    uint2 q[Cfg::NQ];
-                    row(j + 1, q);
-                    recon_hpass<S>(q, xs, fxc, fxp, hcur);
 #pragma unroll
-                    for (int k = 0; k < NP; k++) {
-                        pred[k] = ((hprev[k] * fyc + hcur[k] * fyp + 0x00040004u) >> 3) & 0x1FFF1FFFu;
-                        hprev[k] = hcur[k];
-                    }
+                    for (int t = 0; t < 3; t++) recon_res_row_smem(tp + (it + t) * kResCols, left_in, right_in, rv[t]);
                 } else {
 #pragma unroll
-                    for (int k = 0; k < NP; k++) pred[k] = 0;
+                    for (int t = 0; t < 3; t++) recon_lr_row_smem(buf + 3 * (it + t) * kReconNT, left_in, right_in, rv[t]);
                 }
-                // up_s of the residual (or LR) plane at row Y0 + j (O6), compile-time taps;
-                // lv[0] holds LR row Y0/S + DMIN + it (the window slides one LR row per period)
-                const int ta = tap_d<S>(jj) - DMIN;
-                const int wy = tap_w1<S>(jj);
-                // per LR column t: V = (128-wy) a + wy b (vertical, exact); the
-                // horizontal tap of pixel i is 128 V[d] + w1 (V[d+1] - V[d]).  Scaled
-                // by 4 with the rounding constant and the +256 lane bias folded in, the
-                // value r + 256 lands in the high half-word: one IMAD per pixel and one
-                // PRMT per pixel pair.
-                int base[10], dlt[9];
+            }
+            uint32_t(&hp)[NP] = (j & 1) ? hB : hA;
+            uint32_t(&hc)[NP] = (j & 1) ? hA : hB;
+            recon_hpass8<S>(buf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
+            uint32_t u[NP], x[NP], o[Cfg::BW / 4];
+            recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);
 #pragma unroll
-                for (int t = 0; t < 10; t++) {
-                    const int V = (128 - wy) * lv[ta][t] + wy * lv[ta + 1][t];
-                    base[t] = V * 512 + 4 * (8192 + (256 << 14));
-                }
-#pragma unroll
-                for (int t = 0; t < 9; t++) dlt[t] = base[t + 1] - base[t];
-                uint32_t o[BW / 4];
-#pragma unroll
-                for (int qd = 0; qd < BW / 4; qd++) {
-                    uint32_t pr[2];
-#pragma unroll
-                    for (int hh = 0; hh < 2; hh++) {
-                        const int i0 = 4 * qd + 2 * hh;
-                        const int d0 = tap_d<S>(i0) + 1, d1 = tap_d<S>(i0 + 1) + 1;
-                        const int w0 = tap_w1<S>(i0), w1 = tap_w1<S>(i0 + 1);
-                        // (base + w1 * dlt / 128): dlt is a multiple of 512, so w1*dlt/128 = w1*(dlt/128) exactly
-                        const uint32_t s0 = (uint32_t)(base[d0] + (w0 ? w0 * (dlt[d0] >> 7) : 0));
-                        const uint32_t s1 = (uint32_t)(base[d1] + (w1 ? w1 * (dlt[d1] >> 7) : 0));
-                        uint32_t x = prmt(s0, s1, 0x7632u);  // [r0 + 256, r1 + 256]
-                        x += pred[i0 >> 1];                   // in [1, 766] per lane
-                        pr[hh] = vmin_u16x2(vmax_u16x2(x, 0x01000100u), 0x01FF01FFu);  // clamp to [256, 511]
-                    }
-                    o[qd] = prmt(pr[0], pr[1], 0x6420u);  // low bytes = clamped value (x - 256)
-                }
-                uint2 *dst = reinterpret_cast<uint2 *>(out + c * hrp + (size_t)(Y0 + j) * W + X0);
-#pragma unroll
-                for (int qd = 0; qd < BW / 8; qd++) dst[qd] = make_uint2(o[2 * qd], o[2 * qd + 1]);
+            for (int k = 0; k < NP; k++) {
+                const uint32_t X = u[k] * 64u + hc[k] * fy + hp[k] * fyc + 0x00200020u;
+                x[k] = vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu) >> 6;
             }
 #pragma unroll
-            for (int t = 0; t + 1 < NLR; t++)
-#pragma unroll
-                for (int e = 0; e < 10; e++) lv[t][e] = lv[t + 1][e];
-        }
+            for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6420u);
+            recon_store_row<S>(outc + (size_t)j * W, o);
+        };
+        static_for<RPT>(one);
     }
 }
 
 template <int S>
-__global__ void __launch_bounds__(kReconTX *kReconTY, ReconCfg<S>::MINB)
-    k_recon_step(const StreamDesc *sd, int n, int f, const uint8_t *is_anchor, uint8_t *const *hr_tab,
-                 const int16_t *gold) {
-    using Cfg = ReconCfg<S>;
-    constexpr int BW = Cfg::BW, NP = Cfg::NP;
-    const int sid = blockIdx.z;
-    if (is_anchor[(size_t)sid * n + f]) return;
-    const StreamDesc d = sd[sid];
-    if (d.s != S) return;
-    const int H = d.h * S, W = d.w * S;
-    const int bx = blockIdx.x * kReconTX + threadIdx.x;  // LR block column
-    const int rg = blockIdx.y * kReconTY + threadIdx.y;  // group of RPT HR rows
-    const int X0 = bx * BW, Y0 = rg * Cfg::RPT;
-    if (X0 >= W || Y0 >= H) return;
-    const int bw = d.w / 8;
-    const ns_block_mv mv = d.mv[(size_t)f * (d.h / 8) * bw + (size_t)(Y0 / BW) * bw + bx];
-    const bool key = d.type[f] == NS_KEY;
-    const bool use_lr = key || mv.ref == NS_REF_INTRA;
-    uint8_t *out = hr_tab[d.hr_base + f];
-    const size_t lrp = (size_t)d.h * d.w, hrp = (size_t)H * W;
-    const uint8_t *ref = nullptr;
-    if (!use_lr) {
-        if (mv.ref == NS_REF_GOLDEN) {
-            const int g = gold[(size_t)sid * (n + 1) + f];
-            ref = g >= 0 ? hr_tab[d.hr_base + g] : d.hr_golden;
-        } else {
-            ref = f > 0 ? hr_tab[d.hr_base + f - 1] : d.hr_last;
-        }
-    }
-    // warp geometry (O7): m = s * mv in 1/8 HR pel
-    const int mx = S * mv.mvx, my = S * mv.mvy;
-    const int xs = X0 + (mx >> 3);
-    const uint32_t fx = (uint32_t)(mx & 7), fy = (uint32_t)(my & 7);
-    // packed 2 x 16-bit arithmetic multiplies by a SCALAR (no cross-lane terms)
-    const uint32_t fxp = fx, fyp = fy, fxc = 8u - fx, fyc = 8u - fy;
-    const int iy0 = Y0 + (my >> 3);
-    // every aligned word of the window inside the row -> unconditional cp.async
-    const bool interior = xs >= 0 && (xs & ~7) + 8 * Cfg::NQ <= W;
-    const uint8_t *lr_f = d.lr + (size_t)f * 3 * lrp;
-    const int16_t *res_f = d.res + (size_t)f * 3 * lrp;
-
-    recon_planes<S>(d, use_lr, ref, lr_f, res_f, out, lrp, hrp, H, W, bx, X0, Y0, Y0 / S, xs, iy0, interior, fxc,
-                    fxp, fyc, fyp);
-}
-
-template <int S>
-static size_t recon_smem() {
-    return (size_t)2 * (ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconTX * kReconTY * sizeof(uint2);
-}
-
-template <int S>
-static void recon_launch(dim3 g, cudaStream_t st, const StreamDesc *d_sd, int n, int f, const uint8_t *is_anchor,
-                         uint8_t *const *hr, const int16_t *gold) {
+static void recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f) {
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)recon_smem<S>());
+        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ReconSmem<S>::BYTES);
         // all of the unified L1/shared array as shared memory, so MINB CTAs fit
         cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributePreferredSharedMemoryCarveout,
                              (int)cudaSharedmemCarveoutMaxShared);
         attr = true;
     }
-    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), recon_smem<S>(), st>>>(d_sd, n, f, is_anchor, hr, gold);
+    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f);
 }
 
-cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const int *max_lr_w,
-                              const int *max_lr_h, const uint8_t *is_anchor, uint8_t *const *d_hr_table,
-                              const int16_t *gold_idx, cudaStream_t st) {
+cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
+                              cudaStream_t st) {
     int nl = 0;
     for (int s = 2; s <= 4; s++) nl += max_lr_w[s] > 0;
     KScope ks(F_RECON, st, nl);
@@ -387,11 +440,9 @@ cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const
         const int nbx = max_lr_w[s] / 8;          // LR block columns
         const int nrg = max_lr_h[s] * s / (s == 3 ? 6 : 8);  // groups of RPT HR rows
         dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
-        dim3 b(kReconTX, kReconTY);
-        (void)b;
-        if (s == 2) recon_launch<2>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
-        if (s == 3) recon_launch<3>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
-        if (s == 4) recon_launch<4>(g, st, d_sd, n, f, is_anchor, d_hr_table, gold_idx);
+        if (s == 2) recon_launch<2>(g, st, fd, n, f);
+        if (s == 3) recon_launch<3>(g, st, fd, n, f);
+        if (s == 4) recon_launch<4>(g, st, fd, n, f);
     }
     return cudaGetLastError();
 }

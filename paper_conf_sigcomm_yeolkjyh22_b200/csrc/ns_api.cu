@@ -171,6 +171,7 @@ struct ns_ctx {
     int32_t *rank, *order, *grank, *pos_stream, *cut, *job_count;
     uint8_t *anchor;
     int16_t *gold;
+    FrameDesc *fdesc;
     SrJob *jobs;
     uint16_t *blob_stage;  // device staging for host weight blobs
     size_t blob_stage_elems;
@@ -231,7 +232,7 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     NS_CUDA(cudaSetDevice(device));
     ns_ctx *c = new ns_ctx();
     c->device = device;
-    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2) +
+    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2 + sizeof(FrameDesc)) +
                          (size_t)kMaxJobs * (sizeof(SrJob) + sizeof(uint8_t *) + sizeof(uint32_t)) +
                          kStageSlots * kStageBytes + (64u << 20) + 64 * 1024;
     if (pool_bytes < fixed + (64u << 20)) {
@@ -253,6 +254,7 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     c->pos_stream = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
     c->anchor = (uint8_t *)pool_take(c, kMaxSN);
     c->gold = (int16_t *)pool_take(c, sizeof(int16_t) * (kMaxSN + 4096));
+    c->fdesc = (FrameDesc *)pool_take(c, sizeof(FrameDesc) * kMaxSN);
     c->cut = (int32_t *)pool_take(c, 256);
     c->job_count = (int32_t *)pool_take(c, sizeof(int32_t) * 4096);
     c->jobs = (SrJob *)pool_take(c, sizeof(SrJob) * kMaxJobs);
@@ -621,7 +623,8 @@ static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch,
         maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
     }
     NS_CUDA(launch_golden_index(g.d_sd, S, n, c->gold, st));
-    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(g.d_sd, S, n, f, mw, mh, is_anchor, g.d_hr, c->gold, st));
+    NS_CUDA(launch_frame_desc(g.d_sd, S, n, is_anchor, g.d_hr, c->gold, c->fdesc, st));
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, S, n, f, mw, mh, st));
     NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, maxhr, st));
     return NS_OK;
 }

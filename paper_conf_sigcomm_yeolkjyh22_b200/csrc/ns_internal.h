@@ -30,6 +30,23 @@ struct StreamDesc {
     int32_t use_res_size;
 };
 
+// Per (stream, frame) reconstruction step descriptor, resolved once per chunk
+// after selection (k_frame_desc): a recon CTA reads its 64 B and can start
+// staging at once, instead of walking sd -> type / is_anchor / gold -> hr table.
+struct __align__(16) FrameDesc {
+    const uint8_t *lr_f;       // LR[f] [3][h][w]
+    const int16_t *res_f;      // res[f] [3][h][w]
+    const ns_block_mv *mv_f;   // mv[f] [h/8][w/8]
+    uint8_t *out;              // HR[f]
+    const uint8_t *ref_last;   // HR[f-1] or hr_last
+    const uint8_t *ref_gold;   // HR of the latest KEY/ALTREF < f, or hr_golden
+    int32_t w, h;              // LR size
+    int16_t s;                 // scale
+    uint8_t anchor, key;       // is_anchor[f], type[f] == KEY
+    int32_t pad;
+};
+static_assert(sizeof(FrameDesc) == 64, "FrameDesc is one 64-B record");
+
 // One anchor-SR job (device).
 struct SrJob {
     const uint8_t *lr;     // [3][h][w]
@@ -92,9 +109,11 @@ cudaError_t launch_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, co
                              size_t max_len, cudaStream_t st);
 cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st);
 // max_lr_w / max_lr_h: [5] indexed by scale (0 = no stream of that scale)
-cudaError_t launch_recon_step(const StreamDesc *d_sd, int S, int n, int f, const int *max_lr_w,
-                              const int *max_lr_h, const uint8_t *is_anchor, uint8_t *const *d_hr_table,
-                              const int16_t *gold_idx, cudaStream_t st);
+// fd[s][f] for all streams and frames (after launch_golden_index)
+cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
+                              uint8_t *const *d_hr_table, const int16_t *gold_idx, FrameDesc *fd, cudaStream_t st);
+cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
+                              cudaStream_t st);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
