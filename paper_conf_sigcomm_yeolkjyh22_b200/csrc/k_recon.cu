@@ -78,7 +78,7 @@ struct ReconCfg {
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
     static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
     static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
-    static constexpr int MINB = (S == 3) ? 3 : 2;  // resident CTAs per SM (shared memory)
+    static constexpr int MINB = (S == 3) ? 4 : 3;  // resident CTAs per SM (registers)
 };
 constexpr int kReconTX = 32, kReconTY = 4;
 constexpr int kReconNT = kReconTX * kReconTY;
@@ -87,7 +87,7 @@ constexpr int kResCols = 8 * kReconTX + 16;        // residual tile columns (one
 template <int S>
 struct ReconSmem {
     static constexpr int RROWS = kReconTY * ReconCfg<S>::PER + 2;      // residual tile LR rows
-    static constexpr size_t REF = (size_t)2 * (ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconNT * 8;
+    static constexpr size_t REF = (size_t)(ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconNT * 8;
     static constexpr size_t RES = (size_t)3 * RROWS * kResCols * 2;
     static constexpr size_t BYTES = REF + RES;
 };
@@ -109,7 +109,7 @@ __device__ __forceinline__ void cp_async16(void *dst, const void *src) {
 // across the CTA's threads: conflict-free reads).  W and the word base are
 // multiples of 8, so every word lies wholly inside the row or wholly outside
 // it; an outside word stages the row's first / last word instead, and
-// recon_fix_edges replicates its edge pixel (Z16) after the copy lands: every
+// recon_fix_row replicates its edge pixel (Z16) after the copy lands: every
 // global read stays an asynchronous copy, and none reads past the row.
 template <int S>
 __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int W, bool interior, uint2 *dst,
@@ -122,19 +122,19 @@ __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int 
         cp_async8(dst + i * stride, row + st);
     }
 }
-// After the copies of a non-interior window have landed: replicate the edge
-// pixel into the staged words that lie outside the row (first word at xb).
+// After the copies of one non-interior window row have landed: replicate the
+// edge pixel into the staged words that lie outside the row (first word at xb).
 template <int S>
-__device__ __noinline__ void recon_fix_edges(uint2 *buf, int xb, int W) {
-    using Cfg = ReconCfg<S>;
-#pragma unroll 1
-    for (int i = 0; i < Cfg::NQ; i++) {
+__device__ __forceinline__ void recon_fix_row(uint2 *row, int xb, int W) {
+#pragma unroll
+    for (int i = 0; i < ReconCfg<S>::NQ; i++) {
         const int st = xb + 8 * i;
-        if (st >= 0 && st < W) continue;
-#pragma unroll 1
-        for (int j = 0; j <= Cfg::RPT; j++) {
-            uint2 *q = buf + (j * Cfg::NQ + i) * kReconNT;
-            const uint32_t v = st < 0 ? prmt(q->x, 0u, 0x0000u) : prmt(q->y, 0u, 0x3333u);
+        uint2 *q = row + i * kReconNT;
+        if (st < 0) {
+            const uint32_t v = prmt(q->x, 0u, 0x0000u);
+            *q = make_uint2(v, v);
+        } else if (st >= W) {
+            const uint32_t v = prmt(q->y, 0u, 0x3333u);
             *q = make_uint2(v, v);
         }
     }
@@ -175,22 +175,28 @@ __device__ __forceinline__ void recon_hpass8(const uint2 *buf, int m, uint32_t f
 }
 
 // LR rows of KEY frames / INTRA blocks (Z17) are staged per thread in the
-// thread's (otherwise unused) warp-window slots: LR row t as the three aligned
-// words of columns 8bx-8 .. 8bx+15 (clamped to the row; edges fixed on use).
+// thread's (otherwise unused) warp-window slots, two per LR row: the aligned
+// word of columns 8bx .. 8bx+7, and [columns 8bx-4 .. 8bx-1 | 8bx+8 .. 8bx+11]
+// (clamped to the row; the edge columns are replaced on use when outside, Z16).
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
 __device__ __forceinline__ void recon_lr_row_stage(const uint8_t *plane, int row, int bx, int w, uint2 *dst) {
     const uint8_t *p = plane + (size_t)row * w;
-#pragma unroll
-    for (int k = 0; k < 3; k++) cp_async8(dst + k * kReconNT, p + min(max(8 * (bx - 1 + k), 0), w - 8));
+    cp_async8(dst, p + 8 * bx);
+    uint32_t *e = reinterpret_cast<uint32_t *>(dst + kReconNT);
+    cp_async4(e, p + max(8 * bx - 4, 0));
+    cp_async4(e + 1, p + min(8 * bx + 8, w - 4));
 }
 __device__ __forceinline__ void recon_lr_row_smem(const uint2 *src, bool left_in, bool right_in, int (&v)[10]) {
-    const uint2 l = src[0], q = src[kReconNT], r = src[2 * kReconNT];
+    const uint2 q = src[0], e = src[kReconNT];
 #pragma unroll
     for (int i = 0; i < 4; i++) {
         v[1 + i] = (q.x >> (8 * i)) & 255;
         v[5 + i] = (q.y >> (8 * i)) & 255;
     }
-    v[0] = left_in ? (int)(l.y >> 24) : v[1];
-    v[9] = right_in ? (int)(r.x & 255) : v[8];
+    v[0] = left_in ? (int)(e.x >> 24) : v[1];
+    v[9] = right_in ? (int)(e.y & 255) : v[8];
 }
 
 // Residual-row values for columns 8bx-1 .. 8bx+8 from the staged tile row `p`
@@ -253,6 +259,11 @@ __device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o
                      : "memory");
 }
 
+__device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t r;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+    return r;
+}
 __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
     uint32_t r;
     asm("max.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
@@ -313,7 +324,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     const size_t lrp = (size_t)h * w, hrp = (size_t)H * W;
 
     extern __shared__ __align__(16) uint8_t recon_sm[];
-    uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [2][RPT+1][NQ][NT] warp windows
+    uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [RPT+1][NQ][NT] warp windows
     int16_t *tres = reinterpret_cast<int16_t *>(recon_sm + Sm::REF);   // [3][RROWS][kResCols] residual tile
 
     // cooperative residual tile: tile row r <-> LR row Y0c/S - 1 + r (clamped, Z16),
@@ -348,44 +359,48 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     const uint32_t fxc = use_lr ? 0u : 8u - fx, fyc = use_lr ? 0u : 8u - fy;  // lanes x SCALAR: no cross-lane terms
     const int iy0 = Y0 + (my >> 3);
     const bool interior = xs >= 0 && (xs & ~7) + 8 * NQ <= W;
-    auto stage = [&](int c) {
-        if (!valid) return;
+    // Reference windows live in ONE buffer of RPT+1 rows: row r of plane c+1 is
+    // staged right after plane c's warp pass has read row r, one commit group per
+    // row, so before the pass over row r there are always exactly RPT groups newer
+    // than row r's (wait_group RPT).  LR rows (use_lr threads) alternate between
+    // two small slot sets and ride in the group of row 0.
+    uint2 *wbuf = rsm + tid;
+    auto stage_row = [&](int c, int r) {
+        if (!valid || c >= 3) return;
         if (use_lr) {
-            uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
+            if (r == 0) {
 #pragma unroll
-            for (int t = 0; t < Cfg::PER + 2; t++)
-                recon_lr_row_stage(fd.lr_f + c * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
-                                   buf + 3 * t * kReconNT);
+                for (int t = 0; t < Cfg::PER + 2; t++)
+                    recon_lr_row_stage(fd.lr_f + c * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
+                                       wbuf + ((c & 1) * (Cfg::PER + 2) + t) * 2 * kReconNT);
+            }
             return;
         }
-        const uint8_t *P = ref + c * hrp;
-        uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
-#pragma unroll
-        for (int j = 0; j <= RPT; j++) {
-            const int r = min(max(iy0 + j, 0), H - 1);
-            recon_row_stage<S>(P + (size_t)r * W, xs, W, interior, buf + j * NQ * kReconNT, kReconNT);
-        }
+        const int rr = min(max(iy0 + r, 0), H - 1);
+        recon_row_stage<S>(ref + c * hrp + (size_t)rr * W, xs, W, interior, wbuf + r * NQ * kReconNT, kReconNT);
     };
-    stage(0);
-    asm volatile("cp.async.commit_group;" ::: "memory");
+    for (int r = 0; r <= RPT; r++) {
+        stage_row(0, r);
+        asm volatile("cp.async.commit_group;" ::: "memory");   // the residual tile rides in row 0's group
+    }
     const bool left_in = bx > 0, right_in = 8 * bx + 8 < w;
     const int m = xs & 7;
+    const bool fix = valid && !interior && !use_lr;
     uint8_t *outp = fd.out + (size_t)Y0 * W + X0;
 
 #pragma unroll 1
     for (int c = 0; c < 3; c++) {
-        if (c + 1 < 3) stage(c + 1);
-        asm volatile("cp.async.commit_group;" ::: "memory");
-        asm volatile("cp.async.wait_group 1;" ::: "memory");  // plane c's windows (and at c = 0 the tile) landed
+        asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
         if (c == 0) __syncthreads();                            // the residual tile is cooperative
-        if (!valid) continue;
-        const uint2 *buf = rsm + (size_t)(c & 1) * (RPT + 1) * NQ * kReconNT + tid;
-        if (!interior && !use_lr) recon_fix_edges<S>(const_cast<uint2 *>(buf), xs & ~7, W);
-        // (use_lr threads run the warp pass over their LR words: every weight is 0, so pred = 0)
+        // (use_lr threads run the warp pass over whatever the slots hold: every weight is 0, so pred = 0)
         const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
+        const uint2 *lrb = wbuf + (c & 1) * (Cfg::PER + 2) * 2 * kReconNT;
         uint8_t *outc = outp + c * hrp;
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
-        recon_hpass8<S>(buf, m, fxc, fx, hA);
+        if (fix) recon_fix_row<S>(wbuf, xs & ~7, W);
+        recon_hpass8<S>(wbuf, m, fxc, fx, hA);
+        stage_row(c + 1, 0);
+        asm volatile("cp.async.commit_group;" ::: "memory");
         int rv[3][10];
         auto one = [&](auto jc) {
             constexpr int j = decltype(jc)::value, it = j / S, jj = j % S;
@@ -396,22 +411,26 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                     for (int t = 0; t < 3; t++) recon_res_row_smem(tp + (it + t) * kResCols, left_in, right_in, rv[t]);
                 } else {
 #pragma unroll
-                    for (int t = 0; t < 3; t++) recon_lr_row_smem(buf + 3 * (it + t) * kReconNT, left_in, right_in, rv[t]);
+                    for (int t = 0; t < 3; t++) recon_lr_row_smem(lrb + (it + t) * 2 * kReconNT, left_in, right_in, rv[t]);
                 }
             }
             uint32_t(&hp)[NP] = (j & 1) ? hB : hA;
             uint32_t(&hc)[NP] = (j & 1) ? hA : hB;
-            recon_hpass8<S>(buf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
+            asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
+            if (fix) recon_fix_row<S>(wbuf + (j + 1) * NQ * kReconNT, xs & ~7, W);
+            recon_hpass8<S>(wbuf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
+            stage_row(c + 1, j + 1);
+            asm volatile("cp.async.commit_group;" ::: "memory");
             uint32_t u[NP], x[NP], o[Cfg::BW / 4];
             recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);
 #pragma unroll
             for (int k = 0; k < NP; k++) {
-                const uint32_t X = u[k] * 64u + hc[k] * fy + hp[k] * fyc + 0x00200020u;
+                const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], 64u, 0x00200020u)));
                 x[k] = vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu) >> 6;
             }
 #pragma unroll
             for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6420u);
-            recon_store_row<S>(outc + (size_t)j * W, o);
+            if (valid) recon_store_row<S>(outc + (size_t)j * W, o);
         };
         static_for<RPT>(one);
     }
