@@ -401,38 +401,44 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
         recon_hpass8<S>(wbuf, m, fxc, fx, hA);
         stage_row(c + 1, 0);
         asm volatile("cp.async.commit_group;" ::: "memory");
-        int rv[3][10];
-        auto one = [&](auto jc) {
-            constexpr int j = decltype(jc)::value, it = j / S, jj = j % S;
-            constexpr int ta = tap_d<S>(jj) + 1;
-            if constexpr (jj == 0) {  // a new period: LR rows it .. it + 2 of this thread
-                if (!use_lr) {
+#pragma unroll 1
+        for (int it = 0; it < Cfg::PER; it++) {
+            int rv[3][10];  // LR rows it .. it + 2 of this thread
+            if (!use_lr) {
 #pragma unroll
-                    for (int t = 0; t < 3; t++) recon_res_row_smem(tp + (it + t) * kResCols, left_in, right_in, rv[t]);
-                } else {
+                for (int t = 0; t < 3; t++) recon_res_row_smem(tp + (it + t) * kResCols, left_in, right_in, rv[t]);
+            } else {
 #pragma unroll
-                    for (int t = 0; t < 3; t++) recon_lr_row_smem(lrb + (it + t) * 2 * kReconNT, left_in, right_in, rv[t]);
+                for (int t = 0; t < 3; t++) recon_lr_row_smem(lrb + (it + t) * 2 * kReconNT, left_in, right_in, rv[t]);
+            }
+            auto one = [&](auto jc) {
+                constexpr int jj = decltype(jc)::value;
+                constexpr int ta = tap_d<S>(jj) + 1;
+                const int j = it * S + jj;
+                uint32_t(&hp)[NP] = (jj & 1) ? hB : hA;
+                uint32_t(&hc)[NP] = (jj & 1) ? hA : hB;
+                asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
+                if (fix) recon_fix_row<S>(wbuf + (j + 1) * NQ * kReconNT, xs & ~7, W);
+                recon_hpass8<S>(wbuf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
+                stage_row(c + 1, j + 1);
+                asm volatile("cp.async.commit_group;" ::: "memory");
+                uint32_t u[NP], x[NP], o[Cfg::BW / 4];
+                recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);
+#pragma unroll
+                for (int k = 0; k < NP; k++) {
+                    const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], 64u, 0x00200020u)));
+                    x[k] = vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu) >> 6;
                 }
-            }
-            uint32_t(&hp)[NP] = (j & 1) ? hB : hA;
-            uint32_t(&hc)[NP] = (j & 1) ? hA : hB;
-            asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
-            if (fix) recon_fix_row<S>(wbuf + (j + 1) * NQ * kReconNT, xs & ~7, W);
-            recon_hpass8<S>(wbuf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
-            stage_row(c + 1, j + 1);
-            asm volatile("cp.async.commit_group;" ::: "memory");
-            uint32_t u[NP], x[NP], o[Cfg::BW / 4];
-            recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);
 #pragma unroll
-            for (int k = 0; k < NP; k++) {
-                const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], 64u, 0x00200020u)));
-                x[k] = vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu) >> 6;
-            }
+                for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6420u);
+                if (valid) recon_store_row<S>(outc + (size_t)j * W, o);
+            };
+            static_for<S>(one);
+            if constexpr (S & 1) {  // the period ended on an even row: its warp row is in hB
 #pragma unroll
-            for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6420u);
-            if (valid) recon_store_row<S>(outc + (size_t)j * W, o);
-        };
-        static_for<RPT>(one);
+                for (int k = 0; k < NP; k++) hA[k] = hB[k];
+            }
+        }
     }
 }
 
