@@ -97,6 +97,11 @@ __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
     asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
     return r;
 }
+__device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) {
+    uint32_t r;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
+    return r;
+}
 __device__ __forceinline__ void cp_async8(void *dst, const void *src) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
@@ -122,36 +127,45 @@ __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int 
         cp_async8(dst + i * stride, row + st);
     }
 }
-// After the copies of one non-interior window row have landed: replicate the
-// edge pixel into the staged words that lie outside the row (first word at xb).
+// Load one staged window row (NQ words) into registers; for a non-interior
+// window replicate the edge pixel into the words that lie outside the row
+// (first word at xb).
 template <int S>
-__device__ __forceinline__ void recon_fix_row(uint2 *row, int xb, int W) {
+__device__ __forceinline__ void recon_load_row(const uint2 *row, bool fix, int xb, int W,
+                                               uint2 (&q)[ReconCfg<S>::NQ]) {
 #pragma unroll
-    for (int i = 0; i < ReconCfg<S>::NQ; i++) {
-        const int st = xb + 8 * i;
-        uint2 *q = row + i * kReconNT;
-        if (st < 0) {
-            const uint32_t v = prmt(q->x, 0u, 0x0000u);
-            *q = make_uint2(v, v);
-        } else if (st >= W) {
-            const uint32_t v = prmt(q->y, 0u, 0x3333u);
-            *q = make_uint2(v, v);
+    for (int i = 0; i < ReconCfg<S>::NQ; i++) q[i] = row[i * kReconNT];
+    if (fix) {
+#pragma unroll
+        for (int i = 0; i < ReconCfg<S>::NQ; i++) {
+            const int st = xb + 8 * i;
+            if (st < 0) {
+                const uint32_t v = prmt(q[i].x, 0u, 0x0000u);
+                q[i] = make_uint2(v, v);
+            } else if (st >= W) {
+                const uint32_t v = prmt(q[i].y, 0u, 0x3333u);
+                q[i] = make_uint2(v, v);
+            }
         }
     }
 }
 
-// Horizontal bilinear pass over one staged reference row, scaled by 8:
-// h8[k] = packed pixels (2k, 2k+1) of (R[x](8-fx) + R[x+1]fx + 4) & ~7.
+// Horizontal bilinear pass over one staged reference row, scaled by 8.  Pixel
+// pairs are even/odd interleaved: pair 2g holds pixels (4g, 4g+2) and pair 2g+1
+// pixels (4g+1, 4g+3), so both operands of each pass come from one byte
+// permute of the aligned window word (no per-pair realignment):
+//   h8[2g]   = E_g (8-fx) + O_g fx + 4,  h8[2g+1] = O_g (8-fx) + E'_g fx + 4   (& ~7 per lane)
+// with E_g = [p4g, p4g+2], O_g = [p4g+1, p4g+3], E'_g = [p4g+2, p4g+4].
 template <int S>
-__device__ __forceinline__ void recon_hpass8(const uint2 *buf, int m, uint32_t fxc, uint32_t fx,
+__device__ __forceinline__ void recon_hpass8(const uint2 (&q)[ReconCfg<S>::NQ], int m, uint32_t fxc, uint32_t fx,
                                              uint32_t (&h)[ReconCfg<S>::NP]) {
     using Cfg = ReconCfg<S>;
+    constexpr int NG = Cfg::BW / 4;
     uint32_t w[2 * Cfg::NQ + 2];
 #pragma unroll
     for (int i = 0; i < Cfg::NQ; i++) {
-        const uint2 q = buf[i * kReconNT];
-        w[2 * i] = q.x;
-        w[2 * i + 1] = q.y;
+        w[2 * i] = q[i].x;
+        w[2 * i + 1] = q[i].y;
     }
     w[2 * Cfg::NQ] = 0;
     w[2 * Cfg::NQ + 1] = 0;
@@ -160,19 +174,22 @@ __device__ __forceinline__ void recon_hpass8(const uint2 *buf, int m, uint32_t f
         for (int i = 0; i < 2 * Cfg::NQ + 1; i++) w[i] = w[i + 1];
     }
     const uint32_t sh = 8u * (uint32_t)(m & 3);
-    uint32_t A[Cfg::NP + 2];
+    uint32_t E[NG + 1], O[NG];
 #pragma unroll
-    for (int i = 0; i < Cfg::NA32; i++) {
-        const uint32_t a = __funnelshift_r(w[i], w[i + 1], sh);
-        A[2 * i] = prmt(a, 0u, 0x4140u);
-        if (2 * i + 1 < Cfg::NP + 2) A[2 * i + 1] = prmt(a, 0u, 0x4342u);
+    for (int g = 0; g <= NG; g++) {
+        const uint32_t a = __funnelshift_r(w[g], w[g + 1], sh);
+        E[g] = prmt(a, 0u, 0x4240u);
+        if (g < NG) O[g] = prmt(a, 0u, 0x4341u);
     }
 #pragma unroll
-    for (int k = 0; k < Cfg::NP; k++) {
-        const uint32_t B = __funnelshift_r(A[k], A[k + 1], 16);
-        h[k] = (A[k] * fxc + B * fx + 0x00040004u) & 0xFFF8FFF8u;
+    for (int g = 0; g < NG; g++) {
+        const uint32_t E1 = __funnelshift_r(E[g], E[g + 1], 16);
+        h[2 * g] = (E[g] * fxc + O[g] * fx + 0x00040004u) & 0xFFF8FFF8u;
+        h[2 * g + 1] = (O[g] * fxc + E1 * fx + 0x00040004u) & 0xFFF8FFF8u;
     }
 }
+// pixel (within the thread's row) of lane e of pair k (even/odd interleave)
+__host__ __device__ constexpr int pair_px(int k, int e) { return 4 * (k >> 1) + (k & 1) + 2 * e; }
 
 // LR rows of KEY frames / INTRA blocks (Z17) are staged per thread in the
 // thread's (otherwise unused) warp-window slots, two per LR row: the aligned
@@ -207,7 +224,7 @@ __device__ __forceinline__ void recon_res_row_smem(const int16_t *p, bool left_i
 #pragma unroll
     for (int i = 0; i < 4; i++) {
         v[1 + 2 * i] = (int)(int16_t)(qq[i] & 0xFFFFu);
-        v[2 + 2 * i] = (int)qq[i] >> 16;
+        v[2 + 2 * i] = __mulhi((int)qq[i], 65536);  // arithmetic >> 16 on the FMA pipe
     }
     const int l = p[7], r = p[16];
     v[0] = left_in ? l : v[1];
@@ -236,14 +253,14 @@ __device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[
 #pragma unroll
     for (int t = 0; t < 10; t++) {
         V[t] = WY ? (128 - WY) * a[t] + WY * b[t] : 128 * a[t];
-        base[t] = V[t] * 512 + KB;
+        base[t] = (int)mad_u32((uint32_t)V[t], 512u, (uint32_t)KB);
     }
 #pragma unroll
     for (int k = 0; k < BW / 2; k++) {
         uint32_t sv[2];
 #pragma unroll
         for (int e = 0; e < 2; e++) {
-            const int i = 2 * k + e;
+            const int i = pair_px(k, e);
             const int d = tap_d<S>(i) + 1, w1 = tap_w1<S>(i);
             sv[e] = (uint32_t)(w1 ? base[d] + (4 * w1) * (V[d + 1] - V[d]) : base[d]);
         }
@@ -252,18 +269,14 @@ __device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[
 }
 
 template <int S>
-__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4]) {
+__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4], bool on) {
 #pragma unroll
     for (int q = 0; q < ReconCfg<S>::BW / 8; q++)
-        asm volatile("st.global.v2.b32 [%0], {%1, %2};" ::"l"(dst + 8 * q), "r"(o[2 * q]), "r"(o[2 * q + 1])
+        asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p st.global.v2.b32 [%0], {%1, %2}; }" ::"l"(dst + 8 * q),
+                     "r"(o[2 * q]), "r"(o[2 * q + 1]), "r"((uint32_t)on)
                      : "memory");
 }
 
-__device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) {
-    uint32_t r;
-    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
-    return r;
-}
 __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
     uint32_t r;
     asm("max.u16x2 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
@@ -397,8 +410,11 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
         const uint2 *lrb = wbuf + (c & 1) * (Cfg::PER + 2) * 2 * kReconNT;
         uint8_t *outc = outp + c * hrp;
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
-        if (fix) recon_fix_row<S>(wbuf, xs & ~7, W);
-        recon_hpass8<S>(wbuf, m, fxc, fx, hA);
+        {
+            uint2 q[NQ];
+            recon_load_row<S>(wbuf, fix, xs & ~7, W, q);
+            recon_hpass8<S>(q, m, fxc, fx, hA);
+        }
         stage_row(c + 1, 0);
         asm volatile("cp.async.commit_group;" ::: "memory");
 #pragma unroll 1
@@ -418,20 +434,21 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                 uint32_t(&hp)[NP] = (jj & 1) ? hB : hA;
                 uint32_t(&hc)[NP] = (jj & 1) ? hA : hB;
                 asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
-                if (fix) recon_fix_row<S>(wbuf + (j + 1) * NQ * kReconNT, xs & ~7, W);
-                recon_hpass8<S>(wbuf + (j + 1) * NQ * kReconNT, m, fxc, fx, hc);
+                uint2 q[NQ];
+                recon_load_row<S>(wbuf + (j + 1) * NQ * kReconNT, fix, xs & ~7, W, q);
+                uint32_t u[NP], x[NP], o[Cfg::BW / 4];
+                recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);   // independent of q: covers the load
+                recon_hpass8<S>(q, m, fxc, fx, hc);
                 stage_row(c + 1, j + 1);
                 asm volatile("cp.async.commit_group;" ::: "memory");
-                uint32_t u[NP], x[NP], o[Cfg::BW / 4];
-                recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);
 #pragma unroll
                 for (int k = 0; k < NP; k++) {
                     const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], 64u, 0x00200020u)));
-                    x[k] = vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu) >> 6;
+                    x[k] = __umulhi(vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu), 1u << 26);  // >> 6
                 }
 #pragma unroll
-                for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6420u);
-                if (valid) recon_store_row<S>(outc + (size_t)j * W, o);
+                for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6240u);
+                recon_store_row<S>(outc + (size_t)j * W, o, valid);
             };
             static_for<S>(one);
             if constexpr (S & 1) {  // the period ended on an even row: its warp row is in hB
