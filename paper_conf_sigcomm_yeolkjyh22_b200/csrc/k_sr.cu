@@ -1404,68 +1404,85 @@ __device__ __forceinline__ float act_at(const uint16_t *act, int y, int x, int c
     return __uint_as_float((uint32_t)act[(((size_t)y * (C / 8) + ci / 8) * w + x) * 8 + ci % 8] << 16);
 }
 
-// One thread per out-of-frame position, all C channels.  A CTA covers positions
-// of one band (row -1, row H, col -1, col W), whose upsampler taps are the
-// single valid kernel row/column (ky=2 / ky=0 / kx=2 / kx=0): their weights for
-// the s sub-pixels are staged in shared memory ([s][C][C][3] fp32).
-constexpr int kExtThreads = 128;
-__global__ void __launch_bounds__(kExtThreads) k_uptail_ext_u(const SrJob *jobs, int j0, const int32_t *job_count,
-                                                             const uint16_t *hact, int h, int w, int C, int s,
-                                                             size_t aux_off, float *ext) {
-    extern __shared__ float wsm[];  // [s][C out][C in][3]
-    const int slot = blockIdx.y, job = j0 + slot;
+// u_ext along the four bands.  Along a band only one kernel row (row bands:
+// ky = 2 at Y = -1, ky = 0 at Y = H) or one kernel column (column bands) of the
+// upsampler meets the frame, so u_ext is a 1-D 3-tap conv along the band over
+// the frame's first/last h row (column):
+//   u_ext[c, sp](p) = b_up + sum_{ci, t} W_up[c s^2 + i s + j][ci][ky][kx] h_line[p + t - 1][ci]
+// with (i, j, ky, kx) = (s-1, sp, 2, t) | (0, sp, 0, t) | (sp, s-1, t, 2) | (sp, 0, t, 0)
+// for bands row -1 | row H | col -1 | col W, p the LR coordinate along the band,
+// and HR coordinate s p + sp along it.  One thread per output (c, sp) keeps its
+// 3C weights in registers; the CTA stages 128 + 2 line pixels (fp32,
+// channel-major) and each thread sweeps them 4 positions at a time (6 shared
+// loads per 12 FMAs, all broadcasts).
+template <int C, int S>
+__global__ void __launch_bounds__(C * S) k_uptail_ext_u(const SrJob *jobs, int j0, const int32_t *job_count,
+                                                       const uint16_t *hact, int h, int w, size_t aux_off,
+                                                       float *ext) {
+    constexpr int P = 128;                       // LR positions per CTA
+    __shared__ __align__(16) float hs[C][P + 4];  // line pixels p0-1 .. p0+P (+ pad)
+    const int slot = blockIdx.y, job = j0 + slot, band = blockIdx.z;
     if (job_count && job >= *job_count) return;
-    const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H;
-    // band of this CTA: blocks are laid out band by band
-    const int nbr = (W + 2 + kExtThreads - 1) / kExtThreads, nbc = (H + kExtThreads - 1) / kExtThreads;
-    int band, local_blk = blockIdx.x;
-    if (local_blk < nbr) band = 0;
-    else if ((local_blk -= nbr) < nbr) band = 1;
-    else if ((local_blk -= nbr) < nbc) band = 2;
-    else { local_blk -= nbc; band = 3; }
-    const int bandlen = band < 2 ? W + 2 : H;
-    const int e = local_blk * kExtThreads + threadIdx.x;
+    const int H = h * S, W = w * S, next = 2 * (W + 2) + 2 * H;
+    const int L = band < 2 ? w : h;              // line length (LR)
+    // row bands need p = -1 .. w (HR X = -1 .. W); column bands p = 0 .. h-1
+    const int pfirst = band < 2 ? -1 : 0, plast = band < 2 ? w : h - 1;
+    const int p0 = pfirst + blockIdx.x * P;
+    if (p0 > plast) return;
+    const int tid = threadIdx.x, c = tid / S, sp = tid % S;
+    int i, j;
+    if (band == 0) { i = S - 1; j = sp; }
+    else if (band == 1) { i = 0; j = sp; }
+    else if (band == 2) { i = sp; j = S - 1; }
+    else { i = sp; j = 0; }
     const float *Wup = reinterpret_cast<const float *>(jobs[job].wts + aux_off);
-    const float *bup = Wup + (size_t)s * s * C * C * 9;
-    // stage weights: sub-pixel index sp in 0..s-1 (j' for row bands, i' for column bands)
-    for (int idx = threadIdx.x; idx < s * C * C * 3; idx += blockDim.x) {
-        const int t = idx % 3, ci = (idx / 3) % C, c = (idx / (3 * C)) % C, sp = idx / (3 * C * C);
-        int ip, jp, ky, kx;
-        if (band == 0) { ip = s - 1; jp = sp; ky = 2; kx = t; }
-        else if (band == 1) { ip = 0; jp = sp; ky = 0; kx = t; }
-        else if (band == 2) { ip = sp; jp = s - 1; ky = t; kx = 2; }
-        else { ip = sp; jp = 0; ky = t; kx = 0; }
-        wsm[idx] = Wup[((size_t)(c * s * s + ip * s + jp) * C + ci) * 9 + ky * 3 + kx];
-    }
-    __syncthreads();
-    if (e >= bandlen) return;
-    int Y, X, pos;
-    if (band == 0) { Y = -1; X = e - 1; pos = e; }
-    else if (band == 1) { Y = H; X = e - 1; pos = (W + 2) + e; }
-    else if (band == 2) { Y = e; X = -1; pos = 2 * (W + 2) + e; }
-    else { Y = e; X = W; pos = 2 * (W + 2) + H + e; }
-    const int y = (Y + s) / s - 1, i = Y - s * y, x = (X + s) / s - 1, j = X - s * x;
-    const int sp = band < 2 ? j : i;
+    const float *wrow = Wup + (size_t)(c * S * S + i * S + j) * C * 9;
+    float wr[C][3];
+#pragma unroll
+    for (int ci = 0; ci < C; ci++)
+#pragma unroll
+        for (int t = 0; t < 3; t++) {
+            const int ky = band == 0 ? 2 : band == 1 ? 0 : t, kx = band < 2 ? t : band == 2 ? 2 : 0;
+            wr[ci][t] = wrow[ci * 9 + ky * 3 + kx];
+        }
+    const float bias = Wup[(size_t)S * S * C * C * 9 + c * S * S + i * S + j];
+    // stage the line: element e <-> line pixel p0 - 1 + e (zero outside the frame: the upsampler's padding)
     const uint16_t *act = hact + (size_t)slot * h * (C / 8) * w * 8;
-    float hv[3][32];
+    for (int idx = tid; idx < (P + 2) * (C / 8); idx += C * S) {
+        const int e = idx % (P + 2), g = idx / (P + 2), pp = p0 - 1 + e;
+        float v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (pp >= 0 && pp < L) {
+            const int yy = band == 0 ? 0 : band == 1 ? h - 1 : pp, xx = band < 2 ? pp : band == 2 ? 0 : w - 1;
+            const uint4 q = *reinterpret_cast<const uint4 *>(act + (((size_t)yy * (C / 8) + g) * w + xx) * 8);
+            v[0] = bf_lo(q.x); v[1] = bf_hi(q.x); v[2] = bf_lo(q.y); v[3] = bf_hi(q.y);
+            v[4] = bf_lo(q.z); v[5] = bf_hi(q.z); v[6] = bf_lo(q.w); v[7] = bf_hi(q.w);
+        }
 #pragma unroll
-    for (int t = 0; t < 3; t++) {
-        const int yy = band == 0 ? 0 : band == 1 ? h - 1 : y + t - 1;
-        const int xx = band == 2 ? 0 : band == 3 ? w - 1 : x + t - 1;
-        const bool ok = yy >= 0 && yy < h && xx >= 0 && xx < w;
-#pragma unroll
-        for (int ci = 0; ci < 32; ci++)
-            hv[t][ci] = (ok && ci < C) ? __uint_as_float((uint32_t)act[(((size_t)yy * (C / 8) + ci / 8) * w + xx) * 8 + ci % 8] << 16) : 0.f;
+        for (int k = 0; k < 8; k++) hs[g * 8 + k][e] = v[k];
     }
-    const float *wb = wsm + (size_t)sp * C * C * 3;
-    float *dst = ext + ((size_t)slot * next + pos) * C;
-    for (int c = 0; c < C; c++) {
-        float acc = bup[c * s * s + i * s + j];
-        const float *wr = wb + (size_t)c * C * 3;
+    if (tid < C * 2) hs[tid / 2][P + 2 + tid % 2] = 0.f;
+    __syncthreads();
+    const int pos_base = band == 0 ? 1 : band == 1 ? (W + 2) + 1 : band == 2 ? 2 * (W + 2) : 2 * (W + 2) + H;
+    const int zmin = band < 2 ? -1 : 0, zmax = band < 2 ? W : H - 1;
+    float *dst = ext + (size_t)slot * next * C;
+#pragma unroll 1
+    for (int q = 0; q < P; q += 4) {
+        if (p0 + q > plast) break;
+        float acc[4] = {bias, bias, bias, bias};
 #pragma unroll
-        for (int ci = 0; ci < 32; ci++)
-            if (ci < C) acc += wr[ci * 3 + 0] * hv[0][ci] + wr[ci * 3 + 1] * hv[1][ci] + wr[ci * 3 + 2] * hv[2][ci];
-        dst[c] = acc;
+        for (int ci = 0; ci < C; ci++) {
+            const float4 a4 = *reinterpret_cast<const float4 *>(&hs[ci][q]);
+            const float2 b2 = *reinterpret_cast<const float2 *>(&hs[ci][q + 4]);
+            const float v[6] = {a4.x, a4.y, a4.z, a4.w, b2.x, b2.y};
+#pragma unroll
+            for (int k = 0; k < 4; k++)
+                acc[k] = fmaf(wr[ci][0], v[k], fmaf(wr[ci][1], v[k + 1], fmaf(wr[ci][2], v[k + 2], acc[k])));
+        }
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const int p = p0 + q + k, Z = S * p + sp;
+            if (p <= plast && Z >= zmin && Z <= zmax) dst[(size_t)(pos_base + Z) * C + c] = acc[k];
+        }
     }
 }
 
@@ -1473,9 +1490,16 @@ __global__ void __launch_bounds__(kExtThreads) k_uptail_ext_u(const SrJob *jobs,
 // the out-of-frame tail taps, then the bilinear skip, round, clamp, store.
 __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, int C, int s,
                               size_t aux_off, const float *ext, const float *ring) {
+    __shared__ float swt[3 * 32 * 9];  // W_tail [3][C][9]
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
     const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
+    {
+        const float *aux = reinterpret_cast<const float *>(jobs[job].wts + aux_off);
+        const float *Wt = aux + (size_t)s * s * C * C * 9 + (size_t)s * s * C;
+        for (int k = threadIdx.x; k < 3 * C * 9; k += blockDim.x) swt[k] = Wt[k];
+        __syncthreads();
+    }
     const int e = blockIdx.x * blockDim.x + threadIdx.x;
     if (e >= nring) return;
     int Y, X;
@@ -1484,8 +1508,7 @@ __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_coun
     else if (e < 2 * W + (H - 2)) { Y = 1 + (e - 2 * W); X = 0; }
     else { Y = 1 + (e - 2 * W - (H - 2)); X = W - 1; }
     const SrJob J = jobs[job];
-    const float *aux = reinterpret_cast<const float *>(J.wts + aux_off);
-    const float *Wt = aux + (size_t)s * s * C * C * 9 + (size_t)s * s * C;
+    const float *Wt = swt;
     const float *E = ext + (size_t)slot * next * C;
     const float *tr = ring + ((size_t)slot * nring + e) * 3;
     float t[3] = {tr[0], tr[1], tr[2]};
@@ -1770,15 +1793,10 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         // exact frame-border ring (the tail's zero padding of u)
         KScope ks(F_SR_TAIL, st, 2);
         const int H = h * s, W = w * s, next = 2 * (W + 2) + 2 * H, nring = 2 * W + 2 * (H - 2);
-        const int nbr = (W + 2 + kExtThreads - 1) / kExtThreads, nbc = (H + kExtThreads - 1) / kExtThreads;
-        const size_t wsm = (size_t)s * C * C * 3 * sizeof(float);
-        static bool attr = false;
-        if (!attr) {
-            cudaFuncSetAttribute(k_uptail_ext_u, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024);
-            attr = true;
-        }
-        dim3 g1(2 * nbr + 2 * nbc, nj), g2((nring + 127) / 128, nj);
-        k_uptail_ext_u<<<g1, kExtThreads, wsm, st>>>(jobs, j0, job_count, endout, h, w, C, s, cs.aux_off, a->band);
+        dim3 g1((std::max(w + 2, h) + 127) / 128, nj, 4), g2((nring + 127) / 128, nj);
+        if (s == 2) k_uptail_ext_u<C, 2><<<g1, C * 2, 0, st>>>(jobs, j0, job_count, endout, h, w, cs.aux_off, a->band);
+        else if (s == 3) k_uptail_ext_u<C, 3><<<g1, C * 3, 0, st>>>(jobs, j0, job_count, endout, h, w, cs.aux_off, a->band);
+        else k_uptail_ext_u<C, 4><<<g1, C * 4, 0, st>>>(jobs, j0, job_count, endout, h, w, cs.aux_off, a->band);
         k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, h, w, C, s, cs.aux_off, a->band,
                                           a->band + (size_t)a->nb * next * C);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
