@@ -16,7 +16,8 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libneuroscaler.so")
+# NS_LIB: an alternative in-tree build of the same library (A/B timing of variants)
+LIB_PATH = os.environ.get("NS_LIB") or os.path.join(_HERE, "libneuroscaler.so")
 
 NS_OK, NS_EINVAL, NS_ECUDA, NS_ENOMEM, NS_EUNSUPPORTED = 0, -1, -2, -3, -4
 NS_KEY, NS_ALTREF, NS_NORMAL = 0, 1, 2

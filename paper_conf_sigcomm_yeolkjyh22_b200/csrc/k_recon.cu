@@ -572,12 +572,16 @@ __global__ void k_stats_final(const StreamDesc *sd, int S, int n, double *stats)
 
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
                          uint8_t *const *d_hr_table, size_t max_hr_bytes, double *stats, cudaStream_t st) {
-    KScope ks(F_STATS, st, 3);
+    // max_hr_bytes == 0: no stream carries ground truth, so there is no SSE pass
+    KScope ks(F_STATS, st, max_hr_bytes ? 3 : 1);
     k_stats_meta<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, score, stats);
-    const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
-    dim3 g(blocks < 1 ? 1 : (blocks > 1024 ? 1024 : blocks), S * n);
-    k_stats_sse<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, stats);
-    k_stats_final<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, stats);
+    if (max_hr_bytes) {
+        // one CTA row per (stream, frame), ~4 CTAs per SM-resident wave over the frame
+        const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
+        dim3 g(blocks < 1 ? 1 : (blocks > 64 ? 64 : blocks), S * n);
+        k_stats_sse<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, stats);
+        k_stats_final<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, stats);
+    }
     return cudaGetLastError();
 }
 

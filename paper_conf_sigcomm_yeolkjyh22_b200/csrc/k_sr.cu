@@ -551,6 +551,13 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
 
 // ------------------------------------------------------------------ fused residual block
 constexpr int kRbMmaWarps = 4;
+// h ring depth per tile: the slot of row q+NH is freed by E2(q+2), so the TMA row
+// load (~2,000 cycles measured on the clock64 timeline) gets NH-3 steps of
+// slack.  A/B on B200 (tools/build_variant.sh): NH 5 / 6 / 7 -> body 114.6 /
+// 105.1 / 109.6 ms per c4 step (7 leaves the epilogues more SMEM contention).
+#ifndef NS_RB_NH
+#define NS_RB_NH 6
+#endif
 constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 // h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
 // h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
@@ -574,8 +581,8 @@ struct RbCfg {
     static constexpr uint32_t BIAS_BYTES = C * 4u;
     static constexpr uint32_t W_CONV = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * C * 2u;
-    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int NH = 5;                                 // h ring per tile
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);  // TMA destination: 128-B aligned
+    static constexpr int NH = NS_RB_NH;                          // h ring per tile
     static constexpr int NTS = 2;                                // t slots per tile
     static constexpr uint32_t TILE_BYTES = (NH + NTS) * SLOT;
     static constexpr uint32_t TCOLS = 2 * 3 * NB;                // conv1 + conv2 rings per tile
@@ -792,8 +799,11 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
                     if (warp % 4 == 2 && lane == 0) NS_TR(40 + k, q);
+#ifndef NS_TRACE_NOZERO
                     tmem_zeroN<NB>(acc);
                     tmem_wait_st();
+#endif
+
                     tc_fence_before();
                     mbar_arrive(e1z(k));  // the next conv1 group may start
                     // t slot q%2 was last read by M2(q-2) (another warp's MMAs): completion
@@ -837,8 +847,11 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
+#ifndef NS_TRACE_NOZERO
                     tmem_zeroN<NB>(acc);
                     tmem_wait_st();
+#endif
+
                     tc_fence_before();
                     mbar_arrive(e2z(k));  // the next conv2 group may start
                     const int x = x0k(k) + p;

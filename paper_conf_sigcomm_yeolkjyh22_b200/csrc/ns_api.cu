@@ -732,7 +732,9 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
         if (stats) {
             size_t maxhr = 0;
             for (int s = 0; s < S; s++) maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
-            cudaError_t e = launch_stats(g.d_sd, S, n, anchor, c->score, g.d_hr, maxhr, stats, st);
+            bool any_gt = false;
+            for (int s = 0; s < S; s++) any_gt |= ch[s].gt != nullptr;
+            cudaError_t e = launch_stats(g.d_sd, S, n, anchor, c->score, g.d_hr, any_gt ? maxhr : 0, stats, st);
             if (e != cudaSuccess) { r = cuda_fail(e, "stats"); break; }
         }
     } while (0);
