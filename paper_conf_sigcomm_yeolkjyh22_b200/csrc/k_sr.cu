@@ -558,6 +558,9 @@ constexpr int kRbMmaWarps = 4;
 #ifndef NS_RB_NH
 #define NS_RB_NH 6
 #endif
+#ifndef NS_RB_NTS
+#define NS_RB_NTS 2
+#endif
 constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 // h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
 // h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
@@ -583,11 +586,11 @@ struct RbCfg {
     static constexpr uint32_t SLOT_BYTES = kHalo * C * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);  // TMA destination: 128-B aligned
     static constexpr int NH = NS_RB_NH;                          // h ring per tile
-    static constexpr int NTS = 2;                                // t slots per tile
+    static constexpr int NTS = NS_RB_NTS;                        // t slots per tile (<= 4: e1t rotates over 4)
     static constexpr uint32_t TILE_BYTES = (NH + NTS) * SLOT;
     static constexpr uint32_t TCOLS = 2 * 3 * NB;                // conv1 + conv2 rings per tile
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
-    static constexpr int BPT = 2 * NH + 10;                      // barriers per tile
+    static constexpr int BPT = 2 * NH + 8 + NTS;                 // barriers per tile
     static constexpr int NBAR = 2 * BPT + 1;
     static constexpr uint32_t SMEM = 2 * W_CONV + 2 * TILE_BYTES + NBAR * 8 + 64;
     static_assert(SMEM <= 232448, "shared memory");
@@ -621,7 +624,7 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
     uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + Cfg::NBAR);
     auto hslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
     auto tslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + (NH + i) * Cfg::SLOT; };
-    // per tile: hfull[NH], m1, m2, e1z, e2z, e1t[4], tfree[2], hfree[NH]
+    // per tile: hfull[NH], m1, m2, e1z, e2z, e1t[4], tfree[NTS], hfree[NH]
     constexpr int BPT = Cfg::BPT;
     auto hfull = [&](int k, int i) { return &bars[k * BPT + i]; };
     auto m1bar = [&](int k) { return &bars[k * BPT + NH]; };
@@ -630,7 +633,7 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
     auto e2z = [&](int k) { return &bars[k * BPT + NH + 3]; };
     auto e1t = [&](int k, int i) { return &bars[k * BPT + NH + 4 + i]; };
     auto tfree = [&](int k, int i) { return &bars[k * BPT + NH + 8 + i]; };
-    auto hfree = [&](int k, int i) { return &bars[k * BPT + NH + 10 + i]; };
+    auto hfree = [&](int k, int i) { return &bars[k * BPT + NH + 8 + Cfg::NTS + i]; };
     uint64_t *wbar = &bars[2 * BPT];
 
     const int slot_job = blockIdx.z;
@@ -653,8 +656,7 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
             mbar_init(e1z(k), 128);
             mbar_init(e2z(k), 128);
             for (int i = 0; i < 4; i++) mbar_init(e1t(k, i), 128);
-            mbar_init(tfree(k, 0), 1);
-            mbar_init(tfree(k, 1), 1);
+            for (int i = 0; i < Cfg::NTS; i++) mbar_init(tfree(k, i), 1);
         }
         mbar_init(wbar, 1);
         fence_mbar_init();
@@ -759,7 +761,7 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
                     tc_fence_after();
                     // tfree: t slot q%2 may be overwritten once these MMAs complete
                     mma_rot(tmem + k * Cfg::TCOLS + 3 * NB, tslot(k, q % Cfg::NTS), s_w2, y0 - 3 + q, m2bar(k),
-                            tfree(k, q & 1));
+                            tfree(k, q % Cfg::NTS));
                     if (lane == 0) NS_TR(7 + k, q);
                 }
             }
@@ -808,7 +810,7 @@ __global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constan
                     mbar_arrive(e1z(k));  // the next conv1 group may start
                     // t slot q%2 was last read by M2(q-2) (another warp's MMAs): completion
                     // #((q-4)/2) of tfree[q%2]; M2(q-4) is done, M2(q) cannot be -> exact
-                    if (q >= 4) mbar_wait(tfree(k, q & 1), ((q - 4) >> 1) & 1);
+                    if (q >= 2 + Cfg::NTS) mbar_wait(tfree(k, q % Cfg::NTS), ((q - Cfg::NTS - 2) / Cfg::NTS) & 1);
                     if (q >= 2) {
                         const int xt = x0k(k) - 1 + p;
                         const bool inside = yt >= 0 && yt < a.H && xt >= 0 && xt < a.W;
