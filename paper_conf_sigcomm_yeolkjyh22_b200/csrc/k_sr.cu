@@ -1088,6 +1088,12 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
 // and the other tile's MMAs cover that wait.  The TMA warp also stages the
 // three u8 LR rows r-1..r+1 of each output row r (bilinear skip taps) in a
 // separate ring that the epilogue groups release.
+#ifndef NS_UP_NS
+#define NS_UP_NS 3
+#endif
+#ifndef NS_UP_MMA2
+#define NS_UP_MMA2 0
+#endif
 template <int CIN, int NB, int S>
 struct Up2Cfg {
     static constexpr int KC = CIN / 16, NSTRIP = 9;
@@ -1095,8 +1101,8 @@ struct Up2Cfg {
     static constexpr uint32_t BIAS_BYTES = NB * 4u;
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo5 * CIN * 2u;
-    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int NS = 3;                                    // input ring per tile
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);     // TMA destination: 128-B aligned
+    static constexpr int NS = NS_UP_NS;                             // input ring per tile
     static constexpr int NL = 3;                                    // LR ring per tile
     static constexpr uint32_t LR_BYTES = 9u * kLrBoxW;              // [row 3][plane 3][kLrBoxW]
     static constexpr uint32_t LSLOT = round_up(LR_BYTES, 128);
@@ -1106,7 +1112,7 @@ struct Up2Cfg {
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
     static constexpr int BPT = 2 * NS + 3 + 2 * NL;                // barriers per tile
     static constexpr int NBAR = 2 * BPT + 1;
-    static constexpr int NWARPS = 2 + 2 * S * 4;
+    static constexpr int NWARPS = 2 + 2 * S * 4 + NS_UP_MMA2;      // (+ the second tile's MMA issuer, last)
     static constexpr uint32_t SMEM = W_REGION + 2 * TILE_BYTES + NBAR * 8 + 64;
     static_assert(5 * NB <= 256, "N = 5 nb");
     static_assert(SMEM <= 232448, "shared memory");
@@ -1180,7 +1186,7 @@ __device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>:
 // frame-border ring pixels of sub-row I keep their fp32 t = acc + bias for the
 // exact fix-up (k_uptail_ring)
 template <int NB, int S, int I>
-__device__ __noinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
+__device__ __forceinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
                                                const ConvArgs &a, int x, int r, int lh, int lw, int slot_job) {
     constexpr int base = UpCols<NB, S>::base(I);
     const int HH = lh * S, WW = lw * S;
@@ -1245,13 +1251,9 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     const int nq = y1 - y0 + 4;  // input rows y0-2 .. y1+1
     const int lh = a.H, lw = a.W;
     const int HH = lh * S, WW = lw * S;
-    int x0k[2];
-    bool vk[2];
-    for (int k = 0; k < 2; k++) {
-        const int tix = 2 * blockIdx.x + k;
-        vk[k] = tix * kTile < lw;
-        x0k[k] = tix * kTile;
-    }
+    // tile k of this CTA (computed, not indexed: no local memory)
+    auto x0k = [&](int k) { return (2 * (int)blockIdx.x + k) * kTile; };
+    auto vk = [&](int k) { return (2 * (int)blockIdx.x + k) * kTile < lw; };
     if (tid == 0) {
         for (int k = 0; k < 2; k++) {
             for (int i = 0; i < NS; i++) { mbar_init(hfull(k, i), 1); mbar_init(sfree(k, i), 1); }
@@ -1268,7 +1270,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *s_tmem;
-    if (warp >= 2 && ((warp - 2) / 4) % S == 0) {
+    if (warp >= 2 && warp < 2 + 8 * S && ((warp - 2) / 4) % S == 0) {
         // sub-row-0 group of each tile: zero its accumulator ring (the block of
         // row y0 has no earlier owner whose retirement would have zeroed it)
         const int k = (warp - 2) / 4 / S;
@@ -1291,26 +1293,29 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
             bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, wbar);
             for (int q = 0; q < nq; q++)
                 for (int k = 0; k < 2; k++) {
-                    if (!vk[k]) continue;
+                    if (!vk(k)) continue;
                     const int sl = q % NS;
                     if (q >= NS) mbar_wait(sfree(k, sl), ((q / NS) - 1) & 1);
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
-                    tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k[k] - 2, 0, y0 - 2 + q, slot_job);
+                    tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
                     const int qv = q - 4;  // output row y0 + qv retires at this step
                     if (qv >= 0) {
                         const int ls = qv % NL;
                         if (qv >= NL) mbar_wait(lfree(k, ls), ((qv / NL) - 1) & 1);
                         mbar_arrive_expect_tx(lfull(k, ls), Cfg::LR_BYTES);
-                        tma_load_4d(lslot(k, ls), &tm_lr, lfull(k, ls), x0k[k] - kLrBoxX, 0, y0 + qv - 1, slot_job);
+                        tma_load_4d(lslot(k, ls), &tm_lr, lfull(k, ls), x0k(k) - kLrBoxX, 0, y0 + qv - 1, slot_job);
                     }
                 }
         }
-    } else if (warp == 1) {  // ---- MMA issuer (whole warp, elected lane issues)
+    } else if (warp == 1 || (NS_UP_MMA2 && warp == Cfg::NWARPS - 1)) {
+        // ---- MMA issuer(s) (whole warp, elected lane issues); with NS_UP_MMA2 one
+        // warp per tile, so one tile's epilogue wait never holds the other tile's MMAs
         const uint32_t idesc = idesc_bf16_f32(128, 5 * NB);
+        const int kfirst = NS_UP_MMA2 ? (warp == 1 ? 0 : 1) : 0, klast = NS_UP_MMA2 ? kfirst : 1;
         mbar_wait(wbar, 0);
         for (int q = 0; q < nq; q++)
-            for (int k = 0; k < 2; k++) {
-                if (!vk[k]) continue;
+            for (int k = kfirst; k <= klast; k++) {
+                if (!vk(k)) continue;
                 const int sl = q % NS, yin = y0 - 2 + q;
                 mbar_wait(hfull(k, sl), (q / NS) & 1);
                 if (q >= 1) mbar_wait(edone(k), (q - 1) & 1);  // E(q-1) retired row yin-3 = the block of yin+2
@@ -1335,16 +1340,16 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
         const int grp = (warp - 2) / 4, k = grp / S, g = grp % S;
         const int ew = warp % 4;
         const int p = ew * 32 + lane;
-        const int x = x0k[k] + p;
+        const int x = x0k(k) + p;
         const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
         uint8_t *so = oslot(k, g);
-        if (vk[k]) {
+        if (vk(k)) {
             mbar_wait(wbar, 0);
             float bh[3 * S];
 #pragma unroll
             for (int i = 0; i < 3 * S; i++) bh[i] = s_bias[3 * S * g + i] + 0.5f;
             const uint32_t cbase = (uint32_t)(NB <= 16 ? 0 : 8 * ((3 * S * g) / 8));
-            const int xs_hr = x0k[k] * S, wv = min(kTile, lw - x0k[k]) * S;
+            const int xs_hr = x0k(k) * S, wv = min(kTile, lw - x0k(k)) * S;
             uint8_t *const hr = a.jobs[job].hr + xs_hr;
             for (int q = 0; q < nq; q++) {
                 const int r = y0 - 4 + q;  // LR output row completed at this step
@@ -1368,10 +1373,10 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     mbar_wait(lfull(k, ls), (qv / NL) & 1);
                     const uint8_t *lr = lslot(k, ls);
                     if (x < lw) {
-                        if (g == 0) uptail_group_step<NB, S, 0>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
-                        else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
-                        else if (S > 2 && g == 2) uptail_group_step<NB, S, (S > 2 ? 2 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
-                        else if (S > 3 && g == 3) uptail_group_step<NB, S, (S > 3 ? 3 : 0)>(v, bh, s_bias, lr, r, x, x0k[k], lh, lw, a, so, p, slot_job);
+                        if (g == 0) uptail_group_step<NB, S, 0>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 2 && g == 2) uptail_group_step<NB, S, (S > 2 ? 2 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 3 && g == 3) uptail_group_step<NB, S, (S > 3 ? 3 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
                     }
                     named_bar(3 + grp, 128);  // this group's staging row is complete, its LR reads done
                     if (p == 0) mbar_arrive(lfree(k, ls));
