@@ -375,17 +375,25 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     // Reference windows live in ONE buffer of RPT+1 rows: row r of plane c+1 is
     // staged right after plane c's warp pass has read row r, one commit group per
     // row, so before the pass over row r there are always exactly RPT groups newer
-    // than row r's (wait_group RPT).  LR rows (use_lr threads) alternate between
-    // two small slot sets and ride in the group of row 0.
+    // than row r's (wait_group RPT).  LR rows (use_lr threads) ride in the group
+    // of row 0: when all three planes fit the thread's slots (s = 3, 4) they are
+    // staged at once with plane 0 -- LR may be host memory read across PCIe
+    // (ns_enhance_streams_host), so its latency is paid once, not per plane --
+    // otherwise per plane, alternating between two slot sets.
+    constexpr int LRS = (Cfg::PER + 2) * 2;                 // slots per plane's LR rows
+    constexpr bool LR_ALL = 3 * LRS <= (RPT + 1) * NQ;
+    auto lr_slots = [&](int c) { return (LR_ALL ? c : (c & 1)) * LRS * kReconNT; };
     uint2 *wbuf = rsm + tid;
     auto stage_row = [&](int c, int r) {
         if (!valid || c >= 3) return;
         if (use_lr) {
-            if (r == 0) {
+            if (r == 0 && (!LR_ALL || c == 0)) {
+#pragma unroll 1
+                for (int cc = c; cc < (LR_ALL ? 3 : c + 1); cc++)
 #pragma unroll
-                for (int t = 0; t < Cfg::PER + 2; t++)
-                    recon_lr_row_stage(fd.lr_f + c * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
-                                       wbuf + ((c & 1) * (Cfg::PER + 2) + t) * 2 * kReconNT);
+                    for (int t = 0; t < Cfg::PER + 2; t++)
+                        recon_lr_row_stage(fd.lr_f + cc * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
+                                           wbuf + lr_slots(cc) + t * 2 * kReconNT);
             }
             return;
         }
@@ -407,7 +415,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
         if (c == 0) __syncthreads();                            // the residual tile is cooperative
         // (use_lr threads run the warp pass over whatever the slots hold: every weight is 0, so pred = 0)
         const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
-        const uint2 *lrb = wbuf + (c & 1) * (Cfg::PER + 2) * 2 * kReconNT;
+        const uint2 *lrb = wbuf + lr_slots(c);
         uint8_t *outc = outp + c * hrp;
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
         {

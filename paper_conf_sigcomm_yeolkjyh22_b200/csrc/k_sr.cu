@@ -558,6 +558,9 @@ constexpr int kRbMmaWarps = 4;
 #ifndef NS_RB_NH
 #define NS_RB_NH 6
 #endif
+#ifndef NS_RB_QUAL
+#define NS_RB_QUAL __launch_bounds__(kRbThreads, 1)
+#endif
 #ifndef NS_RB_NTS
 #define NS_RB_NTS 2
 #endif
@@ -612,7 +615,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
 // both tiles' groups while the epilogues run (a drained queue costs the ~300-
 // cycle commit round trip, tools/ubench.cu).
 template <int C>
-__global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
+__global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
     using Cfg = RbCfg<C>;
     constexpr int NB = Cfg::NB, NH = Cfg::NH;
     extern __shared__ __align__(1024) uint8_t smem[];
