@@ -220,7 +220,7 @@ def main():
     ap.add_argument("--config", type=int, default=4)
     ap.add_argument("--streams", type=int, default=0)
     ap.add_argument("--distinct", type=int, default=8, help="distinct generated streams (replicated on device)")
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sr-batch", type=int, default=16)
     args = ap.parse_args()

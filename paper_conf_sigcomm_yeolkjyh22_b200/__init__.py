@@ -303,7 +303,8 @@ class Context:
         """Pool bytes ns_enhance_streams_host carves on first use (two input
         staging buffers of one ~S/8-stream group + the anchors' LR staging)."""
         a = lambda v: (v + 255) // 256 * 256
-        gs = max(1, (streams + 7) // 8)
+        g = int(os.environ.get("NS_HOST_GROUPS", "0")) or 8
+        gs = max(1, (streams + g - 1) // g)
         px = h * w
         per = a(n * 3 * px * 2) + a(n * (px // 64) * 8) + a(n) + a(n * 4)
         return 2 * gs * per + gs * k * a(3 * px) + (1 << 20)

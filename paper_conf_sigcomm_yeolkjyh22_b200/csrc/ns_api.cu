@@ -3,6 +3,7 @@
 // model slots + weight refit, descriptor staging and the
 // multi-stream batcher that drives the kernels.
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <atomic>
@@ -142,6 +143,15 @@ constexpr size_t kStageBytes = 8u << 20;
 constexpr int kMaxSN = 1 << 20;           // max streams x frames per call
 constexpr int kMaxJobs = 1 << 20;
 constexpr int kHostGroups = 8;            // stream groups per ns_enhance_streams_host call
+// (NS_HOST_GROUPS in the environment overrides it: tuning experiments only)
+static int host_groups() {
+    static const int g = [] {
+        const char *e = getenv("NS_HOST_GROUPS");
+        const int v = e ? atoi(e) : 0;
+        return v > 0 ? v : kHostGroups;
+    }();
+    return g;
+}
 
 struct ArenaEntry {
     int h, w, C, s;
@@ -791,7 +801,7 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
     // groups of consecutive streams, ~kHostGroups per call: the first group's
     // upload and the last group's compute are the unhidden fill and drain; global
     // budget mode needs all scores before selecting -> one group
-    const int gs = topk ? std::max(1, (S + kHostGroups - 1) / kHostGroups) : S;
+    const int gs = topk ? std::max(1, (S + host_groups() - 1) / host_groups()) : S;
     // group sizes: gs each, the last one split into halves and quarters
     // (gs/2, gs/4, gs/4): the drain -- the last group's compute after the final
     // upload -- shrinks 4x, and compute (~0.55 of the upload time per stream)
