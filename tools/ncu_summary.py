@@ -59,7 +59,7 @@ def main():
     reps = sys.argv[3:]
     agg = launches(lpath)
     tot = sum(a[1] for a in agg.values())
-    lines = ["# ncu summary (round 1, c4 bench step; `tools/ncu_summary.py`)", "",
+    lines = [f"# ncu summary ({os.path.basename(md).split("_")[0]}, c4 bench step; `tools/ncu_summary.py`)", "",
              f"Launch list: `{os.path.basename(lpath)}` -- `ncu --metrics gpu__time_duration.sum --clock-control none`, "
              "warm-up + 1 timed step of `bench.py` (cold-cache, serialised; shares, not absolute times, compare with "
              "the live CUDA-event breakdown in the bench JSON).", "",
@@ -67,7 +67,7 @@ def main():
     for n, (c, t) in sorted(agg.items(), key=lambda x: -x[1][1]):
         lines.append(f"| `{n}` | {c} | {t * 1e3:.2f} | {t / tot:.1%} |")
     traffic = {}
-    lines += ["", "## `--set full` captures (one launch each: 16 jobs of 1280x720)", "",
+    lines += ["", "## `--set full` captures (one launch each: SR kernels 16 jobs of 1280x720, recon one frame step of 64 streams)", "",
               "| kernel | duration ms | DRAM read GB | DRAM write GB | DRAM % peak | SM % | tensor pipe % | issue % | "
               "occupancy % | regs | top stalls |", "|---|---|---|---|---|---|---|---|---|---|---|"]
     for rep in reps:
