@@ -93,19 +93,38 @@ typedef struct {
     const uint8_t *gt;         /* optional [n][3][s*h][s*w] ground truth for stats   */
 } ns_chunk;
 
-/* Anchor selection mode (§5.1 top-k per chunk; §5.2 global budget). */
-enum { NS_TOPK_PER_STREAM = 0, NS_GLOBAL_BUDGET = 1 };
+/* Anchor selection mode (§5.1 top-k per chunk; §5.2 global budget).
+   NS_GIVEN_ANCHORS: the anchor map was decided elsewhere -- by ns_select_merge
+   over the streams of every GPU (§5.2 global selection across GPUs)
+   -- and is passed in `anchor_in`; `cost` and `budget` are those of that global
+   selection (this call's streams' entries of cost[]), which bound the anchors
+   this call can receive (sum of their cost <= budget).  Only ns_enhance_streams
+   and ns_enhance_streams_host accept it. */
+enum { NS_TOPK_PER_STREAM = 0, NS_GLOBAL_BUDGET = 1, NS_GIVEN_ANCHORS = 2 };
 /* Residual carried from the G_altref pass into the G_normal pass (reading Z2,
    default) or recomputed per group (literal Alg. 1 line 2). */
 enum { NS_CARRY = 0, NS_FRESH = 1 };
+/* Anchor selector (top-k mode only).  NS_SEL_NEUROSCALER: Alg. 1 + Fig. 10.
+   The two real-time baselines of §3:
+     NS_SEL_KEY          "Key SR": key frames only -- the first min(k, #key)
+                         key frames (k = n: every key frame; reading R6);
+     NS_SEL_KEY_UNIFORM  "Key+Uniform SR": key frames, then the equally spaced
+                         frames U = { floor(j*n/k) : 0 <= j < k } (reading R5),
+                         priority (key asc, U asc, rest asc), first k anchors.
+   Per-frame SR is top-k with k = n under any selector.  gain is
+   INT64_MAX for key frames and 0 otherwise under the baselines. */
+enum { NS_SEL_NEUROSCALER = 0, NS_SEL_KEY = 1, NS_SEL_KEY_UNIFORM = 2 };
 
 typedef struct {
-    int32_t mode;              /* NS_TOPK_PER_STREAM | NS_GLOBAL_BUDGET              */
+    int32_t mode;              /* NS_TOPK_PER_STREAM | NS_GLOBAL_BUDGET | NS_GIVEN_ANCHORS */
     int32_t k;                 /* top-k mode: anchors per stream, 0 <= k <= n         */
-    int64_t budget;            /* global mode: T_intv * M in cost units       */
+    int64_t budget;            /* global / given mode: T_intv * M in cost units */
     const int64_t *cost;       /* HOST [S]: T_DNN of one anchor of stream s, >= 1     */
     int32_t group_residual;    /* NS_CARRY | NS_FRESH                                 */
     int32_t use_res_size;      /* 1: score = res_size (P:191 proxy) when non-NULL     */
+    int32_t selector;          /* NS_SEL_* (top-k mode; 0 otherwise)                  */
+    int32_t reserved;          /* 0                                                   */
+    const uint8_t *anchor_in;  /* NS_GIVEN_ANCHORS: DEVICE [S][n] 0/1, else NULL      */
 } ns_select_params;
 
 /* One anchor-SR job: HR = SR_model(LR) (O5). */
@@ -145,6 +164,26 @@ NS_API ns_status ns_model_destroy(ns_model *m);
    global order in NS_GLOBAL_BUDGET mode), is_anchor (0/1). */
 NS_API ns_status ns_select_anchors(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
                             int64_t *gain, int32_t *rank, uint8_t *is_anchor, void *stream);
+
+/* Global anchor selection over streams gathered from every GPU (§5.2: "select
+   anchor frames globally across all streams").
+   Each GPU first runs ns_select_anchors on its own streams (any mode; only the
+   per-stream gain and rank are used), then the callers all-gather, per stream,
+   gain[n], rank[n], type[n], cost and a global stream id, and every GPU calls
+   this with the identical gathered arrays, so every GPU computes the identical
+   selection with no further exchange.  Inputs, all DEVICE, S = streams over all
+   GPUs in any order: gain, rank_in (per-stream rank from ns_select_anchors)
+   int64 / int32 [S][n]; type u8 [S][n]; sid int32 [S] distinct global stream
+   ids (the stream key of the merged order, readings Z5, R7); cost int64 [S] >= 1.
+   The merged order is G_key by (sid, frame), then G_altref, then G_normal, each
+   by (gain desc, sid asc, frame asc); the anchors are its longest prefix with
+   summed cost <= budget (Z7).  Outputs DEVICE [S][n]: rank (global
+   position), is_anchor.  Equals ns_select_anchors in NS_GLOBAL_BUDGET mode over
+   the same streams ordered by sid.  The values of cost/sid are not validated
+   (device data); S * n <= 2^20. */
+NS_API ns_status ns_select_merge(ns_ctx *ctx, int S, int n, const int64_t *gain, const int32_t *rank_in,
+                                 const uint8_t *type, const int32_t *sid, const int64_t *cost, int64_t budget,
+                                 int32_t *rank, uint8_t *is_anchor, void *stream);
 
 /* SR on a host-supplied job list (jobs: HOST array [n_jobs]).  Jobs may mix
    models and resolutions; they are grouped by shape internally. */

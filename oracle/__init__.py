@@ -162,12 +162,21 @@ def psnr(a: np.ndarray, b: np.ndarray) -> float:
     return float(lib().or_psnr(_p(a), _p(b), a.size))
 
 
-def enhance_chunk(chunk, blob, B, C, k, mode=CARRY, hr_last=None, hr_golden=None, use_res_size=False):
-    """The whole hot path for one stream-chunk: score -> gain/select (top-k)
-    -> SR on anchors -> reconstruct.  Returns dict(gain, rank, is_anchor, hr,
-    hr_last, hr_golden)."""
+def enhance_chunk(chunk, blob, B, C, k, mode=CARRY, hr_last=None, hr_golden=None, use_res_size=False,
+                  selector="neuroscaler", is_anchor=None):
+    """The whole hot path for one stream-chunk: score -> gain/select (top-k;
+    selector "neuroscaler" = Alg. 1, "key" / "key_uniform" = the §3 baselines
+    of P:108; or a given anchor map) -> SR on anchors -> reconstruct.  Returns
+    dict(gain, rank, is_anchor, hr, hr_last, hr_golden)."""
     sc = score(chunk.res, chunk.res_size if use_res_size else None)
-    gain, rank, is_anchor = select_topk(list(chunk.type), [int(v) for v in sc], k, mode)
+    if is_anchor is not None:
+        gain, rank, is_anchor = None, None, [int(v) for v in is_anchor]
+    elif selector == "key":
+        gain, rank, is_anchor = select.select_key(list(chunk.type), k)
+    elif selector == "key_uniform":
+        gain, rank, is_anchor = select.select_key_uniform(list(chunk.type), k)
+    else:
+        gain, rank, is_anchor = select_topk(list(chunk.type), [int(v) for v in sc], k, mode)
     s = chunk.scale
     hr = np.zeros((chunk.n, 3, s * chunk.h, s * chunk.w), np.uint8)
     for f in range(chunk.n):

@@ -10,6 +10,8 @@ integers, no numpy arithmetic; one function per step of the paper:
   select_topk          Fig. 10 steps 1-4 for one stream
   select_global        Fig. 10 step 3-4 merged over streams + the budget
                        equation of §5.2
+  select_key           "Key SR" baseline of §3, reading R6
+  select_key_uniform   "Key+Uniform SR" baseline of §3, reading R5
 
 Readings where the paper's text is garbled or silent (SURVEY.md §8(c),
 restated in DESIGN.md): Z1 (loop counter, variable names), Z2 (CARRY is the
@@ -160,3 +162,78 @@ def select_global(streams, cost, budget, mode=CARRY):
         else:
             taking = False                        # strict prefix (Z7)
     return gains, rank, is_anchor
+
+
+def _rank_from_order(n, order, k):
+    rank = [0] * n
+    for pos, f in enumerate(order):
+        rank[f] = pos
+    return rank, [1 if rank[f] < k else 0 for f in range(n)]
+
+
+def select_key(types, k):
+    """Key SR ("applying neural super-resolution only to key frames"):
+    order = key frames ascending, then every other frame ascending; the anchors
+    are the key frames among the first k (reading R6: k = n selects every key
+    frame).  gain = KEY_GAIN for key frames, 0 otherwise."""
+    n = len(types)
+    keys = [f for f in range(n) if types[f] == KEY]
+    order = keys + [f for f in range(n) if types[f] != KEY]
+    rank, is_anchor = _rank_from_order(n, order, min(k, len(keys)))
+    gain = [KEY_GAIN if types[f] == KEY else 0 for f in range(n)]
+    return gain, rank, is_anchor
+
+
+def select_key_uniform(types, k):
+    """Key+Uniform SR ("key frames and equally-spaced normal frames"):
+    U = {floor(j * n / k) : 0 <= j < k}, the k equally spaced frames of the
+    chunk (reading R5); order = key frames ascending, then the frames of U that
+    are not key frames ascending, then the rest ascending; anchors = the first k."""
+    n = len(types)
+    U = set((j * n) // k for j in range(k)) if k > 0 else set()
+    keys = [f for f in range(n) if types[f] == KEY]
+    uni = [f for f in range(n) if types[f] != KEY and f in U]
+    rest = [f for f in range(n) if types[f] != KEY and f not in U]
+    rank, is_anchor = _rank_from_order(n, keys + uni + rest, k)
+    gain = [KEY_GAIN if types[f] == KEY else 0 for f in range(n)]
+    return gain, rank, is_anchor
+
+
+def select_global_sid(streams, sid, cost, budget, mode=CARRY):
+    """Global selection over streams gathered from several GPUs in any order
+    (ns_select_merge): the stream key of the merged order is the global stream
+    id sid[i] (reading R7), i.e. select_global over the streams sorted by sid.
+    Returns per-input-stream lists gain, rank, is_anchor."""
+    perm = sorted(range(len(streams)), key=lambda i: sid[i])
+    g, r, a = select_global([streams[i] for i in perm], [cost[i] for i in perm], budget, mode)
+    out_g, out_r, out_a = [None] * len(streams), [None] * len(streams), [None] * len(streams)
+    for pos, i in enumerate(perm):
+        out_g[i], out_r[i], out_a[i] = g[pos], r[pos], a[pos]
+    return out_g, out_r, out_a
+
+
+def merge_gathered(types, gains, sid, cost, budget):
+    """Fig. 10 steps 3-4 and the budget equation over
+    rows gathered from several GPUs (what ns_select_merge computes): types[i],
+    gains[i] per gathered stream row i (gains from Alg. 1 on the owning GPU),
+    sid[i] its global stream id (reading R7), cost[i] its T_DNN.  Order: key
+    entries by (sid, frame), then G_altref, then G_normal, each by (gain desc,
+    sid asc, frame asc); anchors = the longest prefix within budget (Z7).
+    Returns per-row lists rank, is_anchor."""
+    rows = range(len(types))
+    order = sorted(((i, f) for i in rows for f in range(len(types[i])) if types[i][f] == KEY),
+                   key=lambda e: (sid[e[0]], e[1]))
+    for grp in (ALTREF, NORMAL):
+        order += sorted(((i, f) for i in rows for f in range(len(types[i])) if types[i][f] == grp),
+                        key=lambda e: (-gains[e[0]][e[1]], sid[e[0]], e[1]))
+    rank = [[0] * len(t) for t in types]
+    is_anchor = [[0] * len(t) for t in types]
+    total, taking = 0, True
+    for pos, (i, f) in enumerate(order):
+        rank[i][f] = pos
+        if taking and total + cost[i] <= budget:
+            total += cost[i]
+            is_anchor[i][f] = 1
+        else:
+            taking = False
+    return rank, is_anchor

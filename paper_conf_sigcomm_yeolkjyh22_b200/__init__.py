@@ -22,8 +22,9 @@ LIB_PATH = os.environ.get("NS_LIB") or os.path.join(_HERE, "libneuroscaler.so")
 NS_OK, NS_EINVAL, NS_ECUDA, NS_ENOMEM, NS_EUNSUPPORTED = 0, -1, -2, -3, -4
 NS_KEY, NS_ALTREF, NS_NORMAL = 0, 1, 2
 NS_REF_LAST, NS_REF_GOLDEN, NS_REF_INTRA = 0, 1, 2
-NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET = 0, 1
+NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET, NS_GIVEN_ANCHORS = 0, 1, 2
 NS_CARRY, NS_FRESH = 0, 1
+NS_SEL_NEUROSCALER, NS_SEL_KEY, NS_SEL_KEY_UNIFORM = 0, 1, 2
 
 P = ctypes.c_void_p
 
@@ -36,7 +37,8 @@ class NsChunk(ctypes.Structure):
 
 class NsSelectParams(ctypes.Structure):
     _fields_ = [("mode", ctypes.c_int32), ("k", ctypes.c_int32), ("budget", ctypes.c_int64), ("cost", P),
-                ("group_residual", ctypes.c_int32), ("use_res_size", ctypes.c_int32)]
+                ("group_residual", ctypes.c_int32), ("use_res_size", ctypes.c_int32),
+                ("selector", ctypes.c_int32), ("reserved", ctypes.c_int32), ("anchor_in", P)]
 
 
 class NsProfEntry(ctypes.Structure):
@@ -49,7 +51,7 @@ class NsSrJob(ctypes.Structure):
 
 
 EXPORTS = ["ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_blob_len",
-           "ns_model_destroy", "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
+           "ns_model_destroy", "ns_select_anchors", "ns_select_merge", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
            "ns_enhance_streams_host", "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read"]
 
 _lib = None
@@ -77,6 +79,7 @@ def lib() -> ctypes.CDLL:
         L.ns_model_blob_len.restype = ctypes.c_size_t
         L.ns_model_destroy.argtypes = [P]
         L.ns_select_anchors.argtypes = [P, P, i32, ctypes.POINTER(NsSelectParams), P, P, P, P]
+        L.ns_select_merge.argtypes = [P, i32, i32, P, P, P, P, P, ctypes.c_int64, P, P, P]
         L.ns_sr_anchors.argtypes = [P, P, i32, P]
         L.ns_reconstruct_chunk.argtypes = [P, P, i32, P, P, P]
         L.ns_enhance_streams.argtypes = [P, P, i32, ctypes.POINTER(NsSelectParams), P, P, P, P]
@@ -90,7 +93,7 @@ def lib() -> ctypes.CDLL:
         L.ns_profile_read.argtypes = [P, i32]
         L.ns_profile_read.restype = i32
         for f in ("ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_destroy",
-                  "ns_select_anchors", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
+                  "ns_select_anchors", "ns_select_merge", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
                   "ns_enhance_streams_host"):
             getattr(L, f).restype = i32
         _lib = L
@@ -213,9 +216,12 @@ class Model:
                    "ns_model_set_weights")
 
 
-def _params(mode=NS_TOPK_PER_STREAM, k=0, budget=0, cost=None, fresh=False, use_res_size=False):
+def _params(mode=NS_TOPK_PER_STREAM, k=0, budget=0, cost=None, fresh=False, use_res_size=False,
+            selector=NS_SEL_NEUROSCALER, anchor_in=None):
     p = NsSelectParams()
     p.mode, p.k, p.budget = mode, k, budget
+    p.selector = selector
+    p.anchor_in = _ptr(anchor_in)
     keep = None
     if cost is not None:
         keep = np.ascontiguousarray(cost, np.int64)
@@ -258,6 +264,14 @@ class Context:
         _check(lib().ns_select_anchors(self.handle, arr, len(chunks), ctypes.byref(p), _ptr(gain), _ptr(rank),
                                        _ptr(is_anchor), _stream(stream)), "ns_select_anchors")
         del keep
+
+    def select_merge(self, gain, rank_in, type_, sid, cost, budget, rank, is_anchor, stream=None):
+        """ns_select_merge: global selection over streams gathered from every
+        GPU (device tensors: gain i64 / rank_in i32 / type u8 [S, n], sid i32
+        [S], cost i64 [S]; outputs rank i32 / is_anchor u8 [S, n])."""
+        S, n = int(gain.shape[0]), int(gain.shape[1])
+        _check(lib().ns_select_merge(self.handle, S, n, _ptr(gain), _ptr(rank_in), _ptr(type_), _ptr(sid), _ptr(cost),
+                                     int(budget), _ptr(rank), _ptr(is_anchor), _stream(stream)), "ns_select_merge")
 
     def sr_anchors(self, jobs, stream=None):
         """jobs: list of (model, lr [3,h,w] u8 tensor, hr_out [3,sh,sw] u8 tensor)."""

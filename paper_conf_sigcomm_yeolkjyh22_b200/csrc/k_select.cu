@@ -74,8 +74,8 @@ cudaError_t launch_score(const StreamDesc *d_sd, int S, int n, int max_frame_vec
 //     f by (group, gain desc, frame asc); is_anchor = rank < k.
 constexpr int kSelWarps = 4;
 __global__ void __launch_bounds__(kSelWarps * 32)
-    k_select(const StreamDesc *sd, const int64_t *score, int S, int n, int k, int fresh, int64_t *gain_out,
-             int32_t *rank_out, uint8_t *anchor_out, int32_t *order_out) {
+    k_select(const StreamDesc *sd, const int64_t *score, int S, int n, int k, int fresh, int selector,
+             int64_t *gain_out, int32_t *rank_out, uint8_t *anchor_out, int32_t *order_out) {
     __shared__ int64_t sR[kSelWarps][kMaxFrames];
     __shared__ int64_t sG[kSelWarps][kMaxFrames];
     __shared__ int16_t sNR[kSelWarps][kMaxFrames];
@@ -139,10 +139,32 @@ __global__ void __launch_bounds__(kSelWarps * 32)
             __syncwarp();
         }
     };
-    calc_residual();
-    estimate_gain(NS_ALTREF);
-    if (fresh) calc_residual();
-    estimate_gain(NS_NORMAL);
+    if (selector == NS_SEL_NEUROSCALER) {
+        calc_residual();
+        estimate_gain(NS_ALTREF);
+        if (fresh) calc_residual();
+        estimate_gain(NS_NORMAL);
+    } else {
+        // The real-time baselines of §3.  Frames are re-classed so the
+        // rank rule below orders them (class, frame): 0 = key, 1 = the equally
+        // spaced frames U = {floor(j n / k)} (Key+Uniform, reading R5; f is in U
+        // iff j = ceil(f k / n) < k has floor(j n / k) = f), 2 = the rest.
+        int nkey = 0;
+        for (int f = lane; f < n; f += 32) {
+            int cls = 2;
+            if (T[f] == NS_KEY) {
+                cls = 0;
+                nkey++;
+            } else if (selector == NS_SEL_KEY_UNIFORM && k > 0) {
+                const int j = (f * k + n - 1) / n;
+                if (j < k && (j * n) / k == f) cls = 1;
+            }
+            T[f] = (uint8_t)cls;
+        }
+        nkey = __reduce_add_sync(0xffffffffu, nkey);
+        if (selector == NS_SEL_KEY && k > nkey) k = nkey;  // Key SR: key frames only (reading R6)
+        __syncwarp();
+    }
     for (int f = lane; f < n; f += 32) {
         int cnt = 0;
         const int tf = T[f];
@@ -161,10 +183,11 @@ __global__ void __launch_bounds__(kSelWarps * 32)
 }
 
 cudaError_t launch_select(const StreamDesc *d_sd, const int64_t *score, int S, int n, int k, int fresh,
-                          int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order, cudaStream_t st) {
+                          int selector, int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order,
+                          cudaStream_t st) {
     KScope ks(F_SELECT, st);
-    k_select<<<(S + kSelWarps - 1) / kSelWarps, kSelWarps * 32, 0, st>>>(d_sd, score, S, n, k, fresh, gain, rank,
-                                                                        is_anchor, order);
+    k_select<<<(S + kSelWarps - 1) / kSelWarps, kSelWarps * 32, 0, st>>>(d_sd, score, S, n, k, fresh, selector,
+                                                                        gain, rank, is_anchor, order);
     return cudaGetLastError();
 }
 
@@ -173,17 +196,25 @@ cudaError_t launch_select(const StreamDesc *d_sd, const int64_t *score, int S, i
 // G_normal, each by (gain desc, stream asc, frame asc): its rank inside its own
 // stream plus, for every other stream, a binary search in that stream's
 // sorted order for the entries that precede it.
-__global__ void k_global_rank(const StreamDesc *sd, int S, int n, const int64_t *gain, const int32_t *order,
-                              const int32_t *rank_in, int32_t *grank, int32_t *pos_stream) {
+// FLAT (ns_select_merge): types from a gathered [S][n] array and the stream key
+// sid[s] (global stream ids of the streams of every GPU, reading R7).
+template <bool FLAT>
+__global__ void k_global_rank(const StreamDesc *sd, const uint8_t *type_flat, const int32_t *sid, int S, int n,
+                              const int64_t *gain, const int32_t *order, const int32_t *rank_in, int32_t *grank,
+                              int32_t *pos_stream) {
     const int e = blockIdx.x * blockDim.x + threadIdx.x;
     if (e >= S * n) return;
     const int s = e / n, f = e % n;
-    const int t = sd[s].type[f];
+    auto types = [&](int q) -> const uint8_t * { return FLAT ? type_flat + (size_t)q * n : sd[q].type; };
+    auto key = [&](int q) -> int { return FLAT ? sid[q] : q; };
+    const int t = types(s)[f];
+    const int ks = key(s);
     const int64_t g = gain[e];
     int cnt = rank_in[e];
     for (int s2 = 0; s2 < S; s2++) {
         if (s2 == s) continue;
-        const uint8_t *T2 = sd[s2].type;
+        const uint8_t *T2 = types(s2);
+        const int k2 = key(s2);
         const int32_t *O2 = order + (size_t)s2 * n;
         const int64_t *G2 = gain + (size_t)s2 * n;
         int lo = 0, hi = n;  // first position whose entry does NOT precede (s, f)
@@ -192,7 +223,7 @@ __global__ void k_global_rank(const StreamDesc *sd, int S, int n, const int64_t 
             const int f2 = O2[mid];
             const int t2 = T2[f2];
             const int64_t g2 = G2[f2];
-            const bool prec = (t2 < t) || (t2 == t && (g2 > g || (g2 == g && s2 < s)));
+            const bool prec = (t2 < t) || (t2 == t && (g2 > g || (g2 == g && k2 < ks)));
             if (prec) lo = mid + 1;
             else hi = mid;
         }
@@ -200,6 +231,14 @@ __global__ void k_global_rank(const StreamDesc *sd, int S, int n, const int64_t 
     }
     grank[e] = cnt;
     pos_stream[cnt] = s;
+}
+
+// order[s][rank_in[s][f]] = f: the per-stream priority order from the ranks.
+__global__ void k_order_from_rank(int N, int n, const int32_t *rank_in, int32_t *order) {
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= N) return;
+    const int s = e / n;
+    order[(size_t)s * n + rank_in[e]] = e % n;
 }
 
 // Longest prefix of the global order whose summed cost stays <= budget
@@ -243,7 +282,21 @@ cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *g
     KScope ks(F_GLOBAL, st, 3);
     const int N = S * n;
     // rank currently holds the per-stream rank (written by k_select)
-    k_global_rank<<<(N + 255) / 256, 256, 0, st>>>(d_sd, S, n, gain, order, rank, grank, pos_stream);
+    k_global_rank<false><<<(N + 255) / 256, 256, 0, st>>>(d_sd, nullptr, nullptr, S, n, gain, order, rank, grank,
+                                                           pos_stream);
+    k_global_cut<<<1, 1024, 0, st>>>(N, pos_stream, cost, budget, cut);
+    k_global_mark<<<(N + 255) / 256, 256, 0, st>>>(N, grank, cut, rank, is_anchor);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_merge(int S, int n, const int64_t *gain, const int32_t *rank_in, const uint8_t *type,
+                         const int32_t *sid, const int64_t *cost, int64_t budget, int32_t *order, int32_t *grank,
+                         int32_t *pos_stream, int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st) {
+    KScope ks(F_GLOBAL, st, 4);
+    const int N = S * n;
+    k_order_from_rank<<<(N + 255) / 256, 256, 0, st>>>(N, n, rank_in, order);
+    k_global_rank<true><<<(N + 255) / 256, 256, 0, st>>>(nullptr, type, sid, S, n, gain, order, rank_in, grank,
+                                                          pos_stream);
     k_global_cut<<<1, 1024, 0, st>>>(N, pos_stream, cost, budget, cut);
     k_global_mark<<<(N + 255) / 256, 256, 0, st>>>(N, grank, cut, rank, is_anchor);
     return cudaGetLastError();
@@ -263,8 +316,10 @@ __global__ void k_compact(const StreamDesc *sd, int S, int n, const uint8_t *is_
     int local = 0;
     for (int f = 0; f < n; f++) {
         if (!is_anchor[(size_t)s * n + f]) continue;
-        const int slot = topk ? d.job_base + local : d.job_base + atomicAdd(&job_count[d.group], 1);
+        const int claim = topk ? local : atomicAdd(&job_count[d.group], 1);
         local++;
+        if (claim >= d.job_cap) continue;  // over the bound of a given anchor map: dropped (ns.h)
+        const int slot = d.job_base + claim;
         SrJob j;
         j.lr = d.lr + f * lr_frame;
         j.hr = hr_tab[d.hr_base + f];

@@ -458,7 +458,8 @@ struct Staged {
 static size_t a256(size_t v) { return (v + 255) / 256 * 256; }
 
 static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint8_t *const *hr, const int64_t *cost,
-                               const int *group, const int *job_base, bool use_res_size, Staged *out) {
+                               const int *group, const int *job_base, bool use_res_size, Staged *out,
+                               const int *job_cap = nullptr) {
     Staged g{};
     ns_status r = stage_begin(c, &g.host, &g.dev, &g.slot);
     if (r != NS_OK) return r;
@@ -478,6 +479,7 @@ static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint
         d.hr_base = s * n;
         d.group = group ? group[s] : 0;
         d.job_base = job_base ? job_base[s] : 0;
+        d.job_cap = job_cap ? job_cap[s] : INT32_MAX;
         d.use_res_size = use_res_size ? 1 : 0;
         sd[s] = d;
     }
@@ -502,10 +504,17 @@ static ns_status check_params(const ns_select_params *p, int S, int n) {
     if (!p) return fail(NS_EINVAL, "params is NULL");
     if (p->group_residual != NS_CARRY && p->group_residual != NS_FRESH)
         return fail(NS_EINVAL, "group_residual %d invalid", p->group_residual);
+    if (p->selector != NS_SEL_NEUROSCALER && p->selector != NS_SEL_KEY && p->selector != NS_SEL_KEY_UNIFORM)
+        return fail(NS_EINVAL, "selector %d invalid", p->selector);
+    if (p->mode != NS_TOPK_PER_STREAM && p->selector != NS_SEL_NEUROSCALER)
+        return fail(NS_EINVAL, "the baseline selectors are top-k only");
+    if (p->mode != NS_GIVEN_ANCHORS && p->anchor_in)
+        return fail(NS_EINVAL, "anchor_in is only read in NS_GIVEN_ANCHORS mode");
     if (p->mode == NS_TOPK_PER_STREAM) {
         if (p->k < 0 || p->k > n) return fail(NS_EINVAL, "k = %d not in [0, n = %d]", p->k, n);
-    } else if (p->mode == NS_GLOBAL_BUDGET) {
-        if (!p->cost) return fail(NS_EINVAL, "global mode needs cost[S]");
+    } else if (p->mode == NS_GLOBAL_BUDGET || p->mode == NS_GIVEN_ANCHORS) {
+        if (p->mode == NS_GIVEN_ANCHORS && !p->anchor_in) return fail(NS_EINVAL, "given mode needs anchor_in");
+        if (!p->cost) return fail(NS_EINVAL, "global / given mode needs cost[S]");
         if (p->budget < 0) return fail(NS_EINVAL, "budget < 0");
         for (int s = 0; s < S; s++)
             if (p->cost[s] < 1) return fail(NS_EINVAL, "cost[%d] = %lld < 1", s, (long long)p->cost[s]);
@@ -521,9 +530,14 @@ static ns_status run_select(ns_ctx *c, const Staged &g, const ns_chunk *ch, int 
     int maxv = 0;
     for (int s = 0; s < S; s++) maxv = std::max(maxv, 3 * ch[s].h * ch[s].w / 8);
     NS_CUDA(launch_score(g.d_sd, S, n, maxv, c->score, st));
+    if (p->mode == NS_GIVEN_ANCHORS) {  // decided by ns_select_merge across GPUs
+        if (is_anchor != p->anchor_in)
+            NS_CUDA(cudaMemcpyAsync(is_anchor, p->anchor_in, (size_t)S * n, cudaMemcpyDeviceToDevice, st));
+        return NS_OK;
+    }
     const bool global = p->mode == NS_GLOBAL_BUDGET;
-    NS_CUDA(launch_select(g.d_sd, c->score, S, n, global ? -1 : p->k, p->group_residual == NS_FRESH, gain, rank,
-                          is_anchor, global ? c->order : nullptr, st));
+    NS_CUDA(launch_select(g.d_sd, c->score, S, n, global ? -1 : p->k, p->group_residual == NS_FRESH, p->selector,
+                          gain, rank, is_anchor, global ? c->order : nullptr, st));
     if (global)
         NS_CUDA(launch_global(g.d_sd, S, n, gain, c->order, g.d_cost, p->budget, c->grank, c->pos_stream, c->cut,
                               rank, is_anchor, st));
@@ -537,6 +551,7 @@ extern "C" ns_status ns_select_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
     ns_status r = check_chunks(ch, S, false, &n);
     if (r != NS_OK) return r;
     if ((r = check_params(p, S, n)) != NS_OK) return r;
+    if (p->mode == NS_GIVEN_ANCHORS) return fail(NS_EINVAL, "ns_select_anchors: NS_GIVEN_ANCHORS selects nothing");
     if (!gain || !rank || !is_anchor) return fail(NS_EINVAL, "ns_select_anchors: outputs must be non-NULL");
     cudaStream_t st = (cudaStream_t)stream;
     NS_CUDA(cudaSetDevice(c->device));
@@ -548,6 +563,21 @@ extern "C" ns_status ns_select_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
     r = run_select(c, g, ch, S, n, p, gain, rank, is_anchor, st);
     stage_release(c, g.slot, st);
     return r;
+}
+
+extern "C" ns_status ns_select_merge(ns_ctx *c, int S, int n, const int64_t *gain, const int32_t *rank_in,
+                                     const uint8_t *type, const int32_t *sid, const int64_t *cost, int64_t budget,
+                                     int32_t *rank, uint8_t *is_anchor, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_select_merge: ctx is NULL");
+    if (S < 1 || n < 1 || n > kMaxFrames) return fail(NS_EINVAL, "ns_select_merge: S = %d, n = %d", S, n);
+    if ((size_t)S * n > (size_t)kMaxSN) return fail(NS_EINVAL, "S * n = %zu exceeds %d", (size_t)S * n, kMaxSN);
+    if (budget < 0) return fail(NS_EINVAL, "budget < 0");
+    if (!gain || !rank_in || !type || !sid || !cost || !rank || !is_anchor)
+        return fail(NS_EINVAL, "ns_select_merge: NULL array");
+    NS_CUDA(cudaSetDevice(c->device));
+    NS_CUDA(launch_merge(S, n, gain, rank_in, type, sid, cost, budget, c->order, c->grank, c->pos_stream, c->cut, rank,
+                         is_anchor, (cudaStream_t)stream));
+    return NS_OK;
 }
 
 // ------------------------------------------------------------------ SR
@@ -669,6 +699,9 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
                               uint8_t *const *hr_out, uint8_t *anchor, double *stats, cudaStream_t st,
                               const LrGather *lg, uint64_t *gathered) {
     const bool topk = p->mode == NS_TOPK_PER_STREAM;
+    // exactly k anchors per stream -> fixed job slots; otherwise (budget, given
+    // map, Key SR with fewer key frames than k) slots are claimed per group
+    const bool fixed = topk && p->selector != NS_SEL_KEY;
     // SR shape groups and job slots (multi-stream batcher)
     std::map<std::tuple<int, int, int, int, int>, int> gid;
     std::vector<std::tuple<int, int, int, int, int>> gkey;
@@ -706,19 +739,21 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
         std::vector<int> local(G, 0);
         for (int s = 0; s < S; s++) {
             const int gi = group[s];
-            job_base[s] = topk ? goff[gi] + local[gi]++ * p->k : goff[gi];
+            job_base[s] = fixed ? goff[gi] + local[gi]++ * p->k : goff[gi];
         }
     }
     if (gathered && lg) {  // exact in top-k mode (k frames per stream); upper bound otherwise
         uint64_t b = 0;
-        for (int s = 0; s < S; s++) b += (uint64_t)3 * ch[s].h * ch[s].w * (topk ? p->k : 0);
-        if (!topk) b = (uint64_t)total * lg->stride;
+        for (int s = 0; s < S; s++) b += (uint64_t)3 * ch[s].h * ch[s].w * (fixed ? p->k : 0);
+        if (!fixed) b = (uint64_t)total * lg->stride;
         *gathered += b;
     }
     Staged g;
     ns_status r;
+    std::vector<int> job_cap(S);
+    for (int s = 0; s < S; s++) job_cap[s] = fixed ? p->k : gcount[group[s]];
     if ((r = stage_streams(c, ch, S, n, hr_out, topk ? nullptr : p->cost, group.data(), job_base.data(),
-                           p->use_res_size != 0, &g)) != NS_OK)
+                           p->use_res_size != 0, &g, job_cap.data())) != NS_OK)
         return r;
     if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
     do {
@@ -727,14 +762,15 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
             cudaError_t e = cudaSuccess;
             if (lg) e = cudaMemsetAsync(c->lr_len, 0, sizeof(uint32_t) * total, st);
             if (e == cudaSuccess)
-                e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, topk, p->k, st,
+                e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, fixed, p->k, st,
                                    lg ? lg->stage : nullptr, lg ? lg->stride : 0, c->lr_src, c->lr_len);
             if (e == cudaSuccess && lg) e = launch_lr_gather(c->jobs, c->lr_src, c->lr_len, total, lg->stride, st);
             if (e != cudaSuccess) { r = cuda_fail(e, "compact"); break; }
             for (int gi = 0; gi < G && r == NS_OK; gi++) {
                 int h, w, C, s, B;
                 std::tie(h, w, C, s, B) = gkey[gi];
-                r = run_sr_group(c, h, w, C, s, B, c->jobs + goff[gi], gcount[gi], topk ? nullptr : c->job_count + gi, st);
+                r = run_sr_group(c, h, w, C, s, B, c->jobs + goff[gi], gcount[gi], fixed ? nullptr : c->job_count + gi,
+                                 st);
             }
             if (r != NS_OK) break;
         }

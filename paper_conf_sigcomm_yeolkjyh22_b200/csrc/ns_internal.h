@@ -27,6 +27,7 @@ struct StreamDesc {
     int32_t hr_base;       // index of hr_out[s][0] in the device hr table
     int32_t group;         // SR shape group index (ns_enhance_streams)
     int32_t job_base;      // first SR job slot of this stream in its group
+    int32_t job_cap;       // slots of its group (budget / given modes: claims beyond are dropped)
     int32_t use_res_size;
 };
 
@@ -95,7 +96,12 @@ CompShape model_comp(int n_blocks, int C, int s);
 cudaError_t launch_score(const StreamDesc *d_sd, int S, int n, int max_frame_vec8, int64_t *score,
                          cudaStream_t st);
 cudaError_t launch_select(const StreamDesc *d_sd, const int64_t *score, int S, int n, int k, int fresh,
-                          int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order, cudaStream_t st);
+                          int selector, int64_t *gain, int32_t *rank, uint8_t *is_anchor, int32_t *order,
+                          cudaStream_t st);
+// ns_select_merge: global selection over gathered [S][n] gain / rank / type arrays.
+cudaError_t launch_merge(int S, int n, const int64_t *gain, const int32_t *rank_in, const uint8_t *type,
+                         const int32_t *sid, const int64_t *cost, int64_t budget, int32_t *order, int32_t *grank,
+                         int32_t *pos_stream, int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st);
 cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *gain, const int32_t *order,
                           const int64_t *cost, int64_t budget, int32_t *grank, int32_t *pos_stream,
                           int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st);

@@ -68,3 +68,59 @@ def gather_stats(stats, group=None):
     parts = [torch.zeros_like(stats) for _ in range(dist.get_world_size(group))]
     dist.all_gather(parts, stats.contiguous(), group=group)
     return torch.cat(parts)
+
+
+# ---------------------------------------------------------------- NEXT-1: global selection across GPUs
+def gather_rows(tensors, group=None):
+    """all_gather of per-rank tensors whose first dimension (streams) differs
+    between ranks: every tensor is padded to the largest S_r, gathered, and the
+    valid rows concatenated rank-major.  Returns (gathered tensors, row offset
+    of this rank).  One small exchange per chunk (<= 30k
+    entries); NCCL on GPUs, gloo on CPU.  Data movement only."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return list(tensors), 0
+    world, me = dist.get_world_size(group), dist.get_rank(group)
+    dev = tensors[0].device
+    cnt = torch.tensor([tensors[0].shape[0]], dtype=torch.int64, device=dev)
+    cnts = [torch.zeros_like(cnt) for _ in range(world)]
+    dist.all_gather(cnts, cnt, group=group)
+    cnts = [int(c.item()) for c in cnts]
+    smax = max(cnts)
+    out = []
+    for t in tensors:
+        pad = torch.zeros((smax,) + tuple(t.shape[1:]), dtype=t.dtype, device=dev)
+        pad[: t.shape[0]] = t
+        parts = [torch.empty_like(pad) for _ in range(world)]
+        dist.all_gather(parts, pad, group=group)
+        out.append(torch.cat([p[:c] for p, c in zip(parts, cnts)]))
+    return out, sum(cnts[:me])
+
+
+def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_res_size=False, group=None,
+                               stream=None):
+    """§5.2 global anchor selection over the streams of every GPU:
+    (1) per-stream gains and ranks on this GPU (ns_select_anchors, Alg. 1);
+    (2) all_gather of gain / rank / type / sid / cost rows (gather_rows);
+    (3) ns_select_merge on the gathered rows -- the identical deterministic
+    prefix on every GPU, no further exchange.  Returns this GPU's is_anchor
+    [S_local, n] (device u8) for ns_enhance_streams(mode=NS_GIVEN_ANCHORS,
+    anchor_in=..., cost=cost, budget=budget), and the global rank rows."""
+    import torch
+    from . import NS_TOPK_PER_STREAM
+    S, n = len(chunks), chunks[0].n
+    dev = chunks[0].type.device
+    gain = torch.empty((S, n), dtype=torch.int64, device=dev)
+    rank = torch.empty((S, n), dtype=torch.int32, device=dev)
+    anc = torch.empty((S, n), dtype=torch.uint8, device=dev)
+    ctx.select_anchors(chunks, gain, rank, anc, stream=stream, mode=NS_TOPK_PER_STREAM, k=0, fresh=fresh,
+                       use_res_size=use_res_size)
+    types = torch.stack([c.type for c in chunks])
+    sid_t = torch.as_tensor(list(sid), dtype=torch.int32).to(dev)
+    cost_t = torch.as_tensor(list(cost), dtype=torch.int64).to(dev)
+    (g_all, r_all, t_all, s_all, c_all), off = gather_rows([gain, rank, types, sid_t, cost_t], group)
+    rank_out = torch.empty_like(r_all)
+    anc_all = torch.empty_like(t_all)
+    ctx.select_merge(g_all, r_all, t_all, s_all, c_all, budget, rank_out, anc_all, stream=stream)
+    return anc_all[off: off + S].contiguous(), rank_out[off: off + S].contiguous()

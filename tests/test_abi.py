@@ -64,6 +64,7 @@ def test_invalid_args_no_launch(nslib):
     assert "NULL" in nslib.last_error()
     assert L.ns_reconstruct_chunk(None, None, 1, None, None, None) == nslib.NS_EINVAL
     assert L.ns_sr_anchors(None, None, 1, None) == nslib.NS_EINVAL
+    assert L.ns_select_merge(None, 1, 1, None, None, None, None, None, 0, None, None, None) == nslib.NS_EINVAL
     assert L.ns_model_destroy(None) == nslib.NS_EINVAL
     del h
     assert nslib.launch_count() == before

@@ -65,3 +65,62 @@ def test_gloo_world2_gather_and_max():
         assert t.shape == (6, 8)
         assert t[:3, 0].tolist() == [0.0, 1.0, 2.0] and t[3:, 0].tolist() == [10.0, 11.0, 12.0]
         assert (t[3:, 1:] == 1.0).all() and (t[:3, 1:] == 0.0).all()
+
+
+# ---------------------------------------------------------------- NEXT-1 host logic (gloo, world 2)
+def _merge_worker(rank, world, port, q):
+    """Each rank owns an unequal, interleaved subset of 7 streams; it computes
+    its streams' gains with the oracle (standing in for ns_select_anchors),
+    gathers the rows with shard.gather_rows, and runs the oracle merge on the
+    gathered rows.  Every rank must get the selection of select_global over
+    all streams, and its own rows at the returned offset."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from oracle import select as S
+        streams, cost = _merge_streams()
+        mine = [i for i in range(len(streams)) if (i % 3 == 0) == (rank == 0)]   # 3 vs 4 streams
+        n = len(streams[0][0])
+        gain = torch.tensor([S.select_topk(*streams[i], 0)[0] for i in mine], dtype=torch.int64)
+        rk = torch.tensor([S.select_topk(*streams[i], 0)[1] for i in mine], dtype=torch.int32)
+        ty = torch.tensor([streams[i][0] for i in mine], dtype=torch.uint8)
+        sid = torch.tensor(mine, dtype=torch.int32)
+        co = torch.tensor([cost[i] for i in mine], dtype=torch.int64)
+        (g, r, t, s, c), off = shard.gather_rows([gain, rk, ty, sid, co])
+        assert g.shape == (len(streams), n) and t.dtype == torch.uint8
+        _, a = S.merge_gathered(t.tolist(), g.tolist(), s.tolist(), c.tolist(), 9)
+        q.put((rank, s.tolist(), off, len(mine), a, g.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+def _merge_streams():
+    import random
+    rng = random.Random(3)
+    from oracle import select as S
+    streams = []
+    for _ in range(7):
+        types = [S.KEY] + [rng.choice((S.NORMAL, S.NORMAL, S.ALTREF)) for _ in range(9)]
+        streams.append((types, [rng.randint(1, 50) for _ in range(10)]))
+    return streams, [rng.randint(1, 3) for _ in range(7)]
+
+
+def test_gloo_world2_global_selection_rows():
+    from oracle import select as S
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_merge_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    streams, cost = _merge_streams()
+    gains_all, _, anc_all = S.select_global(streams, cost, 9)
+    (r0, sid0, off0, n0, a0, g0), (r1, sid1, off1, n1, a1, g1) = res
+    assert sid0 == sid1 == [0, 3, 6, 1, 2, 4, 5]          # rank-major rows, unequal counts
+    assert (off0, n0, off1, n1) == (0, 3, 3, 4)
+    assert g0 == g1 == [gains_all[i] for i in sid0]         # gathered gains are every stream's
+    assert a0 == a1 == [anc_all[i] for i in sid0]           # = global selection over all streams
