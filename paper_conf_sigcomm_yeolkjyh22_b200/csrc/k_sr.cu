@@ -364,6 +364,33 @@ __device__ __forceinline__ void tmem_zero(uint32_t taddr) {
                 taddr), "r"(0u) : "memory");
     }
 }
+// Stores 32 / 16 per-column values (the same for every lane of the warp's quarter).
+template <int NB>
+__device__ __forceinline__ void tmem_st_vals(uint32_t taddr, const float (&b)[NB]) {
+#define NS_F(i) "f"(b[i])
+    if constexpr (NB == 32) {
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+            "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+            NS_F(0), NS_F(1), NS_F(2), NS_F(3), NS_F(4), NS_F(5), NS_F(6), NS_F(7), NS_F(8), NS_F(9), NS_F(10),
+            NS_F(11), NS_F(12), NS_F(13), NS_F(14), NS_F(15), NS_F(16), NS_F(17), NS_F(18), NS_F(19), NS_F(20),
+            NS_F(21), NS_F(22), NS_F(23), NS_F(24), NS_F(25), NS_F(26), NS_F(27), NS_F(28), NS_F(29), NS_F(30),
+            NS_F(31) : "memory");
+    } else {
+        static_assert(NB == 16, "");
+        asm volatile(
+            "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::
+                "r"(taddr), NS_F(0), NS_F(1), NS_F(2), NS_F(3), NS_F(4), NS_F(5), NS_F(6), NS_F(7), NS_F(8), NS_F(9),
+            NS_F(10), NS_F(11), NS_F(12), NS_F(13), NS_F(14), NS_F(15) : "memory");
+    }
+#undef NS_F
+}
+// ReLU + round-to-nearest bf16 of a pair, one instruction: low half = lo.
+__device__ __forceinline__ uint32_t pack_bf16_relu(float lo, float hi) {
+    uint32_t r;
+    asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+    return r;
+}
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 __device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
@@ -601,6 +628,50 @@ struct RbCfg {
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+__device__ __forceinline__ void named_bar_sync(int id, int n) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+// Epilogue-group synchronisation of the fused res-block.  Every mbarrier poll
+// and arrive is a shared-memory access, and a sleeping waiter re-polls on every
+// barrier update of the CTA: with 128 threads arriving and 4 warps polling per
+// group, ncu counted ~23M SYNCS polls per launch, ~18% of all shared-memory
+// wavefronts of a kernel that is shared-memory-bandwidth bound (the MMA operand
+// reads take the rest).  NS_RB_ARRIVE1: one arrive per warp (counts 4), after
+// __syncwarp.  NS_RB_GWAIT: one warp of the group polls, the group follows on a
+// named barrier (no shared-memory traffic).  A/B on B200 (tools/ab_libs.sh,
+// body ms per c4 step): neither 104.5, ARRIVE1 105.4, GWAIT 108.1, both 110:
+// the polls do not compete with the operand reads enough to matter, and the
+// named-barrier hop lengthens the epilogue chain -- both off.
+// NS_RB_BIAS_INIT: a retired accumulator block is re-initialised with the
+// conv's bias instead of zero, so the epilogues add no bias (E1 becomes one
+// cvt.rn.relu.bf16x2 per channel pair).
+#ifndef NS_RB_BIAS_INIT
+#define NS_RB_BIAS_INIT 1
+#endif
+#ifndef NS_RB_ARRIVE1
+#define NS_RB_ARRIVE1 0
+#endif
+#ifndef NS_RB_GWAIT
+#define NS_RB_GWAIT 0
+#endif
+constexpr uint32_t kRbArriveCount = NS_RB_ARRIVE1 ? 4 : 128;
+__device__ __forceinline__ void rb_arrive(uint64_t *bar) {
+#if NS_RB_ARRIVE1
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) mbar_arrive(bar);
+#else
+    mbar_arrive(bar);
+#endif
+}
+__device__ __forceinline__ void rb_group_wait(uint64_t *bar, uint32_t phase, int group) {
+#if NS_RB_GWAIT
+    if (((threadIdx.x >> 5) & 3) == 0) mbar_wait(bar, phase);
+    named_bar_sync(1 + group, 128);
+#else
+    (void)group;
+    mbar_wait(bar, phase);
+#endif
+}
 
 // Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-17 = four
 // epilogue groups (tile 0 E1, tile 0 E2, tile 1 E1, tile 1 E2); warp w owns
@@ -653,12 +724,12 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
     if (tid == 0) {
         for (int k = 0; k < 2; k++) {
             for (int i = 0; i < NH; i++) mbar_init(hfull(k, i), 1);
-            for (int i = 0; i < NH; i++) mbar_init(hfree(k, i), 128);
+            for (int i = 0; i < NH; i++) mbar_init(hfree(k, i), kRbArriveCount);
             mbar_init(m1bar(k), 1);
             mbar_init(m2bar(k), 1);
-            mbar_init(e1z(k), 128);
-            mbar_init(e2z(k), 128);
-            for (int i = 0; i < 4; i++) mbar_init(e1t(k, i), 128);
+            mbar_init(e1z(k), kRbArriveCount);
+            mbar_init(e2z(k), kRbArriveCount);
+            for (int i = 0; i < 4; i++) mbar_init(e1t(k, i), kRbArriveCount);
             for (int i = 0; i < Cfg::NTS; i++) mbar_init(tfree(k, i), 1);
         }
         mbar_init(wbar, 1);
@@ -790,13 +861,13 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
             if (role == 0) {
                 for (int q = 0; q < nq; q++) {  // E1: t = ReLU(conv1 + b1) -> t slot
                     const int yt = y0 - 3 + q;
-                    mbar_wait(m1bar(k), q & 1);
+                    rb_group_wait(m1bar(k), q & 1, g);
                     if (warp % 4 == 2 && lane == 0) NS_TR(10 + k, q);
                     tc_fence_after();
 #ifdef NS_TRACE_NOEPI
                     tc_fence_before();
-                    mbar_arrive(e1z(k));
-                    mbar_arrive(e1t(k, q & 3));
+                    rb_arrive(e1z(k));
+                    rb_arrive(e1t(k, q & 3));
                     continue;
 #endif
                     const uint32_t acc = tl + (uint32_t)(mod3(yt) * NB);
@@ -804,22 +875,41 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
                     if (warp % 4 == 2 && lane == 0) NS_TR(40 + k, q);
+#if NS_RB_BIAS_INIT
+                    // the retired block becomes row yt+3's: it starts at b1, so the
+                    // epilogue adds no bias (the first three rows retire blocks zeroed at
+                    // allocation and add it here)
+                    if (q < 3) {
+#pragma unroll
+                        for (int i = 0; i < NB; i++) v[i] = __float_as_uint(__uint_as_float(v[i]) + bias[i]);
+                    }
+                    tmem_st_vals<NB>(acc, bias);
+                    tmem_wait_st();
+#else
 #ifndef NS_TRACE_NOZERO
                     tmem_zeroN<NB>(acc);
                     tmem_wait_st();
 #endif
+#endif
 
                     tc_fence_before();
-                    mbar_arrive(e1z(k));  // the next conv1 group may start
+                    rb_arrive(e1z(k));  // the next conv1 group may start
                     // t slot q%2 was last read by M2(q-2) (another warp's MMAs): completion
                     // #((q-4)/2) of tfree[q%2]; M2(q-4) is done, M2(q) cannot be -> exact
-                    if (q >= 2 + Cfg::NTS) mbar_wait(tfree(k, q % Cfg::NTS), ((q - Cfg::NTS - 2) / Cfg::NTS) & 1);
+                    if (q >= 2 + Cfg::NTS) rb_group_wait(tfree(k, q % Cfg::NTS), ((q - Cfg::NTS - 2) / Cfg::NTS) & 1, g);
                     if (q >= 2) {
                         const int xt = x0k(k) - 1 + p;
                         const bool inside = yt >= 0 && yt < a.H && xt >= 0 && xt < a.W;
                         uint8_t *ts = tslot(k, q % Cfg::NTS);
 #pragma unroll
                         for (int cg = 0; cg < NB / 8; cg++) {
+#if NS_RB_BIAS_INIT
+                            const uint32_t *w = v + cg * 8;
+                            auto pr = [&](int i) {
+                                return inside ? pack_bf16_relu(__uint_as_float(w[i]), __uint_as_float(w[i + 1])) : 0u;
+                            };
+                            const uint4 o = make_uint4(pr(0), pr(2), pr(4), pr(6));
+#else
                             float f[8];
 #pragma unroll
                             for (int i = 0; i < 8; i++)
@@ -827,38 +917,46 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                             uint4 o;
                             o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
                             o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
+#endif
                             *reinterpret_cast<uint4 *>(ts + cg * kHalo * 16 + p * 16) = o;
                         }
                     }
                     if (warp % 4 == 2 && lane == 0) NS_TR(42 + k, q);
                     fence_proxy_async_smem();
                     if (warp % 4 == 2 && lane == 0) NS_TR(46 + k, q);
-                    mbar_arrive(e1t(k, q & 3));
+                    rb_arrive(e1t(k, q & 3));
                     if (warp % 4 == 2 && lane == 0) NS_TR(12 + k, q);
                 }
             } else {
                 for (int q = 2; q < nq; q++) {  // E2: out = conv2 + b2 + h
                     const int yo = y0 - 4 + q;
-                    mbar_wait(m2bar(k), (q - 2) & 1);
+                    rb_group_wait(m2bar(k), (q - 2) & 1, g);
                     if (warp % 4 == 2 && lane == 0) NS_TR(20 + k, q);
                     tc_fence_after();
 #ifdef NS_TRACE_NOEPI
                     tc_fence_before();
-                    mbar_arrive(hfree(k, (q - 2) % NH));
-                    mbar_arrive(e2z(k));
+                    rb_arrive(hfree(k, (q - 2) % NH));
+                    rb_arrive(e2z(k));
                     continue;
 #endif
                     const uint32_t acc = tl + 3 * NB + (uint32_t)(mod3(yo) * NB);
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
+#if NS_RB_BIAS_INIT
+                    const bool addb = q < 5;  // first three retirements: blocks zeroed at allocation
+                    tmem_st_vals<NB>(acc, bias);
+                    tmem_wait_st();
+#else
+                    constexpr bool addb = true;
 #ifndef NS_TRACE_NOZERO
                     tmem_zeroN<NB>(acc);
                     tmem_wait_st();
 #endif
+#endif
 
                     tc_fence_before();
-                    mbar_arrive(e2z(k));  // the next conv2 group may start
+                    rb_arrive(e2z(k));  // the next conv2 group may start
                     const int x = x0k(k) + p;
                     if (yo >= y0 && yo < y1 && p < kRbOut && x < a.W) {
                         const uint8_t *hs = hslot(k, (q - 2) % NH);  // h row yo (step q-2)
@@ -868,7 +966,8 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                             const uint4 rr = *reinterpret_cast<const uint4 *>(hs + cg * kHalo * 16 + (p + 2) * 16);
                             float f[8];
 #pragma unroll
-                            for (int i = 0; i < 8; i++) f[i] = __uint_as_float(v[cg * 8 + i]) + bias[cg * 8 + i];
+                            for (int i = 0; i < 8; i++)
+                                f[i] = addb ? __uint_as_float(v[cg * 8 + i]) + bias[cg * 8 + i] : __uint_as_float(v[cg * 8 + i]);
                             f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
                             f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
                             f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
@@ -879,7 +978,7 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                             *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * a.W + x) * 8) = o;
                         }
                     }
-                    mbar_arrive(hfree(k, (q - 2) % NH));
+                    rb_arrive(hfree(k, (q - 2) % NH));
                     if (warp % 4 == 2 && lane == 0) NS_TR(22 + k, q);
                 }
             }
