@@ -78,7 +78,10 @@ struct ReconCfg {
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
     static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
     static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
-    static constexpr int MINB = (S == 3) ? 4 : 3;  // resident CTAs per SM (registers)
+#ifndef NS_RECON_MINB3
+#define NS_RECON_MINB3 4
+#endif
+    static constexpr int MINB = (S == 3) ? NS_RECON_MINB3 : 3;  // resident CTAs per SM (registers)
 };
 constexpr int kReconTX = 32, kReconTY = 4;
 constexpr int kReconNT = kReconTX * kReconTY;
@@ -89,7 +92,8 @@ struct ReconSmem {
     static constexpr int RROWS = kReconTY * ReconCfg<S>::PER + 2;      // residual tile LR rows
     static constexpr size_t REF = (size_t)(ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconNT * 8;
     static constexpr size_t RES = (size_t)3 * RROWS * kResCols * 2;
-    static constexpr size_t BYTES = REF + RES;
+    static constexpr size_t BAR = REF + RES;                           // mbarrier of the residual tile
+    static constexpr size_t BYTES = BAR + 16;
 };
 
 __device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
@@ -340,18 +344,27 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [RPT+1][NQ][NT] warp windows
     int16_t *tres = reinterpret_cast<int16_t *>(recon_sm + Sm::REF);   // [3][RROWS][kResCols] residual tile
 
-    // cooperative residual tile: tile row r <-> LR row Y0c/S - 1 + r (clamped, Z16),
-    // tile column 8q+e <-> LR column 8 bx0 - 8 + 8q + e (chunks outside the row are
-    // never read: the edge columns are clamped on use)
-    if (!fd.key) {
-        constexpr int CH = kResCols / 8;
-        for (int e = tid; e < 3 * Sm::RROWS * CH; e += kReconNT) {
-            const int c = e / (Sm::RROWS * CH), rr = (e / CH) % Sm::RROWS, q = e % CH;
-            const int col = 8 * bx0 - 8 + 8 * q;
-            if (col < 0 || col >= w) continue;
+    // residual tile: tile row r <-> LR row Y0c/S - 1 + r (clamped, Z16), tile
+    // column t <-> LR column 8 bx0 - 8 + t; the part inside the row arrives as one
+    // bulk copy per (plane, row) issued by warp 0 (columns outside the row are
+    // never read: the edge columns are clamped on use).  One bulk copy per row
+    // instead of per-thread 16-B chunks: the chunk loop's index arithmetic was
+    // ~6% of the kernel's instructions (ncu source counters).
+    uint64_t *tbar = reinterpret_cast<uint64_t *>(recon_sm + Sm::BAR);
+    if (!fd.key && tid < 32) {
+        const int col_lo = max(8 * bx0 - 8, 0), col_hi = min(8 * bx0 - 8 + kResCols, w);
+        const uint32_t bytes = (uint32_t)(col_hi - col_lo) * 2u;
+        if (tid == 0) {
+            mbar_init(tbar, 1);
+            fence_mbar_init();
+            mbar_arrive_expect_tx(tbar, 3 * Sm::RROWS * bytes);
+        }
+        __syncwarp();
+        for (int e = tid; e < 3 * Sm::RROWS; e += 32) {
+            const int c = e / Sm::RROWS, rr = e % Sm::RROWS;
             const int row = min(max(Y0c / S - 1 + rr, 0), h - 1);
-            cp_async16(tres + ((size_t)c * Sm::RROWS + rr) * kResCols + 8 * q,
-                       fd.res_f + c * lrp + (size_t)row * w + col);
+            bulk_load(tres + (size_t)e * kResCols + (col_lo - (8 * bx0 - 8)),
+                      fd.res_f + c * lrp + (size_t)row * w + col_lo, bytes, tbar);
         }
     }
 
@@ -402,7 +415,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     };
     for (int r = 0; r <= RPT; r++) {
         stage_row(0, r);
-        asm volatile("cp.async.commit_group;" ::: "memory");   // the residual tile rides in row 0's group
+        asm volatile("cp.async.commit_group;" ::: "memory");
     }
     const bool left_in = bx > 0, right_in = 8 * bx + 8 < w;
     const int m = xs & 7;
@@ -412,7 +425,10 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
 #pragma unroll 1
     for (int c = 0; c < 3; c++) {
         asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
-        if (c == 0) __syncthreads();                            // the residual tile is cooperative
+        if (c == 0) {
+            __syncthreads();                                    // (orders the tile barrier's init)
+            if (!fd.key) mbar_wait(tbar, 0);                    // the residual tile
+        }
         // (use_lr threads run the warp pass over whatever the slots hold: every weight is 0, so pred = 0)
         const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
         const uint2 *lrb = wbuf + lr_slots(c);
