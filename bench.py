@@ -52,12 +52,15 @@ def cfg_of(args):
     return c
 
 
-def workload_config(cfg, world):
+def workload_config(cfg, world, select="topk"):
     """The `config` object both arms print (same workload, same keys)."""
     S, s, w, h = cfg["streams"], cfg["scale"], cfg["w"], cfg["h"]
+    sel = ("top-k per stream" if select == "topk" else
+           f"global budget k*S*N = {cfg['k'] * S * world} anchors over all GPUs' streams (§5.2, NEXT-1)")
     return {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{s * w}x{s * h} x{s} streams per GPU, "
-                        f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} (top-k per stream)",
-            "streams_per_gpu": S, "frames_per_step_per_gpu": S * cfg["n"], "parallelism": f"streams x{world}"}
+                        f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} ({sel})",
+            "streams_per_gpu": S, "frames_per_step_per_gpu": S * cfg["n"], "parallelism": f"streams x{world}",
+            "select": select}
 
 
 def _gen(a):
@@ -223,6 +226,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sr-batch", type=int, default=16)
+    ap.add_argument("--select", default="topk", choices=["topk", "global"],
+                    help="global: §5.2 selection across all GPUs' streams (per-GPU gains, NCCL all_gather, "
+                         "ns_select_merge, NS_GIVEN_ANCHORS) inside the timed step")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -280,8 +286,17 @@ def main():
     stats = torch.zeros((S, 8), dtype=torch.float64, device=dev)
     stream = torch.cuda.current_stream(dev)
 
+    sids = [rank * S + si for si in range(S)]
+    cost = [1] * S                    # one resolution and model size: equal T_DNN per anchor
+    budget = k * S * world            # the same anchor count as top-k, placed globally
+
     def step():
-        ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, k=k, stream=stream)
+        if args.select == "global":
+            anc, _ = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream)
+            ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, stream=stream,
+                                mode=ns.NS_GIVEN_ANCHORS, anchor_in=anc, cost=cost, budget=budget)
+        else:
+            ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, k=k, stream=stream)
 
     for _ in range(args.warmup):
         step()
@@ -383,7 +398,7 @@ def main():
         ems = shard.max_over_ranks(q0.elapsed_time(q1))
         e2e = {"value": world * S * n * args.e2e_steps / (ems / 1000.0), "unit": UNIT, "h2d_bytes_per_step": moved[0],
                "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
-               "api": "ns_enhance_streams_host (C ABI, pinned host inputs)",
+               "api": "ns_enhance_streams_host (C ABI, pinned host inputs)", "select": "topk",
                "note": "per step: H2D of every stream's residual+MV+type (uploaded in stream groups on the library's "
                        "copy stream, overlapped with compute) and of the anchors' LR frames (gathered after "
                        "selection; non-anchor LR is read only for intra blocks, in place); D2H of the per-stream "
@@ -400,7 +415,7 @@ def main():
                 "vs_baseline": None, "dtype": "bf16",
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
-                "config": dict(workload_config(cfg, world),
+                "config": dict(workload_config(cfg, world, args.select),
                                l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
