@@ -40,7 +40,10 @@ __device__ unsigned long long g_trace[16 * 2 * 1024];
 #define NS_TR_ROLE(r)
 #endif
 
-enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4 };
+// EPI_HEAD: the store epilogue of the head conv, whose input x = LR - 128 has 3
+// real channels: only channel group 0 (8 channels, 16 B/px) is stored and
+// loaded by TMA; group 1 of every ring slot is a zero region written once.
+enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4, EPI_HEAD = 5 };
 constexpr int kSlots = 6;
 constexpr int kRows = 32;   // rows per CTA strip
 
@@ -451,13 +454,22 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     const uint32_t tmem = *s_tmem;
     const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);  // this warp's TMEM lanes
     const SrJob J = a.jobs[job];
+    // EPI_HEAD: TMA fills channel group 0 only; group 1 (at +kHalo*16, the A
+    // descriptor's leading byte offset) stays zero for the whole kernel
+    constexpr uint32_t LOAD_BYTES = (EPI == EPI_HEAD) ? kHalo * 16u : Cfg::SLOT_BYTES;
+    static_assert(EPI != EPI_HEAD || CIN == 16, "head: 3 channels in one group of 8, padded to K = 16");
+    if constexpr (EPI == EPI_HEAD) {
+        for (int i = tid; i < Cfg::NSLOT * kHalo; i += blockDim.x)
+            reinterpret_cast<uint4 *>(s_ring + (i / kHalo) * Cfg::SLOT + kHalo * 16)[i % kHalo] = make_uint4(0, 0, 0, 0);
+        fence_proxy_async_smem();
+    }
     if (tid == 0) {
         prefetch_tmap(&tm_in);
         mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
         bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
         bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
         for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
-            mbar_arrive_expect_tx(&bars[q], Cfg::SLOT_BYTES);
+            mbar_arrive_expect_tx(&bars[q], LOAD_BYTES);
             tma_load_5d(s_ring + q * Cfg::SLOT, &tm_in, &bars[q], 0, x0 - 1, 0, y0 - 1 + q, slot_job);
         }
     }
@@ -512,7 +524,7 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         tc_fence_after();
         if (tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
             const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
-            mbar_arrive_expect_tx(&bars[sl], Cfg::SLOT_BYTES);
+            mbar_arrive_expect_tx(&bars[sl], LOAD_BYTES);
             tma_load_5d(s_ring + sl * Cfg::SLOT, &tm_in, &bars[sl], 0, x0 - 1, 0, y0 - 1 + qn, slot_job);
         }
         const uint32_t acc = tl + (uint32_t)(mod3(r) * NB);
@@ -1658,7 +1670,9 @@ __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_coun
     }
 }
 
-// LR u8 planar [3][h][w] -> bf16 [h][2][w][8]: channels 0..2 = LR - 128 (Z13), 3..15 = 0.
+// LR u8 planar [3][h][w] -> bf16 [h][w][8], channel group 0 of the head input:
+// channels 0..2 = LR - 128 (Z13), 3..7 = 0 (channels 8..15 are the zero region of
+// the head's ring slots, EPI_HEAD).
 __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0,
                           uint8_t *lr8, int wp) {
     const int slot = blockIdx.y, job = j0 + slot;
@@ -1669,14 +1683,11 @@ __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, i
     const uint8_t *L = jobs[job].lr;
     const size_t plane = (size_t)h * w;
     const float r = (float)L[idx] - 128.f, g = (float)L[plane + idx] - 128.f, b = (float)L[2 * plane + idx] - 128.f;
-    uint4 o0, z;
+    uint4 o0;
     o0.x = pack_bf16(r, g);
     o0.y = pack_bf16(b, 0.f);
     o0.z = 0; o0.w = 0;
-    z.x = z.y = z.z = z.w = 0;
-    uint16_t *base = x0 + (((size_t)slot * h + y) * 2) * (size_t)w * 8;
-    *reinterpret_cast<uint4 *>(base + (size_t)x * 8) = o0;
-    *reinterpret_cast<uint4 *>(base + ((size_t)w + x) * 8) = z;
+    *reinterpret_cast<uint4 *>(x0 + (((size_t)slot * h + y) * w + x) * 8) = o0;  // channel group 0 only
     uint8_t *l8 = lr8 + ((size_t)slot * h + y) * 3 * wp + x;
     l8[0] = L[idx];
     l8[wp] = L[plane + idx];
@@ -1734,7 +1745,7 @@ static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u posit
 
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
     const size_t px = (size_t)h * w * nb;
-    size_t b = px * 16 * 2;                  // x0
+    size_t b = px * 8 * 2;                   // x0 (channel group 0 of the head input)
     b += 3 * px * C * 2;                     // h0, hb, tb
     b += band_floats(h, w, C, s) * 4 * nb;   // border bands
     b += (size_t)h * 3 * ((w + 15) / 16 * 16) * nb;  // lr8
@@ -1749,7 +1760,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
         mem += (bytes + 255) / 256 * 256;
         return p;
     };
-    a->x0 = reinterpret_cast<uint16_t *>(take(px * 16 * 2));
+    a->x0 = reinterpret_cast<uint16_t *>(take(px * 8 * 2));
     a->h0 = reinterpret_cast<uint16_t *>(take(px * C * 2));
     a->hb = reinterpret_cast<uint16_t *>(take(px * C * 2));
     a->tb = reinterpret_cast<uint16_t *>(take(px * C * 2));
@@ -1758,7 +1769,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     a->lr8 = take((size_t)h * 3 * a->wp * nb);
     int rc = 0;
     rc |= make_lr8_map(&a->tm_lr8, a->lr8, h, a->wp, nb);
-    rc |= make_act_map(&a->tm_x0, a->x0, h, w, 16, nb, kHalo);
+    rc |= make_act_map(&a->tm_x0, a->x0, h, w, 8, nb, kHalo);
     rc |= make_act_map(&a->tm_h0, a->h0, h, w, C, nb, kHalo);
     rc |= make_act_map(&a->tm_hb, a->hb, h, w, C, nb, kHalo);
     rc |= make_act_map(&a->tm_tb, a->tb, h, w, C, nb, kHalo);
@@ -1876,7 +1887,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
-        if ((e = conv_rot<16, C, EPI_STORE>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
+        if ((e = conv_rot<16, C, EPI_HEAD>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     // residual blocks, fused (conv1 + ReLU + conv2 + skip), ping-pong hb / tb
     const CUtensorMap *hin = &a->tm_h0;

@@ -221,3 +221,33 @@ def test_host_path_new_modes_match_device_path(ctx, kw):
         assert ia0.sum() == S + 1                                 # every key frame, fewer than k
     for a, b in zip(hr0 + st0, hr1 + st1):
         assert np.array_equal(a, b)
+
+
+def test_select_merge_full_size_c5_rows(ctx):
+    """ns_select_merge at the scale of c5 (512 streams x 60 frames, rows from 8
+    GPUs in LPT-like interleaved order, ~8% budget): bit-exact against the oracle
+    merge.  Gains come from ns_select_anchors on small frames (the merge only
+    sees gain / rank / type rows, whatever the resolution)."""
+    S, n = 512, 60
+    rng = np.random.default_rng(77)
+    cs = [synth.make_chunk(20000 + s, 16, 16, 2, n, types=synth.default_types(n, int(rng.integers(8, 20))))
+          for s in range(S)]
+    dcs = [dev_chunk(ns, c, DEV) for c in cs]
+    g, r, _ = _select_gpu(ctx, dcs, k=0)
+    # gathered order: 8 ranks, rank j owns streams with s % 8 == j
+    perm = [s for j in range(8) for s in range(S) if s % 8 == j]
+    pt = torch.tensor(perm, device=DEV)
+    g_all, r_all = g[pt].contiguous(), r[pt].contiguous()
+    t_all = torch.stack([dcs[s].type for s in perm])
+    cost = [1 + (s % 2) * 3 for s in perm]                  # 720p streams cost ~4x a 360p stream (P:120)
+    budget = int(0.08 * n * sum(cost) / 2.5)
+    rank = torch.empty_like(r_all)
+    anc = torch.empty_like(t_all)
+    ctx.select_merge(g_all, r_all, t_all, torch.tensor(perm, dtype=torch.int32, device=DEV),
+                     torch.tensor(cost, dtype=torch.int64, device=DEV), budget, rank, anc)
+    torch.cuda.synchronize()
+    er, ea = OS.merge_gathered(t_all.cpu().tolist(), g_all.cpu().tolist(), perm, cost, budget)
+    assert anc.cpu().tolist() == ea
+    assert rank.cpu().tolist() == er
+    chosen = sum(c for c, row in zip(cost, ea) for v in row if v)
+    assert 0 < chosen <= budget
