@@ -486,6 +486,10 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     const uint32_t idesc = idesc_bf16_f32(128, 3 * NB);
     const int p = warp * 32 + lane;
     const int x = x0 + p;
+    constexpr int RC = (EPI == EPI_RESID) ? NB / 8 : 1;
+    uint4 rnext[RC];  // EPI_RESID: residual row prefetched one step ahead
+#pragma unroll
+    for (int cg = 0; cg < RC; cg++) rnext[cg] = make_uint4(0, 0, 0, 0);
     for (int q = 0; q < n_loads; q++) {
         const int yin = y0 - 1 + q;
         if (tid == 0) {
@@ -510,14 +514,19 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         __syncwarp();
         const int r = yin - 1;  // output row completed by this input row
         const bool valid = r >= y0 && x < a.W;
-        constexpr int RC = (EPI == EPI_RESID) ? NB / 8 : 1;
         uint4 rres[RC];
         if constexpr (EPI == EPI_RESID) {
-            if (valid) {
-                const size_t rb = ((size_t)slot_job * a.H + r) * (NB / 8);
+            // the residual of this row was fetched one step ago; fetch the next
+            // row's now, so its latency is covered by a whole step (ncu: the
+            // same-step load left the end conv 60% long-scoreboard stalls)
+#pragma unroll
+            for (int cg = 0; cg < RC; cg++) rres[cg] = rnext[cg];
+            const int rn = yin;
+            if (rn >= y0 && rn < y1 && x < a.W) {
+                const size_t rb = ((size_t)slot_job * a.H + rn) * (NB / 8);
 #pragma unroll
                 for (int cg = 0; cg < RC; cg++)
-                    rres[cg] = __ldg(reinterpret_cast<const uint4 *>(a.resid + ((rb + cg) * a.W + x) * 8));
+                    rnext[cg] = __ldg(reinterpret_cast<const uint4 *>(a.resid + ((rb + cg) * a.W + x) * 8));
             }
         }
         mbar_wait(&bars[4], q & 1);
