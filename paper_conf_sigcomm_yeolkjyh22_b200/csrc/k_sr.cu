@@ -612,6 +612,13 @@ constexpr int kRbMmaWarps = 4;
 #ifndef NS_RB_NTS
 #define NS_RB_NTS 2
 #endif
+// NS_RB_BULK: each h row of a tile arrives as C/8 one-dimensional bulk copies
+// (one contiguous 16-B x 130-px run per channel group) instead of one tensor
+// box whose innermost extent is 16 B (8 channels); the out-of-frame columns of
+// a tile are zeroed once, out-of-frame rows by the producer.
+#ifndef NS_RB_BULK
+#define NS_RB_BULK 1
+#endif
 constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 // h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
 // h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
@@ -623,6 +630,7 @@ constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 constexpr int kRbOut = kTile - 2;
 struct RbArgs {
     int H, W, n_tiles, rows_per_cta, j0;
+    const uint16_t *in;     // h [job][H][C/8][W][8] (NS_RB_BULK: rows by 1-D bulk copies)
     const SrJob *jobs;
     const int32_t *job_count;
     size_t b1_off, bias1_off, b2_off, bias2_off;
@@ -761,6 +769,16 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
         const int ks = i / (Cfg::SLOT / 16), o = i % (Cfg::SLOT / 16);
         reinterpret_cast<uint4 *>(tslot(ks / Cfg::NTS, ks % Cfg::NTS))[o] = make_uint4(0, 0, 0, 0);
     }
+    // h slot column c <-> x = x0k - 2 + c; in-frame columns [c_lo, c_hi)
+    auto c_lo = [&](int k) { return max(0, 2 - x0k(k)); };
+    auto c_hi = [&](int k) { return min(kHalo, a.W - x0k(k) + 2); };
+#if NS_RB_BULK
+    for (int i = tid; i < 2 * NH * (C / 8) * kHalo; i += blockDim.x) {  // out-of-frame columns stay zero
+        const int c = i % kHalo, cg = (i / kHalo) % (C / 8), sl = (i / (kHalo * (C / 8))) % NH, k = i / (kHalo * (C / 8) * NH);
+        if (c < c_lo(k) || c >= c_hi(k))
+            reinterpret_cast<uint4 *>(hslot(k, sl) + cg * kHalo * 16)[c] = make_uint4(0, 0, 0, 0);
+    }
+#endif
     fence_proxy_async_smem();
     tc_fence_before();
     __syncthreads();
@@ -798,8 +816,27 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     // slot reuse: h row q-NH was last read by E2 at step q-NH+2, which
                     // arrives on hfree[slot] (one completion per reuse: never runs ahead)
                     if (q >= NH) mbar_wait(hfree(k, sl), ((q / NH) - 1) & 1);
+#if NS_RB_BULK
+                    const int yy = y0 - 2 + q, lo = c_lo(k), hi = c_hi(k);
+                    if (yy < 0 || yy >= a.H) {  // zero padding row: in-frame columns to zero
+                        for (int cg = 0; cg < C / 8; cg++)
+                            for (int c = lo; c < hi; c++)
+                                reinterpret_cast<uint4 *>(hslot(k, sl) + cg * kHalo * 16)[c] = make_uint4(0, 0, 0, 0);
+                        fence_proxy_async_smem();
+                        mbar_arrive(hfull(k, sl));
+                    } else {
+                        const uint32_t run = (uint32_t)(hi - lo) * 16u;
+                        mbar_arrive_expect_tx(hfull(k, sl), run * (C / 8));
+                        const uint16_t *src = a.in + (((size_t)slot_job * a.H + yy) * (C / 8) * a.W +
+                                                      (size_t)(x0k(k) - 2 + lo)) * 8;
+                        for (int cg = 0; cg < C / 8; cg++)
+                            bulk_load(hslot(k, sl) + cg * kHalo * 16 + lo * 16, src + (size_t)cg * a.W * 8, run,
+                                      hfull(k, sl));
+                    }
+#else
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
                     tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
+#endif
                     NS_TR(30 + k, q);
                 }
             }
@@ -1908,6 +1945,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         r.H = h; r.W = w; r.j0 = j0; r.jobs = jobs; r.job_count = job_count;
         r.b1_off = l1.b_off; r.bias1_off = l1.bias_off; r.b2_off = l2.b_off; r.bias2_off = l2.bias_off;
         r.out = dst;
+        r.in = hcur;
         if ((e = resblock<C>(*hin, r, nj, st)) != cudaSuccess) return e;
         hin = (dst == a->hb) ? &a->tm_hb : &a->tm_tb;
         hcur = dst;
