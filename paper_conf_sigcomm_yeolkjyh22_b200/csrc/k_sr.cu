@@ -54,6 +54,7 @@ struct ConvArgs {
     const SrJob *jobs;
     const int32_t *job_count;
     size_t b_off, bias_off; // this launch's B operand / bias offsets in the packed model
+    const uint16_t *in;     // bf16 activation in [job][H][CIN/8][W][8] (k_conv_rot, k_uptail2: bulk-copied rows)
     uint16_t *out;          // bf16 activation out (EPI_STORE/RELU/RESID/SHUFFLE)
     const uint16_t *resid;  // EPI_RESID
     int C;                  // channels of the output activation (shuffle: per sub-pixel)
@@ -424,6 +425,56 @@ __device__ __forceinline__ void tmem_zeroN(uint32_t a) {
 
 
 
+#ifndef NS_RB_BULK
+#define NS_RB_BULK 1
+#endif
+#ifndef NS_ROT_BULK
+#define NS_ROT_BULK 1
+#endif
+// (k_uptail2 with bulk-copied rows measured neutral to slightly slower on the
+// same box -- 20.3 vs 19.2-20.3 ms -- so it keeps its tensor box)
+#ifndef NS_UP_BULK
+#define NS_UP_BULK 0
+#endif
+// Activation rows into a ring slot by one-dimensional bulk copies.  The
+// activation layout [job][H][G][W][8] (bf16) holds each channel group's row as
+// one contiguous run of 16 B per pixel, so a tile row segment of ncols pixels
+// starting at x_start is G contiguous runs; the slot layout is [G][ncols][8]
+// (the UMMA K-major core-matrix layout, leading byte offset ncols * 16).  A
+// tensor box over the same data has an innermost extent of 16 B (8 channels),
+// which the TMA unit serves far more slowly (res-block A/B: body 102.4 -> 96.9
+// ms per c4 step).  Columns outside the frame are zeroed once per slot
+// (slot_zero_edges); a row outside the frame gets its in-frame columns zeroed
+// by the producer (generic stores, proxy fence) and a plain arrive.
+__device__ __forceinline__ uint32_t mbar_arrive_state(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+    return 0;
+}
+template <int G>
+__device__ __forceinline__ void slot_zero_edges(uint8_t *slot, int ncols, int W, int x_start, int t, int nt) {
+    const int lo = max(0, -x_start), hi = min(ncols, W - x_start);
+    for (int i = t; i < G * ncols; i += nt) {
+        const int c = i % ncols, g = i / ncols;
+        if (c < lo || c >= hi) reinterpret_cast<uint4 *>(slot + g * ncols * 16)[c] = make_uint4(0, 0, 0, 0);
+    }
+}
+template <int G>
+__device__ __forceinline__ void row_bulk(uint8_t *slot, int ncols, const uint16_t *in, int job, int H, int W, int y,
+                                         int x_start, uint64_t *bar) {
+    const int lo = max(0, -x_start), hi = min(ncols, W - x_start);
+    if (y < 0 || y >= H) {
+        for (int g = 0; g < G; g++)
+            for (int c = lo; c < hi; c++) reinterpret_cast<uint4 *>(slot + g * ncols * 16)[c] = make_uint4(0, 0, 0, 0);
+        fence_proxy_async_smem();
+        mbar_arrive_state(bar);
+        return;
+    }
+    const uint32_t run = (uint32_t)(hi - lo) * 16u;
+    mbar_arrive_expect_tx(bar, run * G);
+    const uint16_t *src = in + (((size_t)job * H + y) * G * W + (size_t)(x_start + lo)) * 8;
+    for (int g = 0; g < G; g++) bulk_load(slot + g * ncols * 16 + lo * 16, src + (size_t)g * W * 8, run, bar);
+}
+
 template <int CIN, int NB, int EPI>
 __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
     using Cfg = RotCfg<CIN, NB>;
@@ -463,14 +514,26 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
             reinterpret_cast<uint4 *>(s_ring + (i / kHalo) * Cfg::SLOT + kHalo * 16)[i % kHalo] = make_uint4(0, 0, 0, 0);
         fence_proxy_async_smem();
     }
+#if NS_ROT_BULK
+    // rows by bulk copies (row_bulk): G channel groups of 16 B per pixel
+    constexpr int G = (EPI == EPI_HEAD) ? 1 : CIN / 8;
+    (void)LOAD_BYTES;
+    for (int sl = 0; sl < Cfg::NSLOT; sl++) slot_zero_edges<G>(s_ring + sl * Cfg::SLOT, kHalo, a.W, x0 - 1, tid, blockDim.x);
+    fence_proxy_async_smem();
+    __syncthreads();
+#endif
     if (tid == 0) {
         prefetch_tmap(&tm_in);
         mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
         bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
         bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
         for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
+#if NS_ROT_BULK
+            row_bulk<G>(s_ring + q * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + q, x0 - 1, &bars[q]);
+#else
             mbar_arrive_expect_tx(&bars[q], LOAD_BYTES);
             tma_load_5d(s_ring + q * Cfg::SLOT, &tm_in, &bars[q], 0, x0 - 1, 0, y0 - 1 + q, slot_job);
+#endif
         }
     }
     // the three accumulator blocks start at zero
@@ -533,8 +596,12 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         tc_fence_after();
         if (tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
             const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
+#if NS_ROT_BULK
+            row_bulk<G>(s_ring + sl * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + qn, x0 - 1, &bars[sl]);
+#else
             mbar_arrive_expect_tx(&bars[sl], LOAD_BYTES);
             tma_load_5d(s_ring + sl * Cfg::SLOT, &tm_in, &bars[sl], 0, x0 - 1, 0, y0 - 1 + qn, slot_job);
+#endif
         }
         const uint32_t acc = tl + (uint32_t)(mod3(r) * NB);
         uint32_t v[NB];
@@ -616,9 +683,7 @@ constexpr int kRbMmaWarps = 4;
 // (one contiguous 16-B x 130-px run per channel group) instead of one tensor
 // box whose innermost extent is 16 B (8 channels); the out-of-frame columns of
 // a tile are zeroed once, out-of-frame rows by the producer.
-#ifndef NS_RB_BULK
-#define NS_RB_BULK 1
-#endif
+
 constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 // h_out = h + conv2(ReLU(conv1(h) + b1)) + b2 (EDSR block) in one kernel:
 // h rows arrive once by TMA, t = ReLU(conv1) never leaves shared memory (it is
@@ -1425,6 +1490,12 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
         mbar_init(wbar, 1);
         fence_mbar_init();
     }
+#if NS_UP_BULK
+    for (int k = 0; k < 2; k++)
+        for (int i = 0; i < NS; i++)
+            slot_zero_edges<CIN / 8>(islot(k, i), kHalo5, a.W, x0k(k) - 2, tid, blockDim.x);
+    fence_proxy_async_smem();
+#endif
     if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
     tc_fence_before();
     __syncthreads();
@@ -1456,8 +1527,13 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     if (!vk(k)) continue;
                     const int sl = q % NS;
                     if (q >= NS) mbar_wait(sfree(k, sl), ((q / NS) - 1) & 1);
+#if NS_UP_BULK
+                    row_bulk<CIN / 8>(islot(k, sl), kHalo5, a.in, slot_job, a.H, a.W, y0 - 2 + q, x0k(k) - 2,
+                                      hfull(k, sl));
+#else
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
                     tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
+#endif
                     const int qv = q - 4;  // output row y0 + qv retires at this step
                     if (qv >= 0) {
                         const int ls = qv % NL;
@@ -1932,7 +2008,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     auto L = [&](int l) { return model_layer(n_blocks, C, s, l); };
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
-        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0;
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0; g.in = a->x0;
         if ((e = conv_rot<16, C, EPI_HEAD>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     // residual blocks, fused (conv1 + ReLU + conv2 + skip), ping-pong hb / tb
@@ -1955,13 +2031,13 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     const CUtensorMap &tm5 = (endout == a->tb) ? a->tm_tb5 : a->tm_hb5;
     {
         ConvArgs g = base; LayerShape ls = L(2 * n_blocks + 1);
-        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = endout; g.resid = a->h0;
+        g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = endout; g.resid = a->h0; g.in = hcur;
         if ((e = conv_rot<C, C, EPI_RESID>(F_SR_END, *hin, g, nj, st)) != cudaSuccess) return e;
     }
     {   // tail o shuffle o upsampler as one 5x5 conv at LR (+ bilinear skip, round, clamp) -> u8 HR
         const CompShape cs = model_comp(n_blocks, C, s);
         ConvArgs g = base;
-        g.b_off = cs.b_off; g.bias_off = cs.bias_off;
+        g.b_off = cs.b_off; g.bias_off = cs.bias_off; g.in = endout;
         {
             const size_t H = (size_t)h * s, W = (size_t)w * s;
             g.ring = a->band + (size_t)a->nb * (2 * (W + 2) + 2 * H) * C;
