@@ -666,12 +666,14 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
 
 // ------------------------------------------------------------------ fused residual block
 constexpr int kRbMmaWarps = 4;
-// h ring depth per tile: the slot of row q+NH is freed by E2(q+2), so the TMA row
-// load (~2,000 cycles measured on the clock64 timeline) gets NH-3 steps of
-// slack.  A/B on B200 (tools/build_variant.sh): NH 5 / 6 / 7 -> body 114.6 /
-// 105.1 / 109.6 ms per c4 step (7 leaves the epilogues more SMEM contention).
+// h ring depth per tile: the slot of row q+NH is freed by E2(q+2), so the row
+// load gets NH-3 steps of slack.  A/B on B200 (tools/build_variant.sh, body ms
+// per c4 step): with tensor-box rows (~2,600-3,200 cycles issue -> landed on the
+// clock64 timeline) NH 5 / 6 / 7 -> 114.6 / 105.1 / 109.6; with bulk-copied
+// rows (~1,400-1,600 cycles) NH 5 / 6 / 7 -> 106.1 / 98.1 / 95.9.  7 is the
+// most that fits (shared memory).
 #ifndef NS_RB_NH
-#define NS_RB_NH 6
+#define NS_RB_NH 7
 #endif
 #ifndef NS_RB_QUAL
 #define NS_RB_QUAL __launch_bounds__(kRbThreads, 1)

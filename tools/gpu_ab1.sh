@@ -1,2 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_parity.py tests/test_gpu_next.py tests/test_gpu_host_path.py -x -q > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
-LIBS="default tools/bin/lib_tma2.so default tools/bin/lib_tma2.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+LIBS="default tools/bin/lib_nh5.so tools/bin/lib_nh7.so default tools/bin/lib_nh5.so tools/bin/lib_nh7.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+python tools/rb_trace2.py > gpurun_out/trace3.txt 2>&1
