@@ -69,6 +69,18 @@ __device__ __forceinline__ void static_for(F &&f) {
     }
 }
 
+// CTA shape: kReconTX LR block columns x kReconTY thread rows (RPT HR rows each)
+#ifndef NS_RECON_TX
+#define NS_RECON_TX 32
+#endif
+#ifndef NS_RECON_TY
+#define NS_RECON_TY 4
+#endif
+constexpr int kReconTX = NS_RECON_TX, kReconTY = NS_RECON_TY;
+constexpr int kReconNT = kReconTX * kReconTY;
+#ifndef NS_RECON_MINB3
+#define NS_RECON_MINB3 (512 / (NS_RECON_TX * NS_RECON_TY))
+#endif
 template <int S>
 struct ReconCfg {
     static constexpr int BW = 8 * S;               // HR pixels per thread row
@@ -78,13 +90,9 @@ struct ReconCfg {
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
     static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
     static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
-#ifndef NS_RECON_MINB3
-#define NS_RECON_MINB3 4
-#endif
-    static constexpr int MINB = (S == 3) ? NS_RECON_MINB3 : 3;  // resident CTAs per SM (registers)
+    // resident CTAs per SM (registers): 512 threads at 128 registers for s = 3
+    static constexpr int MINB = (S == 3) ? NS_RECON_MINB3 : (384 / kReconNT > 0 ? 384 / kReconNT : 1);
 };
-constexpr int kReconTX = 32, kReconTY = 4;
-constexpr int kReconNT = kReconTX * kReconTY;
 constexpr int kResCols = 8 * kReconTX + 16;        // residual tile columns (one 16-B chunk of halo per side)
 
 template <int S>
