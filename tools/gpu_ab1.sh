@@ -1,1 +1,2 @@
-LIBS="default tools/bin/lib_ty8.so tools/bin/lib_tx16ty8.so default tools/bin/lib_ty8.so tools/bin/lib_tx16ty8.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "recon or enhance" > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
+LIBS="default tools/bin/lib_noef.so default tools/bin/lib_noef.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
