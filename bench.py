@@ -226,6 +226,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sr-batch", type=int, default=16)
+    ap.add_argument("--balance", action="store_true",
+                    help="with --select global: anchor-level load balancing across GPUs (shard.plan_anchor_moves; "
+                         "LR out / HR back point-to-point), then ns_sr_anchors + ns_reconstruct_chunk")
     ap.add_argument("--select", default="topk", choices=["topk", "global"],
                     help="global: §5.2 selection across all GPUs' streams (per-GPU gains, NCCL all_gather, "
                          "ns_select_merge, NS_GIVEN_ANCHORS) inside the timed step")
@@ -290,8 +293,27 @@ def main():
     cost = [1] * S                    # one resolution and model size: equal T_DNN per anchor
     budget = k * S * world            # the same anchor count as top-k, placed globally
 
+    models_all = {rank * S + si: models[si] for si in range(S)}
+    if args.balance:  # every GPU keeps every stream's model (weights are small) to serve moved anchors
+        for r in range(world):
+            if r == rank:
+                continue
+            for si in range(S):
+                m = ctx.model(B, C, s)
+                m.set_weights(synth.make_weights(4000 + r * 100000 + si, B, C, s))
+                models_all[r * S + si] = m
+
     def step():
-        if args.select == "global":
+        if args.select == "global" and args.balance:
+            anc, _, allr = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream,
+                                                            return_all=True)
+            anc_h = allr["anchor"].cpu().numpy()
+            sid_h = allr["sid"].cpu().tolist()
+            anchors_all = [[int(f) for f in np.nonzero(anc_h[i])[0]] for i in range(len(sid_h))]
+            shard.balanced_sr_and_reconstruct(ctx, chunks, models_all, sids, anc, hr_out, anchors_all,
+                                              [x // S for x in sid_h], sid_h, allr["cost"].cpu().tolist())
+            ia.copy_(anc)
+        elif args.select == "global":
             anc, _ = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream)
             ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, stream=stream,
                                 mode=ns.NS_GIVEN_ANCHORS, anchor_in=anc, cost=cost, budget=budget)
@@ -415,14 +437,15 @@ def main():
                 "vs_baseline": None, "dtype": "bf16",
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
-                "config": dict(workload_config(cfg, world, args.select),
+                "config": dict(workload_config(cfg, world, args.select), balance=bool(args.balance),
                                l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
                              "anchors_per_step": int(ia_np.sum())},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
-                "quality": {"anchors": float(st[:, 1].sum()), "frames": float(st[:, 0].sum())}}
+                "quality": ({"anchors": float(st[:, 1].sum()), "frames": float(st[:, 0].sum())} if not args.balance
+                            else None)}  # the balanced path (ns_sr_anchors + ns_reconstruct_chunk) computes no stats
         print(json.dumps(line), flush=True)
     ctx.close()
     if world > 1:

@@ -99,7 +99,7 @@ def gather_rows(tensors, group=None):
 
 
 def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_res_size=False, group=None,
-                               stream=None):
+                               stream=None, return_all=False):
     """§5.2 global anchor selection over the streams of every GPU:
     (1) per-stream gains and ranks on this GPU (ns_select_anchors, Alg. 1);
     (2) all_gather of gain / rank / type / sid / cost rows (gather_rows);
@@ -123,4 +123,105 @@ def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_
     rank_out = torch.empty_like(r_all)
     anc_all = torch.empty_like(t_all)
     ctx.select_merge(g_all, r_all, t_all, s_all, c_all, budget, rank_out, anc_all, stream=stream)
+    if return_all:  # every gathered row, for the anchor-level load balancing
+        return (anc_all[off: off + S].contiguous(), rank_out[off: off + S].contiguous(),
+                {"anchor": anc_all, "sid": s_all, "cost": c_all})
     return anc_all[off: off + S].contiguous(), rank_out[off: off + S].contiguous()
+
+
+# ---------------------------------------------------------------- NEXT-1: anchor-level load balancing
+def plan_anchor_moves(anchors, owner, cost, world):
+    """Deterministic anchor-level load balancing across GPUs (§5.2: the
+    scheduler spreads the selected anchor frames' DNN work over the GPUs,
+    P:205-213).  Streams stay on their GPU; single anchor SR jobs
+    move.  anchors[i]: the anchor frames of gathered stream row i; owner[i]: its
+    rank; cost[i]: T_DNN of one of its anchors (> 0).  Greedy: while the most
+    loaded rank (lowest index on ties) has an anchor whose move to the least
+    loaded rank lowers the pair's maximum, move its first such anchor in
+    (row desc, frame desc) order.  Every rank computes the same plan from the
+    same gathered rows.  Returns [(row, frame, src, dst)] in move order."""
+    load = [0] * world
+    on = [[] for _ in range(world)]
+    for i, fr in enumerate(anchors):
+        for f in fr:
+            load[owner[i]] += cost[i]
+            on[owner[i]].append((i, f))
+    for r in range(world):
+        on[r].sort(reverse=True)
+    moves = []
+    while world > 1:
+        hi = min(range(world), key=lambda r: (-load[r], r))
+        lo = min(range(world), key=lambda r: (load[r], r))
+        pick = None
+        for idx, (i, f) in enumerate(on[hi]):
+            if load[lo] + cost[i] < load[hi]:
+                pick = idx
+                break
+        if pick is None:
+            break
+        i, f = on[hi].pop(pick)
+        load[hi] -= cost[i]
+        load[lo] += cost[i]
+        moves.append((i, f, hi, lo))
+    return moves
+
+
+def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anchors_all, owner_all, sid_all, cost_all,
+                                group=None, stream=None):
+    """SR on this GPU's share of the balanced anchor set, then reconstruction of
+    this GPU's streams (ns_sr_anchors + ns_reconstruct_chunk).  anchors_all /
+    owner_all / sid_all / cost_all describe every gathered stream row (host
+    lists, identical on all ranks); chunks / models / sid / is_anchor / hr_out
+    are this GPU's streams (models: dict sid -> Model, holding at least the
+    models of the rows this GPU may serve -- per-stream weights are small and
+    every GPU keeps all of them).  Exported anchors: LR out, HR back; imported
+    anchors: LR in, SR here, HR out -- point-to-point over NCCL (NVLink).
+    Everything is ordered on the current torch stream (stream=None), which the
+    NCCL point-to-point calls synchronise with."""
+    import torch
+    import torch.distributed as dist
+    dist_on = dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1
+    world = dist.get_world_size(group) if dist_on else 1
+    me = dist.get_rank(group) if dist_on else 0
+    moves = plan_anchor_moves(anchors_all, owner_all, cost_all, world)
+    local = {s: li for li, s in enumerate(sid)}
+    exported = {(sid_all[i], f): dst for i, f, src, dst in moves if src == me}
+    jobs = []
+    for li, s in enumerate(sid):
+        row = [i for i in range(len(sid_all)) if sid_all[i] == s][0]
+        for f in anchors_all[row]:
+            if (s, f) not in exported:
+                jobs.append((models[s], chunks[li].lr[f], hr_out[li][f]))
+    imports = []
+    ops = []
+    for i, f, src, dst in moves:          # LR out / in, in the global move order on every rank
+        s = sid_all[i]
+        if src == me:
+            ops.append(dist.P2POp(dist.isend, chunks[local[s]].lr[f].contiguous(), dst, group))
+        elif dst == me:
+            c0 = chunks[0]
+            h, w, sc = c0.h, c0.w, c0.scale
+            lr = torch.empty((3, h, w), dtype=torch.uint8, device=c0.lr.device)
+            hr = torch.empty((3, sc * h, sc * w), dtype=torch.uint8, device=c0.lr.device)
+            imports.append((i, f, src, lr, hr))
+            ops.append(dist.P2POp(dist.irecv, lr, src, group))
+    if ops:
+        for rq in dist.batch_isend_irecv(ops):
+            rq.wait()
+    for i, f, src, lr, hr in imports:
+        jobs.append((models[sid_all[i]], lr, hr))
+    if jobs:
+        ctx.sr_anchors(jobs, stream=stream)
+    ops = []
+    for i, f, src, dst in moves:          # HR back
+        s = sid_all[i]
+        if dst == me:
+            hr = [x for x in imports if x[0] == i and x[1] == f][0][4]
+            ops.append(dist.P2POp(dist.isend, hr, src, group))
+        elif src == me:
+            ops.append(dist.P2POp(dist.irecv, hr_out[local[s]][f], dst, group))
+    if ops:
+        for rq in dist.batch_isend_irecv(ops):
+            rq.wait()
+    ctx.reconstruct_chunk(chunks, is_anchor, hr_out, stream=stream)
+    return moves

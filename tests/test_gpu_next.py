@@ -251,3 +251,33 @@ def test_select_merge_full_size_c5_rows(ctx):
     assert rank.cpu().tolist() == er
     chosen = sum(c for c, row in zip(cost, ea) for v in row if v)
     assert 0 < chosen <= budget
+
+
+def test_balanced_path_single_gpu_equals_given(ctx):
+    """shard.balanced_sr_and_reconstruct (ns_sr_anchors + ns_reconstruct_chunk on
+    the balanced anchor set) on one GPU -- no moves -- gives the frames of the
+    one-call NS_GIVEN_ANCHORS path byte for byte."""
+    from paper_conf_sigcomm_yeolkjyh22_b200 import shard
+    S, n = 4, 10
+    cs = [synth.make_chunk(9990 + s, 48, 24, 2, n, types=synth.default_types(n, 4)) for s in range(S)]
+    m = ctx.model(1, 16, 2)
+    m.set_weights(synth.make_weights(81, 1, 16, 2))
+    anc = torch.zeros((S, n), dtype=torch.uint8, device=DEV)
+    anc[:, 0] = 1
+    anc[0, 4] = anc[2, 7] = anc[3, 3] = 1
+    outs = []
+    for path in ("given", "balanced"):
+        dcs = [dev_chunk(ns, c, DEV, model=m, state=True) for c in cs]
+        hr = [alloc_hr(n, c, DEV, fill=5) for c in cs]
+        if path == "given":
+            ctx.enhance_streams(dcs, hr, mode=ns.NS_GIVEN_ANCHORS, anchor_in=anc, cost=[1] * S, budget=S * n)
+        else:
+            anchors_all = [[f for f in range(n) if anc[s, f]] for s in range(S)]
+            moves = shard.balanced_sr_and_reconstruct(ctx, dcs, {s: m for s in range(S)}, list(range(S)), anc, hr,
+                                                      anchors_all, [0] * S, list(range(S)), [1] * S)
+            assert moves == []
+        torch.cuda.synchronize()
+        outs.append([np.stack([t.cpu().numpy() for t in row]) for row in hr] +
+                    [d.hr_last.cpu().numpy() for d in dcs] + [d.hr_golden.cpu().numpy() for d in dcs])
+    for a, b in zip(*outs):
+        assert np.array_equal(a, b)

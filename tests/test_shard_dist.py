@@ -124,3 +124,98 @@ def test_gloo_world2_global_selection_rows():
     assert (off0, n0, off1, n1) == (0, 3, 3, 4)
     assert g0 == g1 == [gains_all[i] for i in sid0]         # gathered gains are every stream's
     assert a0 == a1 == [anc_all[i] for i in sid0]           # = global selection over all streams
+
+
+# ---------------------------------------------------------------- NEXT-1 anchor-level load balancing
+def test_plan_anchor_moves_balances_and_is_deterministic():
+    import random
+    rng = random.Random(4)
+    for world in (1, 2, 4, 8):
+        for _ in range(20):
+            rows = rng.randint(world, 40)
+            owner = [rng.randrange(world) for _ in range(rows)]
+            cost = [rng.choice((1, 4)) for _ in range(rows)]      # 360p vs 720p anchor
+            anchors = [sorted(rng.sample(range(60), rng.randint(0, 9))) for _ in range(rows)]
+            moves = shard.plan_anchor_moves(anchors, owner, cost, world)
+            assert moves == shard.plan_anchor_moves(anchors, owner, cost, world)
+            load = [0] * world
+            for i, fr in enumerate(anchors):
+                load[owner[i]] += cost[i] * len(fr)
+            before = max(load)
+            seen = set()
+            for i, f, src, dst in moves:
+                assert f in anchors[i] and (i, f) not in seen and src != dst
+                seen.add((i, f))
+                load[src] -= cost[i]
+                load[dst] += cost[i]
+            assert max(load) <= before
+            # no single remaining move (an anchor moves at most once) from the max
+            # to the min rank lowers the max
+            hi, lo = load.index(max(load)), load.index(min(load))
+            unmoved = [(i, f) for i, fr in enumerate(anchors) for f in fr if (i, f) not in seen and owner[i] == hi]
+            assert all(load[lo] + cost[i] >= load[hi] for i, f in unmoved)
+            if world == 1:
+                assert moves == []
+
+
+class _FakeCtx:
+    """Stands in for ns.Context on CPU: 'SR' = nearest x2 upsample + model id."""
+    def __init__(self):
+        self.sr_calls, self.recon_calls = 0, 0
+
+    def sr_anchors(self, jobs, stream=None):
+        self.sr_calls += 1
+        for m, lr, hr in jobs:
+            hr.copy_((lr.repeat_interleave(2, 1).repeat_interleave(2, 2).int() + m) % 256)
+
+    def reconstruct_chunk(self, chunks, is_anchor, hr_out, stream=None):
+        self.recon_calls += 1
+
+
+def _lb_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from types import SimpleNamespace
+        n, h, w = 6, 4, 8
+        S_tot = 5
+        owner_all = [0, 0, 0, 0, 1]                     # rank 0 holds 4 streams, rank 1 one
+        sid_all = list(range(S_tot))
+        cost_all = [1] * S_tot
+        anchors_all = [[0, 3], [0, 2], [0], [0, 5], [0]]
+        mine = [i for i in range(S_tot) if owner_all[i] == rank]
+        g = torch.Generator().manual_seed(9)
+        lr_all = torch.randint(0, 256, (S_tot, n, 3, h, w), generator=g, dtype=torch.int32).to(torch.uint8)
+        chunks = [SimpleNamespace(lr=lr_all[i], h=h, w=w, scale=2) for i in mine]
+        hr_out = [[torch.zeros((3, 2 * h, 2 * w), dtype=torch.uint8) for _ in range(n)] for _ in mine]
+        models = {s: 10 + s for s in sid_all}
+        ia = torch.zeros((len(mine), n), dtype=torch.uint8)
+        ctx = _FakeCtx()
+        moves = shard.balanced_sr_and_reconstruct(ctx, chunks, models, mine, ia, hr_out, anchors_all, owner_all,
+                                                  sid_all, cost_all)
+        ok = True
+        for li, s in enumerate(mine):
+            for f in anchors_all[s]:
+                exp = (lr_all[s, f].repeat_interleave(2, 1).repeat_interleave(2, 2).int() + models[s]) % 256
+                ok &= bool(torch.equal(hr_out[li][f], exp.to(torch.uint8)))
+        q.put((rank, moves, ok, ctx.recon_calls))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_balanced_sr_exchange():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_lb_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    (r0, m0, ok0, rc0), (r1, m1, ok1, rc1) = res
+    assert m0 == m1 and len(m0) == 3                        # loads 7 / 1 -> 4 / 4
+    assert all(src == 0 and dst == 1 for _, _, src, dst in m0)
+    assert ok0 and ok1                                      # every anchor's HR is its own stream's SR
+    assert rc0 == rc1 == 1
