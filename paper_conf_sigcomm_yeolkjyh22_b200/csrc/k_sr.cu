@@ -395,6 +395,9 @@ __device__ __forceinline__ uint32_t pack_bf16_relu(float lo, float hi) {
     asm("cvt.rn.relu.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
     return r;
 }
+__device__ __forceinline__ void tmem_st1(uint32_t taddr, float v) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "f"(v) : "memory");
+}
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 __device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
@@ -433,6 +436,11 @@ __device__ __forceinline__ void tmem_zeroN(uint32_t a) {
 #endif
 // (k_uptail2 with bulk-copied rows measured neutral to slightly slower on the
 // same box -- 20.3 vs 19.2-20.3 ms -- so it keeps its tensor box)
+// NS_UP_BIAS_INIT: uptail2's retired accumulator columns are re-initialised by
+// their own epilogue group with bias + 1/2 (no 3-group barrier per step).
+#ifndef NS_UP_BIAS_INIT
+#define NS_UP_BIAS_INIT 1
+#endif
 #ifndef NS_UP_BULK
 #define NS_UP_BULK 0
 #endif
@@ -1413,7 +1421,7 @@ __device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>:
 // frame-border ring pixels of sub-row I keep their fp32 t = acc + bias for the
 // exact fix-up (k_uptail_ring)
 template <int NB, int S, int I>
-__device__ __forceinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB, S>::LW], const float *s_bias,
+__device__ __forceinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB, S>::LW], const float (&be)[3 * S],
                                                const ConvArgs &a, int x, int r, int lh, int lw, int slot_job) {
     constexpr int base = UpCols<NB, S>::base(I);
     const int HH = lh * S, WW = lw * S;
@@ -1426,7 +1434,10 @@ __device__ __forceinline__ void uptail_ring_store(const uint32_t (&v)[UpCols<NB,
 #pragma unroll
             for (int c = 0; c < 3; c++) {
                 const int n = (I * S + j) * 3 + c;
-                a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] = __uint_as_float(v[n - base]) + s_bias[n];
+                // t = acc + bias: be = bias + 1/2 while the block starts at zero, 0 once it
+                // starts at bias + 1/2
+                a.ring[((size_t)slot_job * (2 * WW + 2 * (HH - 2)) + ri) * 3 + c] =
+                    __uint_as_float(v[n - base]) + be[n - 3 * S * I] - 0.5f;
             }
         }
     }
@@ -1441,7 +1452,7 @@ __device__ __forceinline__ void uptail_group_step(const uint32_t (&v)[UpCols<NB,
     const int ra = min(max(r + oy, 0), lh - 1) - (r - 1), rb = min(max(r + oy + 1, 0), lh - 1) - (r - 1);
     const int cm = max(x - 1, 0) - (x0 - kLrBoxX), c0 = x - (x0 - kLrBoxX), cp = min(x + 1, lw - 1) - (x0 - kLrBoxX);
     uptail_subrow<NB, S, I>(v, bh, lr, ra, rb, cm, c0, cp, so, p);
-    if (r == 0 || r == lh - 1 || x == 0 || x == lw - 1) uptail_ring_store<NB, S, I>(v, s_bias, a, x, r, lh, lw, slot_job);
+    if (r == 0 || r == lh - 1 || x == 0 || x == lw - 1) uptail_ring_store<NB, S, I>(v, bh, a, x, r, lh, lw, slot_job);
 }
 
 template <int CIN, int NB, int S>
@@ -1487,7 +1498,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
             for (int i = 0; i < NL; i++) { mbar_init(lfull(k, i), 1); mbar_init(lfree(k, i), S); }
             mbar_init(mdone(k, 0), 1);
             mbar_init(mdone(k, 1), 1);
-            mbar_init(edone(k), 128);
+            mbar_init(edone(k), NS_UP_BIAS_INIT ? 128 * S : 128);
         }
         mbar_init(wbar, 1);
         fence_mbar_init();
@@ -1597,6 +1608,19 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                 uint32_t v[UpCols<NB, S>::LW];
                 tmem_ldN<UpCols<NB, S>::LW>(acc + cbase, v);
                 tmem_wait_ld();
+#if NS_UP_BIAS_INIT
+                // each group re-initialises its own 3S output columns of the retired
+                // block with bias + 1/2 (the rounding term): no cross-group barrier
+                // before the block is free, and no bias add below.  The first five
+                // retirements read blocks zeroed at allocation and add it here.
+                const bool addb = q < 5;
+#pragma unroll
+                for (int i = 0; i < 3 * S; i++) tmem_st1(acc + (uint32_t)(3 * S * g + i), bh[i]);
+                tmem_wait_st();
+                tc_fence_before();
+                mbar_arrive(edone(k));
+#else
+                constexpr bool addb = true;
                 tc_fence_before();
                 named_bar(1 + k, 128 * S);  // every group of this tile has read the block
                 if (g == 0) {
@@ -1606,15 +1630,19 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     tc_fence_before();
                     mbar_arrive(edone(k));
                 }
+#endif
+                float be[3 * S];  // bias + 1/2 still to add (zero once the block started at it)
+#pragma unroll
+                for (int i = 0; i < 3 * S; i++) be[i] = addb ? bh[i] : 0.f;
                 if (r >= y0) {
                     const int qv = r - y0, ls = qv % NL;
                     mbar_wait(lfull(k, ls), (qv / NL) & 1);
                     const uint8_t *lr = lslot(k, ls);
                     if (x < lw) {
-                        if (g == 0) uptail_group_step<NB, S, 0>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
-                        else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
-                        else if (S > 2 && g == 2) uptail_group_step<NB, S, (S > 2 ? 2 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
-                        else if (S > 3 && g == 3) uptail_group_step<NB, S, (S > 3 ? 3 : 0)>(v, bh, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        if (g == 0) uptail_group_step<NB, S, 0>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 2 && g == 2) uptail_group_step<NB, S, (S > 2 ? 2 : 0)>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
+                        else if (S > 3 && g == 3) uptail_group_step<NB, S, (S > 3 ? 3 : 0)>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
                     }
                     named_bar(3 + grp, 128);  // this group's staging row is complete, its LR reads done
                     if (p == 0) mbar_arrive(lfree(k, ls));

@@ -1,2 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_next.py -x -q > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
-python bench.py --select global --balance --steps 3 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/bal.json 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
+LIBS="default tools/bin/lib_upold.so default tools/bin/lib_upold.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
