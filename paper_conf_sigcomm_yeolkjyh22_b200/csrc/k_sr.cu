@@ -332,6 +332,9 @@ __global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtenso
 // block of row y-1 is complete: the epilogue reads it, applies the fused
 // epilogue, and zeroes it for row y+2.  No im2col, no lane shifts, 128-pixel
 // tiles, N = 96 (C = 32) -> up to 3x the MMA efficiency of N = 32.
+#ifndef NS_ROT_NSLOT
+#define NS_ROT_NSLOT 3  // input ring of k_conv_rot (head, end)
+#endif
 template <int CIN, int NB>
 struct RotCfg {
     static constexpr int KC = CIN / 16;
@@ -340,7 +343,7 @@ struct RotCfg {
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int NSLOT = 3;
+    static constexpr int NSLOT = NS_ROT_NSLOT;  // (4 does not fit the launch: measured failing)
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(3 * NB);
     static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + 128;
     static_assert((3 * NB) % 16 == 0 && 3 * NB <= 256, "N = 3 NB");
@@ -1322,9 +1325,11 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
 // the MMA on input row y waits for the epilogue of row y-3 (previous step),
 // and the other tile's MMAs cover that wait.  The TMA warp also stages the
 // three u8 LR rows r-1..r+1 of each output row r (bilinear skip taps) in a
-// separate ring that the epilogue groups release.
+// separate ring that the epilogue groups release.  Input ring depth: 3 and 4
+// measured equal while the epilogue groups met on a per-step barrier; with the
+// bias-initialised columns (no barrier) 4 wins: 18.2-18.4 -> 16.8-16.9 ms.
 #ifndef NS_UP_NS
-#define NS_UP_NS 3
+#define NS_UP_NS 4
 #endif
 #ifndef NS_UP_MMA2
 #define NS_UP_MMA2 0
