@@ -343,7 +343,7 @@ struct RotCfg {
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int NSLOT = NS_ROT_NSLOT;  // (a 4-slot build failed at run time; not investigated)
+    static constexpr int NSLOT = NS_ROT_NSLOT;  // 3: the barrier array is laid out [0,3) ring, 3 weights, 4 MMA
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(3 * NB);
     static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + 128;
     static_assert((3 * NB) % 16 == 0 && 3 * NB <= 256, "N = 3 NB");
