@@ -1327,9 +1327,10 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
 // three u8 LR rows r-1..r+1 of each output row r (bilinear skip taps) in a
 // separate ring that the epilogue groups release.  Input ring depth: 3 and 4
 // measured equal while the epilogue groups met on a per-step barrier; with the
-// bias-initialised columns (no barrier) 4 wins: 18.2-18.4 -> 16.8-16.9 ms.
+// bias-initialised columns (no barrier): 3 / 4 / 5 / 6 / 7 -> 18.3 / 16.2 /
+// 14.8-15.3 / 15.4-15.5 / 15.5-15.6 ms per c4 step.
 #ifndef NS_UP_NS
-#define NS_UP_NS 4
+#define NS_UP_NS 5
 #endif
 #ifndef NS_UP_MMA2
 #define NS_UP_MMA2 0
