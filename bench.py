@@ -259,7 +259,8 @@ def main():
     t_gen = time.time() - t_gen
 
     host_pool = ns.Context.host_pool_bytes(w, h, n, k, S) if args.e2e_steps > 0 else 0
-    ctx = ns.Context(local, pool_bytes=int((1.2 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)) + host_pool)
+    # two SR arenas: batches alternate between two streams (ns_api.cu run_sr_group)
+    ctx = ns.Context(local, pool_bytes=int((2.4 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)) + host_pool)
     # per-stream content-aware models: distinct weights per stream
     models = []
     for si in range(S):
@@ -453,11 +454,11 @@ def main():
 
 
 def ns_arena_gb(cfg, nb):
-    """SR arena of one shape (csrc/k_sr.cu sr_arena_bytes): x0 (16 ch) + h0/hb/tb
+    """SR arena of one shape (csrc/k_sr.cu sr_arena_bytes): x0 (8 ch) + h0/hb/tb
     (C ch) bf16 + the u8 LR copy + border bands (small)."""
     h, w, C, s = cfg["h"], cfg["w"], cfg["n_ch"], cfg["scale"]
     px = h * w * nb
-    return (px * 16 * 2 + 3 * px * C * 2 + px * 3 + nb * (8 * (w + h) * s * (C + 3) * 4)) / (1 << 30)
+    return (px * 8 * 2 + 3 * px * C * 2 + px * 3 + nb * (8 * (w + h) * s * (C + 3) * 4)) / (1 << 30)
 
 
 if __name__ == "__main__":

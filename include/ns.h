@@ -241,7 +241,7 @@ typedef struct {
     char name[24];
     uint64_t launches;     /* kernels launched                         */
     uint64_t scopes;       /* event-bracketed launch groups             */
-    double total_ms;       /* summed device time of those groups        */
+    double total_ms;       /* device time with >= 1 group running (the union of the groups' intervals) */
 } ns_prof_entry;
 NS_API int ns_profile_enable(int on);
 NS_API int ns_profile_read(ns_prof_entry *out, int max);

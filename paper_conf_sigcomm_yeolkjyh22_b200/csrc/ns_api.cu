@@ -9,6 +9,7 @@
 #include <atomic>
 #include <mutex>
 #include <algorithm>
+#include <deque>
 #include <map>
 #include <tuple>
 #include <vector>
@@ -154,7 +155,7 @@ static int host_groups() {
 }
 
 struct ArenaEntry {
-    int h, w, C, s;
+    int h, w, C, s, idx;   // idx: 0 / 1, the two arenas SR batches alternate between
     SrArena a;
 };
 }  // namespace
@@ -186,11 +187,13 @@ struct ns_ctx {
     uint16_t *blob_stage;  // device staging for host weight blobs
     size_t blob_stage_elems;
     int sr_batch = 16;
-    std::vector<ArenaEntry> arenas;
+    std::deque<ArenaEntry> arenas;   // deque: entries never move
     // host-input path (ns_enhance_streams_host): copy stream, two input staging
     // buffers (group ping-pong) and the anchor-LR gather staging, carved from
     // the pool on first use and grown (bump) if a later call needs more
     cudaStream_t cst = nullptr;
+    cudaStream_t sst = nullptr;          // second SR stream: odd batches, so one batch's tail overlaps the next
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     cudaEvent_t ev_copied[2] = {}, ev_free[2] = {};
     bool hin_used[2] = {};
     uint8_t *hin[2] = {};
@@ -280,9 +283,12 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     }
     c->lr_src = (const uint8_t **)pool_take(c, sizeof(uint8_t *) * kMaxJobs);
     c->lr_len = (uint32_t *)pool_take(c, sizeof(uint32_t) * kMaxJobs);
-    if ((e = cudaStreamCreateWithFlags(&c->cst, cudaStreamNonBlocking)) != cudaSuccess) {
+    if ((e = cudaStreamCreateWithFlags(&c->cst, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&c->sst, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming)) != cudaSuccess) {
         ns_ctx_destroy(c);
-        return cuda_fail(e, "copy stream");
+        return cuda_fail(e, "streams");
     }
     for (int i = 0; i < 2; i++)
         if ((e = cudaEventCreateWithFlags(&c->ev_copied[i], cudaEventDisableTiming)) != cudaSuccess ||
@@ -307,6 +313,9 @@ extern "C" ns_status ns_ctx_destroy(ns_ctx *c) {
         if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
     }
     if (c->cst) cudaStreamDestroy(c->cst);
+    if (c->sst) cudaStreamDestroy(c->sst);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
     if (c->pool) cudaFree(c->pool);
     delete c;
     return NS_OK;
@@ -388,14 +397,36 @@ extern "C" int ns_profile_read(ns_prof_entry *out, int max) {
         memset(&out[f], 0, sizeof(ns_prof_entry));
         snprintf(out[f].name, sizeof(out[f].name), "%s", fam_name(f));
     }
+    // total_ms = the union of the family's event intervals: launch groups of one
+    // family on two streams (alternating SR batches) overlap, and the union is
+    // the device time during which at least one of them ran (= the sum when
+    // they do not overlap)
+    std::vector<std::vector<std::pair<double, double>>> iv(F_COUNT);
     for (auto &r : g_recs) {
-        float ms = 0.f;
+        float a = 0.f, b = 0.f;
         cudaError_t e = cudaEventSynchronize(r.e1);
-        if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, r.e0, r.e1);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&a, g_recs[0].e0, r.e0);
+        if (e == cudaSuccess) e = cudaEventElapsedTime(&b, g_recs[0].e0, r.e1);
         if (e != cudaSuccess) return cuda_fail(e, "ns_profile_read");
         out[r.fam].launches += (uint64_t)r.n;
         out[r.fam].scopes += 1;
-        out[r.fam].total_ms += ms;
+        iv[r.fam].push_back({(double)a, (double)b});
+    }
+    for (int f = 0; f < F_COUNT; f++) {
+        auto &v = iv[f];
+        std::sort(v.begin(), v.end());
+        double tot = 0.0, lo = 0.0, hi = -1e300;
+        for (auto &x : v) {
+            if (x.first > hi) {
+                if (hi > lo) tot += hi - lo;
+                lo = x.first;
+                hi = x.second;
+            } else if (x.second > hi) {
+                hi = x.second;
+            }
+        }
+        if (!v.empty() && hi > lo) tot += hi - lo;
+        out[f].total_ms = tot;
     }
     return (int)F_COUNT;
 }
@@ -581,18 +612,22 @@ extern "C" ns_status ns_select_merge(ns_ctx *c, int S, int n, const int64_t *gai
 }
 
 // ------------------------------------------------------------------ SR
-static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, const SrArena **out) {
+static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int idx, const SrArena **out) {
     for (auto &e : c->arenas)
-        if (e.h == h && e.w == w && e.C == C && e.s == s) {
+        if (e.h == h && e.w == w && e.C == C && e.s == s && e.idx == idx) {
             *out = &e.a;
             return NS_OK;
         }
     const size_t bytes = sr_arena_bytes(h, w, C, s, c->sr_batch);
+    if (idx > 0 && c->used + bytes + 256 > c->pool_bytes) {  // no room for a second arena: one stream
+        *out = nullptr;
+        return NS_OK;
+    }
     uint8_t *mem = pool_take(c, bytes);
     if (!mem)
         return fail(NS_ENOMEM, "SR arena for %dx%d C%d x%d (%d jobs) needs %zu bytes; pool has %zu free", w, h, C, s,
                     c->sr_batch, bytes, c->pool_bytes - c->used);
-    ArenaEntry e{h, w, C, s, {}};
+    ArenaEntry e{h, w, C, s, idx, {}};
     if (sr_arena_init(&e.a, h, w, C, s, c->sr_batch, mem) != 0)
         return fail(NS_ECUDA, "cuTensorMapEncodeTiled failed for the SR arena");
     c->arenas.push_back(e);
@@ -600,15 +635,33 @@ static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, const SrArena 
     return NS_OK;
 }
 
-// jobs (device table) [0, max_jobs) of one shape; job_count (device) may be NULL
+// jobs (device table) [0, max_jobs) of one shape; job_count (device) may be NULL.
+// Batches alternate between `st` (arena 0) and the context's second SR stream
+// (arena 1), forked from and joined back into `st`: a batch's last wave (each
+// SR kernel's final partial wave of CTAs) overlaps the next batch's first.
 static ns_status run_sr_group(ns_ctx *c, int h, int w, int C, int s, int B, const SrJob *d_jobs, int max_jobs,
                               const int32_t *job_count, cudaStream_t st) {
-    const SrArena *a = nullptr;
-    ns_status r = get_arena(c, h, w, C, s, &a);
+    const SrArena *a[2] = {nullptr, nullptr};
+    ns_status r = get_arena(c, h, w, C, s, 0, &a[0]);
     if (r != NS_OK) return r;
-    for (int j0 = 0; j0 < max_jobs; j0 += a->nb) {
-        const int nj = std::min(a->nb, max_jobs - j0);
-        NS_CUDA(sr_run_batch(a, B, d_jobs, j0, nj, job_count, st));
+    const int nbatch = (max_jobs + a[0]->nb - 1) / a[0]->nb;
+#ifndef NS_SR_TWO_STREAMS
+#define NS_SR_TWO_STREAMS 1
+#endif
+    if (NS_SR_TWO_STREAMS && nbatch > 1 && (r = get_arena(c, h, w, C, s, 1, &a[1])) != NS_OK) return r;
+    const bool two = a[1] != nullptr;
+    if (two) {
+        NS_CUDA(cudaEventRecord(c->ev_fork, st));
+        NS_CUDA(cudaStreamWaitEvent(c->sst, c->ev_fork, 0));
+    }
+    for (int i = 0, j0 = 0; j0 < max_jobs; i++, j0 += a[0]->nb) {
+        const int nj = std::min(a[0]->nb, max_jobs - j0);
+        const bool odd = two && (i & 1);
+        NS_CUDA(sr_run_batch(a[odd ? 1 : 0], B, d_jobs, j0, nj, job_count, odd ? c->sst : st));
+    }
+    if (two) {
+        NS_CUDA(cudaEventRecord(c->ev_join, c->sst));
+        NS_CUDA(cudaStreamWaitEvent(st, c->ev_join, 0));
     }
     return NS_OK;
 }
