@@ -356,11 +356,11 @@ cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_
 
 template <int S>
 __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
-    k_recon_step(const FrameDesc *fdesc, int n, int f) {
+    k_recon_step(const FrameDesc *fdesc, int n, int f, int s0) {
     using Cfg = ReconCfg<S>;
     using Sm = ReconSmem<S>;
     constexpr int NP = Cfg::NP, RPT = Cfg::RPT, NQ = Cfg::NQ;
-    const int sid = blockIdx.z;
+    const int sid = s0 + blockIdx.z;
     const FrameDesc fd = fdesc[(size_t)sid * n + f];
     if (fd.anchor || fd.s != S) return;                 // CTA-uniform: anchors already hold SR bytes
     const int w = fd.w, h = fd.h, H = h * S, W = w * S;
@@ -515,7 +515,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
 }
 
 template <int S>
-static void recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f) {
+static void recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ReconSmem<S>::BYTES);
@@ -524,11 +524,11 @@ static void recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, in
                              (int)cudaSharedmemCarveoutMaxShared);
         attr = true;
     }
-    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f);
+    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f, s0);
 }
 
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              cudaStream_t st) {
+                              cudaStream_t st, int s0) {
     int nl = 0;
     for (int s = 2; s <= 4; s++) nl += max_lr_w[s] > 0;
     KScope ks(F_RECON, st, nl);
@@ -537,9 +537,9 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
         const int nbx = max_lr_w[s] / 8;          // LR block columns
         const int nrg = max_lr_h[s] * s / (s == 3 ? 6 : 8);  // groups of RPT HR rows
         dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
-        if (s == 2) recon_launch<2>(g, st, fd, n, f);
-        if (s == 3) recon_launch<3>(g, st, fd, n, f);
-        if (s == 4) recon_launch<4>(g, st, fd, n, f);
+        if (s == 2) recon_launch<2>(g, st, fd, n, f, s0);
+        if (s == 3) recon_launch<3>(g, st, fd, n, f, s0);
+        if (s == 4) recon_launch<4>(g, st, fd, n, f, s0);
     }
     return cudaGetLastError();
 }

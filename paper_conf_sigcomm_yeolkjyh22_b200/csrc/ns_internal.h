@@ -119,7 +119,7 @@ cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *g
 cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
                               uint8_t *const *d_hr_table, const int16_t *gold_idx, FrameDesc *fd, cudaStream_t st);
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              cudaStream_t st);
+                              cudaStream_t st, int s0 = 0);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,

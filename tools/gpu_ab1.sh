@@ -1,1 +1,2 @@
-LIBS="default tools/bin/lib_one.so default tools/bin/lib_one.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
+LIBS="default tools/bin/lib_r1.so default tools/bin/lib_r1.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
