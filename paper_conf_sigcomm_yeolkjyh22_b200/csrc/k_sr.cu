@@ -1954,7 +1954,11 @@ static cudaError_t conv(int fam, const CUtensorMap &tm, ConvArgs args, int nj, c
     return cudaGetLastError();
 }
 
-constexpr int kRotRows = 64;  // rows per CTA strip of the rotated conv
+// (A/B: 64 -> 120 rows 198.8 -> 197.5 ms per c4 step; 120 -> 180 191.9 -> 190.2; 360 no better)
+#ifndef NS_ROT_ROWS
+#define NS_ROT_ROWS 180
+#endif
+constexpr int kRotRows = NS_ROT_ROWS;  // rows per CTA strip of the rotated conv and uptail2
 template <int CIN, int NB, int EPI>
 static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = RotCfg<CIN, NB>;
@@ -1991,7 +1995,14 @@ static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStre
     return cudaGetLastError();
 }
 
-constexpr int kRbRows = 120;
+// Taller strips = fewer halo rows and prologues per CTA; with the two SR streams
+// overlapping each batch's last partial wave, the wave count per launch matters
+// less.  A/B (ms per c4 step, same box): 120 -> 240 rows 198.8 -> 196.2; 240 ->
+// 360 191.9 -> 190.8; 720 no better.
+#ifndef NS_RB_ROWS
+#define NS_RB_ROWS 360
+#endif
+constexpr int kRbRows = NS_RB_ROWS;  // rows per CTA strip of the fused res-block
 template <int C>
 static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, cudaStream_t st) {
     using Cfg = RbCfg<C>;
