@@ -225,7 +225,7 @@ def main():
     ap.add_argument("--distinct", type=int, default=8, help="distinct generated streams (replicated on device)")
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--sr-batch", type=int, default=16)
+    ap.add_argument("--sr-batch", type=int, default=int(os.environ.get("NS_SR_BATCH", "16")))
     ap.add_argument("--balance", action="store_true",
                     help="with --select global: anchor-level load balancing across GPUs (shard.plan_anchor_moves; "
                          "LR out / HR back point-to-point), then ns_sr_anchors + ns_reconstruct_chunk")

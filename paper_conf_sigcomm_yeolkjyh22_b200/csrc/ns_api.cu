@@ -154,6 +154,14 @@ static int host_groups() {
     return g;
 }
 
+// SR batch (jobs per arena); NS_SR_BATCH in the environment overrides it
+// (tuning experiments only)
+static int sr_batch_default() {
+    const char *e = getenv("NS_SR_BATCH");
+    const int v = e ? atoi(e) : 0;
+    return v > 0 ? v : 16;
+}
+
 struct ArenaEntry {
     int h, w, C, s, idx;   // idx: 0 / 1, the two arenas SR batches alternate between
     SrArena a;
@@ -186,7 +194,7 @@ struct ns_ctx {
     SrJob *jobs;
     uint16_t *blob_stage;  // device staging for host weight blobs
     size_t blob_stage_elems;
-    int sr_batch = 16;
+    int sr_batch = sr_batch_default();  // anchors per SR batch (arena size)
     std::deque<ArenaEntry> arenas;   // deque: entries never move
     // host-input path (ns_enhance_streams_host): copy stream, two input staging
     // buffers (group ping-pong) and the anchor-LR gather staging, carved from

@@ -2,7 +2,12 @@
 # A/B of library variants on one box: bench (device path only) per NS_LIB; prints value and family ms.
 # usage: LIBS="default tools/bin/lib_a.so ..." bash tools/ab_libs.sh
 for L in ${LIBS:-default}; do
-  if [ "$L" = default ]; then unset NS_LIB; else export NS_LIB=$PWD/$L; fi
+  unset NS_SR_BATCH
+  case "$L" in
+    default) unset NS_LIB ;;
+    env:*) unset NS_LIB; export ${L#env:} ;;
+    *) export NS_LIB=$PWD/$L ;;
+  esac
   python bench.py --steps ${STEPS:-5} --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab.json 2>gpurun_out/ab.err
   python - "$L" <<'PY'
 import json, sys

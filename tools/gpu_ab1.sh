@@ -1,1 +1,1 @@
-LIBS="default tools/bin/lib_rb720.so tools/bin/lib_rot360.so tools/bin/lib_prev.so default tools/bin/lib_rb720.so tools/bin/lib_rot360.so tools/bin/lib_prev.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+LIBS="default env:NS_SR_BATCH=24 env:NS_SR_BATCH=32 env:NS_SR_BATCH=12 default env:NS_SR_BATCH=24 env:NS_SR_BATCH=32 env:NS_SR_BATCH=12" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
