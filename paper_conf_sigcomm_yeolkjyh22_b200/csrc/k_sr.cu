@@ -1998,9 +1998,11 @@ static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStre
 // Taller strips = fewer halo rows and prologues per CTA; with the two SR streams
 // overlapping each batch's last partial wave, the wave count per launch matters
 // less.  A/B (ms per c4 step, same box): 120 -> 240 rows 198.8 -> 196.2; 240 ->
-// 360 191.9 -> 190.8; 720 no better.
+// 360 191.9 -> 190.8 (within noise); 720 no better.  240 rows = 3 strips =
+// 288 CTAs per 16-job launch, 1.95 waves of 148 SMs, so a launch that runs
+// alone (no overlap) wastes little as well: 240.
 #ifndef NS_RB_ROWS
-#define NS_RB_ROWS 360
+#define NS_RB_ROWS 240
 #endif
 constexpr int kRbRows = NS_RB_ROWS;  // rows per CTA strip of the fused res-block
 template <int C>
