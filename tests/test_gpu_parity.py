@@ -251,6 +251,15 @@ def test_enhance_multistream_mixed(ctx):
     _enhance_vs_oracle(ctx, cs, specs, k=3)
 
 
+def test_enhance_two_sr_batches(ctx):
+    """More anchors of one shape than one SR batch holds (24 > 16): the batches
+    alternate between the caller's stream and the context's second SR stream,
+    each with its own arena (ns_api.cu run_sr_group); the results are the
+    oracle's as for one batch."""
+    cs = [synth.make_chunk(2300 + i, 48, 24, 2, 8, types=synth.default_types(8, 4), with_gt=True) for i in range(6)]
+    _enhance_vs_oracle(ctx, cs, [(1, 16)] * 6, k=4)
+
+
 @pytest.mark.parametrize("k", [0, 8])
 def test_enhance_k_extremes(ctx, k):
     """k = 0 (pure reuse from KEY up-sampling) and k = n (per-frame SR)."""

@@ -1,1 +1,1 @@
-LIBS="default env:NS_SR_BATCH=24 env:NS_SR_BATCH=32 env:NS_SR_BATCH=12 default env:NS_SR_BATCH=24 env:NS_SR_BATCH=32 env:NS_SR_BATCH=12" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "two_sr_batches or enhance" > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
