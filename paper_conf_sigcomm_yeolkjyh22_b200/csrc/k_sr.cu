@@ -44,8 +44,6 @@ __device__ unsigned long long g_trace[16 * 2 * 1024];
 // real channels: only channel group 0 (8 channels, 16 B/px) is stored and
 // loaded by TMA; group 1 of every ring slot is a zero region written once.
 enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4, EPI_HEAD = 5 };
-constexpr int kSlots = 6;
-constexpr int kRows = 32;   // rows per CTA strip
 
 struct ConvArgs {
     int H, W;               // conv spatial dims (input == output)
@@ -69,22 +67,6 @@ __host__ __device__ constexpr uint32_t tmem_cols_for(uint32_t c) {
     return c <= 32 ? 32 : c <= 64 ? 64 : c <= 128 ? 128 : c <= 256 ? 256 : 512;
 }
 
-template <int CIN, int NT, int NSPLIT>
-struct ConvCfg {
-    static constexpr int NTOT = NT * NSPLIT;
-    static constexpr int KC = CIN / 16;
-    static constexpr uint32_t B_BYTES = 9u * CIN * NTOT * 2u;
-    static constexpr uint32_t BIAS_BYTES = NTOT * 4u;
-    static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
-    static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
-    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int ACCB = (NTOT <= 256) ? 2 : 1;
-    static constexpr uint32_t TMEM_COLS = tmem_cols_for(ACCB * NTOT);
-    static constexpr uint32_t SMEM = W_REGION + kSlots * SLOT + 128;
-    static_assert(NT % 16 == 0 && NT >= 16 && NT <= 256, "UMMA M=128 needs N % 16 == 0, 16..256");
-    static_assert(CIN % 16 == 0, "Cin multiple of 16");
-    static_assert(SMEM <= 232448, "shared memory");
-};
 
 __device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
     __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
@@ -101,221 +83,6 @@ __device__ __forceinline__ void up_tap(int X, int s, int len, int &i0, int &i1, 
     w1 = (128 * rem + s) / (2 * s);
     i0 = min(max(x0, 0), len - 1);
     i1 = min(max(x0 + 1, 0), len - 1);
-}
-
-template <int CIN, int NT, int NSPLIT, int EPI>
-__global__ void __launch_bounds__(128) k_conv3x3(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
-    using Cfg = ConvCfg<CIN, NT, NSPLIT>;
-    constexpr int NTOT = Cfg::NTOT;
-    constexpr int ACCB = Cfg::ACCB;
-    extern __shared__ __align__(1024) uint8_t smem[];
-    uint8_t *s_w = smem;
-    const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
-    uint8_t *s_ring = smem + Cfg::W_REGION;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + kSlots * Cfg::SLOT);  // [0,6) ring, 6 w, 7-8 mma
-    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 10);
-
-    const int slot_job = blockIdx.z;
-    const int job = a.j0 + slot_job;
-    if (a.job_count && job >= *a.job_count) return;
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int x0 = blockIdx.x * kTile;
-    const int y0 = blockIdx.y * a.rows_per_cta;
-    const int y1 = min(y0 + a.rows_per_cta, a.H);
-    const int nrows = y1 - y0;
-    const int n_loads = nrows + 2;  // rows y0-1 .. y1
-
-    if (tid == 0) {
-        for (int i = 0; i < 9; i++) mbar_init(&bars[i], 1);
-        fence_mbar_init();
-    }
-    if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
-    tc_fence_before();
-    __syncthreads();
-    tc_fence_after();
-    const uint32_t tmem = *s_tmem;
-    const SrJob J = a.jobs[job];
-
-    if (tid == 0) {
-        prefetch_tmap(&tm_in);
-        mbar_arrive_expect_tx(&bars[6], Cfg::B_BYTES + Cfg::BIAS_BYTES);
-        bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[6]);
-        bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[6]);
-        for (int q = 0; q < 4 && q < n_loads; q++) {
-            mbar_arrive_expect_tx(&bars[q % kSlots], Cfg::SLOT_BYTES);
-            tma_load_5d(s_ring + (q % kSlots) * Cfg::SLOT, &tm_in, &bars[q % kSlots], 0, x0 - 1, 0, y0 - 1 + q,
-                        slot_job);
-        }
-    }
-
-    const uint32_t idesc = idesc_bf16_f32(128, NT);
-    auto issue = [&](int r) {  // MMAs of output row y0 + r (thread 0 only)
-        for (int d = 0; d < 3; d++) {
-            const int q = r + d;
-            mbar_wait(&bars[q % kSlots], (q / kSlots) & 1);
-        }
-        tc_fence_after();
-        const uint32_t acc = tmem + (uint32_t)((r % ACCB) * NTOT);
-        const uint32_t wbase = smem_u32(s_w);
-#pragma unroll
-        for (int sp = 0; sp < NSPLIT; sp++) {
-#pragma unroll
-            for (int tap = 0; tap < 9; tap++) {
-                const int dy = tap / 3, dx = tap % 3;
-                const uint32_t abase = smem_u32(s_ring + ((r + dy) % kSlots) * Cfg::SLOT);
-#pragma unroll
-                for (int kc = 0; kc < Cfg::KC; kc++) {
-                    const uint64_t ad = smem_desc(abase + (uint32_t)(2 * kc * kHalo * 16 + dx * 16), kHalo * 16, 128);
-                    const uint64_t bd =
-                        smem_desc(wbase + (uint32_t)(((sp * 9 + tap) * Cfg::KC + kc) * 2 * NT * 16), NT * 16, 128);
-                    umma_bf16(acc + sp * NT, ad, bd, idesc, (tap | kc) != 0 ? 1u : 0u);
-                }
-            }
-        }
-        umma_commit(&bars[7 + (r % ACCB)]);
-    };
-
-    mbar_wait(&bars[6], 0);  // weights + bias resident (all threads: epilogue reads the bias)
-    if (tid == 0 && ACCB == 2) issue(0);
-
-    const int p = warp * 32 + lane;  // TMEM lane == pixel of the tile
-    const int x = x0 + p;
-    for (int r = 0; r < nrows; r++) {
-        if (tid == 0) {
-            const int q = r + 4;  // prefetch row y0 + r + 3 into the slot freed by MMA(r - 2)
-            if (q < n_loads) {
-                mbar_arrive_expect_tx(&bars[q % kSlots], Cfg::SLOT_BYTES);
-                tma_load_5d(s_ring + (q % kSlots) * Cfg::SLOT, &tm_in, &bars[q % kSlots], 0, x0 - 1, 0,
-                            y0 - 1 + q, slot_job);
-            }
-            if (ACCB == 1) issue(r);
-            else if (r + 1 < nrows) issue(r + 1);
-        }
-        __syncwarp();
-        // residual rows are prefetched before waiting for the MMA (latency overlap)
-        constexpr int RC = (EPI == EPI_RESID) ? NT / 8 : 1;
-        uint4 rres[RC];
-        if constexpr (EPI == EPI_RESID) {
-            if (x < a.W) {
-                const size_t rb = ((size_t)slot_job * a.H + (y0 + r)) * (NT / 8);
-#pragma unroll
-                for (int cg = 0; cg < RC; cg++)
-                    rres[cg] = __ldg(reinterpret_cast<const uint4 *>(a.resid + ((rb + cg) * a.W + x) * 8));
-            }
-        }
-        mbar_wait(&bars[7 + (r % ACCB)], (r / ACCB) & 1);
-        tc_fence_after();
-        const uint32_t acc = tmem + (uint32_t)((r % ACCB) * NTOT) + ((uint32_t)(warp * 32) << 16);
-        const int y = y0 + r;
-
-        if constexpr (EPI == EPI_STORE || EPI == EPI_RELU || EPI == EPI_RESID) {
-            static_assert(NSPLIT == 1, "");
-            constexpr int C = NT;
-            uint32_t v[C];
-            if constexpr (C == 32) {
-                uint32_t (&vv)[32] = *reinterpret_cast<uint32_t(*)[32]>(v);
-                tmem_ld32(acc, vv);
-            } else {
-                uint32_t (&vv)[16] = *reinterpret_cast<uint32_t(*)[16]>(v);
-                tmem_ld16(acc, vv);
-            }
-            tmem_wait_ld();
-            if (x < a.W) {
-                const size_t rowbase = ((size_t)slot_job * a.H + y) * (C / 8);
-#pragma unroll
-                for (int cg = 0; cg < C / 8; cg++) {
-                    float f[8];
-#pragma unroll
-                    for (int i = 0; i < 8; i++) {
-                        f[i] = __uint_as_float(v[cg * 8 + i]) + s_bias[cg * 8 + i];
-                        if (EPI == EPI_RELU) f[i] = fmaxf(f[i], 0.f);
-                    }
-                    const size_t off = ((rowbase + cg) * a.W + x) * 8;
-                    if (EPI == EPI_RESID) {
-                        const uint4 rr = rres[cg];
-                        f[0] += bf_lo(rr.x); f[1] += bf_hi(rr.x);
-                        f[2] += bf_lo(rr.y); f[3] += bf_hi(rr.y);
-                        f[4] += bf_lo(rr.z); f[5] += bf_hi(rr.z);
-                        f[6] += bf_lo(rr.w); f[7] += bf_hi(rr.w);
-                    }
-                    uint4 o;
-                    o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
-                    o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
-                    *reinterpret_cast<uint4 *>(a.out + off) = o;
-                }
-            }
-        } else if constexpr (EPI == EPI_SHUFFLE) {
-            // D column n' = (i*s + j) * C + c  <->  upsampler channel c*s*s + i*s + j
-            // (rows permuted at repack) -> HR pixel (s*y + i, s*x + j), channel c.
-            const int C = a.C, s = a.s;
-            const int Hs = a.H * s, Ws = a.W * s;
-            const int nsub = NTOT / C;
-            for (int sub = 0; sub < nsub; sub++) {
-                const int gsub = a.sub0 + sub;
-                const int i = gsub / s, j = gsub % s;
-                const size_t rowbase = ((size_t)slot_job * Hs + (size_t)(s * y + i)) * (C / 8);
-                if (C == 32) {
-                    uint32_t v[32];
-                    tmem_ld32(acc + sub * 32, v);
-                    tmem_wait_ld();
-                    if (x < a.W) {
-#pragma unroll
-                        for (int cg = 0; cg < 4; cg++) {
-                            const float *b = s_bias + sub * 32 + cg * 8;
-                            uint4 o;
-                            o.x = pack_bf16(__uint_as_float(v[cg * 8 + 0]) + b[0], __uint_as_float(v[cg * 8 + 1]) + b[1]);
-                            o.y = pack_bf16(__uint_as_float(v[cg * 8 + 2]) + b[2], __uint_as_float(v[cg * 8 + 3]) + b[3]);
-                            o.z = pack_bf16(__uint_as_float(v[cg * 8 + 4]) + b[4], __uint_as_float(v[cg * 8 + 5]) + b[5]);
-                            o.w = pack_bf16(__uint_as_float(v[cg * 8 + 6]) + b[6], __uint_as_float(v[cg * 8 + 7]) + b[7]);
-                            *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * Ws + (size_t)(s * x + j)) * 8) = o;
-                        }
-                    }
-                } else {
-                    uint32_t v[16];
-                    tmem_ld16(acc + sub * 16, v);
-                    tmem_wait_ld();
-                    if (x < a.W) {
-#pragma unroll
-                        for (int cg = 0; cg < 2; cg++) {
-                            const float *b = s_bias + sub * 16 + cg * 8;
-                            uint4 o;
-                            o.x = pack_bf16(__uint_as_float(v[cg * 8 + 0]) + b[0], __uint_as_float(v[cg * 8 + 1]) + b[1]);
-                            o.y = pack_bf16(__uint_as_float(v[cg * 8 + 2]) + b[2], __uint_as_float(v[cg * 8 + 3]) + b[3]);
-                            o.z = pack_bf16(__uint_as_float(v[cg * 8 + 4]) + b[4], __uint_as_float(v[cg * 8 + 5]) + b[5]);
-                            o.w = pack_bf16(__uint_as_float(v[cg * 8 + 6]) + b[6], __uint_as_float(v[cg * 8 + 7]) + b[7]);
-                            *reinterpret_cast<uint4 *>(a.out + ((rowbase + cg) * Ws + (size_t)(s * x + j)) * 8) = o;
-                        }
-                    }
-                }
-            }
-        } else {  // EPI_TAIL: out = clamp(floor(up_s(LR) + t + 0.5), 0, 255), u8 planar HR
-            static_assert(NT == 16 && NSPLIT == 1, "");
-            uint32_t v[16];
-            tmem_ld16(acc, v);
-            tmem_wait_ld();
-            if (x < a.W) {
-                const int s = a.s, lh = a.lr_h, lw = a.lr_w;
-                int ya, yb, wy, xa, xb, wx;
-                up_tap(y, s, lh, ya, yb, wy);
-                up_tap(x, s, lw, xa, xb, wx);
-                const size_t plane = (size_t)lh * lw, hplane = (size_t)a.H * a.W;
-#pragma unroll
-                for (int c = 0; c < 3; c++) {
-                    const uint8_t *L = J.lr + c * plane;
-                    const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
-                    const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
-                    const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
-                    const int U = (vv + 8192) >> 14;
-                    const float t = __uint_as_float(v[c]) + s_bias[c];
-                    const float o = floorf((float)U + t + 0.5f);
-                    J.hr[c * hplane + (size_t)y * a.W + x] = (uint8_t)fminf(fmaxf(o, 0.f), 255.f);
-                }
-            }
-        }
-        tc_fence_before();
-        __syncthreads();
-    }
-    if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
 }
 
 // ------------------------------------------------------------------ rotated-accumulator conv
@@ -1934,24 +1701,6 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     rc |= make_act_map(&a->tm_tb5, a->tb, h, w, C, nb, kHalo5);
     rc |= make_act_map(&a->tm_hb5, a->hb, h, w, C, nb, kHalo5);
     return rc;
-}
-
-template <int CIN, int NT, int NSPLIT, int EPI>
-static cudaError_t conv(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
-    using Cfg = ConvCfg<CIN, NT, NSPLIT>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_conv3x3<CIN, NT, NSPLIT, EPI>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
-    args.n_xtiles = (args.W + kTile - 1) / kTile;
-    args.rows_per_cta = kRows;
-    dim3 grid(args.n_xtiles, (args.H + kRows - 1) / kRows, nj);
-    KScope ks(fam, st);
-    k_conv3x3<CIN, NT, NSPLIT, EPI><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
-    return cudaGetLastError();
 }
 
 // (A/B: 64 -> 120 rows 198.8 -> 197.5 ms per c4 step; 120 -> 180 191.9 -> 190.2; 360 no better)
