@@ -60,6 +60,8 @@ struct ConvArgs {
     int sub0;               // shuffle: first sub-pixel of this launch
     int lr_h, lr_w;         // tail: LR dims of the bilinear skip
     float *ring;            // uptail: fp32 t of the HR frame-border ring [job][nring][3]
+    uint8_t *lr8;           // EPI_HEAD with NS_HEAD_BUILD: u8 LR copy [job][H][3][wp] for uptail2
+    int wp;
 };
 
 __host__ __device__ constexpr uint32_t round_up(uint32_t v, uint32_t a) { return (v + a - 1) / a * a; }
@@ -99,6 +101,17 @@ __device__ __forceinline__ void up_tap(int X, int s, int len, int &i0, int &i1, 
 // block of row y-1 is complete: the epilogue reads it, applies the fused
 // epilogue, and zeroes it for row y+2.  No im2col, no lane shifts, 128-pixel
 // tiles, N = 96 (C = 32) -> up to 3x the MMA efficiency of N = 32.
+// NS_HEAD_BUILD: the head conv builds its own input rows (x = LR - 128, bf16,
+// channel group 0) from the u8 LR planes in a dedicated builder warp (warp 4)
+// and writes uptail2's u8 LR copy itself -- no prep pass, no bf16 input copy in
+// HBM.  The builder never stores the conv output, so its proxy fence does not
+// wait on the epilogue's global stores (the reason a same-warp build was slower).
+// Parity green, measured neutral (prep + head 10.76 vs head 10.8 ms per c4 step,
+// union over the two SR streams): one warp of byte loads builds rows no faster
+// than the prep pass + bulk copy deliver them.  Off.
+#ifndef NS_HEAD_BUILD
+#define NS_HEAD_BUILD 0
+#endif
 #ifndef NS_ROT_NSLOT
 #define NS_ROT_NSLOT 3  // input ring of k_conv_rot (head, end)
 #endif
@@ -254,14 +267,17 @@ __device__ __forceinline__ void row_bulk(uint8_t *slot, int ncols, const uint16_
 }
 
 template <int CIN, int NB, int EPI>
-__global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
+__global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128)
+    k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
     using Cfg = RotCfg<CIN, NB>;
+    constexpr bool BUILD = EPI == EPI_HEAD && NS_HEAD_BUILD;  // warp 4 = input-row builder
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *s_w = smem;
     const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
     uint8_t *s_ring = smem + Cfg::W_REGION;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + Cfg::NSLOT * Cfg::SLOT);  // [0,3) ring, 3 w, 4 mma
-    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 6);
+    // [0,3) ring full, 3 weights, 4 MMA done, [5,8) ring empty (BUILD)
+    uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + Cfg::NSLOT * Cfg::SLOT);
+    uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 8);
 
     const int slot_job = blockIdx.z;
     const int job = a.j0 + slot_job;
@@ -273,7 +289,7 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     const int n_loads = y1 - y0 + 2;  // input rows y0-1 .. y1
 
     if (tid == 0) {
-        for (int i = 0; i < 5; i++) mbar_init(&bars[i], 1);
+        for (int i = 0; i < 8; i++) mbar_init(&bars[i], 1);
         fence_mbar_init();
     }
     if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
@@ -296,7 +312,9 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     // rows by bulk copies (row_bulk): G channel groups of 16 B per pixel
     constexpr int G = (EPI == EPI_HEAD) ? 1 : CIN / 8;
     (void)LOAD_BYTES;
-    for (int sl = 0; sl < Cfg::NSLOT; sl++) slot_zero_edges<G>(s_ring + sl * Cfg::SLOT, kHalo, a.W, x0 - 1, tid, blockDim.x);
+    if constexpr (!BUILD)
+        for (int sl = 0; sl < Cfg::NSLOT; sl++)
+            slot_zero_edges<G>(s_ring + sl * Cfg::SLOT, kHalo, a.W, x0 - 1, tid, blockDim.x);
     fence_proxy_async_smem();
     __syncthreads();
 #endif
@@ -305,7 +323,7 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
         bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
         bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
-        for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
+        for (int q = 0; q < Cfg::NSLOT && q < n_loads && !BUILD; q++) {
 #if NS_ROT_BULK
             row_bulk<G>(s_ring + q * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + q, x0 - 1, &bars[q]);
 #else
@@ -314,11 +332,13 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
 #endif
         }
     }
-    // the three accumulator blocks start at zero
-    tmem_zero<NB>(tl);
-    tmem_zero<NB>(tl + NB);
-    tmem_zero<NB>(tl + 2 * NB);
-    tmem_wait_st();
+    // the three accumulator blocks start at zero (the builder warp owns no TMEM lanes)
+    if (warp < 4) {
+        tmem_zero<NB>(tl);
+        tmem_zero<NB>(tl + NB);
+        tmem_zero<NB>(tl + 2 * NB);
+        tmem_wait_st();
+    }
     mbar_wait(&bars[3], 0);
     tc_fence_before();
     __syncthreads();
@@ -331,7 +351,54 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
     uint4 rnext[RC];  // EPI_RESID: residual row prefetched one step ahead
 #pragma unroll
     for (int cg = 0; cg < RC; cg++) rnext[cg] = make_uint4(0, 0, 0, 0);
-    for (int q = 0; q < n_loads; q++) {
+    if (BUILD && warp == 4) {
+        // ---- builder: row q of the ring slot q % NSLOT once MMA(q - NSLOT) has
+        // read it; lane l owns pixels l + 32 i of the 130-pixel row.  The LR
+        // bytes of row q are loaded before the wait for the slot.
+        const size_t plane = (size_t)a.H * a.W;
+        for (int q = 0; q < n_loads; q++) {
+            const int yin = y0 - 1 + q, sl = q % Cfg::NSLOT;
+            uint32_t rgb[5];
+#pragma unroll
+            for (int i = 0; i < 5; i++) {
+                const int px = lane + 32 * i, xx = x0 - 1 + px;
+                rgb[i] = 0xFFFFFFFFu;
+                if (px < kHalo && yin >= 0 && yin < a.H && xx >= 0 && xx < a.W) {
+                    const uint8_t *L = J.lr + (size_t)yin * a.W + xx;
+                    rgb[i] = (uint32_t)__ldg(L) | ((uint32_t)__ldg(L + plane) << 8) |
+                             ((uint32_t)__ldg(L + 2 * plane) << 16);
+                }
+            }
+            if (q >= Cfg::NSLOT) mbar_wait(&bars[5 + sl], ((q / Cfg::NSLOT) - 1) & 1);
+#pragma unroll
+            for (int i = 0; i < 5; i++) {
+                const int px = lane + 32 * i;
+                if (px >= kHalo) continue;
+                uint4 o = make_uint4(0, 0, 0, 0);
+                if (rgb[i] != 0xFFFFFFFFu) {
+                    o.x = pack_bf16((float)(int)(rgb[i] & 255) - 128.f, (float)(int)((rgb[i] >> 8) & 255) - 128.f);
+                    o.y = pack_bf16((float)(int)((rgb[i] >> 16) & 255) - 128.f, 0.f);
+                }
+                *reinterpret_cast<uint4 *>(s_ring + sl * Cfg::SLOT + px * 16) = o;
+            }
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_state(&bars[sl]);
+            if (yin >= y0 && yin < y1) {  // uptail2's u8 LR copy: each pixel of the CTA's own rows once
+#pragma unroll
+                for (int i = 0; i < 5; i++) {
+                    const int px = lane + 32 * i, xx = x0 - 1 + px;
+                    if (px < kHalo && xx >= x0 && xx < x0 + kTile && rgb[i] != 0xFFFFFFFFu) {
+                        uint8_t *l8 = a.lr8 + ((size_t)slot_job * a.H + yin) * 3 * a.wp + xx;
+                        l8[0] = (uint8_t)rgb[i];
+                        l8[a.wp] = (uint8_t)(rgb[i] >> 8);
+                        l8[2 * a.wp] = (uint8_t)(rgb[i] >> 16);
+                    }
+                }
+            }
+        }
+    }
+    for (int q = 0; q < n_loads && (!BUILD || warp < 4); q++) {
         const int yin = y0 - 1 + q;
         if (tid == 0) {
             const int sl = q % Cfg::NSLOT;
@@ -351,6 +418,7 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
                 }
             }
             umma_commit(&bars[4]);
+            if constexpr (BUILD) umma_commit(&bars[5 + sl]);  // the builder may refill the slot
         }
         __syncwarp();
         const int r = yin - 1;  // output row completed by this input row
@@ -372,7 +440,7 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         }
         mbar_wait(&bars[4], q & 1);
         tc_fence_after();
-        if (tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
+        if (!BUILD && tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
             const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
 #if NS_ROT_BULK
             row_bulk<G>(s_ring + sl * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + qn, x0 - 1, &bars[sl]);
@@ -436,7 +504,8 @@ __global__ void __launch_bounds__(128) k_conv_rot(const __grid_constant__ CUtens
         }
         tmem_wait_st();
         tc_fence_before();
-        __syncthreads();
+        if constexpr (BUILD) asm volatile("bar.sync 1, 128;" ::: "memory");  // the 4 MMA/epilogue warps
+        else __syncthreads();
         tc_fence_after();
     }
     if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
@@ -1722,7 +1791,8 @@ static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int n
     args.rows_per_cta = kRotRows;
     dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
     KScope ks(fam, st);
-    k_conv_rot<CIN, NB, EPI><<<grid, 128, Cfg::SMEM, st>>>(tm, args);
+    constexpr int threads = (EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128;
+    k_conv_rot<CIN, NB, EPI><<<grid, threads, Cfg::SMEM, st>>>(tm, args);
     return cudaGetLastError();
 }
 
@@ -1795,18 +1865,21 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
                            const int32_t *job_count, cudaStream_t st) {
     const int h = a->h, w = a->w, s = a->s;
     cudaError_t e;
+#if !NS_HEAD_BUILD
     {
         dim3 g((h * w + 255) / 256, nj);
         KScope ks(F_SR_PREP, st);
         k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
+#endif
     ConvArgs base{};
     base.H = h; base.W = w; base.j0 = j0; base.jobs = jobs; base.job_count = job_count; base.C = C; base.s = s;
     auto L = [&](int l) { return model_layer(n_blocks, C, s, l); };
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0; g.in = a->x0;
+        g.lr8 = a->lr8; g.wp = a->wp;  // NS_HEAD_BUILD: the head writes uptail2's u8 LR copy
         if ((e = conv_rot<16, C, EPI_HEAD>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     // residual blocks, fused (conv1 + ReLU + conv2 + skip), ping-pong hb / tb

@@ -1,1 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "two_sr_batches or enhance" > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
+timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/t3.log 2>&1; echo TESTS $? >> gpurun_out/t3.log
+LIBS="default tools/bin/lib_nobuild.so default tools/bin/lib_nobuild.so" bash tools/ab_libs.sh > gpurun_out/ab1.txt 2>&1
