@@ -77,6 +77,9 @@ __device__ __forceinline__ void static_for(F &&f) {
 #define NS_RECON_TY 4
 #endif
 constexpr int kReconTX = NS_RECON_TX, kReconTY = NS_RECON_TY;
+#ifndef NS_RECON_RPT3
+#define NS_RECON_RPT3 6  // HR rows per thread at s = 3 (a multiple of 3)
+#endif
 constexpr int kReconNT = kReconTX * kReconTY;
 #ifndef NS_RECON_MINB3
 #define NS_RECON_MINB3 (512 / (NS_RECON_TX * NS_RECON_TY))
@@ -88,7 +91,8 @@ struct ReconCfg {
     static constexpr int WIN = BW + 1;             // reference bytes per row
     static constexpr int NQ = (7 + WIN + 7) / 8;   // aligned 64-bit words per row
     static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
-    static constexpr int RPT = (S == 3) ? 6 : 8;   // HR rows per thread: a multiple of S
+    static constexpr int RPT = (S == 3) ? NS_RECON_RPT3 : 8;  // HR rows per thread: a multiple of S
+    static_assert(RPT % S == 0 && (8 * S) % RPT == 0, "a thread's rows lie in one 8x8 LR block row (uniform MV)");
     static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
     // resident CTAs per SM (registers): 512 threads at 128 registers for s = 3
     static constexpr int MINB = (S == 3) ? NS_RECON_MINB3 : (384 / kReconNT > 0 ? 384 / kReconNT : 1);
@@ -535,7 +539,8 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
     for (int s = 2; s <= 4; s++) {
         if (max_lr_w[s] <= 0) continue;
         const int nbx = max_lr_w[s] / 8;          // LR block columns
-        const int nrg = max_lr_h[s] * s / (s == 3 ? 6 : 8);  // groups of RPT HR rows
+        const int rpt = s == 2 ? ReconCfg<2>::RPT : s == 3 ? ReconCfg<3>::RPT : ReconCfg<4>::RPT;
+        const int nrg = (max_lr_h[s] * s + rpt - 1) / rpt;  // groups of RPT HR rows
         dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
         if (s == 2) recon_launch<2>(g, st, fd, n, f, s0);
         if (s == 3) recon_launch<3>(g, st, fd, n, f, s0);
