@@ -219,6 +219,12 @@ __device__ __forceinline__ void tmem_zeroN(uint32_t a) {
 #endif
 // (k_uptail2 with bulk-copied rows measured neutral to slightly slower on the
 // same box -- 20.3 vs 19.2-20.3 ms -- so it keeps its tensor box)
+// NS_UP_OUT2: double-buffered output staging rows in uptail2 (drops one group
+// barrier per step); parity green, measured neutral (sr_up 20.2-20.4 vs
+// 20.1-20.3 ms, union over the two SR streams): off.
+#ifndef NS_UP_OUT2
+#define NS_UP_OUT2 0
+#endif
 // NS_UP_BIAS_INIT: uptail2's retired accumulator columns are re-initialised by
 // their own epilogue group with bias + 1/2 (no 3-group barrier per step).
 #ifndef NS_UP_BIAS_INIT
@@ -1184,7 +1190,8 @@ struct Up2Cfg {
     static constexpr uint32_t LR_BYTES = 9u * kLrBoxW;              // [row 3][plane 3][kLrBoxW]
     static constexpr uint32_t LSLOT = round_up(LR_BYTES, 128);
     static constexpr uint32_t OUTG = round_up(3u * kTile * S, 128);  // per group: [plane][128 s] bytes
-    static constexpr uint32_t TILE_BYTES = NS * SLOT + NL * LSLOT + S * OUTG;
+    static constexpr int NOUT = NS_UP_OUT2 ? 2 : 1;                  // staging rows per group
+    static constexpr uint32_t TILE_BYTES = NS * SLOT + NL * LSLOT + S * NOUT * OUTG;
     static constexpr uint32_t TCOLS = 5 * NB;
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
     static constexpr int BPT = 2 * NS + 3 + 2 * NL;                // barriers per tile
@@ -1311,7 +1318,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
     auto islot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + i * Cfg::SLOT; };
     auto lslot = [&](int k, int i) { return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + i * Cfg::LSLOT; };
     auto oslot = [&](int k, int g) {
-        return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + NL * Cfg::LSLOT + g * Cfg::OUTG;
+        return s_tile + k * Cfg::TILE_BYTES + NS * Cfg::SLOT + NL * Cfg::LSLOT + g * Cfg::NOUT * Cfg::OUTG;
     };
     // per tile: hfull[NS], sfree[NS], mdone[2], edone, lfull[NL], lfree[NL]
     auto hfull = [&](int k, int i) { return &bars[k * BPT + i]; };
@@ -1433,7 +1440,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
         const int p = ew * 32 + lane;
         const int x = x0k(k) + p;
         const uint32_t tl = tmem + ((uint32_t)(ew * 32) << 16) + k * Cfg::TCOLS;
-        uint8_t *so = oslot(k, g);
+        uint8_t *const so0 = oslot(k, g);
         if (vk(k)) {
             mbar_wait(wbar, 0);
             float bh[3 * S];
@@ -1480,6 +1487,10 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     const int qv = r - y0, ls = qv % NL;
                     mbar_wait(lfull(k, ls), (qv / NL) & 1);
                     const uint8_t *lr = lslot(k, ls);
+                    // NS_UP_OUT2: two staging rows per group, alternating by step, so
+                    // the row written at step q is never the one being copied out from
+                    // step q-1 (the barrier of step q orders it) -- no second barrier
+                    uint8_t *const so = so0 + (Cfg::NOUT == 2 ? (q & 1) * Cfg::OUTG : 0);
                     if (x < lw) {
                         if (g == 0) uptail_group_step<NB, S, 0>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
                         else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
@@ -1496,7 +1507,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                             *reinterpret_cast<uint2 *>(dst + (size_t)c * HH * WW + ch * 8) =
                                 *reinterpret_cast<const uint2 *>(so + c * (kTile * S) + ch * 8);
                     }
-                    named_bar(3 + grp, 128);  // staging can be overwritten
+                    if constexpr (Cfg::NOUT == 1) named_bar(3 + grp, 128);  // staging can be overwritten
                 }
             }
         }
