@@ -77,7 +77,7 @@ typedef struct ns_model ns_model;
 typedef struct {
     int32_t w, h;              /* LR size; w % 8 == 0, h % 8 == 0, w,h >= 8         */
     int32_t scale;             /* SR factor s in {2, 3, 4}; must equal model scale   */
-    int32_t n_frames;          /* 1 <= n <= 256                                      */
+    int32_t n_frames;          /* 1 <= n <= 256; per call S <= 65535, S * n <= 2^20  */
     const uint8_t *lr;         /* [n][3][h][w] decoded LR frames                     */
     const int16_t *res;        /* [n][3][h][w] decoded residual                      */
     const ns_block_mv *mv;     /* [n][h/8][w/8]                                      */
@@ -98,8 +98,13 @@ typedef struct {
    over the streams of every GPU (§5.2 global selection across GPUs)
    -- and is passed in `anchor_in`; `cost` and `budget` are those of that global
    selection (this call's streams' entries of cost[]), which bound the anchors
-   this call can receive (sum of their cost <= budget).  Only ns_enhance_streams
-   and ns_enhance_streams_host accept it. */
+   this call can receive (sum of their cost <= budget).  A map that breaks that
+   bound is not an error (it is device data): per SR shape group the anchors
+   take job slots stream by stream, frame by frame, and those beyond the
+   group's min(streams * n, budget / min cost) slots are DEMOTED -- their
+   is_anchor_out entry is cleared and the frame is reconstructed like any
+   other non-anchor frame (deterministic; nothing is left stale).  Only
+   ns_enhance_streams and ns_enhance_streams_host accept it. */
 enum { NS_TOPK_PER_STREAM = 0, NS_GLOBAL_BUDGET = 1, NS_GIVEN_ANCHORS = 2 };
 /* Residual carried from the G_altref pass into the G_normal pass (reading Z2,
    default) or recomputed per group (literal Alg. 1 line 2). */
@@ -167,13 +172,17 @@ NS_API ns_status ns_select_anchors(ns_ctx *ctx, const ns_chunk *chunks, int S, c
 
 /* Global anchor selection over streams gathered from every GPU (§5.2: "select
    anchor frames globally across all streams").
-   Each GPU first runs ns_select_anchors on its own streams (any mode; only the
-   per-stream gain and rank are used), then the callers all-gather, per stream,
-   gain[n], rank[n], type[n], cost and a global stream id, and every GPU calls
-   this with the identical gathered arrays, so every GPU computes the identical
-   selection with no further exchange.  Inputs, all DEVICE, S = streams over all
-   GPUs in any order: gain, rank_in (per-stream rank from ns_select_anchors)
-   int64 / int32 [S][n]; type u8 [S][n]; sid int32 [S] distinct global stream
+   Each GPU first runs ns_select_anchors on its own streams in
+   NS_TOPK_PER_STREAM mode with NS_SEL_NEUROSCALER (any k: only the per-stream
+   Alg. 1 gain is used), then the callers all-gather, per stream, gain[n],
+   type[n], cost and a global stream id, and every GPU calls this with the
+   identical gathered arrays, so every GPU computes the identical selection
+   with no further exchange.  Inputs, all DEVICE, S = streams over all GPUs in
+   any order: gain int64 [S][n]; rank_in int32 [S][n] or NULL -- NOT trusted:
+   each stream's priority order is rebuilt here from (type asc, gain desc,
+   frame asc), which is the rank ns_select_anchors returns in that mode
+   (reading Z5), so a rank array from another mode or selector cannot corrupt
+   the merge; type u8 [S][n]; sid int32 [S] distinct global stream
    ids (the stream key of the merged order, readings Z5, R7); cost int64 [S] >= 1.
    The merged order is G_key by (sid, frame), then G_altref, then G_normal, each
    by (gain desc, sid asc, frame asc); the anchors are its longest prefix with
@@ -192,14 +201,27 @@ NS_API ns_status ns_sr_anchors(ns_ctx *ctx, const ns_sr_job *jobs, int n_jobs, v
 /* Reuse-based reconstruction of every non-anchor frame of S chunks (§2, §6.1).
    is_anchor: DEVICE [S][n].  hr_out: HOST table [S*n] of DEVICE pointers, each
    [3][s*h][s*w]; anchors' entries must already hold the SR output (e.g. from
-   ns_sr_anchors).  hr_out[s][f] must not alias hr_out[s][f-1], hr_last or
-   hr_golden of the same stream (checked) nor the frame serving as GOLDEN
-   (not checked).  Writes hr_last / hr_golden at chunk end. */
+   ns_sr_anchors), so every entry of the table must be distinct (checked:
+   NS_EINVAL; HR rings need ns_enhance_streams), and none may be a stream's
+   hr_last / hr_golden (checked).  Writes hr_last / hr_golden at chunk end. */
 NS_API ns_status ns_reconstruct_chunk(ns_ctx *ctx, const ns_chunk *chunks, int S, const uint8_t *is_anchor,
                                uint8_t *const *hr_out, void *stream);
 
 /* The whole hot path for S streams: select -> SR on anchors (grouped across
-   streams) -> reconstruct.  hr_out: HOST table [S*n] of DEVICE pointers.
+   streams) -> reconstruct.  hr_out: HOST table [S*n] of DEVICE pointers, each
+   [3][s*h][s*w], where frame f of stream s is written.
+   HR rings: a stream's row may repeat entries (e.g. hr_out[s][f] = ring[f % R],
+   R >= 2), so a long chunk of many streams needs O(S * R) HR frames instead of
+   O(S * n).  Rules, all checked (NS_EINVAL):
+     - hr_out[s][f] != hr_out[s][f-1] (frame f reads HR[f-1] as LAST);
+     - no entry is shared with another stream or is any stream's state slot;
+     - a ring stream needs hr_golden (GOLDEN is kept there: HR of the latest
+       KEY/ALTREF is saved into it at the step after it) and no gt.
+   After the call, each entry holds the LAST frame written to it.  Anchors of
+   a ring stream are SR'd into a context-owned anchor cache (carved from the
+   pool on first use: NS_ENOMEM if it does not fit) and copied into their
+   slot at their own frame step (the client "caches [SR anchors] in
+   memory" and reuses them).
    is_anchor_out (DEVICE [S][n]) may be NULL.  stats: DEVICE [S][8] fp64 or
    NULL: {frames, anchors, sum anchor score, total score, SSE vs gt (or -1),
    PSNR vs gt (or -1), 0, 0}. */

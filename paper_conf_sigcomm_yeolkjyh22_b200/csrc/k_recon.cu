@@ -20,7 +20,12 @@ __device__ __forceinline__ void up_tap_r(int X, int s, int len, int &i0, int &i1
 
 // gold[s][f] = latest KEY/ALTREF frame < f of stream s, -1 = the incoming
 // GOLDEN state; gold[s][n] = the GOLDEN after the chunk.
-__global__ void k_golden_index(const StreamDesc *sd, int S, int n, int16_t *gold) {
+// HR rings (nxt != NULL): a KEY/ALTREF frame g is GOLDEN for the frames up to
+// the next KEY/ALTREF gn (inclusive: gn still references g), and after the last
+// one for the rest of the chunk and the chunk-end state.  If its hr_out entry is
+// written again before then (nxt[g] <= min(gn, n-1)) it must be saved into
+// hr_golden: gsv[s][g] = 1.
+__global__ void k_golden_index(const StreamDesc *sd, int S, int n, const int16_t *nxt, int16_t *gold, uint8_t *gsv) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
     const uint8_t *T = sd[s].type;
@@ -30,11 +35,19 @@ __global__ void k_golden_index(const StreamDesc *sd, int S, int n, int16_t *gold
         if (T[f] == NS_KEY || T[f] == NS_ALTREF) g = f;
     }
     gold[(size_t)s * (n + 1) + n] = (int16_t)g;
+    if (!nxt) return;
+    int gn = n;
+    for (int f = n - 1; f >= 0; f--) {
+        const bool golden = T[f] == NS_KEY || T[f] == NS_ALTREF;
+        gsv[(size_t)s * n + f] = golden && nxt[(size_t)s * n + f] <= min(gn, n - 1);
+        if (golden) gn = f;
+    }
 }
 
-cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st) {
+cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, const int16_t *nxt, int16_t *gold_idx,
+                                uint8_t *gsv, cudaStream_t st) {
     KScope ks(F_RECON, st);
-    k_golden_index<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, gold_idx);
+    k_golden_index<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, nxt, gold_idx, gsv);
     return cudaGetLastError();
 }
 
@@ -146,11 +159,13 @@ __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int 
 // Load one staged window row (NQ words) into registers; for a non-interior
 // window replicate the edge pixel into the words that lie outside the row
 // (first word at xb).
+// (on = false: a KEY-frame / INTRA thread, whose warp weights are all 0 and
+// whose slots hold LR rows in flight: nothing is read, so no shared-memory race)
 template <int S>
-__device__ __forceinline__ void recon_load_row(const uint2 *row, bool fix, int xb, int W,
+__device__ __forceinline__ void recon_load_row(const uint2 *row, bool on, bool fix, int xb, int W,
                                                uint2 (&q)[ReconCfg<S>::NQ]) {
 #pragma unroll
-    for (int i = 0; i < ReconCfg<S>::NQ; i++) q[i] = row[i * kReconNT];
+    for (int i = 0; i < ReconCfg<S>::NQ; i++) q[i] = on ? row[i * kReconNT] : make_uint2(0u, 0u);
     if (fix) {
 #pragma unroll
         for (int i = 0; i < ReconCfg<S>::NQ; i++) {
@@ -327,35 +342,62 @@ __device__ __forceinline__ uint32_t vmin_u16x2(uint32_t a, uint32_t b) {
 }
 
 // fd[s][f]: the frame step's pointers resolved once per chunk.
+// HR rings (gsv / asrc non-NULL, ns.h): GOLDEN g is read from hr_out[g] while its
+// entry holds it; if g must be saved (gsv), step g + 1 copies HR[g] into
+// hr_golden -- nothing reads hr_golden during that step, the frames of step g + 1
+// still read hr_out[g] (intact: hr_out[f] != hr_out[f-1]) -- and later steps
+// read the copy.  An anchor SR'd into the anchor cache (asrc) is copied into
+// its entry at its own step.
 __global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *is_anchor, uint8_t *const *hr_tab,
-                             const int16_t *gold, FrameDesc *fd) {
+                             const int16_t *gold, const uint8_t *gsv, const uint8_t *const *asrc, FrameDesc *fd) {
     const int e = blockIdx.x * blockDim.x + threadIdx.x;
     if (e >= S * n) return;
     const int sid = e / n, f = e % n;
     const StreamDesc d = sd[sid];
     const size_t lrp = (size_t)d.h * d.w;
-    FrameDesc o;
+    FrameDesc o{};
     o.lr_f = d.lr + (size_t)f * 3 * lrp;
     o.res_f = d.res + (size_t)f * 3 * lrp;
     o.mv_f = d.mv + (size_t)f * (d.h / 8) * (d.w / 8);
     o.out = hr_tab[d.hr_base + f];
     o.ref_last = f > 0 ? hr_tab[d.hr_base + f - 1] : d.hr_last;
     const int g = gold[(size_t)sid * (n + 1) + f];
-    o.ref_gold = g >= 0 ? hr_tab[d.hr_base + g] : d.hr_golden;
+    const bool saved = g >= 0 && gsv && gsv[(size_t)sid * n + g] && f >= g + 2;
+    o.ref_gold = g >= 0 && !saved ? hr_tab[d.hr_base + g] : d.hr_golden;
+    o.asrc = asrc ? asrc[e] : nullptr;
+    o.gsave_src = nullptr;
+    o.gsave_dst = nullptr;
+    if (gsv && f > 0 && gsv[e - 1]) {
+        o.gsave_src = hr_tab[d.hr_base + f - 1];
+        o.gsave_dst = d.hr_golden;
+    }
     o.w = d.w;
     o.h = d.h;
     o.s = (int16_t)d.s;
     o.anchor = is_anchor[e] ? 1 : 0;
     o.key = d.type[f] == NS_KEY;
-    o.pad = 0;
     fd[e] = o;
 }
 
 cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
-                              uint8_t *const *d_hr_table, const int16_t *gold_idx, FrameDesc *fd, cudaStream_t st) {
+                              uint8_t *const *d_hr_table, const int16_t *gold_idx, const uint8_t *gsv,
+                              const uint8_t *const *asrc, FrameDesc *fd, cudaStream_t st) {
     KScope ks(F_RECON, st);
-    k_frame_desc<<<(S * n + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, gold_idx, fd);
+    k_frame_desc<<<(S * n + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, gold_idx, gsv, asrc, fd);
     return cudaGetLastError();
+}
+
+// Copies the CTA's HR tile (rows y0 .. y1, bytes x0 .. x1 of each of the 3
+// planes) from src to dst in 8-B words (W is a multiple of 8): the HR-ring
+// anchor copy and GOLDEN save, done by the frame step's own CTAs.
+__device__ __forceinline__ void recon_tile_copy(const uint8_t *src, uint8_t *dst, size_t hrp, int W, int x0, int x1,
+                                                int y0, int y1, int tid, int nt) {
+    const int wpr = (x1 - x0) >> 3, rows = y1 - y0, per_plane = wpr * rows;
+    for (int i = tid; i < 3 * per_plane; i += nt) {
+        const int c = i / per_plane, r = (i % per_plane) / wpr, q = i % wpr;
+        const size_t off = (size_t)c * hrp + (size_t)(y0 + r) * W + x0 + 8 * q;
+        *reinterpret_cast<uint2 *>(dst + off) = *reinterpret_cast<const uint2 *>(src + off);
+    }
 }
 
 template <int S>
@@ -366,13 +408,19 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     constexpr int NP = Cfg::NP, RPT = Cfg::RPT, NQ = Cfg::NQ;
     const int sid = s0 + blockIdx.z;
     const FrameDesc fd = fdesc[(size_t)sid * n + f];
-    if (fd.anchor || fd.s != S) return;                 // CTA-uniform: anchors already hold SR bytes
+    if (fd.s != S) return;                              // CTA-uniform
     const int w = fd.w, h = fd.h, H = h * S, W = w * S;
     const int bx0 = blockIdx.x * kReconTX;              // first LR block column of the CTA
     const int Y0c = blockIdx.y * kReconTY * RPT;        // first HR row of the CTA
     if (8 * bx0 >= w || Y0c >= H) return;               // CTA-uniform
     const int tid = threadIdx.y * kReconTX + threadIdx.x;
     const size_t lrp = (size_t)h * w, hrp = (size_t)H * W;
+    if (fd.gsave_src || (fd.anchor && fd.asrc)) {       // HR rings only (k_frame_desc)
+        const int x0 = 8 * S * bx0, x1 = min(8 * S * (bx0 + kReconTX), W), y1 = min(Y0c + kReconTY * RPT, H);
+        if (fd.gsave_src) recon_tile_copy(fd.gsave_src, fd.gsave_dst, hrp, W, x0, x1, Y0c, y1, tid, kReconNT);
+        if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc, fd.out, hrp, W, x0, x1, Y0c, y1, tid, kReconNT);
+    }
+    if (fd.anchor) return;                              // CTA-uniform: the anchor's SR bytes are in place
 
     extern __shared__ __align__(16) uint8_t recon_sm[];
     uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [RPT+1][NQ][NT] warp windows
@@ -464,14 +512,14 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
             __syncthreads();                                    // (orders the tile barrier's init)
             if (!fd.key) mbar_wait(tbar, 0);                    // the residual tile
         }
-        // (use_lr threads run the warp pass over whatever the slots hold: every weight is 0, so pred = 0)
+        // (use_lr threads run the warp pass on zero words: every weight is 0, so pred = 0)
         const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
         const uint2 *lrb = wbuf + lr_slots(c);
         uint8_t *outc = outp + c * hrp;
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
         {
             uint2 q[NQ];
-            recon_load_row<S>(wbuf, fix, xs & ~7, W, q);
+            recon_load_row<S>(wbuf, !use_lr, fix, xs & ~7, W, q);
             recon_hpass8<S>(q, m, fxc, fx, hA);
         }
         stage_row(c + 1, 0);
@@ -494,7 +542,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                 uint32_t(&hc)[NP] = (jj & 1) ? hA : hB;
                 asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
                 uint2 q[NQ];
-                recon_load_row<S>(wbuf + (j + 1) * NQ * kReconNT, fix, xs & ~7, W, q);
+                recon_load_row<S>(wbuf + (j + 1) * NQ * kReconNT, !use_lr, fix, xs & ~7, W, q);
                 uint32_t u[NP], x[NP], o[Cfg::BW / 4];
                 recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);   // independent of q: covers the load
                 recon_hpass8<S>(q, m, fxc, fx, hc);
@@ -519,16 +567,11 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
 }
 
 template <int S>
-static void recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ReconSmem<S>::BYTES);
-        // all of the unified L1/shared array as shared memory, so MINB CTAs fit
-        cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             (int)cudaSharedmemCarveoutMaxShared);
-        attr = true;
-    }
+static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
+    // all of the unified L1/shared array as shared memory, so MINB CTAs fit
+    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, true); e != cudaSuccess) return e;
     k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f, s0);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
@@ -542,15 +585,16 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
         const int rpt = s == 2 ? ReconCfg<2>::RPT : s == 3 ? ReconCfg<3>::RPT : ReconCfg<4>::RPT;
         const int nrg = (max_lr_h[s] * s + rpt - 1) / rpt;  // groups of RPT HR rows
         dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
-        if (s == 2) recon_launch<2>(g, st, fd, n, f, s0);
-        if (s == 3) recon_launch<3>(g, st, fd, n, f, s0);
-        if (s == 4) recon_launch<4>(g, st, fd, n, f, s0);
+        const cudaError_t e = s == 2 ? recon_launch<2>(g, st, fd, n, f, s0)
+                              : s == 3 ? recon_launch<3>(g, st, fd, n, f, s0) : recon_launch<4>(g, st, fd, n, f, s0);
+        if (e != cudaSuccess) return e;
     }
     return cudaGetLastError();
 }
 
 // Chunk-end reference state: hr_last <- HR[n-1], hr_golden <- HR[gold[n]].
-__global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab, const int16_t *gold) {
+__global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab, const int16_t *gold,
+                             const uint8_t *gsv) {
     const int sid = blockIdx.y, which = blockIdx.z;
     const StreamDesc d = sd[sid];
     const size_t nvec = (size_t)3 * d.h * d.s * d.w * d.s / 16;
@@ -560,9 +604,10 @@ __global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab
         dst = d.hr_last;
         src = hr_tab[d.hr_base + n - 1];
     } else {
+        // HR rings: a saved GOLDEN is in hr_golden already (its entry may be gone)
         const int g = gold[(size_t)sid * (n + 1) + n];
         dst = d.hr_golden;
-        src = g >= 0 ? hr_tab[d.hr_base + g] : nullptr;
+        src = g >= 0 && !(gsv && gsv[(size_t)sid * n + g]) ? hr_tab[d.hr_base + g] : nullptr;
     }
     if (!dst || !src || dst == src) return;
     const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
@@ -572,11 +617,11 @@ __global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab
 }
 
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
-                              const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st) {
+                              const int16_t *gold_idx, const uint8_t *gsv, size_t max_hr_bytes, cudaStream_t st) {
     const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
     KScope ks(F_STATE, st);
     dim3 g(blocks < 1 ? 1 : (blocks > 4096 ? 4096 : blocks), S, 2);
-    k_state_copy<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, gold_idx);
+    k_state_copy<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, gold_idx, gsv);
     return cudaGetLastError();
 }
 
@@ -599,14 +644,14 @@ __global__ void k_stats_meta(const StreamDesc *sd, int S, int n, const uint8_t *
 }
 
 __global__ void k_stats_sse(const StreamDesc *sd, int n, uint8_t *const *hr_tab, double *stats) {
-    const int sf = blockIdx.y, sid = sf / n, f = sf % n;
+    const int sf = blockIdx.x, sid = sf / n, f = sf % n;   // (stream, frame) on x: S*n may exceed 65535
     const StreamDesc d = sd[sid];
     if (!d.gt) return;
     const size_t nvec = (size_t)3 * d.h * d.s * d.w * d.s / 16;
     const uint4 *a = reinterpret_cast<const uint4 *>(hr_tab[d.hr_base + f]);
     const uint4 *b = reinterpret_cast<const uint4 *>(d.gt + (size_t)f * nvec * 16);
     unsigned long long acc = 0;
-    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < nvec; i += (size_t)gridDim.x * blockDim.x) {
+    for (size_t i = (size_t)blockIdx.y * blockDim.x + threadIdx.x; i < nvec; i += (size_t)gridDim.y * blockDim.x) {
         const uint4 x = a[i], y = b[i];
         const uint32_t xs[4] = {x.x, x.y, x.z, x.w}, ys[4] = {y.x, y.y, y.z, y.w};
 #pragma unroll
@@ -638,7 +683,7 @@ cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is
     if (max_hr_bytes) {
         // one CTA row per (stream, frame), ~4 CTAs per SM-resident wave over the frame
         const int blocks = (int)((max_hr_bytes / 16 + 255) / 256);
-        dim3 g(blocks < 1 ? 1 : (blocks > 64 ? 64 : blocks), S * n);
+        dim3 g(S * n, blocks < 1 ? 1 : (blocks > 64 ? 64 : blocks));
         k_stats_sse<<<g, 256, 0, st>>>(d_sd, n, d_hr_table, stats);
         k_stats_final<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, stats);
     }

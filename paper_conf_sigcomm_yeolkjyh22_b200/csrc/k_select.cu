@@ -12,19 +12,19 @@ constexpr int64_t kKeyGain = INT64_MAX;  // "equal anchor gain" of key frames (P
 // ---------------------------------------------------------------- K1 score
 // score[s][f] = sum_{c,y,x} |res[f][c][y][x]| ("total residual pixel value",
 // P:191), or the encoded-size proxy res_size[f] when the stream asks for it.
-// Grid (slabs, S*n); 16-B loads of 8 int16; one 64-bit atomic per CTA.
+// Grid (S*n, slabs); 16-B loads of 8 int16; one 64-bit atomic per CTA.
 constexpr int kScoreThreads = 256, kScoreUnroll = 8;
 __global__ void __launch_bounds__(kScoreThreads) k_score(const StreamDesc *sd, int n, int64_t *score) {
-    const int sf = blockIdx.y, s = sf / n, f = sf % n;
+    const int sf = blockIdx.x, s = sf / n, f = sf % n;   // (stream, frame) on x: S*n may exceed 65535
     const StreamDesc d = sd[s];
     if (d.use_res_size && d.res_size) {
-        if (blockIdx.x == 0 && threadIdx.x == 0) score[sf] = (int64_t)d.res_size[f];
+        if (blockIdx.y == 0 && threadIdx.x == 0) score[sf] = (int64_t)d.res_size[f];
         return;
     }
     const size_t nvec = (size_t)3 * d.h * d.w / 8;
     const uint4 *r = reinterpret_cast<const uint4 *>(d.res + (size_t)f * 3 * d.h * d.w);
-    const size_t base = (size_t)blockIdx.x * kScoreThreads * kScoreUnroll + threadIdx.x;
-    if ((size_t)blockIdx.x * kScoreThreads * kScoreUnroll >= nvec) return;
+    const size_t base = (size_t)blockIdx.y * kScoreThreads * kScoreUnroll + threadIdx.x;
+    if ((size_t)blockIdx.y * kScoreThreads * kScoreUnroll >= nvec) return;
     uint4 v[kScoreUnroll];
 #pragma unroll
     for (int i = 0; i < kScoreUnroll; i++) {
@@ -58,7 +58,7 @@ cudaError_t launch_score(const StreamDesc *d_sd, int S, int n, int max_frame_vec
     cudaError_t e = cudaMemsetAsync(score, 0, sizeof(int64_t) * S * n, st);
     if (e != cudaSuccess) return e;
     const int per = kScoreThreads * kScoreUnroll;
-    dim3 g((max_frame_vec8 + per - 1) / per, S * n);
+    dim3 g(S * n, (max_frame_vec8 + per - 1) / per);
     k_score<<<g, kScoreThreads, 0, st>>>(d_sd, n, score);
     return cudaGetLastError();
 }
@@ -233,7 +233,31 @@ __global__ void k_global_rank(const StreamDesc *sd, const uint8_t *type_flat, co
     pos_stream[cnt] = s;
 }
 
-// order[s][rank_in[s][f]] = f: the per-stream priority order from the ranks.
+// Per-stream priority rank of every gathered entry, rebuilt from the entries
+// themselves: the number of frames of the same stream ordered before (s, f) by
+// (type asc, gain desc, frame asc) -- Fig. 10's per-stream order (KEY gain =
+// INT64_MAX, so KEYs order by frame; reading Z5: within a stream this sort is
+// the greedy pick order of Alg. 1).  It equals ns_select_anchors' rank in
+// NS_TOPK_PER_STREAM / NS_SEL_NEUROSCALER mode, and it is a permutation of
+// 0..n-1 for ANY input, so the merge never trusts a caller's rank array.
+__global__ void k_stream_rank(int N, int n, const int64_t *gain, const uint8_t *type, int32_t *rank) {
+    const int e = blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= N) return;
+    const int s = e / n, f = e % n;
+    const uint8_t *T = type + (size_t)s * n;
+    const int64_t *G = gain + (size_t)s * n;
+    const int t = T[f];
+    const int64_t g = G[f];
+    int cnt = 0;
+    for (int f2 = 0; f2 < n; f2++) {
+        const int t2 = T[f2];
+        const int64_t g2 = G[f2];
+        cnt += (t2 < t) || (t2 == t && (g2 > g || (g2 == g && f2 < f)));
+    }
+    rank[e] = cnt;
+}
+
+// order[s][rank[s][f]] = f: the per-stream priority order from the ranks.
 __global__ void k_order_from_rank(int N, int n, const int32_t *rank_in, int32_t *order) {
     const int e = blockIdx.x * blockDim.x + threadIdx.x;
     if (e >= N) return;
@@ -292,10 +316,12 @@ cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *g
 cudaError_t launch_merge(int S, int n, const int64_t *gain, const int32_t *rank_in, const uint8_t *type,
                          const int32_t *sid, const int64_t *cost, int64_t budget, int32_t *order, int32_t *grank,
                          int32_t *pos_stream, int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st) {
-    KScope ks(F_GLOBAL, st, 4);
+    (void)rank_in;  // not trusted: the per-stream ranks are rebuilt from (type, gain, frame) into `rank`
+    KScope ks(F_GLOBAL, st, 5);
     const int N = S * n;
-    k_order_from_rank<<<(N + 255) / 256, 256, 0, st>>>(N, n, rank_in, order);
-    k_global_rank<true><<<(N + 255) / 256, 256, 0, st>>>(nullptr, type, sid, S, n, gain, order, rank_in, grank,
+    k_stream_rank<<<(N + 255) / 256, 256, 0, st>>>(N, n, gain, type, rank);
+    k_order_from_rank<<<(N + 255) / 256, 256, 0, st>>>(N, n, rank, order);
+    k_global_rank<true><<<(N + 255) / 256, 256, 0, st>>>(nullptr, type, sid, S, n, gain, order, rank, grank,
                                                           pos_stream);
     k_global_cut<<<1, 1024, 0, st>>>(N, pos_stream, cost, budget, cut);
     k_global_mark<<<(N + 255) / 256, 256, 0, st>>>(N, grank, cut, rank, is_anchor);
@@ -304,26 +330,79 @@ cudaError_t launch_merge(int S, int n, const int64_t *gain, const int32_t *rank_
 
 // ---------------------------------------------------------------- K3 compaction
 // Anchors of every stream -> SR job table of the stream's shape group.
-// Top-k mode: stream s owns slots [job_base, job_base + k) in frame order
-// (deterministic); global mode: slots are claimed with an atomic per group.
-__global__ void k_compact(const StreamDesc *sd, int S, int n, const uint8_t *is_anchor,
-                          uint8_t *const *hr_tab, SrJob *jobs, int32_t *job_count, int topk, uint8_t *lr_stage,
+// Top-k mode: stream s owns slots [job_base, job_base + k) in frame order.
+// Other modes (global budget, a given anchor map, Key SR): the anchors of a
+// group take consecutive slots stream by stream in the group's list order
+// (k_anchor_count + k_group_scan: deterministic, no atomics); an anchor whose
+// slot would pass the group's job_cap -- only possible for a given map that
+// breaks its budget -- is demoted: is_anchor is cleared and the frame is
+// reconstructed like any other (ns.h NS_GIVEN_ANCHORS).
+// HR rings: an anchor whose hr_out entry an earlier frame of the stream also
+// writes (prv >= 0) cannot be written before the reconstruction runs -- its SR
+// output goes to the group's anchor cache and asrc[s][f] records where, for
+// the frame step that copies it into place.  Every other anchor is SR'd
+// straight into hr_out (always so without rings).
+__global__ void k_anchor_count(int S, int n, const uint8_t *is_anchor, int32_t *acount) {
+    const int s = blockIdx.x * blockDim.x + threadIdx.x;
+    if (s >= S) return;
+    int c = 0;
+    for (int f = 0; f < n; f++) c += is_anchor[(size_t)s * n + f] != 0;
+    acount[s] = c;
+}
+
+// One CTA per group: exclusive scan of the anchor counts over the group's
+// streams in list order -> acount[s] becomes the stream's first slot offset;
+// job_count[g] = the slots the group fills (<= its cap).
+__global__ void __launch_bounds__(1024) k_group_scan(const StreamDesc *sd, const int32_t *glist, const int32_t *goff,
+                                                     int32_t *acount, int32_t *job_count) {
+    __shared__ int32_t buf[1024];
+    __shared__ int32_t carry;
+    const int g = blockIdx.x, i0 = goff[g], i1 = goff[g + 1];
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (int base = i0; base < i1; base += 1024) {
+        const int i = base + threadIdx.x;
+        const int v = i < i1 ? acount[glist[i]] : 0;
+        buf[threadIdx.x] = v;
+        __syncthreads();
+        for (int off = 1; off < 1024; off <<= 1) {
+            const int32_t t = threadIdx.x >= off ? buf[threadIdx.x - off] : 0;
+            __syncthreads();
+            buf[threadIdx.x] += t;
+            __syncthreads();
+        }
+        if (i < i1) acount[glist[i]] = carry + buf[threadIdx.x] - v;
+        __syncthreads();
+        if (threadIdx.x == 0) carry += buf[1023];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0 && i1 > i0) job_count[g] = min(carry, sd[glist[i0]].job_cap);
+}
+
+__global__ void k_compact(const StreamDesc *sd, int S, int n, uint8_t *is_anchor, uint8_t *const *hr_tab,
+                          SrJob *jobs, const int32_t *start, int topk, const int16_t *prv, const uint8_t **asrc,
+                          uint8_t *lr_stage,
                           size_t lr_stride, const uint8_t **lr_src, uint32_t *lr_len) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
     const StreamDesc d = sd[s];
     const size_t lr_frame = (size_t)3 * d.h * d.w;
-    int local = 0;
+    int claim = topk ? 0 : start[s];
     for (int f = 0; f < n; f++) {
-        if (!is_anchor[(size_t)s * n + f]) continue;
-        const int claim = topk ? local : atomicAdd(&job_count[d.group], 1);
-        local++;
-        if (claim >= d.job_cap) continue;  // over the bound of a given anchor map: dropped (ns.h)
-        const int slot = d.job_base + claim;
+        const size_t e = (size_t)s * n + f;
+        if (asrc) asrc[e] = nullptr;
+        if (!is_anchor[e]) continue;
+        if (claim >= d.job_cap) {  // over the bound of a given anchor map: demoted (ns.h)
+            is_anchor[e] = 0;
+            continue;
+        }
+        const int slot = d.job_base + claim++;
         SrJob j;
         j.lr = d.lr + f * lr_frame;
-        j.hr = hr_tab[d.hr_base + f];
+        const bool direct = !prv || prv[e] < 0;
+        j.hr = direct ? hr_tab[d.hr_base + f] : d.acache + (size_t)(slot - d.job_goff) * d.acache_stride;
         j.wts = d.wts;
+        if (!direct) asrc[e] = j.hr;
         if (lr_stage) {  // host-resident LR: gather into device staging, SR reads the copy
             lr_src[slot] = j.lr;
             lr_len[slot] = (uint32_t)lr_frame;
@@ -336,35 +415,37 @@ __global__ void k_compact(const StreamDesc *sd, int S, int n, const uint8_t *is_
 // One CTA row per job, CTAs stride over the frame in 16-B words: wide,
 // coalesced reads of page-locked host memory over PCIe.
 __global__ void k_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len) {
-    const int j = blockIdx.y;
+    const int j = blockIdx.x;   // jobs on x (up to 2^20), CTAs of one job on y
     const uint32_t len = lr_len[j];
     if (len == 0) return;
     const uint4 *src = reinterpret_cast<const uint4 *>(lr_src[j]);
     uint4 *dst = reinterpret_cast<uint4 *>(const_cast<uint8_t *>(jobs[j].lr));
     const uint32_t nw = len / 16;
-    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += gridDim.x * blockDim.x) dst[i] = src[i];
+    for (uint32_t i = blockIdx.y * blockDim.x + threadIdx.x; i < nw; i += gridDim.y * blockDim.x) dst[i] = src[i];
 }
 
 cudaError_t launch_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len, int max_jobs,
                              size_t max_len, cudaStream_t st) {
     KScope ks(F_COMPACT, st);
     const int bx = (int)std::min<size_t>((max_len / 16 + 1023) / 1024, 256);
-    k_lr_gather<<<dim3(std::max(bx, 1), max_jobs), 256, 0, st>>>(jobs, lr_src, lr_len);
+    k_lr_gather<<<dim3(max_jobs, std::max(bx, 1)), 256, 0, st>>>(jobs, lr_src, lr_len);
     return cudaGetLastError();
 }
 
-cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
-                           uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups, int topk,
-                           int k, cudaStream_t st, uint8_t *lr_stage, size_t lr_stride, const uint8_t **lr_src,
-                           uint32_t *lr_len) {
-    (void)k;
-    KScope ks(F_COMPACT, st);
+cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, uint8_t *is_anchor, uint8_t *const *d_hr_table,
+                           SrJob *jobs, int32_t *job_count, int n_groups, const int32_t *glist,
+                           const int32_t *goff, int32_t *acount, int topk, const int16_t *prv,
+                           const uint8_t **asrc, cudaStream_t st, uint8_t *lr_stage, size_t lr_stride,
+                           const uint8_t **lr_src, uint32_t *lr_len) {
+    KScope ks(F_COMPACT, st, topk ? 1 : 3);
     if (!topk) {
         cudaError_t e = cudaMemsetAsync(job_count, 0, sizeof(int32_t) * n_groups, st);
         if (e != cudaSuccess) return e;
+        k_anchor_count<<<(S + 127) / 128, 128, 0, st>>>(S, n, is_anchor, acount);
+        k_group_scan<<<n_groups, 1024, 0, st>>>(d_sd, glist, goff, acount, job_count);
     }
-    k_compact<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, jobs, job_count, topk, lr_stage,
-                                               lr_stride, lr_src, lr_len);
+    k_compact<<<(S + 127) / 128, 128, 0, st>>>(d_sd, S, n, is_anchor, d_hr_table, jobs, acount, topk, prv, asrc,
+                                               lr_stage, lr_stride, lr_src, lr_len);
     return cudaGetLastError();
 }
 

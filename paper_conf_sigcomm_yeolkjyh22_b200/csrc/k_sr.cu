@@ -807,7 +807,7 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                 }
             } else {
                 for (int q = 2; q < nq; q++) {  // conv2 on t row y0-3+q
-                    mbar_wait(e1t(k, q & 3), (q >> 2) & 1);
+                    mbar_wait(e1t(k, (q - 2) & 3), ((q - 2) >> 2) & 1);
                     if (q >= 3) mbar_wait(e2z(k), (q - 3) & 1);
                     if (lane == 0) NS_TR(5 + k, q);
                     tc_fence_after();
@@ -845,7 +845,7 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
 #ifdef NS_TRACE_NOEPI
                     tc_fence_before();
                     rb_arrive(e1z(k));
-                    rb_arrive(e1t(k, q & 3));
+                    if (q >= 2) rb_arrive(e1t(k, (q - 2) & 3));
                     continue;
 #endif
                     const uint32_t acc = tl + (uint32_t)(mod3(yt) * NB);
@@ -902,7 +902,9 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     if (warp % 4 == 2 && lane == 0) NS_TR(42 + k, q);
                     fence_proxy_async_smem();
                     if (warp % 4 == 2 && lane == 0) NS_TR(46 + k, q);
-                    rb_arrive(e1t(k, q & 3));
+                    // t rows y0-3, y0-2 (q < 2) feed no conv2 output: no arrival, so
+                    // every phase of e1t is waited on by M2 (compute-sanitizer synccheck)
+                    if (q >= 2) rb_arrive(e1t(k, (q - 2) & 3));
                     if (warp % 4 == 2 && lane == 0) NS_TR(12 + k, q);
                 }
             } else {
@@ -1791,13 +1793,7 @@ constexpr int kRotRows = NS_ROT_ROWS;  // rows per CTA strip of the rotated conv
 template <int CIN, int NB, int EPI>
 static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = RotCfg<CIN, NB>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_conv_rot<CIN, NB, EPI>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    if (cudaError_t e = ensure_kernel_smem<k_conv_rot<CIN, NB, EPI>>(Cfg::SMEM); e != cudaSuccess) return e;
     args.n_xtiles = (args.W + kTile - 1) / kTile;
     args.rows_per_cta = kRotRows;
     dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
@@ -1810,13 +1806,7 @@ static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int n
 template <int CIN, int NB, int S>
 static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = UpCfg<CIN, NB, S>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_uptail<CIN, NB, S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    if (cudaError_t e = ensure_kernel_smem<k_uptail<CIN, NB, S>>(Cfg::SMEM); e != cudaSuccess) return e;
     args.n_xtiles = (args.W + kTile - 1) / kTile;
     args.rows_per_cta = kRotRows;
     dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
@@ -1838,12 +1828,7 @@ constexpr int kRbRows = NS_RB_ROWS;  // rows per CTA strip of the fused res-bloc
 template <int C>
 static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, cudaStream_t st) {
     using Cfg = RbCfg<C>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_resblock<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    if (cudaError_t e = ensure_kernel_smem<k_resblock<C>>(Cfg::SMEM); e != cudaSuccess) return e;
     RbArgs args = args0;
     args.n_tiles = (args.W + kRbOut - 1) / kRbOut;
     args.rows_per_cta = kRbRows;
@@ -1856,13 +1841,7 @@ static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, 
 template <int CIN, int NB, int S>
 static cudaError_t uptail2(const CUtensorMap &tm, const CUtensorMap &tm_lr, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = Up2Cfg<CIN, NB, S>;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(k_uptail2<CIN, NB, S>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             Cfg::SMEM);
-        if (e != cudaSuccess) return e;
-        attr = true;
-    }
+    if (cudaError_t e = ensure_kernel_smem<k_uptail2<CIN, NB, S>>(Cfg::SMEM); e != cudaSuccess) return e;
     const int ntiles = (args.W + kTile - 1) / kTile;
     args.rows_per_cta = kRotRows;
     dim3 grid((ntiles + 1) / 2, (args.H + kRotRows - 1) / kRotRows, nj);

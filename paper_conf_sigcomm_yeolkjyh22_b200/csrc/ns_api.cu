@@ -12,6 +12,7 @@
 #include <deque>
 #include <map>
 #include <tuple>
+#include <unordered_map>
 #include <vector>
 #include "ns_internal.h"
 
@@ -142,6 +143,7 @@ namespace {
 constexpr int kStageSlots = 4;
 constexpr size_t kStageBytes = 8u << 20;
 constexpr int kMaxSN = 1 << 20;           // max streams x frames per call
+constexpr int kMaxStreams = 65535;        // max streams per call (a grid dimension of the frame step)
 constexpr int kMaxJobs = 1 << 20;
 constexpr int kHostGroups = 8;            // stream groups per ns_enhance_streams_host call
 // (NS_HOST_GROUPS in the environment overrides it: tuning experiments only)
@@ -188,6 +190,9 @@ struct ns_ctx {
     // device scratch (capacity kMaxSN)
     int64_t *score, *gain;
     int32_t *rank, *order, *grank, *pos_stream, *cut, *job_count;
+    int32_t *acount;                     // [kMaxStreams] per-stream anchor counts / first job slots
+    const uint8_t **asrc;                // [kMaxSN] HR rings: anchor sources (anchor cache)
+    uint8_t *gsv;                        // [kMaxSN] HR rings: GOLDEN frames saved into hr_golden
     uint8_t *anchor;
     int16_t *gold;
     FrameDesc *fdesc;
@@ -210,6 +215,10 @@ struct ns_ctx {
     size_t lr_stage_cap = 0;
     const uint8_t **lr_src = nullptr;
     uint32_t *lr_len = nullptr;
+    // ring mode: anchors' SR outputs wait here until their frame step (P:241
+    // "caches it in memory"); carved from the pool on first use, grown on demand
+    uint8_t *acache = nullptr;
+    size_t acache_cap = 0;
 };
 
 static uint8_t *pool_take(ns_ctx *c, size_t bytes) {
@@ -253,7 +262,8 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     NS_CUDA(cudaSetDevice(device));
     ns_ctx *c = new ns_ctx();
     c->device = device;
-    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2 + sizeof(FrameDesc)) +
+    const size_t fixed = (size_t)kMaxSN * (8 + 8 + 4 + 4 + 4 + 4 + 1 + 2 + 2 + 8 + 1 + sizeof(FrameDesc)) +
+                         (size_t)kMaxStreams * (2 + 4) +
                          (size_t)kMaxJobs * (sizeof(SrJob) + sizeof(uint8_t *) + sizeof(uint32_t)) +
                          kStageSlots * kStageBytes + (64u << 20) + 64 * 1024;
     if (pool_bytes < fixed + (64u << 20)) {
@@ -274,7 +284,10 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     c->grank = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
     c->pos_stream = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxSN);
     c->anchor = (uint8_t *)pool_take(c, kMaxSN);
-    c->gold = (int16_t *)pool_take(c, sizeof(int16_t) * (kMaxSN + 4096));
+    c->gold = (int16_t *)pool_take(c, sizeof(int16_t) * ((size_t)kMaxSN + kMaxStreams));
+    c->acount = (int32_t *)pool_take(c, sizeof(int32_t) * kMaxStreams);
+    c->asrc = (const uint8_t **)pool_take(c, sizeof(uint8_t *) * kMaxSN);
+    c->gsv = (uint8_t *)pool_take(c, kMaxSN);
     c->fdesc = (FrameDesc *)pool_take(c, sizeof(FrameDesc) * kMaxSN);
     c->cut = (int32_t *)pool_take(c, 256);
     c->job_count = (int32_t *)pool_take(c, sizeof(int32_t) * 4096);
@@ -445,6 +458,7 @@ static bool al16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
 static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n_out) {
     if (!ch) return fail(NS_EINVAL, "chunks is NULL");
     if (S < 1) return fail(NS_EINVAL, "S = %d < 1", S);
+    if (S > kMaxStreams) return fail(NS_EINVAL, "S = %d exceeds %d streams per call", S, kMaxStreams);
     const int n = ch[0].n_frames;
     if (n < 1 || n > kMaxFrames) return fail(NS_EINVAL, "n_frames %d not in [1, %d]", n, kMaxFrames);
     if ((size_t)S * n > (size_t)kMaxSN) return fail(NS_EINVAL, "S * n = %zu exceeds %d", (size_t)S * n, kMaxSN);
@@ -471,8 +485,18 @@ static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n
     return NS_OK;
 }
 
-static ns_status check_hr_table(const ns_chunk *ch, int S, int n, uint8_t *const *hr) {
+// hr_out[s][f]: non-NULL, 16-B aligned, distinct from hr_out[s][f-1] (the LAST
+// reference frame f reads), from the stream's hr_last / hr_golden, and never
+// shared with another stream.  A stream whose row repeats entries is an HR
+// ring (ring[s] = 1): allowed only where `ring_ok` (ns_enhance_streams), and
+// then it needs hr_golden (GOLDEN is saved there during the chunk) and no
+// ground truth (the quality stats read every frame after the chunk).
+static ns_status check_hr_table(const ns_chunk *ch, int S, int n, uint8_t *const *hr, bool ring_ok,
+                                std::vector<int> *ring) {
     if (!hr) return fail(NS_EINVAL, "hr_out table is NULL");
+    std::unordered_map<const uint8_t *, int> owner;
+    owner.reserve((size_t)S * n * 2);
+    if (ring) ring->assign(S, 0);
     for (int s = 0; s < S; s++)
         for (int f = 0; f < n; f++) {
             uint8_t *p = hr[(size_t)s * n + f];
@@ -480,11 +504,29 @@ static ns_status check_hr_table(const ns_chunk *ch, int S, int n, uint8_t *const
             if (f > 0 && p == hr[(size_t)s * n + f - 1]) return fail(NS_EINVAL, "hr_out[%d][%d] aliases hr_out[%d][%d]", s, f, s, f - 1);
             if (p == ch[s].hr_last || p == ch[s].hr_golden)
                 return fail(NS_EINVAL, "hr_out[%d][%d] aliases the stream's hr_last/hr_golden", s, f);
+            auto it = owner.emplace(p, s);
+            if (!it.second) {
+                if (it.first->second != s)
+                    return fail(NS_EINVAL, "hr_out[%d][%d] is shared with another stream (%d)", s, f, it.first->second);
+                if (!ring_ok)
+                    return fail(NS_EINVAL, "hr_out[%d][%d] repeats an entry of its row: HR rings need ns_enhance_streams", s, f);
+                if (ring) (*ring)[s] = 1;
+            }
         }
+    for (int s = 0; s < S && ring; s++) {
+        if (!(*ring)[s]) continue;
+        if (!ch[s].hr_golden) return fail(NS_EINVAL, "chunk %d: an HR ring needs hr_golden (GOLDEN is kept there)", s);
+        if (ch[s].gt) return fail(NS_EINVAL, "chunk %d: quality stats vs gt need a full hr_out row, not a ring", s);
+    }
+    // state slots must not be shared between streams either
+    for (int s = 0; s < S; s++)
+        for (const uint8_t *q : {(const uint8_t *)ch[s].hr_last, (const uint8_t *)ch[s].hr_golden})
+            if (q && owner.count(q)) return fail(NS_EINVAL, "chunk %d: a state slot is another stream's hr_out", s);
     return NS_OK;
 }
 
-// Builds StreamDesc[S] (+ optional hr table) into a staging slot.
+// Builds StreamDesc[S] (+ optional hr table, cost, SR group stream lists) into
+// a staging slot.
 struct Staged {
     int slot;
     uint8_t *host, *dev;
@@ -492,21 +534,34 @@ struct Staged {
     StreamDesc *d_sd;
     uint8_t **d_hr;
     int64_t *d_cost;
+    int32_t *d_glist, *d_goff;   // SR shape groups: streams of group g = glist[goff[g] .. goff[g+1])
+    int16_t *d_prv, *d_nxt;      // HR rings: previous / next frame writing the same hr_out entry
 };
 
 static size_t a256(size_t v) { return (v + 255) / 256 * 256; }
 
+// Per-stream batcher facts for stage_streams (all optional).
+struct StreamPlan {
+    const int *group = nullptr, *job_base = nullptr, *job_cap = nullptr, *job_goff = nullptr;
+    uint8_t *const *acache = nullptr;    // per stream: its group's anchor cache (ring streams)
+    const size_t *acache_stride = nullptr;
+    const std::vector<int> *glist = nullptr, *goff = nullptr;
+    const std::vector<int16_t> *prv = nullptr, *nxt = nullptr;   // [S*n] (HR rings)
+};
+
 static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint8_t *const *hr, const int64_t *cost,
-                               const int *group, const int *job_base, bool use_res_size, Staged *out,
-                               const int *job_cap = nullptr) {
+                               bool use_res_size, Staged *out, const StreamPlan &pl = StreamPlan()) {
+    const size_t sd_bytes = a256(sizeof(StreamDesc) * S);
+    const size_t hr_bytes = hr ? a256(sizeof(uint8_t *) * (size_t)S * n) : 0;
+    const size_t cost_bytes = cost ? a256(sizeof(int64_t) * S) : 0;
+    const size_t gl_bytes = pl.glist ? a256(sizeof(int32_t) * pl.glist->size()) + a256(sizeof(int32_t) * pl.goff->size()) : 0;
+    const size_t pn_bytes = pl.prv ? 2 * a256(sizeof(int16_t) * (size_t)S * n) : 0;
+    if (sd_bytes + hr_bytes + cost_bytes + gl_bytes + pn_bytes > kStageBytes)
+        return fail(NS_EINVAL, "too many streams x frames for one call (descriptor staging)");
     Staged g{};
     ns_status r = stage_begin(c, &g.host, &g.dev, &g.slot);
     if (r != NS_OK) return r;
     size_t off = 0;
-    const size_t sd_bytes = a256(sizeof(StreamDesc) * S);
-    const size_t hr_bytes = hr ? a256(sizeof(uint8_t *) * (size_t)S * n) : 0;
-    const size_t cost_bytes = cost ? a256(sizeof(int64_t) * S) : 0;
-    if (sd_bytes + hr_bytes + cost_bytes > kStageBytes) return fail(NS_EINVAL, "too many streams for one call (staging)");
     StreamDesc *sd = reinterpret_cast<StreamDesc *>(g.host);
     for (int s = 0; s < S; s++) {
         const ns_chunk &k = ch[s];
@@ -516,10 +571,13 @@ static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint
         d.wts = k.model ? k.model->packed : nullptr;
         d.w = k.w; d.h = k.h; d.s = k.scale; d.n = k.n_frames;
         d.hr_base = s * n;
-        d.group = group ? group[s] : 0;
-        d.job_base = job_base ? job_base[s] : 0;
-        d.job_cap = job_cap ? job_cap[s] : INT32_MAX;
+        d.group = pl.group ? pl.group[s] : 0;
+        d.job_base = pl.job_base ? pl.job_base[s] : 0;
+        d.job_cap = pl.job_cap ? pl.job_cap[s] : INT32_MAX;
+        d.job_goff = pl.job_goff ? pl.job_goff[s] : 0;
         d.use_res_size = use_res_size ? 1 : 0;
+        d.acache = pl.acache ? pl.acache[s] : nullptr;
+        d.acache_stride = pl.acache_stride ? pl.acache_stride[s] : 0;
         sd[s] = d;
     }
     g.d_sd = reinterpret_cast<StreamDesc *>(g.dev);
@@ -533,6 +591,22 @@ static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint
         memcpy(g.host + off, cost, sizeof(int64_t) * S);
         g.d_cost = reinterpret_cast<int64_t *>(g.dev + off);
         off += cost_bytes;
+    }
+    if (pl.glist) {
+        memcpy(g.host + off, pl.glist->data(), sizeof(int32_t) * pl.glist->size());
+        g.d_glist = reinterpret_cast<int32_t *>(g.dev + off);
+        off += a256(sizeof(int32_t) * pl.glist->size());
+        memcpy(g.host + off, pl.goff->data(), sizeof(int32_t) * pl.goff->size());
+        g.d_goff = reinterpret_cast<int32_t *>(g.dev + off);
+        off += a256(sizeof(int32_t) * pl.goff->size());
+    }
+    if (pl.prv) {
+        memcpy(g.host + off, pl.prv->data(), sizeof(int16_t) * (size_t)S * n);
+        g.d_prv = reinterpret_cast<int16_t *>(g.dev + off);
+        off += a256(sizeof(int16_t) * (size_t)S * n);
+        memcpy(g.host + off, pl.nxt->data(), sizeof(int16_t) * (size_t)S * n);
+        g.d_nxt = reinterpret_cast<int16_t *>(g.dev + off);
+        off += a256(sizeof(int16_t) * (size_t)S * n);
     }
     g.used = off;
     *out = g;
@@ -595,7 +669,7 @@ extern "C" ns_status ns_select_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
     cudaStream_t st = (cudaStream_t)stream;
     NS_CUDA(cudaSetDevice(c->device));
     Staged g;
-    if ((r = stage_streams(c, ch, S, n, nullptr, p->mode == NS_GLOBAL_BUDGET ? p->cost : nullptr, nullptr, nullptr,
+    if ((r = stage_streams(c, ch, S, n, nullptr, p->mode == NS_GLOBAL_BUDGET ? p->cost : nullptr,
                            p->use_res_size != 0, &g)) != NS_OK)
         return r;
     if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
@@ -611,7 +685,7 @@ extern "C" ns_status ns_select_merge(ns_ctx *c, int S, int n, const int64_t *gai
     if (S < 1 || n < 1 || n > kMaxFrames) return fail(NS_EINVAL, "ns_select_merge: S = %d, n = %d", S, n);
     if ((size_t)S * n > (size_t)kMaxSN) return fail(NS_EINVAL, "S * n = %zu exceeds %d", (size_t)S * n, kMaxSN);
     if (budget < 0) return fail(NS_EINVAL, "budget < 0");
-    if (!gain || !rank_in || !type || !sid || !cost || !rank || !is_anchor)
+    if (!gain || !type || !sid || !cost || !rank || !is_anchor)
         return fail(NS_EINVAL, "ns_select_merge: NULL array");
     NS_CUDA(cudaSetDevice(c->device));
     NS_CUDA(launch_merge(S, n, gain, rank_in, type, sid, cost, budget, c->order, c->grank, c->pos_stream, c->cut, rank,
@@ -715,7 +789,8 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
 
 // ------------------------------------------------------------------ reconstruct
 static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n,
-                                 const uint8_t *is_anchor, cudaStream_t st) {
+                                 const uint8_t *is_anchor, const uint8_t *const *asrc, cudaStream_t st) {
+    uint8_t *gsv = g.d_nxt ? c->gsv : nullptr;   // HR rings: GOLDEN saves
     int mw[5] = {0, 0, 0, 0, 0}, mh[5] = {0, 0, 0, 0, 0};
     size_t maxhr = 0;
     for (int s = 0; s < S; s++) {
@@ -723,29 +798,10 @@ static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch,
         mh[ch[s].scale] = std::max(mh[ch[s].scale], ch[s].h);
         maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
     }
-    NS_CUDA(launch_golden_index(g.d_sd, S, n, c->gold, st));
-    NS_CUDA(launch_frame_desc(g.d_sd, S, n, is_anchor, g.d_hr, c->gold, c->fdesc, st));
-// (measured neutral: 198.7-198.9 vs 198.1-199.9 ms per c4 step -- off)
-#ifndef NS_RECON_TWO_STREAMS
-#define NS_RECON_TWO_STREAMS 0
-#endif
-    if (NS_RECON_TWO_STREAMS && S >= 2) {
-        // streams are independent chains: the first half steps on `st`, the
-        // second on the context's second stream, so one chain's launch gaps and
-        // last partial wave overlap the other's frame step
-        const int h0 = S / 2;
-        NS_CUDA(cudaEventRecord(c->ev_fork, st));
-        NS_CUDA(cudaStreamWaitEvent(c->sst, c->ev_fork, 0));
-        for (int f = 0; f < n; f++) {
-            NS_CUDA(launch_recon_step(c->fdesc, h0, n, f, mw, mh, st, 0));
-            NS_CUDA(launch_recon_step(c->fdesc, S - h0, n, f, mw, mh, c->sst, h0));
-        }
-        NS_CUDA(cudaEventRecord(c->ev_join, c->sst));
-        NS_CUDA(cudaStreamWaitEvent(st, c->ev_join, 0));
-    } else {
-        for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, S, n, f, mw, mh, st));
-    }
-    NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, maxhr, st));
+    NS_CUDA(launch_golden_index(g.d_sd, S, n, g.d_nxt, c->gold, gsv, st));
+    NS_CUDA(launch_frame_desc(g.d_sd, S, n, is_anchor, g.d_hr, c->gold, gsv, asrc, c->fdesc, st));
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, S, n, f, mw, mh, st));
+    NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, gsv, maxhr, st));
     return NS_OK;
 }
 
@@ -756,13 +812,13 @@ extern "C" ns_status ns_reconstruct_chunk(ns_ctx *c, const ns_chunk *ch, int S, 
     ns_status r = check_chunks(ch, S, false, &n);
     if (r != NS_OK) return r;
     if (!is_anchor) return fail(NS_EINVAL, "ns_reconstruct_chunk: is_anchor is NULL");
-    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    if ((r = check_hr_table(ch, S, n, hr_out, false, nullptr)) != NS_OK) return r;
     cudaStream_t st = (cudaStream_t)stream;
     NS_CUDA(cudaSetDevice(c->device));
     Staged g;
-    if ((r = stage_streams(c, ch, S, n, hr_out, nullptr, nullptr, nullptr, false, &g)) != NS_OK) return r;
+    if ((r = stage_streams(c, ch, S, n, hr_out, nullptr, false, &g)) != NS_OK) return r;
     if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
-    r = run_reconstruct(c, g, ch, S, n, is_anchor, st);
+    r = run_reconstruct(c, g, ch, S, n, is_anchor, nullptr, st);
     stage_release(c, g.slot, st);
     return r;
 }
@@ -777,15 +833,15 @@ struct LrGather {
 
 static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const ns_select_params *p,
                               uint8_t *const *hr_out, uint8_t *anchor, double *stats, cudaStream_t st,
-                              const LrGather *lg, uint64_t *gathered) {
+                              const LrGather *lg, uint64_t *gathered, const std::vector<int> &ring) {
     const bool topk = p->mode == NS_TOPK_PER_STREAM;
     // exactly k anchors per stream -> fixed job slots; otherwise (budget, given
-    // map, Key SR with fewer key frames than k) slots are claimed per group
+    // map, Key SR with fewer key frames than k) slots are assigned per group
     const bool fixed = topk && p->selector != NS_SEL_KEY;
     // SR shape groups and job slots (multi-stream batcher)
     std::map<std::tuple<int, int, int, int, int>, int> gid;
     std::vector<std::tuple<int, int, int, int, int>> gkey;
-    std::vector<int> group(S), job_base(S), gcount, goff;
+    std::vector<int> group(S), job_base(S), job_goff(S), gcount, goff;
     std::vector<int> gstreams;
     int64_t min_cost = INT64_MAX;
     if (!topk)
@@ -815,11 +871,75 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
     if (total > kMaxJobs) return fail(NS_EINVAL, "too many SR jobs (%d)", total);
     if (lg && (size_t)total * lg->stride > c->lr_stage_cap)
         return fail(NS_EINVAL, "anchor LR staging too small (%d jobs)", total);
+    // the streams of each group in stream order (deterministic slot assignment)
+    std::vector<int> glist, gl_off(G + 1, 0);
+    for (int s = 0; s < S; s++) gl_off[group[s] + 1]++;
+    for (int gi = 0; gi < G; gi++) gl_off[gi + 1] += gl_off[gi];
+    glist.resize(S);
     {
-        std::vector<int> local(G, 0);
+        std::vector<int> fill(gl_off.begin(), gl_off.end() - 1), local(G, 0);
         for (int s = 0; s < S; s++) {
             const int gi = group[s];
+            glist[fill[gi]++] = s;
             job_base[s] = fixed ? goff[gi] + local[gi]++ * p->k : goff[gi];
+            job_goff[s] = goff[gi];
+        }
+    }
+    // every SR arena and the anchor cache are reserved before anything is
+    // enqueued, so a pool that is too small fails with nothing launched
+    ns_status r;
+    if (total > 0)
+        for (int gi = 0; gi < G; gi++) {
+            int h, w, C, s, B;
+            std::tie(h, w, C, s, B) = gkey[gi];
+            const SrArena *a0 = nullptr, *a1 = nullptr;
+            if ((r = get_arena(c, h, w, C, s, 0, &a0)) != NS_OK) return r;
+            if (gcount[gi] > a0->nb && (r = get_arena(c, h, w, C, s, 1, &a1)) != NS_OK) return r;
+        }
+    const bool any_ring = std::find(ring.begin(), ring.end(), 1) != ring.end();
+    std::vector<uint8_t *> acache(S, nullptr);
+    std::vector<size_t> astride(S, 0);
+    if (any_ring && total > 0) {
+        std::vector<size_t> gbase(G), gstride(G);
+        size_t need = 0;
+        for (int gi = 0; gi < G; gi++) {
+            int h, w, C, s, B;
+            std::tie(h, w, C, s, B) = gkey[gi];
+            gstride[gi] = a256((size_t)3 * h * s * w * s);
+            gbase[gi] = need;
+            need += gstride[gi] * gcount[gi];
+        }
+        if (need > c->acache_cap) {
+            NS_CUDA(cudaStreamSynchronize(st));  // a smaller cache may still be read (not the steady state)
+            if (!(c->acache = pool_take(c, need)))
+                return fail(NS_ENOMEM, "HR ring: pool too small for the anchor cache (%zu bytes)", need);
+            c->acache_cap = need;
+        }
+        for (int s = 0; s < S; s++) {
+            acache[s] = c->acache + gbase[group[s]];
+            astride[s] = gstride[group[s]];
+        }
+    }
+    // HR rings: for every frame the previous / next frame of its stream that
+    // writes the same hr_out entry (-1 / n: none)
+    std::vector<int16_t> prv, nxt;
+    if (any_ring) {
+        prv.assign((size_t)S * n, -1);
+        nxt.assign((size_t)S * n, (int16_t)n);
+        std::unordered_map<const uint8_t *, int> last;
+        for (int s = 0; s < S; s++) {
+            last.clear();
+            for (int f = 0; f < n; f++) {
+                const size_t e = (size_t)s * n + f;
+                auto it = last.find(hr_out[e]);
+                if (it != last.end()) {
+                    prv[e] = (int16_t)it->second;
+                    nxt[(size_t)s * n + it->second] = (int16_t)f;
+                    it->second = f;
+                } else {
+                    last.emplace(hr_out[e], f);
+                }
+            }
         }
     }
     if (gathered && lg) {  // exact in top-k mode (k frames per stream); upper bound otherwise
@@ -829,11 +949,22 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
         *gathered += b;
     }
     Staged g;
-    ns_status r;
     std::vector<int> job_cap(S);
     for (int s = 0; s < S; s++) job_cap[s] = fixed ? p->k : gcount[group[s]];
-    if ((r = stage_streams(c, ch, S, n, hr_out, topk ? nullptr : p->cost, group.data(), job_base.data(),
-                           p->use_res_size != 0, &g, job_cap.data())) != NS_OK)
+    StreamPlan pl;
+    pl.group = group.data();
+    pl.job_base = job_base.data();
+    pl.job_cap = job_cap.data();
+    pl.job_goff = job_goff.data();
+    pl.acache = acache.data();
+    pl.acache_stride = astride.data();
+    pl.glist = &glist;
+    pl.goff = &gl_off;
+    if (any_ring) {
+        pl.prv = &prv;
+        pl.nxt = &nxt;
+    }
+    if ((r = stage_streams(c, ch, S, n, hr_out, topk ? nullptr : p->cost, p->use_res_size != 0, &g, pl)) != NS_OK)
         return r;
     if ((r = stage_end(c, g.slot, g.used, st)) != NS_OK) return r;
     do {
@@ -842,8 +973,10 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
             cudaError_t e = cudaSuccess;
             if (lg) e = cudaMemsetAsync(c->lr_len, 0, sizeof(uint32_t) * total, st);
             if (e == cudaSuccess)
-                e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, fixed, p->k, st,
-                                   lg ? lg->stage : nullptr, lg ? lg->stride : 0, c->lr_src, c->lr_len);
+                e = launch_compact(g.d_sd, S, n, anchor, g.d_hr, c->jobs, c->job_count, G, g.d_glist, g.d_goff,
+                                   c->acount, fixed, g.d_prv, any_ring ? c->asrc : nullptr, st,
+                                   lg ? lg->stage : nullptr,
+                                   lg ? lg->stride : 0, c->lr_src, c->lr_len);
             if (e == cudaSuccess && lg) e = launch_lr_gather(c->jobs, c->lr_src, c->lr_len, total, lg->stride, st);
             if (e != cudaSuccess) { r = cuda_fail(e, "compact"); break; }
             for (int gi = 0; gi < G && r == NS_OK; gi++) {
@@ -854,7 +987,8 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
             }
             if (r != NS_OK) break;
         }
-        if ((r = run_reconstruct(c, g, ch, S, n, anchor, st)) != NS_OK) break;
+        if ((r = run_reconstruct(c, g, ch, S, n, anchor, any_ring && total > 0 ? c->asrc : nullptr, st)) != NS_OK)
+            break;
         if (stats) {
             size_t maxhr = 0;
             for (int s = 0; s < S; s++) maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
@@ -875,10 +1009,11 @@ extern "C" ns_status ns_enhance_streams(ns_ctx *c, const ns_chunk *ch, int S, co
     ns_status r = check_chunks(ch, S, true, &n);
     if (r != NS_OK) return r;
     if ((r = check_params(p, S, n)) != NS_OK) return r;
-    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    std::vector<int> ring;
+    if ((r = check_hr_table(ch, S, n, hr_out, true, &ring)) != NS_OK) return r;
     NS_CUDA(cudaSetDevice(c->device));
     return enhance_impl(c, ch, S, n, p, hr_out, is_anchor_out ? is_anchor_out : c->anchor, stats,
-                        (cudaStream_t)stream, nullptr, nullptr);
+                        (cudaStream_t)stream, nullptr, nullptr, ring);
 }
 
 // ------------------------------------------------------------------ host-input path
@@ -906,7 +1041,8 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
     ns_status r = check_chunks(ch, S, true, &n);
     if (r != NS_OK) return r;
     if ((r = check_params(p, S, n)) != NS_OK) return r;
-    if ((r = check_hr_table(ch, S, n, hr_out)) != NS_OK) return r;
+    std::vector<int> ring;
+    if ((r = check_hr_table(ch, S, n, hr_out, true, &ring)) != NS_OK) return r;
     for (int s = 0; s < S; s++)
         if (!host_mapped(ch[s].lr) || !host_mapped(ch[s].res) || !host_mapped(ch[s].mv) || !host_mapped(ch[s].type) ||
             !host_mapped(ch[s].res_size))
@@ -1003,8 +1139,9 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
         NS_CUDA(cudaEventRecord(c->ev_copied[b], c->cst));
         NS_CUDA(cudaStreamWaitEvent(st, c->ev_copied[b], 0));
         LrGather lg{c->lr_stage, lr_stride};
+        const std::vector<int> gring(ring.begin() + g0, ring.begin() + g0 + cnt);
         r = enhance_impl(c, dch.data(), cnt, n, p, hr_out + (size_t)g0 * n, anchor + (size_t)g0 * n,
-                         stats ? stats + (size_t)8 * g0 : nullptr, st, &lg, &moved);
+                         stats ? stats + (size_t)8 * g0 : nullptr, st, &lg, &moved, gring);
         if (r != NS_OK) return r;
         NS_CUDA(cudaEventRecord(c->ev_free[b], st));
         c->hin_used[b] = true;

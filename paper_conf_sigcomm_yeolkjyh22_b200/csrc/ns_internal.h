@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstddef>
+#include <atomic>
 #include "../../include/ns.h"
 
 namespace ns {
@@ -27,8 +28,11 @@ struct StreamDesc {
     int32_t hr_base;       // index of hr_out[s][0] in the device hr table
     int32_t group;         // SR shape group index (ns_enhance_streams)
     int32_t job_base;      // first SR job slot of this stream in its group
-    int32_t job_cap;       // slots of its group (budget / given modes: claims beyond are dropped)
+    int32_t job_cap;       // slots of its group; a given anchor map's anchors beyond it are demoted (ns.h)
     int32_t use_res_size;
+    int32_t job_goff;      // first job slot of the stream's SR shape group
+    uint8_t *acache;       // HR rings: the group's anchor cache (job slot j at acache + (j - job_goff) * stride)
+    uint64_t acache_stride;
 };
 
 // Per (stream, frame) reconstruction step descriptor, resolved once per chunk
@@ -40,13 +44,18 @@ struct __align__(16) FrameDesc {
     const ns_block_mv *mv_f;   // mv[f] [h/8][w/8]
     uint8_t *out;              // HR[f]
     const uint8_t *ref_last;   // HR[f-1] or hr_last
-    const uint8_t *ref_gold;   // HR of the latest KEY/ALTREF < f, or hr_golden
+    const uint8_t *ref_gold;   // HR of the latest KEY/ALTREF g < f (its copy in hr_golden from step
+                               // g+2 on when g was saved), or hr_golden
+    const uint8_t *asrc;       // an anchor whose slot an earlier frame uses (HR ring): its SR output
+                               // in the anchor cache, copied to out at this step
+    const uint8_t *gsave_src;  // f-1 is a KEY/ALTREF frame whose ring slot is reused while it is still
+    uint8_t *gsave_dst;        // GOLDEN: HR[f-1] is saved into hr_golden (= gsave_dst) at this step
     int32_t w, h;              // LR size
     int16_t s;                 // scale
     uint8_t anchor, key;       // is_anchor[f], type[f] == KEY
-    int32_t pad;
+    int32_t pad0, pad1, pad2;
 };
-static_assert(sizeof(FrameDesc) == 64, "FrameDesc is one 64-B record");
+static_assert(sizeof(FrameDesc) == 96, "FrameDesc is one 96-B record");
 
 // One anchor-SR job (device).
 struct SrJob {
@@ -105,23 +114,39 @@ cudaError_t launch_merge(int S, int n, const int64_t *gain, const int32_t *rank_
 cudaError_t launch_global(const StreamDesc *d_sd, int S, int n, const int64_t *gain, const int32_t *order,
                           const int64_t *cost, int64_t budget, int32_t *grank, int32_t *pos_stream,
                           int32_t *cut, int32_t *rank, uint8_t *is_anchor, cudaStream_t st);
-cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
-                           uint8_t *const *d_hr_table, SrJob *jobs, int32_t *job_count, int n_groups, int topk,
-                           int k, cudaStream_t st, uint8_t *lr_stage = nullptr, size_t lr_stride = 0,
-                           const uint8_t **lr_src = nullptr, uint32_t *lr_len = nullptr);
+// Anchors -> SR job slots.  topk: stream s owns slots [job_base, job_base + k).
+// Otherwise slots are assigned deterministically, stream by stream in each
+// group's list order (glist / goff: the streams of group g are
+// glist[goff[g] .. goff[g+1])), and anchors beyond the group's job_cap are
+// demoted (is_anchor cleared: the frame is reconstructed instead).  acount:
+// [S] scratch.  HR rings (else both NULL): prv [S][n] = the previous frame of
+// the stream writing the same hr_out entry (-1: none); an anchor with prv >= 0
+// is SR'd into the anchor cache and asrc[s][f] records where.
+cudaError_t launch_compact(const StreamDesc *d_sd, int S, int n, uint8_t *is_anchor, uint8_t *const *d_hr_table,
+                           SrJob *jobs, int32_t *job_count, int n_groups, const int32_t *glist,
+                           const int32_t *goff, int32_t *acount, int topk, const int16_t *prv,
+                           const uint8_t **asrc, cudaStream_t st,
+                           uint8_t *lr_stage = nullptr, size_t lr_stride = 0, const uint8_t **lr_src = nullptr,
+                           uint32_t *lr_len = nullptr);
 // Copies every filled job's LR frame (lr_len[j] > 0) from lr_src[j] (host-mapped
 // memory) to jobs[j].lr (device staging set by launch_compact).
 cudaError_t launch_lr_gather(const SrJob *jobs, const uint8_t *const *lr_src, const uint32_t *lr_len, int max_jobs,
                              size_t max_len, cudaStream_t st);
-cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, int16_t *gold_idx, cudaStream_t st);
+// gold [S][n+1]; HR rings (nxt [S][n] = the next frame writing the same hr_out
+// entry, n: none): gsv [S][n] = 1 for a KEY/ALTREF frame that must be saved into
+// hr_golden because its slot is reused while it is GOLDEN; nxt = NULL: no saves.
+cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, const int16_t *nxt, int16_t *gold_idx,
+                                uint8_t *gsv, cudaStream_t st);
 // max_lr_w / max_lr_h: [5] indexed by scale (0 = no stream of that scale)
 // fd[s][f] for all streams and frames (after launch_golden_index)
+// gsv / asrc: from launch_golden_index / launch_compact for HR rings, else NULL
 cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
-                              uint8_t *const *d_hr_table, const int16_t *gold_idx, FrameDesc *fd, cudaStream_t st);
+                              uint8_t *const *d_hr_table, const int16_t *gold_idx, const uint8_t *gsv,
+                              const uint8_t *const *asrc, FrameDesc *fd, cudaStream_t st);
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
                               cudaStream_t st, int s0 = 0);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
-                              const int16_t *gold_idx, size_t max_hr_bytes, cudaStream_t st);
+                              const int16_t *gold_idx, const uint8_t *gsv, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
                          uint8_t *const *d_hr_table, size_t max_hr_bytes, double *stats, cudaStream_t st);
 cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint8_t *packed, cudaStream_t st);
@@ -142,6 +167,26 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);
 // shape).  job_count (device) may be NULL; otherwise CTAs of jobs >= *job_count exit.
 cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                          const int32_t *job_count, cudaStream_t st);
+
+// Sets a kernel's dynamic shared memory limit (and, optionally, the all-shared
+// L1 carveout) once per DEVICE: function attributes belong to the context of
+// the device current at the call, and a process may drive several devices
+// (ns.h: one context per device).  One flag word per kernel instantiation
+// (template on the kernel pointer), bit d = device d done; thread-safe.
+template <auto K>
+cudaError_t ensure_kernel_smem(int bytes, bool max_carveout = false) {
+    static std::atomic<unsigned long long> done{0};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const unsigned long long bit = 1ull << (dev & 63);
+    if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+    e = cudaFuncSetAttribute(K, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess && max_carveout)
+        e = cudaFuncSetAttribute(K, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+    if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_release);
+    return e;
+}
 
 // Kernel families for ns_launch_count / ns_profile_read.
 enum Fam { F_SCORE = 0, F_SELECT, F_GLOBAL, F_COMPACT, F_SR_PREP, F_SR_HEAD, F_SR_BODY, F_SR_END, F_SR_UP,

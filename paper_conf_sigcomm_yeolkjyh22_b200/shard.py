@@ -99,33 +99,43 @@ def gather_rows(tensors, group=None):
 
 
 def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_res_size=False, group=None,
-                               stream=None, return_all=False):
+                               stream=None, return_all=False, n=None, device=None):
     """§5.2 global anchor selection over the streams of every GPU:
     (1) per-stream gains and ranks on this GPU (ns_select_anchors, Alg. 1);
     (2) all_gather of gain / rank / type / sid / cost rows (gather_rows);
     (3) ns_select_merge on the gathered rows -- the identical deterministic
     prefix on every GPU, no further exchange.  Returns this GPU's is_anchor
     [S_local, n] (device u8) for ns_enhance_streams(mode=NS_GIVEN_ANCHORS,
-    anchor_in=..., cost=cost, budget=budget), and the global rank rows."""
+    anchor_in=..., cost=cost, budget=budget), and the global rank rows.
+    A rank may own no streams (chunks == []): it then passes n and device, and
+    still takes part in the gather and the merge."""
     import torch
     from . import NS_TOPK_PER_STREAM
-    S, n = len(chunks), chunks[0].n
-    dev = chunks[0].type.device
-    gain = torch.empty((S, n), dtype=torch.int64, device=dev)
-    rank = torch.empty((S, n), dtype=torch.int32, device=dev)
-    anc = torch.empty((S, n), dtype=torch.uint8, device=dev)
-    ctx.select_anchors(chunks, gain, rank, anc, stream=stream, mode=NS_TOPK_PER_STREAM, k=0, fresh=fresh,
-                       use_res_size=use_res_size)
-    types = torch.stack([c.type for c in chunks])
-    sid_t = torch.as_tensor(list(sid), dtype=torch.int32).to(dev)
-    cost_t = torch.as_tensor(list(cost), dtype=torch.int64).to(dev)
-    (g_all, r_all, t_all, s_all, c_all), off = gather_rows([gain, rank, types, sid_t, cost_t], group)
+    S = len(chunks)
+    n = chunks[0].n if S else int(n)
+    dev = chunks[0].type.device if S else torch.device(device)
+    gain = torch.zeros((S, n), dtype=torch.int64, device=dev)
+    rank = torch.zeros((S, n), dtype=torch.int32, device=dev)
+    anc = torch.zeros((S, n), dtype=torch.uint8, device=dev)
+    if S:
+        ctx.select_anchors(chunks, gain, rank, anc, stream=stream, mode=NS_TOPK_PER_STREAM, k=0, fresh=fresh,
+                           use_res_size=use_res_size)
+        types = torch.stack([c.type for c in chunks])
+    else:
+        types = torch.zeros((0, n), dtype=torch.uint8, device=dev)
+    sid_t = torch.as_tensor(list(sid), dtype=torch.int32).reshape(-1).to(dev)
+    cost_t = torch.as_tensor(list(cost), dtype=torch.int64).reshape(-1).to(dev)
+    # (w, h, scale) of every row: the anchor exchange sizes each moved frame by
+    # its own stream's shape (mixed-resolution fleets, SURVEY §8(d) c5)
+    shape_t = torch.as_tensor([[c.w, c.h, c.scale] for c in chunks], dtype=torch.int32).reshape(-1, 3).to(dev)
+    (g_all, r_all, t_all, s_all, c_all, sh_all), off = gather_rows([gain, rank, types, sid_t, cost_t, shape_t],
+                                                                   group)
     rank_out = torch.empty_like(r_all)
     anc_all = torch.empty_like(t_all)
     ctx.select_merge(g_all, r_all, t_all, s_all, c_all, budget, rank_out, anc_all, stream=stream)
     if return_all:  # every gathered row, for the anchor-level load balancing
         return (anc_all[off: off + S].contiguous(), rank_out[off: off + S].contiguous(),
-                {"anchor": anc_all, "sid": s_all, "cost": c_all})
+                {"anchor": anc_all, "sid": s_all, "cost": c_all, "shape": sh_all})
     return anc_all[off: off + S].contiguous(), rank_out[off: off + S].contiguous()
 
 
@@ -167,7 +177,7 @@ def plan_anchor_moves(anchors, owner, cost, world):
 
 
 def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anchors_all, owner_all, sid_all, cost_all,
-                                group=None, stream=None):
+                                group=None, stream=None, shape_all=None, device=None):
     """SR on this GPU's share of the balanced anchor set, then reconstruction of
     this GPU's streams (ns_sr_anchors + ns_reconstruct_chunk).  anchors_all /
     owner_all / sid_all / cost_all describe every gathered stream row (host
@@ -177,7 +187,10 @@ def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anc
     every GPU keeps all of them).  Exported anchors: LR out, HR back; imported
     anchors: LR in, SR here, HR out -- point-to-point over NCCL (NVLink).
     Everything is ordered on the current torch stream (stream=None), which the
-    NCCL point-to-point calls synchronise with."""
+    NCCL point-to-point calls synchronise with.  shape_all[i] = (w, h, scale)
+    of row i (select_global_across_ranks(return_all=True)["shape"]): an
+    imported anchor's LR / HR buffers take its source stream's shape.  A rank
+    with no streams (chunks == []) passes `device` and still serves imports."""
     import torch
     import torch.distributed as dist
     dist_on = dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1
@@ -199,10 +212,13 @@ def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anc
         if src == me:
             ops.append(dist.P2POp(dist.isend, chunks[local[s]].lr[f].contiguous(), dst, group))
         elif dst == me:
-            c0 = chunks[0]
-            h, w, sc = c0.h, c0.w, c0.scale
-            lr = torch.empty((3, h, w), dtype=torch.uint8, device=c0.lr.device)
-            hr = torch.empty((3, sc * h, sc * w), dtype=torch.uint8, device=c0.lr.device)
+            if shape_all is not None:
+                w, h, sc = (int(v) for v in shape_all[i])
+            else:  # uniform fleets: every row has this rank's shape
+                w, h, sc = chunks[0].w, chunks[0].h, chunks[0].scale
+            dev = chunks[0].lr.device if chunks else torch.device(device)
+            lr = torch.empty((3, h, w), dtype=torch.uint8, device=dev)
+            hr = torch.empty((3, sc * h, sc * w), dtype=torch.uint8, device=dev)
             imports.append((i, f, src, lr, hr))
             ops.append(dist.P2POp(dist.irecv, lr, src, group))
     if ops:
@@ -223,5 +239,6 @@ def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anc
     if ops:
         for rq in dist.batch_isend_irecv(ops):
             rq.wait()
-    ctx.reconstruct_chunk(chunks, is_anchor, hr_out, stream=stream)
+    if chunks:
+        ctx.reconstruct_chunk(chunks, is_anchor, hr_out, stream=stream)
     return moves

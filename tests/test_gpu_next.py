@@ -131,6 +131,31 @@ def test_select_merge_bit_exact(ctx):
             assert list(gr[s]) == rank[j].cpu().tolist()
 
 
+def test_select_merge_does_not_trust_rank_in(ctx):
+    """ns_select_merge rebuilds each stream's priority order from (type, gain
+    desc, frame asc) (ns.h): a rank array from a baseline selector, a garbage
+    one (values >= n, negative) or NULL give the same merge as the true ranks."""
+    S, n = 5, 16
+    cs = [synth.make_chunk(9800 + s, 32, 24, 3, n, types=synth.default_types(n, 5)) for s in range(S)]
+    dcs = [dev_chunk(ns, c, DEV) for c in cs]
+    g, r, _ = _select_gpu(ctx, dcs, k=0)
+    t_all = torch.stack([d.type for d in dcs])
+    sid = torch.arange(S, dtype=torch.int32, device=DEV)
+    co = torch.tensor([1, 2, 1, 3, 1], dtype=torch.int64, device=DEV)
+    _, rk, _ = _select_gpu(ctx, dcs, k=3, selector=ns.NS_SEL_KEY_UNIFORM)
+    bad = torch.randint(-1000, 1000, r.shape, dtype=torch.int32, device=DEV)
+    outs = []
+    for rin in (r, rk, bad, None):
+        rank = torch.empty_like(r)
+        anc = torch.empty_like(t_all)
+        ctx.select_merge(g, rin, t_all, sid, co, 17, rank, anc)
+        torch.cuda.synchronize()
+        outs.append((rank.cpu().tolist(), anc.cpu().tolist()))
+    er, ea = OS.merge_gathered(t_all.cpu().tolist(), g.cpu().tolist(), list(range(S)), [1, 2, 1, 3, 1], 17)
+    for o in outs:
+        assert o == (er, ea)
+
+
 def test_enhance_given_anchors_equals_global(ctx):
     """Per-shard whole path on the merged anchor map == one global call."""
     S, n = 6, 10

@@ -219,3 +219,57 @@ def test_gloo_world2_balanced_sr_exchange():
     assert all(src == 0 and dst == 1 for _, _, src, dst in m0)
     assert ok0 and ok1                                      # every anchor's HR is its own stream's SR
     assert rc0 == rc1 == 1
+
+
+def _lb_worker_mixed(rank, world, port, q):
+    """Mixed resolutions (c5-like fleets) and a rank that owns no stream: the
+    imported anchors' buffers take their source stream's shape (shape_all)."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from types import SimpleNamespace
+        n = 6
+        shapes = [(8, 4, 2), (16, 8, 2), (8, 4, 2), (24, 8, 2)]   # (w, h, scale) per stream
+        S_tot = len(shapes)
+        owner_all = [0] * S_tot                         # rank 1 owns nothing
+        sid_all = list(range(S_tot))
+        cost_all = [1, 4, 1, 6]
+        anchors_all = [[0, 3], [0, 2], [0], [0, 5]]
+        mine = [i for i in range(S_tot) if owner_all[i] == rank]
+        g = torch.Generator().manual_seed(11)
+        lr_all = [torch.randint(0, 256, (n, 3, h, w), generator=g, dtype=torch.int32).to(torch.uint8)
+                  for (w, h, _) in shapes]
+        chunks = [SimpleNamespace(lr=lr_all[i], w=shapes[i][0], h=shapes[i][1], scale=2) for i in mine]
+        hr_out = [[torch.zeros((3, 2 * shapes[i][1], 2 * shapes[i][0]), dtype=torch.uint8) for _ in range(n)]
+                  for i in mine]
+        models = {s: 20 + s for s in sid_all}
+        ia = torch.zeros((len(mine), n), dtype=torch.uint8)
+        ctx = _FakeCtx()
+        moves = shard.balanced_sr_and_reconstruct(ctx, chunks, models, mine, ia, hr_out, anchors_all, owner_all,
+                                                  sid_all, cost_all, shape_all=shapes, device="cpu")
+        ok = True
+        for li, s in enumerate(mine):
+            for f in anchors_all[s]:
+                exp = (lr_all[s][f].repeat_interleave(2, 1).repeat_interleave(2, 2).int() + models[s]) % 256
+                ok &= bool(torch.equal(hr_out[li][f], exp.to(torch.uint8)))
+        q.put((rank, moves, ok, ctx.recon_calls))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_balanced_mixed_shapes_empty_rank():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_lb_worker_mixed, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    (r0, m0, ok0, rc0), (r1, m1, ok1, rc1) = res
+    assert m0 == m1 and len(m0) > 0
+    assert {shapes_i for shapes_i, *_ in m0} & {1, 3}       # large-frame rows moved too
+    assert ok0 and ok1
+    assert (rc0, rc1) == (1, 0)                             # the empty rank reconstructs nothing

@@ -1,0 +1,6 @@
+#!/bin/bash
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.limit --format=csv > gpurun_out/smi.txt
+lscpu | head -20 > gpurun_out/lscpu.txt; nproc >> gpurun_out/lscpu.txt
+bash tools/gpu_sanitize.sh
+python bench.py --no-cpu-baseline --e2e-steps 0 > gpurun_out/b0.log 2>&1
