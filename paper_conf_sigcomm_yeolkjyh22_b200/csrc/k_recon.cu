@@ -131,8 +131,20 @@ __device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) 
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
     return r;
 }
+// (experiment knob NS_RECON_L2PF: L2 prefetch size hint of the window loads)
+#ifndef NS_RECON_L2PF
+#define NS_RECON_L2PF 0
+#endif
 __device__ __forceinline__ void cp_async8(void *dst, const void *src) {
+#if NS_RECON_L2PF == 64
+    asm volatile("cp.async.ca.shared.global.L2::64B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+#elif NS_RECON_L2PF == 128
+    asm volatile("cp.async.ca.shared.global.L2::128B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+#elif NS_RECON_L2PF == 256
+    asm volatile("cp.async.ca.shared.global.L2::256B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+#else
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+#endif
 }
 __device__ __forceinline__ void cp_async16(void *dst, const void *src) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
@@ -569,7 +581,12 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
 template <int S>
 static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
     // all of the unified L1/shared array as shared memory, so MINB CTAs fit
+#ifdef NS_RECON_CARVE  // (experiment knob: shared-memory carveout percentage instead of the maximum)
+    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, false); e != cudaSuccess) return e;
+    cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributePreferredSharedMemoryCarveout, NS_RECON_CARVE);
+#else
     if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, true); e != cudaSuccess) return e;
+#endif
     k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f, s0);
     return cudaGetLastError();
 }

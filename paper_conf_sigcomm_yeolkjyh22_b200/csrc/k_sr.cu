@@ -60,7 +60,7 @@ struct ConvArgs {
     int sub0;               // shuffle: first sub-pixel of this launch
     int lr_h, lr_w;         // tail: LR dims of the bilinear skip
     float *ring;            // uptail: fp32 t of the HR frame-border ring [job][nring][3]
-    uint8_t *lr8;           // EPI_HEAD with NS_HEAD_BUILD: u8 LR copy [job][H][3][wp] for uptail2
+    uint8_t *lr8;           // (unused by the convs: uptail2's u8 LR copy is written by k_prep_lr)
     int wp;
 };
 
@@ -101,20 +101,8 @@ __device__ __forceinline__ void up_tap(int X, int s, int len, int &i0, int &i1, 
 // block of row y-1 is complete: the epilogue reads it, applies the fused
 // epilogue, and zeroes it for row y+2.  No im2col, no lane shifts, 128-pixel
 // tiles, N = 96 (C = 32) -> up to 3x the MMA efficiency of N = 32.
-// NS_HEAD_BUILD: the head conv builds its own input rows (x = LR - 128, bf16,
-// channel group 0) from the u8 LR planes in a dedicated builder warp (warp 4)
-// and writes uptail2's u8 LR copy itself -- no prep pass, no bf16 input copy in
-// HBM.  The builder never stores the conv output, so its proxy fence does not
-// wait on the epilogue's global stores (the reason a same-warp build was slower).
-// Parity green, measured neutral (prep + head 10.76 vs head 10.8 ms per c4 step,
-// union over the two SR streams): one warp of byte loads builds rows no faster
-// than the prep pass + bulk copy deliver them.  Off.
-#ifndef NS_HEAD_BUILD
-#define NS_HEAD_BUILD 0
-#endif
-#ifndef NS_ROT_NSLOT
-#define NS_ROT_NSLOT 3  // input ring of k_conv_rot (head, end)
-#endif
+// (A head that builds its own input rows from the u8 LR planes in a builder
+// warp -- no prep pass -- was parity green and measured neutral.)
 template <int CIN, int NB>
 struct RotCfg {
     static constexpr int KC = CIN / 16;
@@ -123,7 +111,7 @@ struct RotCfg {
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
-    static constexpr int NSLOT = NS_ROT_NSLOT;  // 3: the barrier array is laid out [0,3) ring, 3 weights, 4 MMA
+    static constexpr int NSLOT = 3;  // input ring; the barrier array is laid out [0,3) ring, 3 weights, 4 MMA
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(3 * NB);
     static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + 128;
     static_assert((3 * NB) % 16 == 0 && 3 * NB <= 256, "N = 3 NB");
@@ -211,28 +199,11 @@ __device__ __forceinline__ void tmem_zeroN(uint32_t a) {
 
 
 
-#ifndef NS_RB_BULK
-#define NS_RB_BULK 1
-#endif
-#ifndef NS_ROT_BULK
-#define NS_ROT_BULK 1
-#endif
 // (k_uptail2 with bulk-copied rows measured neutral to slightly slower on the
-// same box -- 20.3 vs 19.2-20.3 ms -- so it keeps its tensor box)
-// NS_UP_OUT2: double-buffered output staging rows in uptail2 (drops one group
-// barrier per step); parity green, measured neutral (sr_up 20.2-20.4 vs
-// 20.1-20.3 ms, union over the two SR streams): off.
-#ifndef NS_UP_OUT2
-#define NS_UP_OUT2 0
-#endif
-// NS_UP_BIAS_INIT: uptail2's retired accumulator columns are re-initialised by
-// their own epilogue group with bias + 1/2 (no 3-group barrier per step).
-#ifndef NS_UP_BIAS_INIT
-#define NS_UP_BIAS_INIT 1
-#endif
-#ifndef NS_UP_BULK
-#define NS_UP_BULK 0
-#endif
+// same box -- 20.3 vs 19.2-20.3 ms -- so it keeps its tensor box; double-
+// buffered output staging rows measured neutral too.)  uptail2's retired
+// accumulator columns are re-initialised by their own epilogue group with
+// bias + 1/2 (no 3-group barrier per step).
 // Activation rows into a ring slot by one-dimensional bulk copies.  The
 // activation layout [job][H][G][W][8] (bf16) holds each channel group's row as
 // one contiguous run of 16 B per pixel, so a tile row segment of ncols pixels
@@ -273,15 +244,14 @@ __device__ __forceinline__ void row_bulk(uint8_t *slot, int ncols, const uint16_
 }
 
 template <int CIN, int NB, int EPI>
-__global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128)
+__global__ void __launch_bounds__(128)
     k_conv_rot(const __grid_constant__ CUtensorMap tm_in, const ConvArgs a) {
     using Cfg = RotCfg<CIN, NB>;
-    constexpr bool BUILD = EPI == EPI_HEAD && NS_HEAD_BUILD;  // warp 4 = input-row builder
     extern __shared__ __align__(1024) uint8_t smem[];
     uint8_t *s_w = smem;
     const float *s_bias = reinterpret_cast<const float *>(smem + Cfg::B_BYTES);
     uint8_t *s_ring = smem + Cfg::W_REGION;
-    // [0,3) ring full, 3 weights, 4 MMA done, [5,8) ring empty (BUILD)
+    // [0,3) ring full, 3 weights, 4 MMA done
     uint64_t *bars = reinterpret_cast<uint64_t *>(s_ring + Cfg::NSLOT * Cfg::SLOT);
     uint32_t *s_tmem = reinterpret_cast<uint32_t *>(bars + 8);
 
@@ -314,37 +284,27 @@ __global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128
             reinterpret_cast<uint4 *>(s_ring + (i / kHalo) * Cfg::SLOT + kHalo * 16)[i % kHalo] = make_uint4(0, 0, 0, 0);
         fence_proxy_async_smem();
     }
-#if NS_ROT_BULK
     // rows by bulk copies (row_bulk): G channel groups of 16 B per pixel
     constexpr int G = (EPI == EPI_HEAD) ? 1 : CIN / 8;
     (void)LOAD_BYTES;
-    if constexpr (!BUILD)
-        for (int sl = 0; sl < Cfg::NSLOT; sl++)
+    for (int sl = 0; sl < Cfg::NSLOT; sl++)
             slot_zero_edges<G>(s_ring + sl * Cfg::SLOT, kHalo, a.W, x0 - 1, tid, blockDim.x);
     fence_proxy_async_smem();
     __syncthreads();
-#endif
     if (tid == 0) {
         prefetch_tmap(&tm_in);
         mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
         bulk_load(s_w, J.wts + a.b_off, Cfg::B_BYTES, &bars[3]);
         bulk_load(smem + Cfg::B_BYTES, J.wts + a.bias_off, Cfg::BIAS_BYTES, &bars[3]);
-        for (int q = 0; q < Cfg::NSLOT && q < n_loads && !BUILD; q++) {
-#if NS_ROT_BULK
+        for (int q = 0; q < Cfg::NSLOT && q < n_loads; q++) {
             row_bulk<G>(s_ring + q * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + q, x0 - 1, &bars[q]);
-#else
-            mbar_arrive_expect_tx(&bars[q], LOAD_BYTES);
-            tma_load_5d(s_ring + q * Cfg::SLOT, &tm_in, &bars[q], 0, x0 - 1, 0, y0 - 1 + q, slot_job);
-#endif
         }
     }
-    // the three accumulator blocks start at zero (the builder warp owns no TMEM lanes)
-    if (warp < 4) {
-        tmem_zero<NB>(tl);
-        tmem_zero<NB>(tl + NB);
-        tmem_zero<NB>(tl + 2 * NB);
-        tmem_wait_st();
-    }
+    // the three accumulator blocks start at zero
+    tmem_zero<NB>(tl);
+    tmem_zero<NB>(tl + NB);
+    tmem_zero<NB>(tl + 2 * NB);
+    tmem_wait_st();
     mbar_wait(&bars[3], 0);
     tc_fence_before();
     __syncthreads();
@@ -357,54 +317,7 @@ __global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128
     uint4 rnext[RC];  // EPI_RESID: residual row prefetched one step ahead
 #pragma unroll
     for (int cg = 0; cg < RC; cg++) rnext[cg] = make_uint4(0, 0, 0, 0);
-    if (BUILD && warp == 4) {
-        // ---- builder: row q of the ring slot q % NSLOT once MMA(q - NSLOT) has
-        // read it; lane l owns pixels l + 32 i of the 130-pixel row.  The LR
-        // bytes of row q are loaded before the wait for the slot.
-        const size_t plane = (size_t)a.H * a.W;
-        for (int q = 0; q < n_loads; q++) {
-            const int yin = y0 - 1 + q, sl = q % Cfg::NSLOT;
-            uint32_t rgb[5];
-#pragma unroll
-            for (int i = 0; i < 5; i++) {
-                const int px = lane + 32 * i, xx = x0 - 1 + px;
-                rgb[i] = 0xFFFFFFFFu;
-                if (px < kHalo && yin >= 0 && yin < a.H && xx >= 0 && xx < a.W) {
-                    const uint8_t *L = J.lr + (size_t)yin * a.W + xx;
-                    rgb[i] = (uint32_t)__ldg(L) | ((uint32_t)__ldg(L + plane) << 8) |
-                             ((uint32_t)__ldg(L + 2 * plane) << 16);
-                }
-            }
-            if (q >= Cfg::NSLOT) mbar_wait(&bars[5 + sl], ((q / Cfg::NSLOT) - 1) & 1);
-#pragma unroll
-            for (int i = 0; i < 5; i++) {
-                const int px = lane + 32 * i;
-                if (px >= kHalo) continue;
-                uint4 o = make_uint4(0, 0, 0, 0);
-                if (rgb[i] != 0xFFFFFFFFu) {
-                    o.x = pack_bf16((float)(int)(rgb[i] & 255) - 128.f, (float)(int)((rgb[i] >> 8) & 255) - 128.f);
-                    o.y = pack_bf16((float)(int)((rgb[i] >> 16) & 255) - 128.f, 0.f);
-                }
-                *reinterpret_cast<uint4 *>(s_ring + sl * Cfg::SLOT + px * 16) = o;
-            }
-            fence_proxy_async_smem();
-            __syncwarp();
-            if (lane == 0) mbar_arrive_state(&bars[sl]);
-            if (yin >= y0 && yin < y1) {  // uptail2's u8 LR copy: each pixel of the CTA's own rows once
-#pragma unroll
-                for (int i = 0; i < 5; i++) {
-                    const int px = lane + 32 * i, xx = x0 - 1 + px;
-                    if (px < kHalo && xx >= x0 && xx < x0 + kTile && rgb[i] != 0xFFFFFFFFu) {
-                        uint8_t *l8 = a.lr8 + ((size_t)slot_job * a.H + yin) * 3 * a.wp + xx;
-                        l8[0] = (uint8_t)rgb[i];
-                        l8[a.wp] = (uint8_t)(rgb[i] >> 8);
-                        l8[2 * a.wp] = (uint8_t)(rgb[i] >> 16);
-                    }
-                }
-            }
-        }
-    }
-    for (int q = 0; q < n_loads && (!BUILD || warp < 4); q++) {
+    for (int q = 0; q < n_loads; q++) {
         const int yin = y0 - 1 + q;
         if (tid == 0) {
             const int sl = q % Cfg::NSLOT;
@@ -424,7 +337,6 @@ __global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128
                 }
             }
             umma_commit(&bars[4]);
-            if constexpr (BUILD) umma_commit(&bars[5 + sl]);  // the builder may refill the slot
         }
         __syncwarp();
         const int r = yin - 1;  // output row completed by this input row
@@ -446,14 +358,9 @@ __global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128
         }
         mbar_wait(&bars[4], q & 1);
         tc_fence_after();
-        if (!BUILD && tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
+        if (tid == 0 && q + Cfg::NSLOT < n_loads) {  // the slot MMA(q) read is free again
             const int sl = q % Cfg::NSLOT, qn = q + Cfg::NSLOT;
-#if NS_ROT_BULK
             row_bulk<G>(s_ring + sl * Cfg::SLOT, kHalo, a.in, slot_job, a.H, a.W, y0 - 1 + qn, x0 - 1, &bars[sl]);
-#else
-            mbar_arrive_expect_tx(&bars[sl], LOAD_BYTES);
-            tma_load_5d(s_ring + sl * Cfg::SLOT, &tm_in, &bars[sl], 0, x0 - 1, 0, y0 - 1 + qn, slot_job);
-#endif
         }
         const uint32_t acc = tl + (uint32_t)(mod3(r) * NB);
         uint32_t v[NB];
@@ -510,8 +417,7 @@ __global__ void __launch_bounds__((EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128
         }
         tmem_wait_st();
         tc_fence_before();
-        if constexpr (BUILD) asm volatile("bar.sync 1, 128;" ::: "memory");  // the 4 MMA/epilogue warps
-        else __syncthreads();
+        __syncthreads();
         tc_fence_after();
     }
     if (warp == 0) tmem_dealloc(tmem, Cfg::TMEM_COLS);
@@ -525,16 +431,7 @@ constexpr int kRbMmaWarps = 4;
 // clock64 timeline) NH 5 / 6 / 7 -> 114.6 / 105.1 / 109.6; with bulk-copied
 // rows (~1,400-1,600 cycles) NH 5 / 6 / 7 -> 106.1 / 98.1 / 95.9.  7 is the
 // most that fits (shared memory).
-#ifndef NS_RB_NH
-#define NS_RB_NH 7
-#endif
-#ifndef NS_RB_QUAL
-#define NS_RB_QUAL __launch_bounds__(kRbThreads, 1)
-#endif
-#ifndef NS_RB_NTS
-#define NS_RB_NTS 2
-#endif
-// NS_RB_BULK: each h row of a tile arrives as C/8 one-dimensional bulk copies
+// Each h row of a tile arrives as C/8 one-dimensional bulk copies
 // (one contiguous 16-B x 130-px run per channel group) instead of one tensor
 // box whose innermost extent is 16 B (8 channels); the out-of-frame columns of
 // a tile are zeroed once, out-of-frame rows by the producer.
@@ -550,7 +447,7 @@ constexpr int kRbThreads = 32 * (1 + kRbMmaWarps + 16);
 constexpr int kRbOut = kTile - 2;
 struct RbArgs {
     int H, W, n_tiles, rows_per_cta, j0;
-    const uint16_t *in;     // h [job][H][C/8][W][8] (NS_RB_BULK: rows by 1-D bulk copies)
+    const uint16_t *in;     // h [job][H][C/8][W][8] (rows by 1-D bulk copies)
     const SrJob *jobs;
     const int32_t *job_count;
     size_t b1_off, bias1_off, b2_off, bias2_off;
@@ -564,8 +461,8 @@ struct RbCfg {
     static constexpr uint32_t W_CONV = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * C * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);  // TMA destination: 128-B aligned
-    static constexpr int NH = NS_RB_NH;                          // h ring per tile
-    static constexpr int NTS = NS_RB_NTS;                        // t slots per tile (<= 4: e1t rotates over 4)
+    static constexpr int NH = 7;                                 // h ring per tile
+    static constexpr int NTS = 2;                                // t slots per tile (<= 4: e1t rotates over 4; 3 measured slower)
     static constexpr uint32_t TILE_BYTES = (NH + NTS) * SLOT;
     static constexpr uint32_t TCOLS = 2 * 3 * NB;                // conv1 + conv2 rings per tile
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
@@ -585,8 +482,8 @@ __device__ __forceinline__ void named_bar_sync(int id, int n) {
 // barrier update of the CTA: with 128 threads arriving and 4 warps polling per
 // group, ncu counted ~23M SYNCS polls per launch, ~18% of all shared-memory
 // wavefronts of a kernel that is shared-memory-bandwidth bound (the MMA operand
-// reads take the rest).  NS_RB_ARRIVE1: one arrive per warp (counts 4), after
-// __syncwarp.  NS_RB_GWAIT: one warp of the group polls, the group follows on a
+// reads take the rest).  Tried: one arrive per warp (counts 4), after
+// __syncwarp; and one warp of the group polls, the group follows on a
 // named barrier (no shared-memory traffic).  A/B on B200 (tools/ab_libs.sh,
 // body ms per c4 step): neither 104.5, ARRIVE1 105.4, GWAIT 108.1, both 110:
 // the polls do not compete with the operand reads enough to matter, and the
@@ -594,32 +491,13 @@ __device__ __forceinline__ void named_bar_sync(int id, int n) {
 // NS_RB_BIAS_INIT: a retired accumulator block is re-initialised with the
 // conv's bias instead of zero, so the epilogues add no bias (E1 becomes one
 // cvt.rn.relu.bf16x2 per channel pair).
-#ifndef NS_RB_BIAS_INIT
-#define NS_RB_BIAS_INIT 1
-#endif
-#ifndef NS_RB_ARRIVE1
-#define NS_RB_ARRIVE1 0
-#endif
-#ifndef NS_RB_GWAIT
-#define NS_RB_GWAIT 0
-#endif
-constexpr uint32_t kRbArriveCount = NS_RB_ARRIVE1 ? 4 : 128;
+constexpr uint32_t kRbArriveCount = 128;
 __device__ __forceinline__ void rb_arrive(uint64_t *bar) {
-#if NS_RB_ARRIVE1
-    __syncwarp();
-    if ((threadIdx.x & 31) == 0) mbar_arrive(bar);
-#else
     mbar_arrive(bar);
-#endif
 }
 __device__ __forceinline__ void rb_group_wait(uint64_t *bar, uint32_t phase, int group) {
-#if NS_RB_GWAIT
-    if (((threadIdx.x >> 5) & 3) == 0) mbar_wait(bar, phase);
-    named_bar_sync(1 + group, 128);
-#else
     (void)group;
     mbar_wait(bar, phase);
-#endif
 }
 
 // Warp roles: warp 0 = TMA producer, warp 1 = MMA issuer, warps 2-17 = four
@@ -635,7 +513,7 @@ __device__ __forceinline__ void rb_group_wait(uint64_t *bar, uint32_t phase, int
 // both tiles' groups while the epilogues run (a drained queue costs the ~300-
 // cycle commit round trip, tools/ubench.cu).
 template <int C>
-__global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
+__global__ void __launch_bounds__(kRbThreads, 1) k_resblock(const __grid_constant__ CUtensorMap tm_in, const RbArgs a) {
     using Cfg = RbCfg<C>;
     constexpr int NB = Cfg::NB, NH = Cfg::NH;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -692,13 +570,11 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
     // h slot column c <-> x = x0k - 2 + c; in-frame columns [c_lo, c_hi)
     auto c_lo = [&](int k) { return max(0, 2 - x0k(k)); };
     auto c_hi = [&](int k) { return min(kHalo, a.W - x0k(k) + 2); };
-#if NS_RB_BULK
     for (int i = tid; i < 2 * NH * (C / 8) * kHalo; i += blockDim.x) {  // out-of-frame columns stay zero
         const int c = i % kHalo, cg = (i / kHalo) % (C / 8), sl = (i / (kHalo * (C / 8))) % NH, k = i / (kHalo * (C / 8) * NH);
         if (c < c_lo(k) || c >= c_hi(k))
             reinterpret_cast<uint4 *>(hslot(k, sl) + cg * kHalo * 16)[c] = make_uint4(0, 0, 0, 0);
     }
-#endif
     fence_proxy_async_smem();
     tc_fence_before();
     __syncthreads();
@@ -736,7 +612,6 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     // slot reuse: h row q-NH was last read by E2 at step q-NH+2, which
                     // arrives on hfree[slot] (one completion per reuse: never runs ahead)
                     if (q >= NH) mbar_wait(hfree(k, sl), ((q / NH) - 1) & 1);
-#if NS_RB_BULK
                     const int yy = y0 - 2 + q, lo = c_lo(k), hi = c_hi(k);
                     if (yy < 0 || yy >= a.H) {  // zero padding row: in-frame columns to zero
                         for (int cg = 0; cg < C / 8; cg++)
@@ -753,10 +628,6 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                             bulk_load(hslot(k, sl) + cg * kHalo * 16 + lo * 16, src + (size_t)cg * a.W * 8, run,
                                       hfull(k, sl));
                     }
-#else
-                    mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
-                    tma_load_5d(hslot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
-#endif
                     NS_TR(30 + k, q);
                 }
             }
@@ -853,7 +724,6 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
                     if (warp % 4 == 2 && lane == 0) NS_TR(40 + k, q);
-#if NS_RB_BIAS_INIT
                     // the retired block becomes row yt+3's: it starts at b1, so the
                     // epilogue adds no bias (the first three rows retire blocks zeroed at
                     // allocation and add it here)
@@ -863,12 +733,6 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     }
                     tmem_st_vals<NB>(acc, bias);
                     tmem_wait_st();
-#else
-#ifndef NS_TRACE_NOZERO
-                    tmem_zeroN<NB>(acc);
-                    tmem_wait_st();
-#endif
-#endif
 
                     tc_fence_before();
                     rb_arrive(e1z(k));  // the next conv1 group may start
@@ -881,21 +745,11 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                         uint8_t *ts = tslot(k, q % Cfg::NTS);
 #pragma unroll
                         for (int cg = 0; cg < NB / 8; cg++) {
-#if NS_RB_BIAS_INIT
                             const uint32_t *w = v + cg * 8;
                             auto pr = [&](int i) {
                                 return inside ? pack_bf16_relu(__uint_as_float(w[i]), __uint_as_float(w[i + 1])) : 0u;
                             };
                             const uint4 o = make_uint4(pr(0), pr(2), pr(4), pr(6));
-#else
-                            float f[8];
-#pragma unroll
-                            for (int i = 0; i < 8; i++)
-                                f[i] = inside ? fmaxf(__uint_as_float(v[cg * 8 + i]) + bias[cg * 8 + i], 0.f) : 0.f;
-                            uint4 o;
-                            o.x = pack_bf16(f[0], f[1]); o.y = pack_bf16(f[2], f[3]);
-                            o.z = pack_bf16(f[4], f[5]); o.w = pack_bf16(f[6], f[7]);
-#endif
                             *reinterpret_cast<uint4 *>(ts + cg * kHalo * 16 + p * 16) = o;
                         }
                     }
@@ -923,17 +777,9 @@ __global__ void NS_RB_QUAL k_resblock(const __grid_constant__ CUtensorMap tm_in,
                     uint32_t v[NB];
                     tmem_ldN<NB>(acc, v);
                     tmem_wait_ld();
-#if NS_RB_BIAS_INIT
                     const bool addb = q < 5;  // first three retirements: blocks zeroed at allocation
                     tmem_st_vals<NB>(acc, bias);
                     tmem_wait_st();
-#else
-                    constexpr bool addb = true;
-#ifndef NS_TRACE_NOZERO
-                    tmem_zeroN<NB>(acc);
-                    tmem_wait_st();
-#endif
-#endif
 
                     tc_fence_before();
                     rb_arrive(e2z(k));  // the next conv2 group may start
@@ -1173,12 +1019,6 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
 // measured equal while the epilogue groups met on a per-step barrier; with the
 // bias-initialised columns (no barrier): 3 / 4 / 5 / 6 / 7 -> 18.3 / 16.2 /
 // 14.8-15.3 / 15.4-15.5 / 15.5-15.6 ms per c4 step.
-#ifndef NS_UP_NS
-#define NS_UP_NS 5
-#endif
-#ifndef NS_UP_MMA2
-#define NS_UP_MMA2 0
-#endif
 template <int CIN, int NB, int S>
 struct Up2Cfg {
     static constexpr int KC = CIN / 16, NSTRIP = 9;
@@ -1187,18 +1027,18 @@ struct Up2Cfg {
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo5 * CIN * 2u;
     static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);     // TMA destination: 128-B aligned
-    static constexpr int NS = NS_UP_NS;                             // input ring per tile
+    static constexpr int NS = 5;                                    // input ring per tile
     static constexpr int NL = 3;                                    // LR ring per tile
     static constexpr uint32_t LR_BYTES = 9u * kLrBoxW;              // [row 3][plane 3][kLrBoxW]
     static constexpr uint32_t LSLOT = round_up(LR_BYTES, 128);
     static constexpr uint32_t OUTG = round_up(3u * kTile * S, 128);  // per group: [plane][128 s] bytes
-    static constexpr int NOUT = NS_UP_OUT2 ? 2 : 1;                  // staging rows per group
+    static constexpr int NOUT = 1;                                  // staging rows per group
     static constexpr uint32_t TILE_BYTES = NS * SLOT + NL * LSLOT + S * NOUT * OUTG;
     static constexpr uint32_t TCOLS = 5 * NB;
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(2 * TCOLS);
     static constexpr int BPT = 2 * NS + 3 + 2 * NL;                // barriers per tile
     static constexpr int NBAR = 2 * BPT + 1;
-    static constexpr int NWARPS = 2 + 2 * S * 4 + NS_UP_MMA2;      // (+ the second tile's MMA issuer, last)
+    static constexpr int NWARPS = 2 + 2 * S * 4;
     static constexpr uint32_t SMEM = W_REGION + 2 * TILE_BYTES + NBAR * 8 + 64;
     static_assert(5 * NB <= 256, "N = 5 nb");
     static_assert(SMEM <= 232448, "shared memory");
@@ -1349,17 +1189,11 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
             for (int i = 0; i < NL; i++) { mbar_init(lfull(k, i), 1); mbar_init(lfree(k, i), S); }
             mbar_init(mdone(k, 0), 1);
             mbar_init(mdone(k, 1), 1);
-            mbar_init(edone(k), NS_UP_BIAS_INIT ? 128 * S : 128);
+            mbar_init(edone(k), 128 * S);
         }
         mbar_init(wbar, 1);
         fence_mbar_init();
     }
-#if NS_UP_BULK
-    for (int k = 0; k < 2; k++)
-        for (int i = 0; i < NS; i++)
-            slot_zero_edges<CIN / 8>(islot(k, i), kHalo5, a.W, x0k(k) - 2, tid, blockDim.x);
-    fence_proxy_async_smem();
-#endif
     if (warp == 0) tmem_alloc(s_tmem, Cfg::TMEM_COLS);
     tc_fence_before();
     __syncthreads();
@@ -1391,13 +1225,8 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     if (!vk(k)) continue;
                     const int sl = q % NS;
                     if (q >= NS) mbar_wait(sfree(k, sl), ((q / NS) - 1) & 1);
-#if NS_UP_BULK
-                    row_bulk<CIN / 8>(islot(k, sl), kHalo5, a.in, slot_job, a.H, a.W, y0 - 2 + q, x0k(k) - 2,
-                                      hfull(k, sl));
-#else
                     mbar_arrive_expect_tx(hfull(k, sl), Cfg::SLOT_BYTES);
                     tma_load_5d(islot(k, sl), &tm_in, hfull(k, sl), 0, x0k(k) - 2, 0, y0 - 2 + q, slot_job);
-#endif
                     const int qv = q - 4;  // output row y0 + qv retires at this step
                     if (qv >= 0) {
                         const int ls = qv % NL;
@@ -1407,11 +1236,11 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     }
                 }
         }
-    } else if (warp == 1 || (NS_UP_MMA2 && warp == Cfg::NWARPS - 1)) {
-        // ---- MMA issuer(s) (whole warp, elected lane issues); with NS_UP_MMA2 one
-        // warp per tile, so one tile's epilogue wait never holds the other tile's MMAs
+    } else if (warp == 1) {
+        // ---- MMA issuer (whole warp, elected lane issues), both tiles; one issuer
+        // per tile measured slower
         const uint32_t idesc = idesc_bf16_f32(128, 5 * NB);
-        const int kfirst = NS_UP_MMA2 ? (warp == 1 ? 0 : 1) : 0, klast = NS_UP_MMA2 ? kfirst : 1;
+        const int kfirst = 0, klast = 1;
         mbar_wait(wbar, 0);
         for (int q = 0; q < nq; q++)
             for (int k = kfirst; k <= klast; k++) {
@@ -1459,7 +1288,6 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                 uint32_t v[UpCols<NB, S>::LW];
                 tmem_ldN<UpCols<NB, S>::LW>(acc + cbase, v);
                 tmem_wait_ld();
-#if NS_UP_BIAS_INIT
                 // each group re-initialises its own 3S output columns of the retired
                 // block with bias + 1/2 (the rounding term): no cross-group barrier
                 // before the block is free, and no bias add below.  The first five
@@ -1470,18 +1298,6 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                 tmem_wait_st();
                 tc_fence_before();
                 mbar_arrive(edone(k));
-#else
-                constexpr bool addb = true;
-                tc_fence_before();
-                named_bar(1 + k, 128 * S);  // every group of this tile has read the block
-                if (g == 0) {
-                    tc_fence_after();
-                    tmem_zeroN<NB>(acc);
-                    tmem_wait_st();
-                    tc_fence_before();
-                    mbar_arrive(edone(k));
-                }
-#endif
                 float be[3 * S];  // bias + 1/2 still to add (zero once the block started at it)
 #pragma unroll
                 for (int i = 0; i < 3 * S; i++) be[i] = addb ? bh[i] : 0.f;
@@ -1489,10 +1305,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                     const int qv = r - y0, ls = qv % NL;
                     mbar_wait(lfull(k, ls), (qv / NL) & 1);
                     const uint8_t *lr = lslot(k, ls);
-                    // NS_UP_OUT2: two staging rows per group, alternating by step, so
-                    // the row written at step q is never the one being copied out from
-                    // step q-1 (the barrier of step q orders it) -- no second barrier
-                    uint8_t *const so = so0 + (Cfg::NOUT == 2 ? (q & 1) * Cfg::OUTG : 0);
+                    uint8_t *const so = so0;
                     if (x < lw) {
                         if (g == 0) uptail_group_step<NB, S, 0>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
                         else if (S > 1 && g == 1) uptail_group_step<NB, S, (S > 1 ? 1 : 0)>(v, be, s_bias, lr, r, x, x0k(k), lh, lw, a, so, p, slot_job);
@@ -1509,7 +1322,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                             *reinterpret_cast<uint2 *>(dst + (size_t)c * HH * WW + ch * 8) =
                                 *reinterpret_cast<const uint2 *>(so + c * (kTile * S) + ch * 8);
                     }
-                    if constexpr (Cfg::NOUT == 1) named_bar(3 + grp, 128);  // staging can be overwritten
+                    named_bar(3 + grp, 128);  // staging can be overwritten
                 }
             }
         }
@@ -1786,10 +1599,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
 }
 
 // (A/B: 64 -> 120 rows 198.8 -> 197.5 ms per c4 step; 120 -> 180 191.9 -> 190.2; 360 no better)
-#ifndef NS_ROT_ROWS
-#define NS_ROT_ROWS 180
-#endif
-constexpr int kRotRows = NS_ROT_ROWS;  // rows per CTA strip of the rotated conv and uptail2
+constexpr int kRotRows = 180;  // rows per CTA strip of the rotated conv and uptail2
 template <int CIN, int NB, int EPI>
 static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = RotCfg<CIN, NB>;
@@ -1798,7 +1608,7 @@ static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int n
     args.rows_per_cta = kRotRows;
     dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
     KScope ks(fam, st);
-    constexpr int threads = (EPI == EPI_HEAD && NS_HEAD_BUILD) ? 160 : 128;
+    constexpr int threads = 128;
     k_conv_rot<CIN, NB, EPI><<<grid, threads, Cfg::SMEM, st>>>(tm, args);
     return cudaGetLastError();
 }
@@ -1821,10 +1631,7 @@ static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStre
 // 360 191.9 -> 190.8 (within noise); 720 no better.  240 rows = 3 strips =
 // 288 CTAs per 16-job launch, 1.95 waves of 148 SMs, so a launch that runs
 // alone (no overlap) wastes little as well: 240.
-#ifndef NS_RB_ROWS
-#define NS_RB_ROWS 240
-#endif
-constexpr int kRbRows = NS_RB_ROWS;  // rows per CTA strip of the fused res-block
+constexpr int kRbRows = 240;  // rows per CTA strip of the fused res-block
 template <int C>
 static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, cudaStream_t st) {
     using Cfg = RbCfg<C>;
@@ -1855,21 +1662,18 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
                            const int32_t *job_count, cudaStream_t st) {
     const int h = a->h, w = a->w, s = a->s;
     cudaError_t e;
-#if !NS_HEAD_BUILD
     {
         dim3 g((h * w + 255) / 256, nj);
         KScope ks(F_SR_PREP, st);
         k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
-#endif
     ConvArgs base{};
     base.H = h; base.W = w; base.j0 = j0; base.jobs = jobs; base.job_count = job_count; base.C = C; base.s = s;
     auto L = [&](int l) { return model_layer(n_blocks, C, s, l); };
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
         g.b_off = ls.b_off; g.bias_off = ls.bias_off; g.out = a->h0; g.in = a->x0;
-        g.lr8 = a->lr8; g.wp = a->wp;  // NS_HEAD_BUILD: the head writes uptail2's u8 LR copy
         if ((e = conv_rot<16, C, EPI_HEAD>(F_SR_HEAD, a->tm_x0, g, nj, st)) != cudaSuccess) return e;
     }
     // residual blocks, fused (conv1 + ReLU + conv2 + skip), ping-pong hb / tb

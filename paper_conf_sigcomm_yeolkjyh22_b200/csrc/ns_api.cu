@@ -727,10 +727,7 @@ static ns_status run_sr_group(ns_ctx *c, int h, int w, int C, int s, int B, cons
     ns_status r = get_arena(c, h, w, C, s, 0, &a[0]);
     if (r != NS_OK) return r;
     const int nbatch = (max_jobs + a[0]->nb - 1) / a[0]->nb;
-#ifndef NS_SR_TWO_STREAMS
-#define NS_SR_TWO_STREAMS 1
-#endif
-    if (NS_SR_TWO_STREAMS && nbatch > 1 && (r = get_arena(c, h, w, C, s, 1, &a[1])) != NS_OK) return r;
+    if (nbatch > 1 && (r = get_arena(c, h, w, C, s, 1, &a[1])) != NS_OK) return r;
     const bool two = a[1] != nullptr;
     if (two) {
         NS_CUDA(cudaEventRecord(c->ev_fork, st));
