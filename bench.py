@@ -233,6 +233,9 @@ def main():
                     help="global: §5.2 selection across all GPUs' streams (per-GPU gains, NCCL all_gather, "
                          "ns_select_merge, NS_GIVEN_ANCHORS) inside the timed step")
     ap.add_argument("--ring", type=int, default=3, help="config 5: HR frames per stream (ring)")
+    ap.add_argument("--encode", action="store_true",
+                    help="after timing: hybrid-encode one step's SR anchors (ns_encode_anchors, §6.1) and report "
+                         "anchors/s and bytes per anchor")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -431,6 +434,20 @@ def main():
                        "selection; non-anchor LR is read only for intra blocks, in place); D2H of the per-stream "
                        "stats and anchor map; HR frames stay in HBM for the downstream encoder"}
 
+    hybrid = None
+    if args.encode:  # §6.1 hybrid encoding of the last step's anchors (off the timed hot path)
+        ia_host = ia.cpu().numpy()
+        ctx.encode_anchors(chunks[:1], ia_host[:1], hr_out[:1])          # encoder setup, warm-up
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        pk = ctx.encode_anchors(chunks, ia_host, hr_out)
+        t_enc = time.perf_counter() - t0
+        na = int(ia_host.sum())
+        hybrid = {"anchors": na, "seconds": t_enc, "anchors_per_s": na / t_enc,
+                  "mean_anchor_bytes": (sum(len(p) for p in pk) - 16 * S * n) / max(na, 1),
+                  "quality": ns.hybrid_quality(k, n), "codec": "JPEG 4:4:4 (nvJPEG), Table 2 quality",
+                  "package_bytes": sum(len(p) for p in pk)}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r = cpu_sample(cfg, pool[0], synth.make_weights(4000, B, C, s))
@@ -449,6 +466,7 @@ def main():
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
                              "anchors_per_step": int(ia_np.sum())},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+                "hybrid_encode": hybrid,
                 # real-time check: one n-frame chunk of every stream (n/60 s of
                 # 60 fps video) must finish within its own duration
                 "realtime": {"chunk_ms": ms / args.steps, "chunk_video_ms": 1000.0 * n / 60.0,

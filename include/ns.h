@@ -56,8 +56,17 @@ typedef enum {
     NS_EUNSUPPORTED = -4   /* device is not sm_100 / shape not supported        */
 } ns_status;
 
-/* Frame types exported by the decoder (G_key, G_altref, G_normal). */
-typedef enum { NS_KEY = 0, NS_ALTREF = 1, NS_NORMAL = 2 } ns_frame_type;
+/* Frame types exported by the decoder (G_key, G_altref, G_normal).
+   Codec neutrality (§9): "to support the H.26x codecs, we only need to
+   replace the VPx-/AV1-specific frame groups (G_key, G_altref, G_normal) with
+   the H.26x-specific groups (G_I, G_P, G_B)" -- the same three tiers, so an
+   H.26x decoder exports I as the key tier (reset points, selected first), P
+   as the high-reference tier and B as the normal tier (reading R8, DESIGN.md
+   §3; GOLDEN is then the latest I/P frame in decode order). */
+typedef enum {
+    NS_KEY = 0, NS_ALTREF = 1, NS_NORMAL = 2,
+    NS_I = NS_KEY, NS_P = NS_ALTREF, NS_B = NS_NORMAL
+} ns_frame_type;
 
 /* Reference index of a block ("reference index"). */
 typedef enum { NS_REF_LAST = 0, NS_REF_GOLDEN = 1, NS_REF_INTRA = 2 } ns_ref;
@@ -249,6 +258,48 @@ NS_API ns_status ns_enhance_streams(ns_ctx *ctx, const ns_chunk *chunks, int S, 
 NS_API ns_status ns_enhance_streams_host(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
                                          uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats,
                                          uint64_t *h2d_bytes, void *stream);
+
+/* ------------------------------------------------------------------ hybrid encoding
+   Hybrid encoding of the super-resolved anchors (§6.1 "Hybrid video encoding",
+   P:233-239).  The ingest video is reused as it is (its
+   bitstream is outside this library: decoding and re-encoding video are out
+   of scope); only the SR anchor frames are compressed, with an image codec --
+   baseline JPEG through nvJPEG, 4:4:4 (the HR frames carry three
+   full-resolution planes, reading Z18) -- and every frame of every chunk gets
+   a header: "A new header attached to each frame contains the frame type
+   (i.e., anchor or non-anchor frame) and the super-resolved frame for an
+   anchor frame".  Package of one stream = n_frames x
+   (ns_hybrid_header, then `bytes` of JPEG for an anchor, nothing otherwise). */
+#define NS_HYBRID_MAGIC 0x4648534Eu   /* "NSHF" little-endian */
+typedef struct {
+    uint32_t magic;    /* NS_HYBRID_MAGIC                                       */
+    uint32_t stream;   /* stream index within the call                          */
+    uint16_t frame;    /* frame index within the chunk                          */
+    uint8_t anchor;    /* 1: the JPEG of the super-resolved frame follows        */
+    uint8_t quality;   /* JPEG quality it was coded at (0 for a non-anchor)     */
+    uint32_t bytes;    /* payload bytes after this header                       */
+} ns_hybrid_header;   /* 16 bytes */
+
+/* Table 2, JPEG column: the quality for a chunk with n_anchors of
+   n_frames frames as anchors -- fraction <= 5%: 95; <= 7.5%: 90; <= 10%: 80;
+   above 10% JPEG "cannot meet the bitrate constraint": -1.  Also -1
+   for invalid counts.  Host only. */
+NS_API int ns_hybrid_quality(int n_anchors, int n_frames);
+
+/* Encodes the anchors of S chunks after ns_enhance_streams and packages them.
+   is_anchor: HOST [S][n] (e.g. a copy of is_anchor_out); hr_out: HOST table
+   [S*n] of DEVICE pointers as passed to ns_enhance_streams (only the anchors'
+   entries are read, so they must still hold their frames: with HR rings, call
+   this before a later frame reuses an anchor's entry).  quality: 1..100, or
+   0 = Table 2 per stream (NS_EUNSUPPORTED if a stream's anchor fraction is
+   above 10%).  out: HOST buffer of out_cap bytes; the S packages are written
+   back to back and out_len (HOST [S]) receives each one's size; NS_ENOMEM if
+   out_cap is too small (out_len then holds what was needed so far).  Not on
+   the GPU hot path: the encoder is created on first use and the call returns
+   once every bitstream is in `out` (it synchronises `stream`). */
+NS_API ns_status ns_encode_anchors(ns_ctx *ctx, const ns_chunk *chunks, int S, const uint8_t *is_anchor,
+                                   uint8_t *const *hr_out, int quality, uint8_t *out, size_t out_cap,
+                                   size_t *out_len, void *stream);
 
 /* Number of this library's kernel launches enqueued by the calling thread
    since the last reset (for the bench's gpu_launches claim). */

@@ -21,6 +21,7 @@ LIB_PATH = os.environ.get("NS_LIB") or os.path.join(_HERE, "libneuroscaler.so")
 
 NS_OK, NS_EINVAL, NS_ECUDA, NS_ENOMEM, NS_EUNSUPPORTED = 0, -1, -2, -3, -4
 NS_KEY, NS_ALTREF, NS_NORMAL = 0, 1, 2
+NS_I, NS_P, NS_B = NS_KEY, NS_ALTREF, NS_NORMAL      # H.26x groups G_I, G_P, G_B
 NS_REF_LAST, NS_REF_GOLDEN, NS_REF_INTRA = 0, 1, 2
 NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET, NS_GIVEN_ANCHORS = 0, 1, 2
 NS_CARRY, NS_FRESH = 0, 1
@@ -52,7 +53,16 @@ class NsSrJob(ctypes.Structure):
 
 EXPORTS = ["ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_blob_len",
            "ns_model_destroy", "ns_select_anchors", "ns_select_merge", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
-           "ns_enhance_streams_host", "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read"]
+           "ns_enhance_streams_host", "ns_launch_count", "ns_last_error", "ns_profile_enable", "ns_profile_read",
+           "ns_hybrid_quality", "ns_encode_anchors"]
+
+NS_HYBRID_MAGIC = 0x4648534E
+
+
+class NsHybridHeader(ctypes.Structure):
+    """ns_hybrid_header (include/ns.h): per-frame header of the hybrid package."""
+    _fields_ = [("magic", ctypes.c_uint32), ("stream", ctypes.c_uint32), ("frame", ctypes.c_uint16),
+                ("anchor", ctypes.c_uint8), ("quality", ctypes.c_uint8), ("bytes", ctypes.c_uint32)]
 
 _lib = None
 
@@ -92,9 +102,12 @@ def lib() -> ctypes.CDLL:
         L.ns_profile_enable.restype = i32
         L.ns_profile_read.argtypes = [P, i32]
         L.ns_profile_read.restype = i32
+        L.ns_hybrid_quality.argtypes = [i32, i32]
+        L.ns_hybrid_quality.restype = i32
+        L.ns_encode_anchors.argtypes = [P, P, i32, P, P, i32, P, ctypes.c_size_t, P, P]
         for f in ("ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_destroy",
                   "ns_select_anchors", "ns_select_merge", "ns_sr_anchors", "ns_reconstruct_chunk", "ns_enhance_streams",
-                  "ns_enhance_streams_host"):
+                  "ns_enhance_streams_host", "ns_encode_anchors"):
             getattr(L, f).restype = i32
         _lib = L
     return _lib
@@ -103,6 +116,23 @@ def lib() -> ctypes.CDLL:
 def _check(rc: int, where: str):
     if rc != NS_OK:
         raise NsError(rc, where, lib().ns_last_error().decode())
+
+
+def hybrid_quality(n_anchors: int, n_frames: int) -> int:
+    """Table 2's JPEG quality for a chunk's anchor fraction (-1: above 10%)."""
+    return int(lib().ns_hybrid_quality(n_anchors, n_frames))
+
+
+def parse_hybrid(pkg: bytes):
+    """Splits one stream's hybrid package into [(header, payload bytes)]."""
+    out, pos, hs = [], 0, ctypes.sizeof(NsHybridHeader)
+    while pos < len(pkg):
+        h = NsHybridHeader.from_buffer_copy(pkg[pos:pos + hs])
+        if h.magic != NS_HYBRID_MAGIC:
+            raise ValueError(f"bad hybrid header magic at byte {pos}")
+        out.append((h, pkg[pos + hs:pos + hs + h.bytes]))
+        pos += hs + h.bytes
+    return out
 
 
 def last_error() -> str:
@@ -311,6 +341,27 @@ class Context:
                "ns_enhance_streams_host")
         del keep
         return int(moved.value)
+
+    def encode_anchors(self, chunks, is_anchor, hr_out, quality=0, out_cap=None, stream=None):
+        """ns_encode_anchors (§6.1 hybrid encoding): JPEG of every anchor +
+        per-frame headers.  is_anchor: [S, n] array-like (host copy is made);
+        hr_out as for enhance_streams.  Returns a list of S `bytes` packages."""
+        arr = self._chunks(chunks)
+        tab = self._hr_table(hr_out)
+        ia = np.ascontiguousarray(np.asarray(is_anchor, dtype=np.uint8))
+        S = len(chunks)
+        if out_cap is None:
+            px = sum(c.n * 3 * (c.scale * c.h) * (c.scale * c.w) for c in chunks)
+            out_cap = px // 2 + 64 * S * chunks[0].n + (1 << 20)
+        buf = (ctypes.c_uint8 * out_cap)()
+        lens = (ctypes.c_size_t * S)()
+        _check(lib().ns_encode_anchors(self.handle, arr, S, ia.ctypes.data, tab, int(quality), buf, out_cap, lens,
+                                       _stream(stream)), "ns_encode_anchors")
+        raw, out, pos = bytes(buf), [], 0
+        for s in range(S):
+            out.append(raw[pos:pos + lens[s]])
+            pos += lens[s]
+        return out
 
     @staticmethod
     def host_pool_bytes(w: int, h: int, n: int, k: int, streams: int) -> int:

@@ -12,7 +12,7 @@ CSRC = os.path.join(HERE, "csrc")
 ROOT = os.path.dirname(HERE)
 LIB = os.path.join(HERE, "libneuroscaler.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["ns_api.cu", "k_select.cu", "k_recon.cu", "k_sr.cu"]
+SOURCES = ["ns_api.cu", "k_select.cu", "k_recon.cu", "k_sr.cu", "ns_hybrid.cu"]
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
          "-I", os.path.join(ROOT, "include"), "-Xptxas", "-v"]
@@ -39,7 +39,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         objs = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
     tmp = LIB + ".tmp"
     subprocess.check_call([NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs,
-                           "-lcuda" if False else "-lcudart_static", "-Xcompiler", "-fPIC"])
+                           "-lcudart_static", "-lnvjpeg", "-Xcompiler", "-fPIC"])
     os.replace(tmp, LIB)
     return LIB
 

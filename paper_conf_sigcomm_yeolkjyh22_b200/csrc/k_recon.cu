@@ -131,20 +131,9 @@ __device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) 
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(c));
     return r;
 }
-// (experiment knob NS_RECON_L2PF: L2 prefetch size hint of the window loads)
-#ifndef NS_RECON_L2PF
-#define NS_RECON_L2PF 0
-#endif
+// (an L2 prefetch-size hint, .L2::128B / 256B, on these copies measured neutral)
 __device__ __forceinline__ void cp_async8(void *dst, const void *src) {
-#if NS_RECON_L2PF == 64
-    asm volatile("cp.async.ca.shared.global.L2::64B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-#elif NS_RECON_L2PF == 128
-    asm volatile("cp.async.ca.shared.global.L2::128B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-#elif NS_RECON_L2PF == 256
-    asm volatile("cp.async.ca.shared.global.L2::256B [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-#else
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-#endif
 }
 __device__ __forceinline__ void cp_async16(void *dst, const void *src) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
@@ -311,35 +300,17 @@ __device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[
     }
 }
 
-// NS_RECON_STORE_EF: the output rows (1.56 GB per 64-frame launch, read back
-// only by the next frame step, long after they would have left L2) are stored
-// with an L2 evict-first policy, so they do not push out the reference-window
-// and residual halo lines neighbouring CTAs still read.  Measured neutral to
-// slightly slower (recon 65.0-65.5 vs 64.5-65.0 ms): off.
-#ifndef NS_RECON_STORE_EF
-#define NS_RECON_STORE_EF 0
-#endif
-__device__ __forceinline__ uint64_t l2_evict_first_policy() {
-    uint64_t pol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-    return pol;
-}
+// Output rows: each thread stores its BW bytes per row as 8-B stores.  (Staging
+// the warp's row in shared memory and storing whole 16-B chunks -- the pattern
+// a store-only probe ran 2.2x faster, tools/mem_probe.cu -- measured slower in
+// this kernel: +11% instructions for stores that were not its bottleneck.)
 template <int S>
-__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4], bool on,
-                                                uint64_t pol) {
+__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4], bool on) {
 #pragma unroll
-    for (int q = 0; q < ReconCfg<S>::BW / 8; q++) {
-#if NS_RECON_STORE_EF
-        asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p st.global.L2::cache_hint.v2.b32 [%0], {%1, %2}, %4; }"
-                     ::"l"(dst + 8 * q), "r"(o[2 * q]), "r"(o[2 * q + 1]), "r"((uint32_t)on), "l"(pol)
-                     : "memory");
-#else
-        (void)pol;
+    for (int q = 0; q < ReconCfg<S>::BW / 8; q++)
         asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p st.global.v2.b32 [%0], {%1, %2}; }" ::"l"(dst + 8 * q),
                      "r"(o[2 * q]), "r"(o[2 * q + 1]), "r"((uint32_t)on)
                      : "memory");
-#endif
-    }
 }
 
 __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
@@ -515,7 +486,6 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     const int m = xs & 7;
     const bool fix = valid && !interior && !use_lr;
     uint8_t *outp = fd.out + (size_t)Y0 * W + X0;
-    const uint64_t pol = l2_evict_first_policy();
 
 #pragma unroll 1
     for (int c = 0; c < 3; c++) {
@@ -567,7 +537,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                 }
 #pragma unroll
                 for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6240u);
-                recon_store_row<S>(outc + (size_t)j * W, o, valid, pol);
+                recon_store_row<S>(outc + (size_t)j * W, o, valid);
             };
             static_for<S>(one);
             if constexpr (S & 1) {  // the period ended on an even row: its warp row is in hB
@@ -578,15 +548,20 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     }
 }
 
+// Carveout: just enough shared memory for MINB resident CTAs, the rest of the
+// 256-KB array stays L1 (the window words of neighbouring threads overlap and
+// hit there): the maximum-shared carveout (28 KB of L1) vs this (60 KB) measured
+// 70.2 vs 62.8 ms of reconstruction per c4 step (tools/ab_libs.sh, one box).
+template <int S>
+constexpr int recon_carveout_pct() {
+    return (int)((ReconCfg<S>::MINB * (ReconSmem<S>::BYTES + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
+}
+
 template <int S>
 static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
-    // all of the unified L1/shared array as shared memory, so MINB CTAs fit
-#ifdef NS_RECON_CARVE  // (experiment knob: shared-memory carveout percentage instead of the maximum)
-    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, false); e != cudaSuccess) return e;
-    cudaFuncSetAttribute(k_recon_step<S>, cudaFuncAttributePreferredSharedMemoryCarveout, NS_RECON_CARVE);
-#else
-    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, true); e != cudaSuccess) return e;
-#endif
+    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, recon_carveout_pct<S>());
+        e != cudaSuccess)
+        return e;
     k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f, s0);
     return cudaGetLastError();
 }

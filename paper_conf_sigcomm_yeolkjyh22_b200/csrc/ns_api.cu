@@ -219,6 +219,7 @@ struct ns_ctx {
     // "caches it in memory"); carved from the pool on first use, grown on demand
     uint8_t *acache = nullptr;
     size_t acache_cap = 0;
+    HybridEncoder *hybrid = nullptr;     // nvJPEG encoder (ns_encode_anchors), created on first use
 };
 
 static uint8_t *pool_take(ns_ctx *c, size_t bytes) {
@@ -333,6 +334,7 @@ extern "C" ns_status ns_ctx_destroy(ns_ctx *c) {
         if (c->ev_copied[i]) cudaEventDestroy(c->ev_copied[i]);
         if (c->ev_free[i]) cudaEventDestroy(c->ev_free[i]);
     }
+    hybrid_destroy(c->hybrid);
     if (c->cst) cudaStreamDestroy(c->cst);
     if (c->sst) cudaStreamDestroy(c->sst);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -1144,5 +1146,67 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
         c->hin_used[b] = true;
     }
     if (h2d_bytes) *h2d_bytes = moved;
+    return NS_OK;
+}
+
+// ------------------------------------------------------------------ hybrid encoding (§6.1, NEXT-3)
+extern "C" int ns_hybrid_quality(int n_anchors, int n_frames) { return hybrid_quality_table2(n_anchors, n_frames); }
+
+extern "C" ns_status ns_encode_anchors(ns_ctx *c, const ns_chunk *ch, int S, const uint8_t *is_anchor,
+                                       uint8_t *const *hr_out, int quality, uint8_t *out, size_t out_cap,
+                                       size_t *out_len, void *stream) {
+    if (!c) return fail(NS_EINVAL, "ns_encode_anchors: ctx is NULL");
+    int n = 0;
+    ns_status r = check_chunks(ch, S, false, &n);
+    if (r != NS_OK) return r;
+    if (!is_anchor || !hr_out || !out_len || (!out && out_cap)) return fail(NS_EINVAL, "ns_encode_anchors: NULL argument");
+    if (quality < 0 || quality > 100) return fail(NS_EINVAL, "ns_encode_anchors: quality %d not in [0, 100]", quality);
+    std::vector<int> q(S);
+    for (int s = 0; s < S; s++) {
+        int a = 0;
+        for (int f = 0; f < n; f++) {
+            a += is_anchor[(size_t)s * n + f] != 0;
+            if (is_anchor[(size_t)s * n + f] && !hr_out[(size_t)s * n + f])
+                return fail(NS_EINVAL, "ns_encode_anchors: hr_out[%d][%d] is NULL", s, f);
+        }
+        q[s] = quality ? quality : hybrid_quality_table2(a, n);
+        if (q[s] < 1)
+            return fail(NS_EUNSUPPORTED, "stream %d: anchor fraction %d/%d above 10%%: JPEG cannot meet the bitrate "
+                                         "constraint (Table 2, P:679); pass an explicit quality", s, a, n);
+    }
+    NS_CUDA(cudaSetDevice(c->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    char err[256];
+    if (!c->hybrid && hybrid_create(c->device, st, &c->hybrid, err, sizeof(err)) != 0) return fail(NS_ECUDA, "%s", err);
+    size_t pos = 0;
+    bool full = false;
+    for (int s = 0; s < S; s++) {
+        const size_t start = pos;
+        const int H = ch[s].h * ch[s].scale, W = ch[s].w * ch[s].scale;
+        for (int f = 0; f < n; f++) {
+            ns_hybrid_header hd{};
+            hd.magic = NS_HYBRID_MAGIC;
+            hd.stream = (uint32_t)s;
+            hd.frame = (uint16_t)f;
+            hd.anchor = is_anchor[(size_t)s * n + f] ? 1 : 0;
+            hd.quality = hd.anchor ? (uint8_t)q[s] : 0;
+            size_t len = 0;
+            const size_t hpos = pos;
+            pos += sizeof(hd);
+            if (hd.anchor) {
+                const size_t cap = (!full && pos <= out_cap) ? out_cap - pos : 0;
+                const int rc = hybrid_encode_frame(c->hybrid, hr_out[(size_t)s * n + f], H, W, q[s], out + pos,
+                                                   cap, &len, st, err, sizeof(err));
+                if (rc < 0) return fail(NS_ECUDA, "%s", err);
+                if (rc > 0) full = true;
+            }
+            hd.bytes = (uint32_t)len;
+            if (!full && hpos + sizeof(hd) <= out_cap) memcpy(out + hpos, &hd, sizeof(hd));
+            else full = true;
+            pos += len;
+        }
+        out_len[s] = pos - start;
+    }
+    if (full || pos > out_cap) return fail(NS_ENOMEM, "ns_encode_anchors: out_cap %zu < %zu bytes", out_cap, pos);
     return NS_OK;
 }

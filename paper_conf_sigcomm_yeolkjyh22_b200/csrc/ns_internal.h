@@ -168,13 +168,14 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);
 cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
                          const int32_t *job_count, cudaStream_t st);
 
-// Sets a kernel's dynamic shared memory limit (and, optionally, the all-shared
-// L1 carveout) once per DEVICE: function attributes belong to the context of
-// the device current at the call, and a process may drive several devices
-// (ns.h: one context per device).  One flag word per kernel instantiation
-// (template on the kernel pointer), bit d = device d done; thread-safe.
+// Sets a kernel's dynamic shared memory limit (and, optionally, the preferred
+// shared-memory carveout in percent of the unified L1/shared array) once per
+// DEVICE: function attributes belong to the context of the device current at
+// the call, and a process may drive several devices (ns.h: one context per
+// device).  One flag word per kernel instantiation (template on the kernel
+// pointer), bit d = device d done; thread-safe.
 template <auto K>
-cudaError_t ensure_kernel_smem(int bytes, bool max_carveout = false) {
+cudaError_t ensure_kernel_smem(int bytes, int carveout_pct = -1) {
     static std::atomic<unsigned long long> done{0};
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -182,11 +183,19 @@ cudaError_t ensure_kernel_smem(int bytes, bool max_carveout = false) {
     const unsigned long long bit = 1ull << (dev & 63);
     if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
     e = cudaFuncSetAttribute(K, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
-    if (e == cudaSuccess && max_carveout)
-        e = cudaFuncSetAttribute(K, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
+    if (e == cudaSuccess && carveout_pct >= 0)
+        e = cudaFuncSetAttribute(K, cudaFuncAttributePreferredSharedMemoryCarveout, carveout_pct);
     if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_release);
     return e;
 }
+
+// Hybrid encoding (ns_hybrid.cu, nvJPEG)
+int hybrid_quality_table2(int n_anchors, int n_frames);
+struct HybridEncoder;
+int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *err, size_t errlen);
+void hybrid_destroy(HybridEncoder *e);
+int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int quality, uint8_t *dst, size_t cap,
+                        size_t *len, cudaStream_t stream, char *err, size_t errlen);
 
 // Kernel families for ns_launch_count / ns_profile_read.
 enum Fam { F_SCORE = 0, F_SELECT, F_GLOBAL, F_COMPACT, F_SR_PREP, F_SR_HEAD, F_SR_BODY, F_SR_END, F_SR_UP,

@@ -68,3 +68,29 @@ def test_invalid_args_no_launch(nslib):
     assert L.ns_model_destroy(None) == nslib.NS_EINVAL
     del h
     assert nslib.launch_count() == before
+
+
+def test_hybrid_quality_is_table2(nslib):
+    """ns_hybrid_quality = Table 2's JPEG column (tests/golden/table2_jpeg_quality.json,
+    PAPER.md:668-677): the band edges are inclusive upper bounds."""
+    import json
+    g = json.load(open(os.path.join(ROOT, "tests", "golden", "table2_jpeg_quality.json")))
+    by = {r["fraction"]: r["jpeg"] for r in g["rows"]}
+
+    def band(a, n):  # the paper's bands, evaluated exactly in rationals
+        from fractions import Fraction as Fr
+        f = Fr(a, n)
+        if f <= Fr(5, 100):
+            return by["f <= 5%"]
+        if f <= Fr(75, 1000):
+            return by["5% < f <= 7.5%"]
+        if f <= Fr(10, 100):
+            return by["7.5% < f <= 10%"]
+        return None
+    for n in (1, 8, 20, 40, 60, 120, 256):
+        for a in range(0, n + 1):
+            exp = band(a, n)
+            assert nslib.hybrid_quality(a, n) == (-1 if exp is None else exp), (a, n)
+    assert nslib.hybrid_quality(5, 60) == 80          # the configs' k = 5 of 60 (8.3%)
+    assert nslib.hybrid_quality(3, 60) == 95 and nslib.hybrid_quality(4, 60) == 90
+    assert nslib.hybrid_quality(-1, 60) == -1 and nslib.hybrid_quality(1, 0) == -1

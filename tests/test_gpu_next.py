@@ -306,3 +306,26 @@ def test_balanced_path_single_gpu_equals_given(ctx):
                     [d.hr_last.cpu().numpy() for d in dcs] + [d.hr_golden.cpu().numpy() for d in dcs])
     for a, b in zip(*outs):
         assert np.array_equal(a, b)
+
+
+def test_select_h26x_groups(ctx):
+    """Codec neutrality (§9): H.26x chunks carry G_I / G_P / G_B frame
+    groups in place of G_key / G_altref / G_normal -- an IBBPBBP... decode-order
+    GOP with a second I frame; the selection equals the oracle's over the same
+    three tiers, I frames first, then P by gain, then B by gain."""
+    n = 30
+    t = np.full(n, ns.NS_B, np.uint8)
+    t[0::3] = ns.NS_P
+    t[0] = t[15] = ns.NS_I
+    dcs, cs = [], []
+    for s in range(4):
+        c = synth.make_chunk(9700 + s, 32, 16, 2, n, types=t)
+        cs.append(c)
+        dcs.append(dev_chunk(ns, c, DEV))
+    for k in (1, 2, 5, 12, 30):
+        g, r, a = (x.cpu().numpy() for x in _select_gpu(ctx, dcs, k=k))
+        for s, c in enumerate(cs):
+            eg, er, ea = oracle.select_topk(list(c.type), [int(v) for v in oracle.score(c.res)], k)
+            assert list(g[s]) == eg and list(r[s]) == er and list(a[s]) == ea, (k, s)
+            if k >= 2:
+                assert a[s][0] and a[s][15]          # both I frames before any P or B
