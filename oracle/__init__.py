@@ -50,6 +50,8 @@ def lib():
         L.or_warp_plane.argtypes = [P, i, i, i, P, i, P]
         L.or_reconstruct.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P]
         L.or_reconstruct.restype = i
+        L.or_reconstruct_i420.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P]
+        L.or_reconstruct_i420.restype = i
         L.or_conv3x3.argtypes = [P, i, i, i, P, P, i, P]
         L.or_pixel_shuffle.argtypes = [P, i, i, i, i, P]
         L.or_blob_len.argtypes = [i, i, i]
@@ -115,6 +117,42 @@ def reconstruct(chunk, is_anchor, hr_anchor, hr_last=None, hr_golden=None, s=Non
     if rc != 0:
         raise RuntimeError(f"or_reconstruct failed: {rc}")
     return hr, last, gold
+
+
+def reconstruct_i420(chunk, is_anchor, hr_anchor, hr_last=None, hr_golden=None, s=None):
+    """O8 on a YUV 4:2:0 chunk (NEXT-2, reading R9).  hr_anchor: u8 [n][s*h*s*w*3/2]
+    holding the anchors' SR frames.  Returns (hr, hr_last, hr_golden)."""
+    s = chunk.scale if s is None else s
+    n, h, w = chunk.n, chunk.h, chunk.w
+    hr = np.array(hr_anchor, np.uint8, copy=True, order="C")
+    assert hr.shape == (n, s * h * s * w * 3 // 2)
+    ia = np.ascontiguousarray(is_anchor, np.uint8)
+    last = None if hr_last is None else np.array(hr_last, np.uint8, copy=True, order="C")
+    gold = None if hr_golden is None else np.array(hr_golden, np.uint8, copy=True, order="C")
+    rc = lib().or_reconstruct_i420(w, h, s, n, _p(np.ascontiguousarray(chunk.lr)),
+                                   _p(np.ascontiguousarray(chunk.res)), _p(np.ascontiguousarray(chunk.mv)),
+                                   _p(np.ascontiguousarray(chunk.type)), _p(ia), _p(hr), _p(last), _p(gold))
+    if rc != 0:
+        raise RuntimeError(f"or_reconstruct_i420 failed: {rc}")
+    return hr, last, gold
+
+
+def i420_planes(flat: np.ndarray, h: int, w: int):
+    """Flat 4:2:0 frame -> (Y [h][w], U [h/2][w/2], V [h/2][w/2]) views."""
+    P = h * w
+    return flat[:P].reshape(h, w), flat[P:P + P // 4].reshape(h // 2, w // 2), flat[P + P // 4:].reshape(h // 2, w // 2)
+
+
+def sr_forward_i420(lr_flat: np.ndarray, blob, B: int, C: int, s: int, h: int, w: int) -> np.ndarray:
+    """SR of a 4:2:0 anchor (reading R10): the 4:4:4 net (O5) on (Y, up_2(U),
+    up_2(V)) -- chroma brought to luma resolution with the O6 upsample -- then
+    the HR chroma planes back to 4:2:0 by the rounded 2x2 average
+    floor((a + b + c + d + 2) / 4).  Returns the flat HR 4:2:0 frame."""
+    y, u, v = i420_planes(np.asarray(lr_flat), h, w)
+    full = np.stack([y, upsample(u, 2), upsample(v, 2)]).astype(np.uint8)
+    hr = sr_forward(full, blob, B, C, s).astype(np.int64)
+    cs = (hr[1:, 0::2, 0::2] + hr[1:, 1::2, 0::2] + hr[1:, 0::2, 1::2] + hr[1:, 1::2, 1::2] + 2) >> 2
+    return np.concatenate([hr[0].ravel(), cs.reshape(-1)]).astype(np.uint8)
 
 
 def conv3x3(x: np.ndarray, wt: np.ndarray, bias: np.ndarray | None) -> np.ndarray:

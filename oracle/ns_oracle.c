@@ -20,6 +20,7 @@
  *   or_upsample         O6: fixed-point bilinear x s upsample (Z15, Z16)
  *   or_warp_plane       O7: 1/8-pel two-pass bilinear warp of an HR plane (Z14)
  *   or_reconstruct      O8: reuse-based reconstruction of a chunk
+ *   or_reconstruct_i420 O8 on YUV 4:2:0 frames, chroma MC at 1/16 pel (NEXT-2; R9)
  *   or_conv3x3          3x3 cross-correlation, zero padding 1 (EDSR conv, P:306 / [89])
  *   or_pixel_shuffle    PyTorch-order pixel shuffle (EDSR upsampler)
  *   or_sr_forward       O5: the whole SR DNN on one LR frame ("8 residual
@@ -183,6 +184,86 @@ int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t 
     if (hr_last && n > 0) memmove(hr_last, hr + (size_t)(n - 1) * 3 * hr_plane, 3 * hr_plane);
     if (hr_golden && golden && golden != hr_golden) memmove(hr_golden, golden, 3 * hr_plane);
     free(in); free(up_lr); free(up_res); free(pred);
+    return 0;
+}
+
+/* ---------------------------------------------------------------- O8 in YUV 4:2:0 (NEXT-2) */
+/* The codec's own colour format (VP9 profile 0 streams are YUV 4:2:0; SURVEY
+   Z18 / §8(f) NEXT-2).  A frame is Y [h][w], then U and V [h/2][w/2]; HR the
+   same at s x.  Reading R9, VP9's rule for 4:2:0: a block's
+   chroma motion vector is its luma vector taken at twice the precision, i.e.
+   the same number in 1/16 chroma pel (libvpx's chroma MC is the 1/16-pel
+   bilinear/8-tap family; here bilinear, as O7).  So for an HR chroma pixel
+   (X, Y) of the LR block (X / 4s, Y / 4s) with m = s * mv:
+     ix = X + floor(m_x / 16), fx = m_x mod 16 (same for y);
+     h(r) = (R[r][ix] (16 - fx) + R[r][ix+1] fx + 8) >> 4 for r = iy, iy+1;
+     pred = (h(iy) (16 - fy) + h(iy+1) fy + 8) >> 4
+   (= libvpx taps {128 - 8f, 8f} with FILTER_BITS 7), edge-replicated (Z16).
+   Luma is O7 unchanged; up_s (O6) runs per plane at its own size. */
+static uint8_t warp_px16(const uint8_t *ref, int H, int W, int X, int Y, int mx, int my)
+{
+    int ix = X + (int)floor_div(mx, 16), fx = mx - 16 * (int)floor_div(mx, 16);
+    int iy = Y + (int)floor_div(my, 16), fy = my - 16 * (int)floor_div(my, 16);
+    int xa = clampi(ix, 0, W - 1), xb = clampi(ix + 1, 0, W - 1);
+    int ya = clampi(iy, 0, H - 1), yb = clampi(iy + 1, 0, H - 1);
+    int h0 = (ref[(size_t)ya * W + xa] * (16 - fx) + ref[(size_t)ya * W + xb] * fx + 8) >> 4;
+    int h1 = (ref[(size_t)yb * W + xa] * (16 - fx) + ref[(size_t)yb * W + xb] * fx + 8) >> 4;
+    return (uint8_t)((h0 * (16 - fy) + h1 * fy + 8) >> 4);
+}
+
+/* Same decode-order rules as or_reconstruct (O8), per plane of the 4:2:0 frame.
+   lr, res: [n][h*w*3/2]; hr: [n][s*h*s*w*3/2]; hr_last, hr_golden one HR frame. */
+int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int16_t *res,
+                        const or_mv *mv, const uint8_t *type, const uint8_t *is_anchor,
+                        uint8_t *hr, uint8_t *hr_last, uint8_t *hr_golden)
+{
+    const int H = s * h, W = s * w, bw = w / 8;
+    const size_t lrf = (size_t)h * w * 3 / 2, hrf = (size_t)H * W * 3 / 2;
+    int32_t *in = (int32_t *)malloc((size_t)h * w * sizeof(int32_t));
+    int32_t *up_lr = (int32_t *)malloc((size_t)H * W * sizeof(int32_t));
+    int32_t *up_res = (int32_t *)malloc((size_t)H * W * sizeof(int32_t));
+    if (!in || !up_lr || !up_res) { free(in); free(up_lr); free(up_res); return -3; }
+    const uint8_t *golden = hr_golden;
+    for (int f = 0; f < n; f++) {
+        uint8_t *out = hr + (size_t)f * hrf;
+        const uint8_t *last = f > 0 ? hr + (size_t)(f - 1) * hrf : hr_last;
+        if (!is_anchor[f]) {
+            const or_mv *mvf = mv + (size_t)f * (h / 8) * bw;
+            for (int c = 0; c < 3; c++) {
+                /* plane geometry: luma full size, chroma half size; offset in the frame */
+                const int ph = c ? h / 2 : h, pw = c ? w / 2 : w, PH = s * ph, PW = s * pw;
+                const size_t lo = c == 0 ? 0 : (size_t)h * w + (size_t)(c - 1) * ph * pw;
+                const size_t ho = c == 0 ? 0 : (size_t)H * W + (size_t)(c - 1) * PH * PW;
+                const int blk = c ? 4 * s : 8 * s;            /* HR pixels per LR block side */
+                const uint8_t *lrp = lr + (size_t)f * lrf + lo;
+                const int16_t *rp = res + (size_t)f * lrf + lo;
+                uint8_t *op = out + ho;
+                for (size_t i = 0; i < (size_t)ph * pw; i++) in[i] = lrp[i];
+                or_upsample(in, ph, pw, s, up_lr);
+                if (type[f] == OR_KEY) {
+                    for (size_t i = 0; i < (size_t)PH * PW; i++) op[i] = (uint8_t)up_lr[i];
+                    continue;
+                }
+                for (size_t i = 0; i < (size_t)ph * pw; i++) in[i] = rp[i];
+                or_upsample(in, ph, pw, s, up_res);
+                for (int Y = 0; Y < PH; Y++)
+                    for (int X = 0; X < PW; X++) {
+                        const or_mv *b = &mvf[(size_t)(Y / blk) * bw + X / blk];
+                        size_t i = (size_t)Y * PW + X;
+                        if (b->ref == OR_INTRA) { op[i] = (uint8_t)up_lr[i]; continue; }
+                        const uint8_t *r = (b->ref == OR_GOLDEN ? golden : last);
+                        if (!r) { free(in); free(up_lr); free(up_res); return -1; }
+                        int p = c ? warp_px16(r + ho, PH, PW, X, Y, s * b->mvx, s * b->mvy)
+                                  : warp_px(r + ho, PH, PW, X, Y, s * b->mvx, s * b->mvy);
+                        op[i] = (uint8_t)clampi(p + up_res[i], 0, 255);
+                    }
+            }
+        }
+        if (type[f] == OR_KEY || type[f] == OR_ALTREF) golden = out;
+    }
+    if (hr_last && n > 0) memmove(hr_last, hr + (size_t)(n - 1) * hrf, hrf);
+    if (hr_golden && golden && golden != hr_golden) memmove(hr_golden, golden, hrf);
+    free(in); free(up_lr); free(up_res);
     return 0;
 }
 

@@ -308,6 +308,142 @@ def make_chunk(seed: int, w: int, h: int, scale: int, n: int, *, types=None,
                  res_size=res_size, gt=gt)
 
 
+def _codec_predict16(ref: np.ndarray, mvx_b: np.ndarray, mvy_b: np.ndarray) -> np.ndarray:
+    """Encoder-side 4:2:0 chroma prediction of the synthetic codec: the block's
+    luma vector read in 1/16 chroma pel (VP9's 4:2:0 rule), two-pass bilinear
+    with 16 phases on the 4x4 chroma block, edge-replicated borders."""
+    C, H, W = ref.shape
+    bh, bw = mvx_b.shape
+    ix = np.floor_divide(mvx_b, 16).astype(np.int64); fx = (mvx_b - 16 * ix).astype(np.int32)
+    iy = np.floor_divide(mvy_b, 16).astype(np.int64); fy = (mvy_b - 16 * iy).astype(np.int32)
+    m = int(max(np.abs(ix).max(initial=0), np.abs(iy).max(initial=0))) + 2
+    pad = np.pad(ref, ((0, 0), (m, m), (m, m)), mode="edge").astype(np.int32)
+    win = np.lib.stride_tricks.sliding_window_view(pad, (5, 5), axis=(1, 2))
+    oy = (np.arange(bh) * 4)[:, None] + iy + m
+    ox = (np.arange(bw) * 4)[None, :] + ix + m
+    wv = win[:, oy, ox]                                   # [C][bh][bw][5][5]
+    fx_ = fx[None, :, :, None, None]; fy_ = fy[None, :, :, None, None]
+    hrow = (wv[..., :, :4] * (16 - fx_) + wv[..., :, 1:] * fx_ + 8) >> 4
+    out = (hrow[..., :4, :] * (16 - fy_) + hrow[..., 1:, :] * fy_ + 8) >> 4
+    return out.transpose(0, 1, 3, 2, 4).reshape(C, H, W).astype(np.int64)
+
+
+@dataclasses.dataclass
+class ChunkI420:
+    """One stream's chunk in YUV 4:2:0 (NEXT-2): per frame Y [h][w] then U, V
+    [h/2][w/2], flattened; the rest as Chunk."""
+    w: int
+    h: int
+    scale: int
+    lr: np.ndarray        # u8  [n][h*w*3/2]
+    res: np.ndarray       # i16 [n][h*w*3/2]
+    mv: np.ndarray        # MV_DTYPE [n][h/8][w/8] (luma vectors, 1/8 LR luma pel)
+    type: np.ndarray
+    res_size: np.ndarray
+    gt: np.ndarray | None = None   # u8 [n][s*h*s*w*3/2]
+    fmt: str = "i420"
+
+    @property
+    def n(self) -> int:
+        return int(self.type.shape[0])
+
+
+def to_i420(planes: np.ndarray) -> np.ndarray:
+    """[3][H][W] -> flat Y | U | V with chroma = rounded 2x2 box average (input
+    conversion of the synthetic source only)."""
+    y = planes[0].astype(np.int64)
+    c = planes[1:].astype(np.int64)
+    cs = (c[:, 0::2, 0::2] + c[:, 1::2, 0::2] + c[:, 0::2, 1::2] + c[:, 1::2, 1::2] + 2) >> 2
+    return np.concatenate([y.ravel(), cs.reshape(-1)])
+
+
+def make_chunk_i420(seed: int, w: int, h: int, scale: int, n: int, *, types=None, altref_every: int | None = 16,
+                    profile: int | None = None, intra_frac: float = 0.02, golden_frac: float = 0.15,
+                    jitter: float = 0.3, with_gt: bool = False) -> ChunkI420:
+    """The synthetic codec loop of make_chunk in YUV 4:2:0: luma exactly as
+    there, chroma planes at half resolution predicted with the block's luma
+    vector read in 1/16 chroma pel (_codec_predict16)."""
+    assert w % 8 == 0 and h % 8 == 0 and n >= 1
+    rng = np.random.default_rng(seed)
+    prof = PROFILES[(seed % len(PROFILES)) if profile is None else profile]
+    if types is None:
+        types = default_types(n, altref_every)
+    types = np.asarray(types, np.uint8)
+    scene = _Scene(rng, w, h, n, prof, scale)
+    bh, bw = h // 8, w // 8
+    P = h * w
+    lr = np.empty((n, P * 3 // 2), np.uint8)
+    res = np.empty((n, P * 3 // 2), np.int16)
+    mv = np.zeros((n, bh, bw), MV_DTYPE)
+    gt = np.empty((n, scale * scale * P * 3 // 2), np.uint8) if with_gt else None
+
+    def planes(flat):
+        y = flat[:P].reshape(1, h, w)
+        c = flat[P:].reshape(2, h // 2, w // 2)
+        return y, c
+
+    golden = -1
+    for f in range(n):
+        if with_gt:
+            g = np.clip(np.round(scene.render(f, scale)), 0, 255)
+            gt[f] = to_i420(g)
+            target = _box_down(g, scale)
+        else:
+            target = scene.render(f, 1)
+        tflat = to_i420(np.clip(np.round(target), 0, 255)).astype(np.float64)
+        if types[f] == NS_KEY:
+            rq = _quant(tflat - 128.0, 2)
+            lr[f] = np.clip(128 + rq.astype(np.int32), 0, 255)
+            res[f] = rq
+            mv[f]["ref"] = NS_REF_INTRA
+        else:
+            q = 2 if types[f] == NS_ALTREF else 4
+            u = rng.random((bh, bw))
+            ref = np.where(u < intra_frac, NS_REF_INTRA,
+                           np.where(u < intra_frac + golden_frac, NS_REF_GOLDEN, NS_REF_LAST)).astype(np.uint8)
+            if golden < 0 or f == 0:
+                ref[ref == NS_REF_GOLDEN] = NS_REF_LAST
+            if f == 0:
+                ref[:] = NS_REF_INTRA
+            mvx_l, mvy_l = scene.block_motion(f, f - 1, bh, bw)
+            mvx_g, mvy_g = scene.block_motion(f, max(golden, 0), bh, bw)
+            mvx = np.where(ref == NS_REF_GOLDEN, mvx_g, mvx_l)
+            mvy = np.where(ref == NS_REF_GOLDEN, mvy_g, mvy_l)
+            jm = rng.random((bh, bw)) < jitter
+            mvx = mvx + jm * rng.integers(-1, 2, (bh, bw))
+            jm = rng.random((bh, bw)) < jitter
+            mvy = mvy + jm * rng.integers(-1, 2, (bh, bw))
+            mvx = np.clip(mvx, -32768, 32767)
+            mvy = np.clip(mvy, -32768, 32767)
+            mvx[ref == NS_REF_INTRA] = 0
+            mvy[ref == NS_REF_INTRA] = 0
+            pred = np.empty(P * 3 // 2, np.int64)
+            refpx_y = np.repeat(np.repeat(ref, 8, 0), 8, 1)
+            refpx_c = np.repeat(np.repeat(ref, 4, 0), 4, 1)
+            for which, rp_ in ((NS_REF_LAST, f - 1), (NS_REF_GOLDEN, golden)):
+                if rp_ < 0 or not (ref == which).any():
+                    continue
+                ry, rc = planes(lr[rp_])
+                py = _codec_predict(ry, mvx, mvy)[0]
+                pc = _codec_predict16(rc, mvx, mvy)
+                cur = np.concatenate([py.ravel(), pc.reshape(-1)])
+                sel = np.concatenate([(refpx_y == which).ravel(), np.tile((refpx_c == which).ravel(), 2)])
+                pred[sel] = cur[sel]
+            intra = np.concatenate([(refpx_y == NS_REF_INTRA).ravel(), np.tile((refpx_c == NS_REF_INTRA).ravel(), 2)])
+            pred[intra] = 128
+            rq = _quant(tflat - pred, q)
+            lr[f] = np.clip(pred + rq.astype(np.int64), 0, 255)
+            res[f] = rq
+            mv[f]["mvx"] = mvx
+            mv[f]["mvy"] = mvy
+            mv[f]["ref"] = ref
+        if types[f] in (NS_KEY, NS_ALTREF):
+            golden = f
+    nz = np.abs(res.astype(np.int64))
+    res_size = (1 + (np.log2(1 + nz).sum(axis=1) / 8.0)).astype(np.uint32)
+    return ChunkI420(w=w, h=h, scale=scale, lr=lr, res=res, mv=mv, type=types, res_size=res_size, gt=gt)
+
+
 def _to_bf16_bits(x: np.ndarray) -> np.ndarray:
     """float32 -> bf16 bit pattern, round-to-nearest-even."""
     u = np.ascontiguousarray(x, np.float32).view(np.uint32).astype(np.uint64)
