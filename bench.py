@@ -233,6 +233,8 @@ def main():
                     help="global: §5.2 selection across all GPUs' streams (per-GPU gains, NCCL all_gather, "
                          "ns_select_merge, NS_GIVEN_ANCHORS) inside the timed step")
     ap.add_argument("--ring", type=int, default=3, help="config 5: HR frames per stream (ring)")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N > 1 (gloo + NS_BENCH_SHARE_GPU=1: N ranks on one GPU)")
     ap.add_argument("--encode", action="store_true",
                     help="after timing: hybrid-encode one step's SR anchors (ns_encode_anchors, §6.1) and report "
                          "anchors/s and bytes per anchor")
@@ -250,8 +252,9 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = gpu_of(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        init_dist(args, local)
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
     cfg = cfg_of(args)
@@ -440,13 +443,13 @@ def main():
         ctx.encode_anchors(chunks[:1], ia_host[:1], hr_out[:1])          # encoder setup, warm-up
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
-        pk = ctx.encode_anchors(chunks, ia_host, hr_out)
+        pkgs = ctx.encode_anchors(chunks, ia_host, hr_out)
         t_enc = time.perf_counter() - t0
         na = int(ia_host.sum())
         hybrid = {"anchors": na, "seconds": t_enc, "anchors_per_s": na / t_enc,
-                  "mean_anchor_bytes": (sum(len(p) for p in pk) - 16 * S * n) / max(na, 1),
+                  "mean_anchor_bytes": (sum(len(p) for p in pkgs) - 16 * S * n) / max(na, 1),
                   "quality": ns.hybrid_quality(k, n), "codec": "JPEG 4:4:4 (nvJPEG), Table 2 quality",
-                  "package_bytes": sum(len(p) for p in pk)}
+                  "package_bytes": sum(len(p) for p in pkgs)}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -480,6 +483,23 @@ def main():
         dist.destroy_process_group()
 
 
+def gpu_of(local_rank):
+    """The device of this rank: LOCAL_RANK, or -- NS_BENCH_SHARE_GPU=1, a test of
+    the multi-rank path on a one-GPU box -- every rank on device 0."""
+    return 0 if os.environ.get("NS_BENCH_SHARE_GPU") == "1" else local_rank
+
+
+def init_dist(args, device):
+    """NCCL over NVLink between GPUs; --backend gloo (CPU collectives) lets
+    several ranks share one GPU (NCCL rejects two ranks on one device)."""
+    import torch
+    import torch.distributed as dist
+    if args.backend == "nccl":
+        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{device}"))
+    else:
+        dist.init_process_group("gloo")
+
+
 # ---------------------------------------------------------------- c5: mixed fleet
 K4_PX = 3840 * 2160
 
@@ -510,8 +530,9 @@ def run_c5(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = gpu_of(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
+        init_dist(args, local)
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
     cfg = cfg_of(args)
@@ -589,7 +610,8 @@ def run_c5(args):
     prof = ns.profile_read()
     ms = shard.max_over_ranks(ms_local)
     px4k_local = sum(n * 9 * x["w"] * x["h"] for x in mine) / K4_PX      # 4K-equivalent frames per step
-    tot = torch.tensor([px4k_local, float(S), float(sum(n for _ in mine))], dtype=torch.float64, device=dev)
+    tot = torch.tensor([px4k_local, float(S), float(sum(n for _ in mine))], dtype=torch.float64,
+                       device=dev if args.backend == "nccl" else "cpu")
     if world > 1:
         dist.all_reduce(tot)
     px4k, S_all, frames = (float(v) for v in tot.cpu().tolist())

@@ -81,6 +81,18 @@ typedef struct {
 typedef struct ns_ctx ns_ctx;
 typedef struct ns_model ns_model;
 
+/* Frame formats (codec-faithful formats).
+   NS_FMT_444:  three full-resolution planes per frame (reading Z18), the
+                layouts given below.
+   NS_FMT_I420: the codec's YUV 4:2:0 -- Y [h][w], then U, V [h/2][w/2] per LR
+                frame (lr u8, res int16), the same at s x per HR frame.  Motion
+                vectors stay one per 8x8 luma block; the chroma planes use the
+                block's vector read in 1/16 chroma pel (VP9's 4:2:0 rule,
+                reading R9) with the 16-phase bilinear.  An anchor is SR'd by
+                the 4:4:4 net on (Y, up_2(U), up_2(V)) and its HR chroma taken
+                back to 4:2:0 by the rounded 2x2 average (reading R10). */
+enum { NS_FMT_444 = 0, NS_FMT_I420 = 1 };
+
 /* One stream's chunk (= GOP of n_frames frames) as the decoder exports it
    (frame type and residual; reference index, MV). */
 typedef struct {
@@ -100,6 +112,7 @@ typedef struct {
                                   overwritten with the chunk's last KEY/ALTREF HR.
                                   May be NULL under the same condition.            */
     const uint8_t *gt;         /* optional [n][3][s*h][s*w] ground truth for stats   */
+    int32_t format;            /* NS_FMT_444 (0, the layouts above) | NS_FMT_I420   */
 } ns_chunk;
 
 /* Anchor selection mode (§5.1 top-k per chunk; §5.2 global budget).
@@ -144,9 +157,10 @@ typedef struct {
 /* One anchor-SR job: HR = SR_model(LR) (O5). */
 typedef struct {
     const ns_model *model;
-    const uint8_t *lr;         /* [3][h][w] */
+    const uint8_t *lr;         /* [3][h][w] (NS_FMT_I420: Y, U, V planes of 4:2:0)     */
     int32_t w, h;
-    uint8_t *hr_out;           /* [3][s*h][s*w] */
+    uint8_t *hr_out;           /* [3][s*h][s*w] (NS_FMT_I420: 4:2:0 at s x)          */
+    int32_t format;            /* NS_FMT_444 | NS_FMT_I420                           */
 } ns_sr_job;
 
 /* Creates a context on `device` with a device memory pool of pool_bytes

@@ -26,6 +26,7 @@ NS_REF_LAST, NS_REF_GOLDEN, NS_REF_INTRA = 0, 1, 2
 NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET, NS_GIVEN_ANCHORS = 0, 1, 2
 NS_CARRY, NS_FRESH = 0, 1
 NS_SEL_NEUROSCALER, NS_SEL_KEY, NS_SEL_KEY_UNIFORM = 0, 1, 2
+NS_FMT_444, NS_FMT_I420 = 0, 1
 
 P = ctypes.c_void_p
 
@@ -33,7 +34,7 @@ P = ctypes.c_void_p
 class NsChunk(ctypes.Structure):
     _fields_ = [("w", ctypes.c_int32), ("h", ctypes.c_int32), ("scale", ctypes.c_int32), ("n_frames", ctypes.c_int32),
                 ("lr", P), ("res", P), ("mv", P), ("type", P), ("res_size", P), ("model", P),
-                ("hr_last", P), ("hr_golden", P), ("gt", P)]
+                ("hr_last", P), ("hr_golden", P), ("gt", P), ("format", ctypes.c_int32)]
 
 
 class NsSelectParams(ctypes.Structure):
@@ -48,7 +49,8 @@ class NsProfEntry(ctypes.Structure):
 
 
 class NsSrJob(ctypes.Structure):
-    _fields_ = [("model", P), ("lr", P), ("w", ctypes.c_int32), ("h", ctypes.c_int32), ("hr_out", P)]
+    _fields_ = [("model", P), ("lr", P), ("w", ctypes.c_int32), ("h", ctypes.c_int32), ("hr_out", P),
+                ("format", ctypes.c_int32)]
 
 
 EXPORTS = ["ns_ctx_create", "ns_ctx_destroy", "ns_model_create", "ns_model_set_weights", "ns_model_blob_len",
@@ -186,6 +188,7 @@ class DeviceChunk:
     hr_last: "object" = None   # uint8 [3,sH,sW]
     hr_golden: "object" = None
     gt: "object" = None        # uint8 [n,3,sH,sW]
+    format: int = NS_FMT_444   # NS_FMT_I420: lr/res [n, h*w*3/2], HR frames s*h*s*w*3/2 bytes
 
     @property
     def n(self) -> int:
@@ -194,11 +197,11 @@ class DeviceChunk:
     def to_c(self) -> NsChunk:
         return NsChunk(self.w, self.h, self.scale, self.n, _ptr(self.lr), _ptr(self.res), _ptr(self.mv),
                        _ptr(self.type), _ptr(self.res_size), self.model.handle if self.model else None,
-                       _ptr(self.hr_last), _ptr(self.hr_golden), _ptr(self.gt))
+                       _ptr(self.hr_last), _ptr(self.hr_golden), _ptr(self.gt), int(self.format))
 
     @staticmethod
     def from_numpy(lr, res, mv, types, w, h, scale, device, res_size=None, gt=None, model=None,
-                   hr_last=None, hr_golden=None) -> "DeviceChunk":
+                   hr_last=None, hr_golden=None, format=NS_FMT_444) -> "DeviceChunk":
         """Copies host arrays (mv as a structured or raw 8-byte array) to `device`."""
         import torch
         mvb = np.ascontiguousarray(mv).view(np.uint8).reshape(mv.shape[0], h // 8, w // 8, 8)
@@ -206,7 +209,7 @@ class DeviceChunk:
         rs = None if res_size is None else t(np.asarray(res_size).astype(np.int32))
         return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
                            model=model, res_size=rs, gt=None if gt is None else t(gt),
-                           hr_last=hr_last, hr_golden=hr_golden)
+                           hr_last=hr_last, hr_golden=hr_golden, format=format)
 
 
     @staticmethod
@@ -304,10 +307,16 @@ class Context:
                                      int(budget), _ptr(rank), _ptr(is_anchor), _stream(stream)), "ns_select_merge")
 
     def sr_anchors(self, jobs, stream=None):
-        """jobs: list of (model, lr [3,h,w] u8 tensor, hr_out [3,sh,sw] u8 tensor)."""
+        """jobs: list of (model, lr [3,h,w] u8 tensor, hr_out [3,sh,sw] u8 tensor), or
+        (model, lr, hr_out, w, h, format) for a 4:2:0 frame (flat tensors)."""
         arr = (NsSrJob * len(jobs))()
-        for i, (m, lr, hr) in enumerate(jobs):
-            arr[i] = NsSrJob(m.handle, _ptr(lr), int(lr.shape[-1]), int(lr.shape[-2]), _ptr(hr))
+        for i, job in enumerate(jobs):
+            if len(job) == 3:
+                m, lr, hr = job
+                w, h, fmt = int(lr.shape[-1]), int(lr.shape[-2]), NS_FMT_444
+            else:
+                m, lr, hr, w, h, fmt = job
+            arr[i] = NsSrJob(m.handle, _ptr(lr), int(w), int(h), _ptr(hr), int(fmt))
         _check(lib().ns_sr_anchors(self.handle, arr, len(jobs), _stream(stream)), "ns_sr_anchors")
 
     @staticmethod

@@ -339,8 +339,9 @@ __global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *
     const StreamDesc d = sd[sid];
     const size_t lrp = (size_t)d.h * d.w;
     FrameDesc o{};
-    o.lr_f = d.lr + (size_t)f * 3 * lrp;
-    o.res_f = d.res + (size_t)f * 3 * lrp;
+    o.lr_f = d.lr + (size_t)f * d.lr_frame;
+    o.res_f = d.res + (size_t)f * d.lr_frame;
+    (void)lrp;
     o.mv_f = d.mv + (size_t)f * (d.h / 8) * (d.w / 8);
     o.out = hr_tab[d.hr_base + f];
     o.ref_last = f > 0 ? hr_tab[d.hr_base + f - 1] : d.hr_last;
@@ -359,6 +360,7 @@ __global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *
     o.s = (int16_t)d.s;
     o.anchor = is_anchor[e] ? 1 : 0;
     o.key = d.type[f] == NS_KEY;
+    o.fmt = d.fmt;
     fd[e] = o;
 }
 
@@ -374,9 +376,9 @@ cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_
 // planes) from src to dst in 8-B words (W is a multiple of 8): the HR-ring
 // anchor copy and GOLDEN save, done by the frame step's own CTAs.
 __device__ __forceinline__ void recon_tile_copy(const uint8_t *src, uint8_t *dst, size_t hrp, int W, int x0, int x1,
-                                                int y0, int y1, int tid, int nt) {
+                                                int y0, int y1, int tid, int nt, int planes) {
     const int wpr = (x1 - x0) >> 3, rows = y1 - y0, per_plane = wpr * rows;
-    for (int i = tid; i < 3 * per_plane; i += nt) {
+    for (int i = tid; i < planes * per_plane; i += nt) {
         const int c = i / per_plane, r = (i % per_plane) / wpr, q = i % wpr;
         const size_t off = (size_t)c * hrp + (size_t)(y0 + r) * W + x0 + 8 * q;
         *reinterpret_cast<uint2 *>(dst + off) = *reinterpret_cast<const uint2 *>(src + off);
@@ -398,10 +400,13 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     if (8 * bx0 >= w || Y0c >= H) return;               // CTA-uniform
     const int tid = threadIdx.y * kReconTX + threadIdx.x;
     const size_t lrp = (size_t)h * w, hrp = (size_t)H * W;
+    // planes stepped here: 3 (4:4:4), or the luma plane of a 4:2:0 frame (its
+    // chroma planes step in k_recon_c420)
+    const int np_ = fd.fmt == NS_FMT_I420 ? 1 : 3;
     if (fd.gsave_src || (fd.anchor && fd.asrc)) {       // HR rings only (k_frame_desc)
         const int x0 = 8 * S * bx0, x1 = min(8 * S * (bx0 + kReconTX), W), y1 = min(Y0c + kReconTY * RPT, H);
-        if (fd.gsave_src) recon_tile_copy(fd.gsave_src, fd.gsave_dst, hrp, W, x0, x1, Y0c, y1, tid, kReconNT);
-        if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc, fd.out, hrp, W, x0, x1, Y0c, y1, tid, kReconNT);
+        if (fd.gsave_src) recon_tile_copy(fd.gsave_src, fd.gsave_dst, hrp, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
+        if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc, fd.out, hrp, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
     }
     if (fd.anchor) return;                              // CTA-uniform: the anchor's SR bytes are in place
 
@@ -422,10 +427,10 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
         if (tid == 0) {
             mbar_init(tbar, 1);
             fence_mbar_init();
-            mbar_arrive_expect_tx(tbar, 3 * Sm::RROWS * bytes);
+            mbar_arrive_expect_tx(tbar, np_ * Sm::RROWS * bytes);
         }
         __syncwarp();
-        for (int e = tid; e < 3 * Sm::RROWS; e += 32) {
+        for (int e = tid; e < np_ * Sm::RROWS; e += 32) {
             const int c = e / Sm::RROWS, rr = e % Sm::RROWS;
             const int row = min(max(Y0c / S - 1 + rr, 0), h - 1);
             bulk_load(tres + (size_t)e * kResCols + (col_lo - (8 * bx0 - 8)),
@@ -463,11 +468,11 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     auto lr_slots = [&](int c) { return (LR_ALL ? c : (c & 1)) * LRS * kReconNT; };
     uint2 *wbuf = rsm + tid;
     auto stage_row = [&](int c, int r) {
-        if (!valid || c >= 3) return;
+        if (!valid || c >= np_) return;
         if (use_lr) {
             if (r == 0 && (!LR_ALL || c == 0)) {
 #pragma unroll 1
-                for (int cc = c; cc < (LR_ALL ? 3 : c + 1); cc++)
+                for (int cc = c; cc < (LR_ALL ? np_ : c + 1); cc++)
 #pragma unroll
                     for (int t = 0; t < Cfg::PER + 2; t++)
                         recon_lr_row_stage(fd.lr_f + cc * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
@@ -488,7 +493,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
     uint8_t *outp = fd.out + (size_t)Y0 * W + X0;
 
 #pragma unroll 1
-    for (int c = 0; c < 3; c++) {
+    for (int c = 0; c < np_; c++) {
         asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
         if (c == 0) {
             __syncthreads();                                    // (orders the tile barrier's init)
@@ -566,10 +571,92 @@ static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, in
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- 4:2:0 chroma (NEXT-2)
+// One frame step of the U and V planes of the NS_FMT_I420 streams (readings R9,
+// R10; oracle or_reconstruct_i420).  An HR chroma pixel (X, Y) lies in the LR
+// block (X / 4s, Y / 4s); its motion is the block's luma vector read in 1/16
+// chroma pel, m = s mv: pred = 16-phase two-pass bilinear of the reference
+// chroma plane (edge replicated), plus up_s of the chroma residual plane, clamped;
+// KEY frames and INTRA blocks take up_s of the LR chroma plane.  A thread owns
+// two horizontally adjacent pixels (they share the block: 4s is even) of both
+// planes over kC420Rows rows, so the block's vector, the O6 taps and the warp
+// geometry are computed once per row for four outputs.  Plain integer code:
+// the chroma planes are half the luma plane's pixels.
+constexpr int kC420TX = 64, kC420TY = 2, kC420Rows = 4;
+
+__device__ __forceinline__ int c420_bilin16(const uint8_t *R, int PH, int PW, int X, int Y, int mx, int my) {
+    const int ix = X + (mx >> 4), fx = mx & 15, iy = Y + (my >> 4), fy = my & 15;
+    const int xa = min(max(ix, 0), PW - 1), xb = min(max(ix + 1, 0), PW - 1);
+    const int ya = min(max(iy, 0), PH - 1), yb = min(max(iy + 1, 0), PH - 1);
+    const int h0 = (R[(size_t)ya * PW + xa] * (16 - fx) + R[(size_t)ya * PW + xb] * fx + 8) >> 4;
+    const int h1 = (R[(size_t)yb * PW + xa] * (16 - fx) + R[(size_t)yb * PW + xb] * fx + 8) >> 4;
+    return (h0 * (16 - fy) + h1 * fy + 8) >> 4;
+}
+
+template <class T>
+__device__ __forceinline__ int c420_up(const T *P, int pw, int y0, int y1, int wy, int x0, int x1, int wx) {
+    const int v = (128 - wy) * ((128 - wx) * (int)P[(size_t)y0 * pw + x0] + wx * (int)P[(size_t)y0 * pw + x1]) +
+                  wy * ((128 - wx) * (int)P[(size_t)y1 * pw + x0] + wx * (int)P[(size_t)y1 * pw + x1]);
+    return (v + 8192) >> 14;   // floor((v + 8192) / 2^14) (arithmetic shift)
+}
+
+template <int S>
+__global__ void __launch_bounds__(kC420TX * kC420TY) k_recon_c420(const FrameDesc *fdesc, int n, int f, int s0) {
+    const int sid = s0 + blockIdx.z;
+    const FrameDesc fd = fdesc[(size_t)sid * n + f];
+    if (fd.s != S || fd.fmt != NS_FMT_I420) return;                 // CTA-uniform
+    const int w = fd.w, h = fd.h, H = S * h, W = S * w;
+    const int pw = w / 2, ph = h / 2, PW = W / 2, PH = H / 2;       // chroma planes (LR, HR)
+    const int X = 2 * (blockIdx.x * kC420TX + threadIdx.x);
+    const int Yb = (blockIdx.y * kC420TY + threadIdx.y) * kC420Rows;
+    if (X >= PW || Yb >= PH) return;
+    const size_t lrp = (size_t)h * w, hrp = (size_t)H * W, cl = lrp / 4, ch = hrp / 4;
+    const int Ye = min(Yb + kC420Rows, PH);
+    // HR rings: the GOLDEN save and the anchor copy of the chroma planes
+    auto copy2 = [&](const uint8_t *src, uint8_t *dst) {
+        for (int c = 0; c < 2; c++)
+            for (int Y = Yb; Y < Ye; Y++) {
+                const size_t o = hrp + c * ch + (size_t)Y * PW + X;
+                *reinterpret_cast<uint16_t *>(dst + o) = *reinterpret_cast<const uint16_t *>(src + o);
+            }
+    };
+    if (fd.gsave_src) copy2(fd.gsave_src, fd.gsave_dst);
+    if (fd.anchor) {
+        if (fd.asrc) copy2(fd.asrc, fd.out);
+        return;
+    }
+    constexpr int BLK = 4 * S;                                      // HR chroma pixels per LR block side
+    int xa[2], xb[2], wx[2];
+    for (int e = 0; e < 2; e++) up_tap_r(X + e, S, pw, xa[e], xb[e], wx[e]);
+    for (int Y = Yb; Y < Ye; Y++) {
+        const ns_block_mv mv = fd.mv_f[(size_t)(Y / BLK) * (w / 8) + X / BLK];
+        const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;
+        const uint8_t *ref = mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last;
+        int ya, yb, wy;
+        up_tap_r(Y, S, ph, ya, yb, wy);
+        for (int c = 0; c < 2; c++) {
+            uint8_t o[2];
+            for (int e = 0; e < 2; e++) {
+                int v;
+                if (use_lr) {
+                    v = c420_up(fd.lr_f + lrp + c * cl, pw, ya, yb, wy, xa[e], xb[e], wx[e]);
+                } else {
+                    const int r = c420_up(fd.res_f + lrp + c * cl, pw, ya, yb, wy, xa[e], xb[e], wx[e]);
+                    const int p = c420_bilin16(ref + hrp + c * ch, PH, PW, X + e, Y, S * mv.mvx, S * mv.mvy);
+                    v = min(max(p + r, 0), 255);
+                }
+                o[e] = (uint8_t)v;
+            }
+            *reinterpret_cast<uint16_t *>(fd.out + hrp + c * ch + (size_t)Y * PW + X) =
+                (uint16_t)(o[0] | (o[1] << 8));
+        }
+    }
+}
+
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              cudaStream_t st, int s0) {
+                              const int *has_i420, cudaStream_t st, int s0) {
     int nl = 0;
-    for (int s = 2; s <= 4; s++) nl += max_lr_w[s] > 0;
+    for (int s = 2; s <= 4; s++) nl += (max_lr_w[s] > 0) + (has_i420[s] != 0);
     KScope ks(F_RECON, st, nl);
     for (int s = 2; s <= 4; s++) {
         if (max_lr_w[s] <= 0) continue;
@@ -580,6 +667,15 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
         const cudaError_t e = s == 2 ? recon_launch<2>(g, st, fd, n, f, s0)
                               : s == 3 ? recon_launch<3>(g, st, fd, n, f, s0) : recon_launch<4>(g, st, fd, n, f, s0);
         if (e != cudaSuccess) return e;
+        if (has_i420[s]) {  // the chroma planes of the 4:2:0 streams of this scale, same frame step
+            const int PW = max_lr_w[s] * s / 2, PH = max_lr_h[s] * s / 2;
+            dim3 gc((PW / 2 + kC420TX - 1) / kC420TX, (PH + kC420TY * kC420Rows - 1) / (kC420TY * kC420Rows), S);
+            dim3 bc(kC420TX, kC420TY);
+            if (s == 2) k_recon_c420<2><<<gc, bc, 0, st>>>(fd, n, f, s0);
+            else if (s == 3) k_recon_c420<3><<<gc, bc, 0, st>>>(fd, n, f, s0);
+            else k_recon_c420<4><<<gc, bc, 0, st>>>(fd, n, f, s0);
+            if (cudaError_t e2 = cudaGetLastError(); e2 != cudaSuccess) return e2;
+        }
     }
     return cudaGetLastError();
 }
@@ -589,7 +685,7 @@ __global__ void k_state_copy(const StreamDesc *sd, int n, uint8_t *const *hr_tab
                              const uint8_t *gsv) {
     const int sid = blockIdx.y, which = blockIdx.z;
     const StreamDesc d = sd[sid];
-    const size_t nvec = (size_t)3 * d.h * d.s * d.w * d.s / 16;
+    const size_t nvec = (size_t)d.hr_frame / 16;
     uint8_t *dst;
     const uint8_t *src;
     if (which == 0) {
@@ -639,7 +735,7 @@ __global__ void k_stats_sse(const StreamDesc *sd, int n, uint8_t *const *hr_tab,
     const int sf = blockIdx.x, sid = sf / n, f = sf % n;   // (stream, frame) on x: S*n may exceed 65535
     const StreamDesc d = sd[sid];
     if (!d.gt) return;
-    const size_t nvec = (size_t)3 * d.h * d.s * d.w * d.s / 16;
+    const size_t nvec = (size_t)d.hr_frame / 16;
     const uint4 *a = reinterpret_cast<const uint4 *>(hr_tab[d.hr_base + f]);
     const uint4 *b = reinterpret_cast<const uint4 *>(d.gt + (size_t)f * nvec * 16);
     unsigned long long acc = 0;
@@ -661,7 +757,7 @@ __global__ void k_stats_sse(const StreamDesc *sd, int n, uint8_t *const *hr_tab,
 __global__ void k_stats_final(const StreamDesc *sd, int S, int n, double *stats) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S || !sd[s].gt) return;
-    const double N = 3.0 * sd[s].h * sd[s].s * sd[s].w * sd[s].s * n;
+    const double N = (double)sd[s].hr_frame * n;
     const double sse = stats[(size_t)s * 8 + 4];
     double p = sse == 0.0 ? 100.0 : 10.0 * log10(255.0 * 255.0 / (sse / N));
     stats[(size_t)s * 8 + 5] = p > 100.0 ? 100.0 : p;

@@ -21,8 +21,8 @@ __global__ void __launch_bounds__(kScoreThreads) k_score(const StreamDesc *sd, i
         if (blockIdx.y == 0 && threadIdx.x == 0) score[sf] = (int64_t)d.res_size[f];
         return;
     }
-    const size_t nvec = (size_t)3 * d.h * d.w / 8;
-    const uint4 *r = reinterpret_cast<const uint4 *>(d.res + (size_t)f * 3 * d.h * d.w);
+    const size_t nvec = (size_t)d.lr_frame / 8;   // 3 h w (4:4:4) or h w 3/2 (4:2:0): all planes
+    const uint4 *r = reinterpret_cast<const uint4 *>(d.res + (size_t)f * d.lr_frame);
     const size_t base = (size_t)blockIdx.y * kScoreThreads * kScoreUnroll + threadIdx.x;
     if ((size_t)blockIdx.y * kScoreThreads * kScoreUnroll >= nvec) return;
     uint4 v[kScoreUnroll];
@@ -386,7 +386,7 @@ __global__ void k_compact(const StreamDesc *sd, int S, int n, uint8_t *is_anchor
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
     const StreamDesc d = sd[s];
-    const size_t lr_frame = (size_t)3 * d.h * d.w;
+    const size_t lr_frame = (size_t)d.lr_frame;
     int claim = topk ? 0 : start[s];
     for (int f = 0; f < n; f++) {
         const size_t e = (size_t)s * n + f;

@@ -43,7 +43,7 @@ __device__ unsigned long long g_trace[16 * 2 * 1024];
 // EPI_HEAD: the store epilogue of the head conv, whose input x = LR - 128 has 3
 // real channels: only channel group 0 (8 channels, 16 B/px) is stored and
 // loaded by TMA; group 1 of every ring slot is a zero region written once.
-enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_SHUFFLE = 3, EPI_TAIL = 4, EPI_HEAD = 5 };
+enum { EPI_STORE = 0, EPI_RELU = 1, EPI_RESID = 2, EPI_HEAD = 5 };
 
 struct ConvArgs {
     int H, W;               // conv spatial dims (input == output)
@@ -53,15 +53,17 @@ struct ConvArgs {
     const int32_t *job_count;
     size_t b_off, bias_off; // this launch's B operand / bias offsets in the packed model
     const uint16_t *in;     // bf16 activation in [job][H][CIN/8][W][8] (k_conv_rot, k_uptail2: bulk-copied rows)
-    uint16_t *out;          // bf16 activation out (EPI_STORE/RELU/RESID/SHUFFLE)
+    uint16_t *out;          // bf16 activation out (EPI_STORE/RELU/RESID)
     const uint16_t *resid;  // EPI_RESID
     int C;                  // channels of the output activation (shuffle: per sub-pixel)
     int s;                  // scale (shuffle / tail)
     int sub0;               // shuffle: first sub-pixel of this launch
     int lr_h, lr_w;         // tail: LR dims of the bilinear skip
     float *ring;            // uptail: fp32 t of the HR frame-border ring [job][nring][3]
-    uint8_t *lr8;           // (unused by the convs: uptail2's u8 LR copy is written by k_prep_lr)
+    uint8_t *lr8;           // u8 copy of the net's input planes [job][H][3][wp] (k_prep_lr), k_uptail's skip taps
     int wp;
+    uint8_t *hr_tmp;        // NS_FMT_I420 batches: the HR output goes here ([slot][3][H][W]) and is packed
+    size_t hr_tmp_frame;    // to 4:2:0 into jobs[].hr afterwards (k_pack420); NULL: straight to jobs[].hr
 };
 
 __host__ __device__ constexpr uint32_t round_up(uint32_t v, uint32_t a) { return (v + a - 1) / a * a; }
@@ -374,24 +376,7 @@ __global__ void __launch_bounds__(128)
         tmem_wait_ld();
         tmem_zero<NB>(acc);  // row r's block becomes row r+3's
         if (valid) {
-            if constexpr (EPI == EPI_TAIL) {
-                const int s = a.s, lh = a.lr_h, lw = a.lr_w;
-                int ya, yb, wy, xa, xb, wx;
-                up_tap(r, s, lh, ya, yb, wy);
-                up_tap(x, s, lw, xa, xb, wx);
-                const size_t plane = (size_t)lh * lw, hplane = (size_t)a.H * a.W;
-#pragma unroll
-                for (int c = 0; c < 3; c++) {
-                    const uint8_t *L = J.lr + c * plane;
-                    const int p00 = L[(size_t)ya * lw + xa], p01 = L[(size_t)ya * lw + xb];
-                    const int p10 = L[(size_t)yb * lw + xa], p11 = L[(size_t)yb * lw + xb];
-                    const int vv = (128 - wy) * ((128 - wx) * p00 + wx * p01) + wy * ((128 - wx) * p10 + wx * p11);
-                    const int U = (vv + 8192) >> 14;
-                    const float t = __uint_as_float(v[c]) + s_bias[c];
-                    const float o = floorf((float)U + t + 0.5f);
-                    J.hr[c * hplane + (size_t)r * a.W + x] = (uint8_t)fminf(fmaxf(o, 0.f), 255.f);
-                }
-            } else {
+            {
                 const size_t rowbase = ((size_t)slot_job * a.H + r) * (NB / 8);
 #pragma unroll
                 for (int cg = 0; cg < NB / 8; cg++) {
@@ -880,6 +865,7 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
     const uint32_t tmem = *s_tmem;
     const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);
     const SrJob J = a.jobs[job];
+    uint8_t *const hr_dst = a.hr_tmp ? a.hr_tmp + (size_t)slot_job * a.hr_tmp_frame : J.hr;
     if (tid == 0) {
         prefetch_tmap(&tm_in);
         mbar_arrive_expect_tx(&bars[3], Cfg::B_BYTES + Cfg::BIAS_BYTES);
@@ -926,15 +912,16 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
         __syncwarp();
         const int r = yin - 2;  // LR output row completed by this input row
         const bool valid_row = r >= y0;
-        // bilinear-skip taps for this lane (O6, compile-time sub-pixel weights)
+        // bilinear-skip taps for this lane (O6, compile-time sub-pixel weights), from
+        // the batch's u8 copy of the net's input planes (k_prep_lr: [job][H][3][wp])
         int Lv[3][3][3];
         if (valid_row && x < lw) {
 #pragma unroll
             for (int c = 0; c < 3; c++) {
-                const uint8_t *L = J.lr + (size_t)c * lh * lw;
 #pragma unroll
                 for (int dy = 0; dy < 3; dy++) {
-                    const uint8_t *Lr = L + (size_t)min(max(r + dy - 1, 0), lh - 1) * lw;
+                    const uint8_t *Lr =
+                        a.lr8 + (((size_t)slot_job * lh + min(max(r + dy - 1, 0), lh - 1)) * 3 + c) * a.wp;
 #pragma unroll
                     for (int dx = 0; dx < 3; dx++) Lv[c][dy][dx] = Lr[min(max(x + dx - 1, 0), lw - 1)];
                 }
@@ -997,7 +984,7 @@ __global__ void __launch_bounds__(128) k_uptail(const __grid_constant__ CUtensor
             for (int e = tid; e < 3 * S * CH; e += 128) {
                 const int ch = e % CH, ri = e / CH, c = ri / S, i = ri % S;
                 if (ch * 8 < wv)
-                    *reinterpret_cast<uint2 *>(J.hr + (size_t)c * HH * WW + (size_t)(S * r + i) * WW + xs_hr + ch * 8) =
+                    *reinterpret_cast<uint2 *>(hr_dst + (size_t)c * HH * WW + (size_t)(S * r + i) * WW + xs_hr + ch * 8) =
                         *reinterpret_cast<const uint2 *>(s_out + ri * (kTile * S) + ch * 8);
             }
         }
@@ -1279,7 +1266,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
             for (int i = 0; i < 3 * S; i++) bh[i] = s_bias[3 * S * g + i] + 0.5f;
             const uint32_t cbase = (uint32_t)(NB <= 16 ? 0 : 8 * ((3 * S * g) / 8));
             const int xs_hr = x0k(k) * S, wv = min(kTile, lw - x0k(k)) * S;
-            uint8_t *const hr = a.jobs[job].hr + xs_hr;
+            uint8_t *const hr = (a.hr_tmp ? a.hr_tmp + (size_t)slot_job * a.hr_tmp_frame : a.jobs[job].hr) + xs_hr;
             for (int q = 0; q < nq; q++) {
                 const int r = y0 - 4 + q;  // LR output row completed at this step
                 mbar_wait(mdone(k, q & 1), (q >> 1) & 1);
@@ -1443,7 +1430,8 @@ __global__ void __launch_bounds__(C * S) k_uptail_ext_u(const SrJob *jobs, int j
 // One thread per ring pixel: t = (composed t from the uptail epilogue) minus
 // the out-of-frame tail taps, then the bilinear skip, round, clamp, store.
 __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, int C, int s,
-                              size_t aux_off, const float *ext, const float *ring) {
+                              size_t aux_off, const float *ext, const float *ring, const uint8_t *lr8, int wp,
+                              uint8_t *hr_tmp) {
     __shared__ float swt[3 * 32 * 9];  // W_tail [3][C][9]
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
@@ -1480,21 +1468,38 @@ __global__ void k_uptail_ring(const SrJob *jobs, int j0, const int32_t *job_coun
     int ya, yb, wy, xa, xb, wx;
     up_tap(Y, s, h, ya, yb, wy);
     up_tap(X, s, w, xa, xb, wx);
+    // the skip taps come from the batch's u8 LR copy (k_prep_lr: the net's input
+    // planes, i.e. after the 4:2:0 chroma upsample for NS_FMT_I420)
+    uint8_t *const dst = hr_tmp ? hr_tmp + (size_t)slot * 3 * H * W : J.hr;
+    const uint8_t *L8 = lr8 + (size_t)slot * h * 3 * wp;
     for (int c = 0; c < 3; c++) {
-        const uint8_t *L = J.lr + (size_t)c * h * w;
-        const int v = (128 - wy) * ((128 - wx) * L[(size_t)ya * w + xa] + wx * L[(size_t)ya * w + xb]) +
-                      wy * ((128 - wx) * L[(size_t)yb * w + xa] + wx * L[(size_t)yb * w + xb]);
+        auto L = [&](int yy, int xx) { return (int)L8[((size_t)yy * 3 + c) * wp + xx]; };
+        const int v = (128 - wy) * ((128 - wx) * L(ya, xa) + wx * L(ya, xb)) +
+                      wy * ((128 - wx) * L(yb, xa) + wx * L(yb, xb));
         const int U = (v + 8192) >> 14;
         const float o = fminf(fmaxf(floorf((float)U + t[c] + 0.5f), 0.f), 255.f);
-        J.hr[(size_t)c * H * W + (size_t)Y * W + X] = (uint8_t)o;
+        dst[(size_t)c * H * W + (size_t)Y * W + X] = (uint8_t)o;
     }
 }
 
 // LR u8 planar [3][h][w] -> bf16 [h][w][8], channel group 0 of the head input:
 // channels 0..2 = LR - 128 (Z13), 3..7 = 0 (channels 8..15 are the zero region of
 // the head's ring slots, EPI_HEAD).
+// NS_FMT_I420: the input is Y [h][w], U, V [h/2][w/2]; the net takes the
+// chroma planes at luma resolution, upsampled x2 with the O6 definition
+// (integer bilinear, half-pixel centres, Q7 weights, one round-half-up;
+// reading R10), computed here on the fly.
+__device__ __forceinline__ int up2_px(const uint8_t *P, int ph, int pw, int y, int x) {
+    int ya, yb, wy, xa, xb, wx;
+    up_tap(y, 2, ph, ya, yb, wy);
+    up_tap(x, 2, pw, xa, xb, wx);
+    const int v = (128 - wy) * ((128 - wx) * P[(size_t)ya * pw + xa] + wx * P[(size_t)ya * pw + xb]) +
+                  wy * ((128 - wx) * P[(size_t)yb * pw + xa] + wx * P[(size_t)yb * pw + xb]);
+    return (v + 8192) >> 14;
+}
+
 __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0,
-                          uint8_t *lr8, int wp) {
+                          uint8_t *lr8, int wp, int fmt) {
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
     const int idx = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1502,16 +1507,46 @@ __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, i
     const int y = idx / w, x = idx % w;
     const uint8_t *L = jobs[job].lr;
     const size_t plane = (size_t)h * w;
-    const float r = (float)L[idx] - 128.f, g = (float)L[plane + idx] - 128.f, b = (float)L[2 * plane + idx] - 128.f;
+    int p0 = L[idx], p1, p2;
+    if (fmt == NS_FMT_I420) {
+        p1 = up2_px(L + plane, h / 2, w / 2, y, x);
+        p2 = up2_px(L + plane + plane / 4, h / 2, w / 2, y, x);
+    } else {
+        p1 = L[plane + idx];
+        p2 = L[2 * plane + idx];
+    }
     uint4 o0;
-    o0.x = pack_bf16(r, g);
-    o0.y = pack_bf16(b, 0.f);
+    o0.x = pack_bf16((float)p0 - 128.f, (float)p1 - 128.f);
+    o0.y = pack_bf16((float)p2 - 128.f, 0.f);
     o0.z = 0; o0.w = 0;
     *reinterpret_cast<uint4 *>(x0 + (((size_t)slot * h + y) * w + x) * 8) = o0;  // channel group 0 only
     uint8_t *l8 = lr8 + ((size_t)slot * h + y) * 3 * wp + x;
-    l8[0] = L[idx];
-    l8[wp] = L[plane + idx];
-    l8[2 * wp] = L[2 * plane + idx];
+    l8[0] = (uint8_t)p0;
+    l8[wp] = (uint8_t)p1;
+    l8[2 * wp] = (uint8_t)p2;
+}
+
+// NS_FMT_I420 output: the net's full-resolution HR [3][H][W] (hr_tmp) -> jobs[].hr
+// as 4:2:0: Y as is, U and V by the rounded 2x2 average floor((a+b+c+d+2)/4)
+// (reading R10).  One thread per 2x2 quad (4 Y bytes + 1 U + 1 V).
+__global__ void k_pack420(const SrJob *jobs, int j0, const int32_t *job_count, int H, int W, const uint8_t *hr_tmp) {
+    const int slot = blockIdx.y, job = j0 + slot;
+    if (job_count && job >= *job_count) return;
+    const int q = blockIdx.x * blockDim.x + threadIdx.x;
+    const int QW = W / 2, QH = H / 2;
+    if (q >= QW * QH) return;
+    const int qy = q / QW, qx = q % QW;
+    const size_t P = (size_t)H * W;
+    const uint8_t *src = hr_tmp + (size_t)slot * 3 * P;
+    uint8_t *dst = jobs[job].hr;
+    const size_t i00 = (size_t)(2 * qy) * W + 2 * qx, i10 = i00 + W;
+    *reinterpret_cast<uint16_t *>(dst + i00) = *reinterpret_cast<const uint16_t *>(src + i00);
+    *reinterpret_cast<uint16_t *>(dst + i10) = *reinterpret_cast<const uint16_t *>(src + i10);
+    for (int c = 1; c < 3; c++) {
+        const uint8_t *S = src + c * P;
+        const int v = S[i00] + S[i00 + 1] + S[i10] + S[i10 + 1] + 2;
+        dst[P + (size_t)(c - 1) * (P / 4) + (size_t)qy * QW + qx] = (uint8_t)(v >> 2);
+    }
 }
 
 // ------------------------------------------------------------------ host side
@@ -1563,17 +1598,18 @@ static size_t band_floats(int h, int w, int C, int s) {  // out-of-frame u posit
     return (2 * (W + 2) + 2 * H) * C + (2 * W + 2 * (H - 2)) * 3;
 }
 
-size_t sr_arena_bytes(int h, int w, int C, int s, int nb) {
+size_t sr_arena_bytes(int h, int w, int C, int s, int nb, int fmt) {
     const size_t px = (size_t)h * w * nb;
     size_t b = px * 8 * 2;                   // x0 (channel group 0 of the head input)
     b += 3 * px * C * 2;                     // h0, hb, tb
     b += band_floats(h, w, C, s) * 4 * nb;   // border bands
     b += (size_t)h * 3 * ((w + 15) / 16 * 16) * nb;  // lr8
-    return b + 6 * 256;
+    if (fmt == NS_FMT_I420) b += (size_t)3 * s * s * px;  // hr_tmp
+    return b + 7 * 256;
 }
 
-int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) {
-    a->h = h; a->w = w; a->C = C; a->s = s; a->nb = nb;
+int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, int fmt, uint8_t *mem) {
+    a->h = h; a->w = w; a->C = C; a->s = s; a->nb = nb; a->fmt = fmt;
     const size_t px = (size_t)h * w * nb;
     auto take = [&](size_t bytes) {
         uint8_t *p = mem;
@@ -1587,6 +1623,7 @@ int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem) 
     a->band = reinterpret_cast<float *>(take(band_floats(h, w, C, s) * 4 * nb));
     a->wp = (w + 15) / 16 * 16;
     a->lr8 = take((size_t)h * 3 * a->wp * nb);
+    a->hr_tmp = fmt == NS_FMT_I420 ? take((size_t)3 * s * s * px) : nullptr;
     int rc = 0;
     rc |= make_lr8_map(&a->tm_lr8, a->lr8, h, a->wp, nb);
     rc |= make_act_map(&a->tm_x0, a->x0, h, w, 8, nb, kHalo);
@@ -1665,11 +1702,15 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     {
         dim3 g((h * w + 255) / 256, nj);
         KScope ks(F_SR_PREP, st);
-        k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp);
+        k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp, a->fmt);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     ConvArgs base{};
     base.H = h; base.W = w; base.j0 = j0; base.jobs = jobs; base.job_count = job_count; base.C = C; base.s = s;
+    base.hr_tmp = a->hr_tmp;  // NS_FMT_I420: full-resolution output, packed to 4:2:0 at the end
+    base.lr8 = a->lr8;        // the u8 net-input planes (the upsampler's bilinear skip)
+    base.wp = a->wp;
+    base.hr_tmp_frame = (size_t)3 * h * s * w * s;
     auto L = [&](int l) { return model_layer(n_blocks, C, s, l); };
     {   // head: conv(x; W_head) -> h0
         ConvArgs g = base; LayerShape ls = L(0);
@@ -1719,7 +1760,14 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
         else if (s == 3) k_uptail_ext_u<C, 3><<<g1, C * 3, 0, st>>>(jobs, j0, job_count, endout, h, w, cs.aux_off, a->band);
         else k_uptail_ext_u<C, 4><<<g1, C * 4, 0, st>>>(jobs, j0, job_count, endout, h, w, cs.aux_off, a->band);
         k_uptail_ring<<<g2, 128, 0, st>>>(jobs, j0, job_count, h, w, C, s, cs.aux_off, a->band,
-                                          a->band + (size_t)a->nb * next * C);
+                                          a->band + (size_t)a->nb * next * C, a->lr8, a->wp, a->hr_tmp);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    }
+    if (a->fmt == NS_FMT_I420) {  // full-resolution HR -> 4:2:0 (reading R10)
+        KScope ks(F_SR_TAIL, st);
+        const int H = h * s, W = w * s;
+        dim3 g((H / 2 * (W / 2) + 255) / 256, nj);
+        k_pack420<<<g, 256, 0, st>>>(jobs, j0, job_count, H, W, a->hr_tmp);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
     }
     return cudaSuccess;

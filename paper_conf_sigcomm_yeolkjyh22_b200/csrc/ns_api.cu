@@ -158,6 +158,14 @@ static int host_groups() {
 
 // SR batch (jobs per arena); NS_SR_BATCH in the environment overrides it
 // (tuning experiments only)
+// stream parts of the SR / reconstruction overlap (1 = off); NS_OVERLAP_PARTS in
+// the environment overrides it (tuning experiments only)
+static int overlap_parts_default() {
+    const char *e = getenv("NS_OVERLAP_PARTS");
+    const int v = e ? atoi(e) : 0;
+    return v > 0 ? v : 1;
+}
+
 static int sr_batch_default() {
     const char *e = getenv("NS_SR_BATCH");
     const int v = e ? atoi(e) : 0;
@@ -165,7 +173,7 @@ static int sr_batch_default() {
 }
 
 struct ArenaEntry {
-    int h, w, C, s, idx;   // idx: 0 / 1, the two arenas SR batches alternate between
+    int h, w, C, s, fmt, idx;   // idx: 0 / 1, the two arenas SR batches alternate between
     SrArena a;
 };
 }  // namespace
@@ -206,6 +214,9 @@ struct ns_ctx {
     // the pool on first use and grown (bump) if a later call needs more
     cudaStream_t cst = nullptr;
     cudaStream_t sst = nullptr;          // second SR stream: odd batches, so one batch's tail overlaps the next
+    cudaStream_t rst = nullptr;          // reconstruction stream of the SR / reconstruction overlap
+    cudaEvent_t ev_part[2] = {}, ev_rjoin = nullptr;
+    int overlap_parts = overlap_parts_default();
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     cudaEvent_t ev_copied[2] = {}, ev_free[2] = {};
     bool hin_used[2] = {};
@@ -307,6 +318,10 @@ extern "C" ns_status ns_ctx_create(int device, size_t pool_bytes, ns_ctx **out) 
     c->lr_len = (uint32_t *)pool_take(c, sizeof(uint32_t) * kMaxJobs);
     if ((e = cudaStreamCreateWithFlags(&c->cst, cudaStreamNonBlocking)) != cudaSuccess ||
         (e = cudaStreamCreateWithFlags(&c->sst, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&c->rst, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&c->ev_part[0], cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&c->ev_part[1], cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&c->ev_rjoin, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming)) != cudaSuccess) {
         ns_ctx_destroy(c);
@@ -337,6 +352,10 @@ extern "C" ns_status ns_ctx_destroy(ns_ctx *c) {
     hybrid_destroy(c->hybrid);
     if (c->cst) cudaStreamDestroy(c->cst);
     if (c->sst) cudaStreamDestroy(c->sst);
+    if (c->rst) cudaStreamDestroy(c->rst);
+    for (int i = 0; i < 2; i++)
+        if (c->ev_part[i]) cudaEventDestroy(c->ev_part[i]);
+    if (c->ev_rjoin) cudaEventDestroy(c->ev_rjoin);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
     if (c->ev_join) cudaEventDestroy(c->ev_join);
     if (c->pool) cudaFree(c->pool);
@@ -456,6 +475,17 @@ extern "C" int ns_profile_read(ns_prof_entry *out, int max) {
 
 // ------------------------------------------------------------------ validation
 static bool al16(const void *p) { return ((uintptr_t)p & 15u) == 0; }
+// elements per LR / residual frame and bytes per HR frame (all planes)
+static size_t lr_frame_elems(const ns_chunk &k) {
+    const size_t p = (size_t)k.h * k.w;
+    return k.format == NS_FMT_I420 ? p * 3 / 2 : 3 * p;
+}
+static size_t hr_frame_bytes(const ns_chunk &k) {
+    const size_t p = (size_t)k.h * k.scale * k.w * k.scale;
+    return k.format == NS_FMT_I420 ? p * 3 / 2 : 3 * p;
+}
+// SR shape group: (h, w, C, s, B, format)
+typedef std::tuple<int, int, int, int, int, int> GroupKey;
 
 static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n_out) {
     if (!ch) return fail(NS_EINVAL, "chunks is NULL");
@@ -471,6 +501,8 @@ static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n
             return fail(NS_EINVAL, "chunk %d: w=%d h=%d must be positive multiples of 8", s, c.w, c.h);
         if (c.w > 8192 || c.h > 8192) return fail(NS_EINVAL, "chunk %d: w/h > 8192", s);
         if (c.scale < 2 || c.scale > 4) return fail(NS_EINVAL, "chunk %d: scale %d not in {2,3,4}", s, c.scale);
+        if (c.format != NS_FMT_444 && c.format != NS_FMT_I420)
+            return fail(NS_EINVAL, "chunk %d: format %d not NS_FMT_444 / NS_FMT_I420", s, c.format);
         if (!c.lr || !c.res || !c.mv || !c.type) return fail(NS_EINVAL, "chunk %d: lr/res/mv/type must be non-NULL", s);
         if (!al16(c.res) || !al16(c.lr) || !al16(c.mv)) return fail(NS_EINVAL, "chunk %d: lr/res/mv must be 16-B aligned", s);
         if (c.gt && !al16(c.gt)) return fail(NS_EINVAL, "chunk %d: gt must be 16-B aligned", s);
@@ -578,6 +610,9 @@ static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint
         d.job_cap = pl.job_cap ? pl.job_cap[s] : INT32_MAX;
         d.job_goff = pl.job_goff ? pl.job_goff[s] : 0;
         d.use_res_size = use_res_size ? 1 : 0;
+        d.fmt = k.format;
+        d.lr_frame = (int64_t)lr_frame_elems(k);
+        d.hr_frame = (int64_t)hr_frame_bytes(k);
         d.acache = pl.acache ? pl.acache[s] : nullptr;
         d.acache_stride = pl.acache_stride ? pl.acache_stride[s] : 0;
         sd[s] = d;
@@ -643,7 +678,7 @@ static ns_status check_params(const ns_select_params *p, int S, int n) {
 static ns_status run_select(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n, const ns_select_params *p,
                             int64_t *gain, int32_t *rank, uint8_t *is_anchor, cudaStream_t st) {
     int maxv = 0;
-    for (int s = 0; s < S; s++) maxv = std::max(maxv, 3 * ch[s].h * ch[s].w / 8);
+    for (int s = 0; s < S; s++) maxv = std::max(maxv, (int)(lr_frame_elems(ch[s]) / 8));
     NS_CUDA(launch_score(g.d_sd, S, n, maxv, c->score, st));
     if (p->mode == NS_GIVEN_ANCHORS) {  // decided by ns_select_merge across GPUs
         if (is_anchor != p->anchor_in)
@@ -696,13 +731,13 @@ extern "C" ns_status ns_select_merge(ns_ctx *c, int S, int n, const int64_t *gai
 }
 
 // ------------------------------------------------------------------ SR
-static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int idx, const SrArena **out) {
+static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int fmt, int idx, const SrArena **out) {
     for (auto &e : c->arenas)
-        if (e.h == h && e.w == w && e.C == C && e.s == s && e.idx == idx) {
+        if (e.h == h && e.w == w && e.C == C && e.s == s && e.fmt == fmt && e.idx == idx) {
             *out = &e.a;
             return NS_OK;
         }
-    const size_t bytes = sr_arena_bytes(h, w, C, s, c->sr_batch);
+    const size_t bytes = sr_arena_bytes(h, w, C, s, c->sr_batch, fmt);
     if (idx > 0 && c->used + bytes + 256 > c->pool_bytes) {  // no room for a second arena: one stream
         *out = nullptr;
         return NS_OK;
@@ -711,8 +746,8 @@ static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int idx, const
     if (!mem)
         return fail(NS_ENOMEM, "SR arena for %dx%d C%d x%d (%d jobs) needs %zu bytes; pool has %zu free", w, h, C, s,
                     c->sr_batch, bytes, c->pool_bytes - c->used);
-    ArenaEntry e{h, w, C, s, idx, {}};
-    if (sr_arena_init(&e.a, h, w, C, s, c->sr_batch, mem) != 0)
+    ArenaEntry e{h, w, C, s, fmt, idx, {}};
+    if (sr_arena_init(&e.a, h, w, C, s, c->sr_batch, fmt, mem) != 0)
         return fail(NS_ECUDA, "cuTensorMapEncodeTiled failed for the SR arena");
     c->arenas.push_back(e);
     *out = &c->arenas.back().a;
@@ -723,13 +758,15 @@ static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int idx, const
 // Batches alternate between `st` (arena 0) and the context's second SR stream
 // (arena 1), forked from and joined back into `st`: a batch's last wave (each
 // SR kernel's final partial wave of CTAs) overlaps the next batch's first.
-static ns_status run_sr_group(ns_ctx *c, int h, int w, int C, int s, int B, const SrJob *d_jobs, int max_jobs,
+static ns_status run_sr_group(ns_ctx *c, const GroupKey &key, const SrJob *d_jobs, int max_jobs,
                               const int32_t *job_count, cudaStream_t st) {
+    int h, w, C, s, B, fmt;
+    std::tie(h, w, C, s, B, fmt) = key;
     const SrArena *a[2] = {nullptr, nullptr};
-    ns_status r = get_arena(c, h, w, C, s, 0, &a[0]);
+    ns_status r = get_arena(c, h, w, C, s, fmt, 0, &a[0]);
     if (r != NS_OK) return r;
     const int nbatch = (max_jobs + a[0]->nb - 1) / a[0]->nb;
-    if (nbatch > 1 && (r = get_arena(c, h, w, C, s, 1, &a[1])) != NS_OK) return r;
+    if (nbatch > 1 && (r = get_arena(c, h, w, C, s, fmt, 1, &a[1])) != NS_OK) return r;
     const bool two = a[1] != nullptr;
     if (two) {
         NS_CUDA(cudaEventRecord(c->ev_fork, st));
@@ -760,11 +797,22 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
     cudaStream_t st = (cudaStream_t)stream;
     NS_CUDA(cudaSetDevice(c->device));
     // group by shape
-    std::map<std::tuple<int, int, int, int, int>, std::vector<int>> groups;
     for (int j = 0; j < n_jobs; j++)
-        groups[std::make_tuple(jobs[j].h, jobs[j].w, jobs[j].model->C, jobs[j].model->s, jobs[j].model->n_blocks)]
+        if (jobs[j].format != NS_FMT_444 && jobs[j].format != NS_FMT_I420)
+            return fail(NS_EINVAL, "job %d: format %d invalid", j, jobs[j].format);
+    std::map<GroupKey, std::vector<int>> groups;
+    for (int j = 0; j < n_jobs; j++)
+        groups[GroupKey(jobs[j].h, jobs[j].w, jobs[j].model->C, jobs[j].model->s, jobs[j].model->n_blocks,
+                        jobs[j].format)]
             .push_back(j);
     ns_status r = NS_OK;
+    for (auto &kv : groups) {  // every arena first: a pool that is too small fails with nothing launched
+        int h, w, C, s, B, fmt;
+        std::tie(h, w, C, s, B, fmt) = kv.first;
+        const SrArena *a0 = nullptr, *a1 = nullptr;
+        if ((r = get_arena(c, h, w, C, s, fmt, 0, &a0)) != NS_OK) return r;
+        if ((int)kv.second.size() > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, &a1)) != NS_OK) return r;
+    }
     for (auto &kv : groups) {
         const auto &idx = kv.second;
         if (idx.size() * sizeof(SrJob) > kStageBytes) return fail(NS_EINVAL, "too many SR jobs in one call");
@@ -777,9 +825,7 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
             hj[i] = SrJob{J.lr, J.hr_out, J.model->packed};
         }
         if ((r = stage_end(c, slot, idx.size() * sizeof(SrJob), st)) != NS_OK) return r;
-        int h, w, C, s, B;
-        std::tie(h, w, C, s, B) = kv.first;
-        r = run_sr_group(c, h, w, C, s, B, reinterpret_cast<const SrJob *>(dev), (int)idx.size(), nullptr, st);
+        r = run_sr_group(c, kv.first, reinterpret_cast<const SrJob *>(dev), (int)idx.size(), nullptr, st);
         stage_release(c, slot, st);
         if (r != NS_OK) return r;
     }
@@ -787,21 +833,46 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
 }
 
 // ------------------------------------------------------------------ reconstruct
-static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n,
-                                 const uint8_t *is_anchor, const uint8_t *const *asrc, cudaStream_t st) {
-    uint8_t *gsv = g.d_nxt ? c->gsv : nullptr;   // HR rings: GOLDEN saves
-    int mw[5] = {0, 0, 0, 0, 0}, mh[5] = {0, 0, 0, 0, 0};
+// Reconstruction in three parts so that the whole path can overlap it with SR:
+// the per-chunk descriptors (all streams), the frame steps of streams
+// [s0, s0 + cnt), and the chunk-end state (all streams).
+struct ReconGeom {
+    int mw[5] = {0, 0, 0, 0, 0}, mh[5] = {0, 0, 0, 0, 0}, i420[5] = {0, 0, 0, 0, 0};
     size_t maxhr = 0;
-    for (int s = 0; s < S; s++) {
-        mw[ch[s].scale] = std::max(mw[ch[s].scale], ch[s].w);
-        mh[ch[s].scale] = std::max(mh[ch[s].scale], ch[s].h);
-        maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
+};
+static ReconGeom recon_geom(const ns_chunk *ch, int s0, int cnt) {
+    ReconGeom gm;
+    for (int s = s0; s < s0 + cnt; s++) {
+        gm.mw[ch[s].scale] = std::max(gm.mw[ch[s].scale], ch[s].w);
+        gm.mh[ch[s].scale] = std::max(gm.mh[ch[s].scale], ch[s].h);
+        gm.i420[ch[s].scale] |= ch[s].format == NS_FMT_I420;
+        gm.maxhr = std::max(gm.maxhr, hr_frame_bytes(ch[s]));
     }
+    return gm;
+}
+static ns_status recon_prepare(ns_ctx *c, const Staged &g, int S, int n, const uint8_t *is_anchor,
+                               const uint8_t *const *asrc, cudaStream_t st) {
+    uint8_t *gsv = g.d_nxt ? c->gsv : nullptr;   // HR rings: GOLDEN saves
     NS_CUDA(launch_golden_index(g.d_sd, S, n, g.d_nxt, c->gold, gsv, st));
     NS_CUDA(launch_frame_desc(g.d_sd, S, n, is_anchor, g.d_hr, c->gold, gsv, asrc, c->fdesc, st));
-    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, S, n, f, mw, mh, st));
-    NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, gsv, maxhr, st));
     return NS_OK;
+}
+static ns_status recon_steps(ns_ctx *c, const ns_chunk *ch, int s0, int cnt, int n, cudaStream_t st) {
+    const ReconGeom gm = recon_geom(ch, s0, cnt);
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, cnt, n, f, gm.mw, gm.mh, gm.i420, st, s0));
+    return NS_OK;
+}
+static ns_status recon_finish(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n, cudaStream_t st) {
+    NS_CUDA(launch_state_copy(g.d_sd, S, n, g.d_hr, c->gold, g.d_nxt ? c->gsv : nullptr, recon_geom(ch, 0, S).maxhr,
+                              st));
+    return NS_OK;
+}
+static ns_status run_reconstruct(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n,
+                                 const uint8_t *is_anchor, const uint8_t *const *asrc, cudaStream_t st) {
+    ns_status r;
+    if ((r = recon_prepare(c, g, S, n, is_anchor, asrc, st)) != NS_OK) return r;
+    if ((r = recon_steps(c, ch, 0, S, n, st)) != NS_OK) return r;
+    return recon_finish(c, g, ch, S, n, st);
 }
 
 extern "C" ns_status ns_reconstruct_chunk(ns_ctx *c, const ns_chunk *ch, int S, const uint8_t *is_anchor,
@@ -838,15 +909,15 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
     // map, Key SR with fewer key frames than k) slots are assigned per group
     const bool fixed = topk && p->selector != NS_SEL_KEY;
     // SR shape groups and job slots (multi-stream batcher)
-    std::map<std::tuple<int, int, int, int, int>, int> gid;
-    std::vector<std::tuple<int, int, int, int, int>> gkey;
+    std::map<GroupKey, int> gid;
+    std::vector<GroupKey> gkey;
     std::vector<int> group(S), job_base(S), job_goff(S), gcount, goff;
     std::vector<int> gstreams;
     int64_t min_cost = INT64_MAX;
     if (!topk)
         for (int s = 0; s < S; s++) min_cost = std::min(min_cost, p->cost[s]);
     for (int s = 0; s < S; s++) {
-        auto key = std::make_tuple(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks);
+        const GroupKey key(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks, ch[s].format);
         auto it = gid.find(key);
         if (it == gid.end()) {
             it = gid.emplace(key, (int)gkey.size()).first;
@@ -889,11 +960,11 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
     ns_status r;
     if (total > 0)
         for (int gi = 0; gi < G; gi++) {
-            int h, w, C, s, B;
-            std::tie(h, w, C, s, B) = gkey[gi];
+            int h, w, C, s, B, fmt;
+            std::tie(h, w, C, s, B, fmt) = gkey[gi];
             const SrArena *a0 = nullptr, *a1 = nullptr;
-            if ((r = get_arena(c, h, w, C, s, 0, &a0)) != NS_OK) return r;
-            if (gcount[gi] > a0->nb && (r = get_arena(c, h, w, C, s, 1, &a1)) != NS_OK) return r;
+            if ((r = get_arena(c, h, w, C, s, fmt, 0, &a0)) != NS_OK) return r;
+            if (gcount[gi] > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, &a1)) != NS_OK) return r;
         }
     const bool any_ring = std::find(ring.begin(), ring.end(), 1) != ring.end();
     std::vector<uint8_t *> acache(S, nullptr);
@@ -902,9 +973,9 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
         std::vector<size_t> gbase(G), gstride(G);
         size_t need = 0;
         for (int gi = 0; gi < G; gi++) {
-            int h, w, C, s, B;
-            std::tie(h, w, C, s, B) = gkey[gi];
-            gstride[gi] = a256((size_t)3 * h * s * w * s);
+            int h, w, C, s, B, fmt;
+            std::tie(h, w, C, s, B, fmt) = gkey[gi];
+            gstride[gi] = a256((size_t)h * s * w * s * (fmt == NS_FMT_I420 ? 3 : 6) / 2);
             gbase[gi] = need;
             need += gstride[gi] * gcount[gi];
         }
@@ -943,7 +1014,7 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
     }
     if (gathered && lg) {  // exact in top-k mode (k frames per stream); upper bound otherwise
         uint64_t b = 0;
-        for (int s = 0; s < S; s++) b += (uint64_t)3 * ch[s].h * ch[s].w * (fixed ? p->k : 0);
+        for (int s = 0; s < S; s++) b += (uint64_t)lr_frame_elems(ch[s]) * (fixed ? p->k : 0);
         if (!fixed) b = (uint64_t)total * lg->stride;
         *gathered += b;
     }
@@ -978,19 +1049,45 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
                                    lg ? lg->stride : 0, c->lr_src, c->lr_len);
             if (e == cudaSuccess && lg) e = launch_lr_gather(c->jobs, c->lr_src, c->lr_len, total, lg->stride, st);
             if (e != cudaSuccess) { r = cuda_fail(e, "compact"); break; }
-            for (int gi = 0; gi < G && r == NS_OK; gi++) {
-                int h, w, C, s, B;
-                std::tie(h, w, C, s, B) = gkey[gi];
-                r = run_sr_group(c, h, w, C, s, B, c->jobs + goff[gi], gcount[gi], fixed ? nullptr : c->job_count + gi,
-                                 st);
+        }
+        const uint8_t *const *asrc = any_ring && total > 0 ? c->asrc : nullptr;
+        // SR of stream part p overlaps the reconstruction of part p - 1 (fixed top-k
+        // job slots are contiguous per stream in each shape group): the frame steps
+        // of a part run on the context's reconstruction stream once its anchors
+        // are done; the chunk-end state and the stats wait for all of them.
+        const int parts = (fixed && total > 0) ? std::max(1, std::min(c->overlap_parts, S)) : 1;
+        if (parts == 1) {
+            for (int gi = 0; gi < G && r == NS_OK && total > 0; gi++)
+                r = run_sr_group(c, gkey[gi], c->jobs + goff[gi], gcount[gi], fixed ? nullptr : c->job_count + gi, st);
+            if (r != NS_OK) break;
+            if ((r = run_reconstruct(c, g, ch, S, n, anchor, asrc, st)) != NS_OK) break;
+        } else {
+            if ((r = recon_prepare(c, g, S, n, anchor, asrc, st)) != NS_OK) break;
+            for (int pi = 0; pi < parts && r == NS_OK; pi++) {
+                const int s0 = (int)((int64_t)S * pi / parts), s1 = (int)((int64_t)S * (pi + 1) / parts);
+                for (int gi = 0; gi < G && r == NS_OK; gi++) {  // this part's job range of group gi
+                    int lo = INT32_MAX, hi = -1;
+                    for (int s = s0; s < s1; s++)
+                        if (group[s] == gi) {
+                            lo = std::min(lo, job_base[s]);
+                            hi = std::max(hi, job_base[s] + p->k);
+                        }
+                    if (hi > lo) r = run_sr_group(c, gkey[gi], c->jobs + lo, hi - lo, nullptr, st);
+                }
+                if (r != NS_OK) break;
+                cudaError_t e = cudaEventRecord(c->ev_part[pi & 1], st);
+                if (e == cudaSuccess) e = cudaStreamWaitEvent(c->rst, c->ev_part[pi & 1], 0);
+                if (e != cudaSuccess) { r = cuda_fail(e, "overlap fork"); break; }
+                r = recon_steps(c, ch, s0, s1 - s0, n, c->rst);
             }
             if (r != NS_OK) break;
+            NS_CUDA(cudaEventRecord(c->ev_rjoin, c->rst));
+            NS_CUDA(cudaStreamWaitEvent(st, c->ev_rjoin, 0));
+            if ((r = recon_finish(c, g, ch, S, n, st)) != NS_OK) break;
         }
-        if ((r = run_reconstruct(c, g, ch, S, n, anchor, any_ring && total > 0 ? c->asrc : nullptr, st)) != NS_OK)
-            break;
         if (stats) {
             size_t maxhr = 0;
-            for (int s = 0; s < S; s++) maxhr = std::max(maxhr, (size_t)3 * ch[s].w * ch[s].scale * ch[s].h * ch[s].scale);
+            for (int s = 0; s < S; s++) maxhr = std::max(maxhr, hr_frame_bytes(ch[s]));
             bool any_gt = false;
             for (int s = 0; s < S; s++) any_gt |= ch[s].gt != nullptr;
             cudaError_t e = launch_stats(g.d_sd, S, n, anchor, c->score, g.d_hr, any_gt ? maxhr : 0, stats, st);
@@ -1029,7 +1126,8 @@ static bool host_mapped(const void *p) {
 // bytes of one stream's uploaded inputs in a staging buffer (256-B aligned pieces)
 static size_t host_stream_bytes(const ns_chunk &k) {
     const size_t n = (size_t)k.n_frames, px = (size_t)k.h * k.w;
-    return a256(n * 3 * px * 2) + a256(n * (px / 64) * sizeof(ns_block_mv)) + a256(n) + (k.res_size ? a256(n * 4) : 0);
+    return a256(n * lr_frame_elems(k) * 2) + a256(n * (px / 64) * sizeof(ns_block_mv)) + a256(n) +
+           (k.res_size ? a256(n * 4) : 0);
 }
 
 extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int S, const ns_select_params *p,
@@ -1078,13 +1176,13 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
         cap = std::max(cap, b);
         max_jobs = std::max(max_jobs, jobs);
     }
-    for (int s = 0; s < S; s++) lr_stride = std::max(lr_stride, a256((size_t)3 * ch[s].h * ch[s].w));
+    for (int s = 0; s < S; s++) lr_stride = std::max(lr_stride, a256(lr_frame_elems(ch[s])));
     if (!topk) {  // one group; job slots as enhance_impl lays them out: per SR shape, min(streams * n, budget / min cost)
         int64_t min_cost = INT64_MAX;
         for (int s = 0; s < S; s++) min_cost = std::min(min_cost, p->cost[s]);
-        std::map<std::tuple<int, int, int, int, int>, int> cnt;
+        std::map<GroupKey, int> cnt;
         for (int s = 0; s < S; s++)
-            cnt[std::make_tuple(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks)]++;
+            cnt[GroupKey(ch[s].h, ch[s].w, ch[s].model->C, ch[s].scale, ch[s].model->n_blocks, ch[s].format)]++;
         int64_t t = 0;
         for (auto &kv : cnt) t += std::min<int64_t>((int64_t)kv.second * n, p->budget / std::max<int64_t>(min_cost, 1));
         max_jobs = (int)std::min<int64_t>(t, kMaxJobs);
@@ -1117,7 +1215,7 @@ extern "C" ns_status ns_enhance_streams_host(ns_ctx *c, const ns_chunk *ch, int 
             const ns_chunk &k = ch[g0 + i];
             const size_t nf = (size_t)k.n_frames, px = (size_t)k.h * k.w;
             dch[i] = k;
-            const size_t rb = nf * 3 * px * 2, mb = nf * (px / 64) * sizeof(ns_block_mv);
+            const size_t rb = nf * lr_frame_elems(k) * 2, mb = nf * (px / 64) * sizeof(ns_block_mv);
             NS_CUDA(cudaMemcpyAsync(dst, k.res, rb, cudaMemcpyHostToDevice, c->cst));
             dch[i].res = reinterpret_cast<const int16_t *>(dst);
             dst += a256(rb);
@@ -1195,8 +1293,8 @@ extern "C" ns_status ns_encode_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
             pos += sizeof(hd);
             if (hd.anchor) {
                 const size_t cap = (!full && pos <= out_cap) ? out_cap - pos : 0;
-                const int rc = hybrid_encode_frame(c->hybrid, hr_out[(size_t)s * n + f], H, W, q[s], out + pos,
-                                                   cap, &len, st, err, sizeof(err));
+                const int rc = hybrid_encode_frame(c->hybrid, hr_out[(size_t)s * n + f], H, W, ch[s].format, q[s],
+                                                   out + pos, cap, &len, st, err, sizeof(err));
                 if (rc < 0) return fail(NS_ECUDA, "%s", err);
                 if (rc > 0) full = true;
             }

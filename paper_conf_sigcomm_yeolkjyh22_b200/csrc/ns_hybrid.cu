@@ -79,8 +79,8 @@ int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *er
 // Encodes one HR frame [3][H][W] (device, planar) at `quality` and appends the
 // bitstream at dst (host) if it fits in cap; *len = its size.  Returns 0, 1 if
 // it does not fit (len still set), -1 on an nvjpeg error.
-int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int quality, uint8_t *dst, size_t cap,
-                        size_t *len, cudaStream_t stream, char *err, size_t errlen) {
+int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int fmt, int quality, uint8_t *dst,
+                        size_t cap, size_t *len, cudaStream_t stream, char *err, size_t errlen) {
     nvjpegStatus_t s = NVJPEG_STATUS_SUCCESS;
     if (quality != e->quality) {
         s = nvjpegEncoderParamsSetQuality(e->prm, quality, stream);
@@ -92,11 +92,22 @@ int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int q
     }
     nvjpegImage_t img{};
     const size_t plane = (size_t)H * W;
-    for (int c = 0; c < 3; c++) {
-        img.channel[c] = const_cast<uint8_t *>(hr) + c * plane;
-        img.pitch[c] = (size_t)W;
+    if (fmt == NS_FMT_I420) {  // the codec's own planes: Y, then U, V at half resolution, coded as 4:2:0
+        img.channel[0] = const_cast<uint8_t *>(hr);
+        img.channel[1] = const_cast<uint8_t *>(hr) + plane;
+        img.channel[2] = const_cast<uint8_t *>(hr) + plane + plane / 4;
+        img.pitch[0] = (size_t)W;
+        img.pitch[1] = img.pitch[2] = (size_t)W / 2;
+        s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_420, stream);
+        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncodeYUV(e->h, e->st, e->prm, &img, NVJPEG_CSS_420, W, H, stream);
+        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_444, stream);
+    } else {
+        for (int c = 0; c < 3; c++) {
+            img.channel[c] = const_cast<uint8_t *>(hr) + c * plane;
+            img.pitch[c] = (size_t)W;
+        }
+        s = nvjpegEncodeImage(e->h, e->st, e->prm, &img, NVJPEG_INPUT_RGB, W, H, stream);
     }
-    s = nvjpegEncodeImage(e->h, e->st, e->prm, &img, NVJPEG_INPUT_RGB, W, H, stream);
     if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncodeRetrieveBitstream(e->h, e->st, nullptr, len, stream);
     if (s != NVJPEG_STATUS_SUCCESS) {
         snprintf(err, errlen, "nvjpegEncodeImage %dx%d: %s", W, H, nvj_err(s));

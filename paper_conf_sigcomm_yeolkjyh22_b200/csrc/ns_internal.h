@@ -31,6 +31,9 @@ struct StreamDesc {
     int32_t job_cap;       // slots of its group; a given anchor map's anchors beyond it are demoted (ns.h)
     int32_t use_res_size;
     int32_t job_goff;      // first job slot of the stream's SR shape group
+    int32_t fmt;           // NS_FMT_444 | NS_FMT_I420
+    int64_t lr_frame;      // elements per LR / residual frame: 3 h w, or h w 3/2 (I420)
+    int64_t hr_frame;      // bytes per HR frame: 3 H W, or H W 3/2 (I420)
     uint8_t *acache;       // HR rings: the group's anchor cache (job slot j at acache + (j - job_goff) * stride)
     uint64_t acache_stride;
 };
@@ -53,7 +56,8 @@ struct __align__(16) FrameDesc {
     int32_t w, h;              // LR size
     int16_t s;                 // scale
     uint8_t anchor, key;       // is_anchor[f], type[f] == KEY
-    int32_t pad0, pad1, pad2;
+    int32_t fmt;               // NS_FMT_444 | NS_FMT_I420 (k_recon_step: luma only; k_recon_c420: chroma)
+    int32_t pad1, pad2;
 };
 static_assert(sizeof(FrameDesc) == 96, "FrameDesc is one 96-B record");
 
@@ -143,8 +147,11 @@ cudaError_t launch_golden_index(const StreamDesc *d_sd, int S, int n, const int1
 cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor,
                               uint8_t *const *d_hr_table, const int16_t *gold_idx, const uint8_t *gsv,
                               const uint8_t *const *asrc, FrameDesc *fd, cudaStream_t st);
+// max_lr_w / max_lr_h: [5] per scale; has_i420[5]: a 4:2:0 stream of that scale
+// (its chroma planes then step in k_recon_c420 in the same frame step)
+// streams [s0, s0 + S) of the frame-descriptor table
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              cudaStream_t st, int s0 = 0);
+                              const int *has_i420, cudaStream_t st, int s0 = 0);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, const uint8_t *gsv, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,
@@ -154,6 +161,8 @@ cudaError_t launch_repack(const uint16_t *blob, int n_blocks, int C, int s, uint
 // SR (k_sr.cu)
 struct SrArena {
     int h, w, C, s, nb;        // shape and batch capacity (jobs per batch)
+    int fmt;                   // NS_FMT_444 | NS_FMT_I420 (input conversion, output packing)
+    uint8_t *hr_tmp;           // I420: the net's full-resolution HR output [job][3][sH][sW], packed to 4:2:0 after
     uint16_t *x0, *h0, *hb, *tb;       // bf16 activations, layout [job][H][C/8][W][8]
     float *band;                       // border fix-up: u on the HR frame-edge bands
     uint8_t *lr8;                      // u8 LR copy [job][H][3][wp] (upsampler skip taps), wp = W rounded to 16
@@ -161,8 +170,8 @@ struct SrArena {
     CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_tb5, tm_hb5;   // *5: 132-px boxes (5x5 conv)
     CUtensorMap tm_lr8;                // box: kLrBoxW px x 3 planes x 3 rows
 };
-size_t sr_arena_bytes(int h, int w, int C, int s, int nb);
-int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, uint8_t *mem);  // 0 ok
+size_t sr_arena_bytes(int h, int w, int C, int s, int nb, int fmt);
+int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, int fmt, uint8_t *mem);  // 0 ok
 // Runs the whole net on jobs [j0, j0+nj) of a device job table (all of one
 // shape).  job_count (device) may be NULL; otherwise CTAs of jobs >= *job_count exit.
 cudaError_t sr_run_batch(const SrArena *a, int n_blocks, const SrJob *jobs, int j0, int nj,
@@ -194,8 +203,8 @@ int hybrid_quality_table2(int n_anchors, int n_frames);
 struct HybridEncoder;
 int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *err, size_t errlen);
 void hybrid_destroy(HybridEncoder *e);
-int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int quality, uint8_t *dst, size_t cap,
-                        size_t *len, cudaStream_t stream, char *err, size_t errlen);
+int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int fmt, int quality, uint8_t *dst,
+                        size_t cap, size_t *len, cudaStream_t stream, char *err, size_t errlen);
 
 // Kernel families for ns_launch_count / ns_profile_read.
 enum Fam { F_SCORE = 0, F_SELECT, F_GLOBAL, F_COMPACT, F_SR_PREP, F_SR_HEAD, F_SR_BODY, F_SR_END, F_SR_UP,

@@ -65,6 +65,8 @@ def gather_stats(stats, group=None):
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
         return stats
+    if dist.get_backend(group) == "gloo":
+        stats = stats.cpu()
     parts = [torch.zeros_like(stats) for _ in range(dist.get_world_size(group))]
     dist.all_gather(parts, stats.contiguous(), group=group)
     return torch.cat(parts)

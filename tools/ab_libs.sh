@@ -2,7 +2,7 @@
 # A/B of library variants on one box: bench (device path only) per NS_LIB; prints value and family ms.
 # usage: LIBS="default tools/bin/lib_a.so ..." bash tools/ab_libs.sh
 for L in ${LIBS:-default}; do
-  unset NS_SR_BATCH
+  unset NS_SR_BATCH NS_OVERLAP_PARTS NS_HOST_GROUPS
   case "$L" in
     default) unset NS_LIB ;;
     env:*) unset NS_LIB; export ${L#env:} ;;
