@@ -214,7 +214,7 @@ class DeviceChunk:
 
     @staticmethod
     def pinned_from_numpy(lr, res, mv, types, w, h, scale, res_size=None, model=None,
-                          hr_last=None, hr_golden=None) -> "DeviceChunk":
+                          hr_last=None, hr_golden=None, format=NS_FMT_444) -> "DeviceChunk":
         """Host chunk for ns_enhance_streams_host: inputs in page-locked host
         memory (torch pinned tensors); hr_last / hr_golden stay on the device."""
         import torch
@@ -222,7 +222,7 @@ class DeviceChunk:
         t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
         rs = None if res_size is None else t(np.asarray(res_size).astype(np.int32))
         return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
-                           model=model, res_size=rs, hr_last=hr_last, hr_golden=hr_golden)
+                           model=model, res_size=rs, hr_last=hr_last, hr_golden=hr_golden, format=format)
 
 
 class Model:
@@ -354,21 +354,32 @@ class Context:
     def encode_anchors(self, chunks, is_anchor, hr_out, quality=0, out_cap=None, stream=None):
         """ns_encode_anchors (§6.1 hybrid encoding): JPEG of every anchor +
         per-frame headers.  is_anchor: [S, n] array-like (host copy is made);
-        hr_out as for enhance_streams.  Returns a list of S `bytes` packages."""
+        hr_out as for enhance_streams.  Returns a list of S `bytes` packages.
+        The host buffer starts at a quarter of the anchors' raw size and is
+        grown to the size the library reports if that is too small."""
         arr = self._chunks(chunks)
         tab = self._hr_table(hr_out)
         ia = np.ascontiguousarray(np.asarray(is_anchor, dtype=np.uint8))
         S = len(chunks)
+        hdr = ctypes.sizeof(NsHybridHeader)
+        grow = out_cap is None
         if out_cap is None:
-            px = sum(c.n * 3 * (c.scale * c.h) * (c.scale * c.w) for c in chunks)
-            out_cap = px // 2 + 64 * S * chunks[0].n + (1 << 20)
-        buf = (ctypes.c_uint8 * out_cap)()
+            raw = sum(int(ia[i].sum()) * (3 if c.format == NS_FMT_444 else 1.5) * (c.scale * c.h) * (c.scale * c.w)
+                      for i, c in enumerate(chunks))
+            out_cap = int(raw // 4) + hdr * S * int(ia.shape[1]) + (1 << 16)
         lens = (ctypes.c_size_t * S)()
-        _check(lib().ns_encode_anchors(self.handle, arr, S, ia.ctypes.data, tab, int(quality), buf, out_cap, lens,
-                                       _stream(stream)), "ns_encode_anchors")
-        raw, out, pos = bytes(buf), [], 0
+        for attempt in range(2):
+            buf = np.empty(max(out_cap, 1), np.uint8)
+            rc = lib().ns_encode_anchors(self.handle, arr, S, ia.ctypes.data, tab, int(quality), buf.ctypes.data,
+                                         out_cap, lens, _stream(stream))
+            if rc == NS_ENOMEM and grow and attempt == 0 and sum(lens) > out_cap:
+                out_cap = int(sum(lens)) + (1 << 16)
+                continue
+            _check(rc, "ns_encode_anchors")
+            break
+        out, pos = [], 0
         for s in range(S):
-            out.append(raw[pos:pos + lens[s]])
+            out.append(buf[pos:pos + lens[s]].tobytes())
             pos += lens[s]
         return out
 

@@ -7,6 +7,7 @@
 // Host-side glue; the encoder object lives in the context (created on first
 // use, not on the hot path).
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <nvjpeg.h>
 #include "ns_internal.h"
@@ -66,7 +67,10 @@ int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *er
     if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsCreate(e->h, &e->prm, stream);
     // the three planes are full resolution (reading Z18): keep them so
     if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_444, stream);
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetOptimizedHuffman(e->prm, 1, stream);
+    // optimized Huffman tables cost a second pass over the coefficients; off unless asked for
+    // (NS_JPEG_OPT_HUFFMAN=1: a tuning experiment)
+    const char *oh = getenv("NS_JPEG_OPT_HUFFMAN");
+    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetOptimizedHuffman(e->prm, oh && atoi(oh) ? 1 : 0, stream);
     if (s != NVJPEG_STATUS_SUCCESS) {
         snprintf(err, errlen, "nvjpeg encoder setup: %s", nvj_err(s));
         hybrid_destroy(e);

@@ -119,3 +119,40 @@ def test_host_path_rejects_pageable_memory(ctx):
     with pytest.raises(ns.NsError) as ei:
         ctx.enhance_streams_host([hc], hr, k=1)
     assert ei.value.status == ns.NS_EINVAL and "page-locked" in str(ei.value)
+
+
+def test_host_path_i420_matches_device_path(ctx):
+    """4:2:0 streams (NS_FMT_I420) through the host-input path: the uploaded
+    residual frames and the gathered anchor LR frames have the 4:2:0 sizes;
+    results equal the device-input path byte for byte."""
+    n, k = 10, 2
+    cs = [synth.make_chunk_i420(7300 + i, w, h, s, n, types=synth.default_types(n, 4))
+          for i, (w, h, s) in enumerate([(64, 32, 2), (48, 24, 3), (64, 32, 2)])]
+    outs = {}
+    for path in ("device", "host"):
+        dcs, hrs = [], []
+        for i, c in enumerate(cs):
+            m = ctx.model(1, 16, c.scale)
+            m.set_weights(synth.make_weights(7300 + i, 1, 16, c.scale))
+            size = c.scale * c.h * c.scale * c.w * 3 // 2
+            last = torch.zeros(size, dtype=torch.uint8, device=DEV)
+            gold = torch.zeros(size, dtype=torch.uint8, device=DEV)
+            mk = ns.DeviceChunk.from_numpy if path == "device" else ns.DeviceChunk.pinned_from_numpy
+            kw = dict(device=DEV) if path == "device" else {}
+            dcs.append(mk(c.lr, c.res, c.mv, c.type, c.w, c.h, c.scale, model=m, hr_last=last, hr_golden=gold,
+                          format=ns.NS_FMT_I420, **kw))
+            hrs.append([torch.full((size,), 7, dtype=torch.uint8, device=DEV) for _ in range(n)])
+        ia = torch.zeros((len(cs), n), dtype=torch.uint8, device=DEV)
+        if path == "device":
+            ctx.enhance_streams(dcs, hrs, is_anchor_out=ia, k=k)
+        else:
+            ctx.enhance_streams_host(dcs, hrs, is_anchor_out=ia, k=k)
+        torch.cuda.synchronize()
+        outs[path] = (ia.cpu().numpy(), [np.stack([t.cpu().numpy() for t in r]) for r in hrs],
+                      [d.hr_last.cpu().numpy() for d in dcs])
+    d, h = outs["device"], outs["host"]
+    assert np.array_equal(d[0], h[0])
+    for a, b in zip(d[1], h[1]):
+        assert np.array_equal(a, b)
+    for a, b in zip(d[2], h[2]):
+        assert np.array_equal(a, b)
