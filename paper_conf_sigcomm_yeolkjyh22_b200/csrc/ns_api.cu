@@ -1276,11 +1276,20 @@ extern "C" ns_status ns_encode_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
     cudaStream_t st = (cudaStream_t)stream;
     char err[256];
     if (!c->hybrid && hybrid_create(c->device, st, &c->hybrid, err, sizeof(err)) != 0) return fail(NS_ECUDA, "%s", err);
-    size_t pos = 0;
+    // every anchor, stream-major, frame order
+    std::vector<HybridFrame> fr;
+    for (int s = 0; s < S; s++)
+        for (int f = 0; f < n; f++)
+            if (is_anchor[(size_t)s * n + f])
+                fr.push_back(HybridFrame{hr_out[(size_t)s * n + f], ch[s].h * ch[s].scale, ch[s].w * ch[s].scale,
+                                         ch[s].format, q[s]});
+    std::vector<std::vector<uint8_t>> bits;
+    if (hybrid_encode_frames(c->hybrid, (int)fr.size(), fr.data(), bits, st, err, sizeof(err)) != 0)
+        return fail(NS_ECUDA, "%s", err);
+    size_t pos = 0, ai = 0;
     bool full = false;
     for (int s = 0; s < S; s++) {
         const size_t start = pos;
-        const int H = ch[s].h * ch[s].scale, W = ch[s].w * ch[s].scale;
         for (int f = 0; f < n; f++) {
             ns_hybrid_header hd{};
             hd.magic = NS_HYBRID_MAGIC;
@@ -1288,20 +1297,16 @@ extern "C" ns_status ns_encode_anchors(ns_ctx *c, const ns_chunk *ch, int S, con
             hd.frame = (uint16_t)f;
             hd.anchor = is_anchor[(size_t)s * n + f] ? 1 : 0;
             hd.quality = hd.anchor ? (uint8_t)q[s] : 0;
-            size_t len = 0;
-            const size_t hpos = pos;
-            pos += sizeof(hd);
-            if (hd.anchor) {
-                const size_t cap = (!full && pos <= out_cap) ? out_cap - pos : 0;
-                const int rc = hybrid_encode_frame(c->hybrid, hr_out[(size_t)s * n + f], H, W, ch[s].format, q[s],
-                                                   out + pos, cap, &len, st, err, sizeof(err));
-                if (rc < 0) return fail(NS_ECUDA, "%s", err);
-                if (rc > 0) full = true;
+            const std::vector<uint8_t> *pl = hd.anchor ? &bits[ai++] : nullptr;
+            hd.bytes = pl ? (uint32_t)pl->size() : 0u;
+            const size_t need = sizeof(hd) + hd.bytes;
+            if (!full && pos + need <= out_cap) {
+                memcpy(out + pos, &hd, sizeof(hd));
+                if (pl && !pl->empty()) memcpy(out + pos + sizeof(hd), pl->data(), pl->size());
+            } else {
+                full = true;
             }
-            hd.bytes = (uint32_t)len;
-            if (!full && hpos + sizeof(hd) <= out_cap) memcpy(out + hpos, &hd, sizeof(hd));
-            else full = true;
-            pos += len;
+            pos += need;
         }
         out_len[s] = pos - start;
     }

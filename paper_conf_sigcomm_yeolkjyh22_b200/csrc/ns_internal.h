@@ -5,6 +5,7 @@
 #include <cstdint>
 #include <cstddef>
 #include <atomic>
+#include <vector>
 #include "../../include/ns.h"
 
 namespace ns {
@@ -203,8 +204,12 @@ int hybrid_quality_table2(int n_anchors, int n_frames);
 struct HybridEncoder;
 int hybrid_create(int device, cudaStream_t stream, HybridEncoder **out, char *err, size_t errlen);
 void hybrid_destroy(HybridEncoder *e);
-int hybrid_encode_frame(HybridEncoder *e, const uint8_t *hr, int H, int W, int fmt, int quality, uint8_t *dst,
-                        size_t cap, size_t *len, cudaStream_t stream, char *err, size_t errlen);
+struct HybridFrame {
+    const uint8_t *hr;   // HR frame planes (device)
+    int H, W, fmt, quality;
+};
+int hybrid_encode_frames(HybridEncoder *e, int n, const HybridFrame *fr, std::vector<std::vector<uint8_t>> &out,
+                         cudaStream_t stream, char *err, size_t errlen);
 
 // Kernel families for ns_launch_count / ns_profile_read.
 enum Fam { F_SCORE = 0, F_SELECT, F_GLOBAL, F_COMPACT, F_SR_PREP, F_SR_HEAD, F_SR_BODY, F_SR_END, F_SR_UP,
