@@ -50,25 +50,27 @@ def cfg_of(args):
     return c
 
 
-def workload_config(cfg, world, select="topk"):
+def workload_config(cfg, world, select="topk", fmt="444"):
     """The `config` object both arms print (same workload, same keys)."""
     S, s, w, h = cfg["streams"], cfg["scale"], cfg["w"], cfg["h"]
     sel = ("top-k per stream" if select == "topk" else
            f"global budget k*S*N = {cfg['k'] * S * world} anchors over all GPUs' streams (§5.2, NEXT-1)")
+    fm = "" if fmt == "444" else ", YUV 4:2:0 (NEXT-2)"
     return {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{s * w}x{s * h} x{s} streams per GPU, "
-                        f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} ({sel})",
+                        f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} ({sel}){fm}",
             "streams_per_gpu": S, "frames_per_step_per_gpu": S * cfg["n"], "parallelism": f"streams x{world}",
-            "select": select}
+            "select": select, "format": fmt}
 
 
 def _gen(a):
-    seed, w, h, s, n, alt = a
-    return synth.make_chunk(seed, w, h, s, n, types=synth.default_types(n, alt))
+    seed, w, h, s, n, alt = a[:6]
+    mk = synth.make_chunk_i420 if len(a) > 6 and a[6] == "i420" else synth.make_chunk
+    return mk(seed, w, h, s, n, types=synth.default_types(n, alt))
 
 
-def gen_pool(cfg, n_distinct, rank):
+def gen_pool(cfg, n_distinct, rank, fmt="444"):
     seeds = [1000 * 4 + rank * 100000 + i for i in range(n_distinct)]
-    args = [(sd, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"]) for sd in seeds]
+    args = [(sd, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"], fmt) for sd in seeds]
     procs = min(len(args), max(1, (os.cpu_count() or 1)))
     if procs > 1:
         import multiprocessing as mp
@@ -185,13 +187,14 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------- GPU arm
-def algorithmic(cfg, types, ia, S, n):
+def algorithmic(cfg, types, ia, S, n, fmt="444"):
     """Algorithmic FLOPs / bytes per kernel family over one step (DESIGN.md
     "Roofline"): the defined convs only; reconstruct = ref 3 B + write 3 B +
     residual 6/s^2 B + MV 0.125/s^2 B per HR pixel of a non-anchor inter frame,
     LR 3/s^2 B + write 3 B for a non-anchor KEY frame."""
     B, C, s, h, w = cfg["n_blocks"], cfg["n_ch"], cfg["scale"], cfg["h"], cfg["w"]
     px, hpx = h * w, h * w * s * s
+    pl = 1.5 if fmt == "i420" else 3.0   # planes' worth of samples per pixel (4:2:0: Y + U/4 + V/4)
     anchors = int(ia.sum())
     conv = lambda cin, cout: 2.0 * 9 * cin * cout
     # sr_up = the composed tail o shuffle o upsampler kernel: algorithmic FLOPs are
@@ -206,11 +209,11 @@ def algorithmic(cfg, types, ia, S, n):
             if ia[si, f]:
                 continue
             if types[si][f] == synth.NS_KEY:
-                rec_bytes += hpx * 3 + px * 3
+                rec_bytes += hpx * pl + px * pl
             else:
-                rec_bytes += hpx * 6 + px * 6 + px * 8 / 64.0
-    by = {"recon": rec_bytes, "score": S * n * px * 6.0, "state": S * 2 * 2 * hpx * 3.0,
-          "sr_prep": anchors * px * (3 + 32)}
+                rec_bytes += hpx * 2 * pl + px * 2 * pl + px * 8 / 64.0
+    by = {"recon": rec_bytes, "score": S * n * px * 2 * pl, "state": S * 2 * 2 * hpx * pl,
+          "sr_prep": anchors * px * (pl + 32)}
     return fl, by
 
 
@@ -233,6 +236,8 @@ def main():
                     help="global: §5.2 selection across all GPUs' streams (per-GPU gains, NCCL all_gather, "
                          "ns_select_merge, NS_GIVEN_ANCHORS) inside the timed step")
     ap.add_argument("--ring", type=int, default=3, help="config 5: HR frames per stream (ring)")
+    ap.add_argument("--format", default="444", choices=["444", "i420"],
+                    help="frame format of the streams (i420: YUV 4:2:0, NEXT-2)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N > 1 (gloo + NS_BENCH_SHARE_GPU=1: N ranks on one GPU)")
     ap.add_argument("--encode", action="store_true",
@@ -264,12 +269,14 @@ def main():
     P = min(args.distinct, S)
 
     t_gen = time.time()
-    pool = gen_pool(cfg, P, rank)
+    i420 = args.format == "i420"
+    pool = gen_pool(cfg, P, rank, args.format)
     t_gen = time.time() - t_gen
 
     host_pool = ns.Context.host_pool_bytes(w, h, n, k, S) if args.e2e_steps > 0 else 0
     # two SR arenas: batches alternate between two streams (ns_api.cu run_sr_group)
-    ctx = ns.Context(local, pool_bytes=int((2.4 * ns_arena_gb(cfg, args.sr_batch) + 2) * (1 << 30)) + host_pool)
+    ctx = ns.Context(local, pool_bytes=int((2.4 * ns_arena_gb(cfg, args.sr_batch, args.format) + 2) * (1 << 30)) +
+                     host_pool)
     # per-stream content-aware models: distinct weights per stream
     models = []
     for si in range(S):
@@ -277,8 +284,10 @@ def main():
         m.set_weights(synth.make_weights(4000 + rank * 100000 + si, B, C, s))
         models.append(m)
     # device inputs: P generated chunks, copied to S distinct device buffers
-    lr_d = torch.empty((S, n, 3, h, w), dtype=torch.uint8, device=dev)
-    res_d = torch.empty((S, n, 3, h, w), dtype=torch.int16, device=dev)
+    LRF = (h * w * 3 // 2,) if i420 else (3, h, w)      # one LR / residual frame
+    HRF = (H * W * 3 // 2,) if i420 else (3, H, W)      # one HR frame
+    lr_d = torch.empty((S, n) + LRF, dtype=torch.uint8, device=dev)
+    res_d = torch.empty((S, n) + LRF, dtype=torch.int16, device=dev)
     mv_d = torch.empty((S, n, h // 8, w // 8, 8), dtype=torch.uint8, device=dev)
     ty_d = torch.empty((S, n), dtype=torch.uint8, device=dev)
     for si in range(P):
@@ -290,10 +299,12 @@ def main():
     for si in range(P, S):
         lr_d[si].copy_(lr_d[si % P]); res_d[si].copy_(res_d[si % P])
         mv_d[si].copy_(mv_d[si % P]); ty_d[si].copy_(ty_d[si % P])
-    hr = torch.empty((S, n, 3, H, W), dtype=torch.uint8, device=dev)
-    state = torch.zeros((S, 2, 3, H, W), dtype=torch.uint8, device=dev)
+    hr = torch.empty((S, n) + HRF, dtype=torch.uint8, device=dev)
+    state = torch.zeros((S, 2) + HRF, dtype=torch.uint8, device=dev)
+    fmt_c = ns.NS_FMT_I420 if i420 else ns.NS_FMT_444
     chunks = [ns.DeviceChunk(w=w, h=h, scale=s, lr=lr_d[si], res=res_d[si], mv=mv_d[si], type=ty_d[si],
-                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1]) for si in range(S)]
+                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1], format=fmt_c)
+              for si in range(S)]
     hr_out = [[hr[si, f] for f in range(n)] for si in range(S)]
     ia = torch.zeros((S, n), dtype=torch.uint8, device=dev)
     stats = torch.zeros((S, 8), dtype=torch.float64, device=dev)
@@ -364,7 +375,7 @@ def main():
 
     # rooflines from the live per-family event timing
     pk = peaks()
-    fl, by = algorithmic(cfg, types, ia_np, S, n)
+    fl, by = algorithmic(cfg, types, ia_np, S, n, args.format)
     rl = {}
     for fam, (nl, ng, tms) in prof.items():
         if nl == 0 or tms <= 0:
@@ -403,7 +414,7 @@ def main():
     # anchors' LR frames; then the step's result (stats, anchor map) is read back.
     e2e = None
     if args.e2e_steps > 0:
-        hpool = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, w, h, s) for c in pool]
+        hpool = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, w, h, s, format=fmt_c) for c in pool]
         hchunks = []
         for si in range(S):
             hc = dataclasses.replace(hpool[si % P], model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1])
@@ -452,7 +463,7 @@ def main():
                   "package_bytes": sum(len(p) for p in pkgs)}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not i420:
         r = cpu_sample(cfg, pool[0], synth.make_weights(4000, B, C, s))
         cpu = {kk: r[kk] for kk in ("value", "unit", "cores", "kind", "sample")}
 
@@ -462,7 +473,7 @@ def main():
                 "vs_baseline": None, "dtype": "bf16",
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
-                "config": dict(workload_config(cfg, world, args.select), balance=bool(args.balance),
+                "config": dict(workload_config(cfg, world, args.select, args.format), balance=bool(args.balance),
                                l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
@@ -645,12 +656,13 @@ def run_c5(args):
         dist.destroy_process_group()
 
 
-def ns_arena_gb(cfg, nb):
+def ns_arena_gb(cfg, nb, fmt="444"):
     """SR arena of one shape (csrc/k_sr.cu sr_arena_bytes): x0 (8 ch) + h0/hb/tb
     (C ch) bf16 + the u8 LR copy + border bands (small)."""
     h, w, C, s = cfg["h"], cfg["w"], cfg["n_ch"], cfg["scale"]
     px = h * w * nb
-    return (px * 8 * 2 + 3 * px * C * 2 + px * 3 + nb * (8 * (w + h) * s * (C + 3) * 4)) / (1 << 30)
+    return (px * 8 * 2 + 3 * px * C * 2 + px * 3 + nb * (8 * (w + h) * s * (C + 3) * 4) +
+            (3 * s * s * px if fmt == "i420" else 0)) / (1 << 30)
 
 
 if __name__ == "__main__":

@@ -85,7 +85,8 @@ typedef struct ns_model ns_model;
    NS_FMT_444:  three full-resolution planes per frame (reading Z18), the
                 layouts given below.
    NS_FMT_I420: the codec's YUV 4:2:0 -- Y [h][w], then U, V [h/2][w/2] per LR
-                frame (lr u8, res int16), the same at s x per HR frame.  Motion
+                frame (lr u8, res int16), the same at s x per HR frame; w and
+                h multiples of 16 (whole 8x8 chroma blocks).  Motion
                 vectors stay one per 8x8 luma block; the chroma planes use the
                 block's vector read in 1/16 chroma pel (VP9's 4:2:0 rule,
                 reading R9) with the 16-phase bilinear.  An anchor is SR'd by

@@ -97,26 +97,43 @@ constexpr int kReconNT = kReconTX * kReconTY;
 #ifndef NS_RECON_MINB3
 #define NS_RECON_MINB3 (512 / (NS_RECON_TX * NS_RECON_TY))
 #endif
-template <int S>
+// Plane geometry of a reconstruction thread.  Luma (and every 4:4:4 plane):
+// a thread owns one LR block column = 8 LR / 8s HR pixels, motion at 1/8 pel.
+// 4:2:0 chroma (CH, reading R9): the block is 4 x 4 LR / 4s x 4s HR chroma
+// pixels, motion = the luma vector read in 1/16 chroma pel.
+template <int S, bool CH = false>
 struct ReconCfg {
-    static constexpr int BW = 8 * S;               // HR pixels per thread row
-    static constexpr int NP = BW / 2;              // 16-bit pairs per row
-    static constexpr int WIN = BW + 1;             // reference bytes per row
-    static constexpr int NQ = (7 + WIN + 7) / 8;   // aligned 64-bit words per row
-    static constexpr int NA32 = (WIN + 3) / 4;     // aligned 32-bit window words
+    static constexpr int LRB = CH ? 4 : 8;          // LR pixels per block side in this plane
+    static constexpr int BW = LRB * S;              // HR pixels per thread row
+    static constexpr int NP = BW / 2;               // 16-bit pairs per row
+    static constexpr int WIN = BW + 1;              // reference bytes per row
+    static constexpr int NQ = (7 + WIN + 7) / 8;    // aligned 64-bit words per row
+    static constexpr int PB = CH ? 4 : 3;           // sub-pel bits of the motion (1/8 or 1/16)
+    static constexpr int NLR = LRB + 2;             // LR columns an output row's O6 taps touch
     static constexpr int RPT = (S == 3) ? NS_RECON_RPT3 : 8;  // HR rows per thread: a multiple of S
-    static_assert(RPT % S == 0 && (8 * S) % RPT == 0, "a thread's rows lie in one 8x8 LR block row (uniform MV)");
-    static constexpr int PER = RPT / S;            // periods of the vertical O6 taps
+    static_assert(RPT % S == 0 && BW % RPT == 0, "a thread's rows lie in one block row (uniform MV)");
+    static_assert(BW % 4 == 0, "pixel quads of the even/odd pair interleave");
+    static constexpr int PER = RPT / S;             // periods of the vertical O6 taps
     // resident CTAs per SM (registers): 512 threads at 128 registers for s = 3
     static constexpr int MINB = (S == 3) ? NS_RECON_MINB3 : (384 / kReconNT > 0 ? 384 / kReconNT : 1);
+    static constexpr int RES_COLS = LRB * kReconTX + 16;   // residual tile columns (16-B halo chunk per side)
+    static constexpr int NPL = CH ? 2 : 3;          // planes a CTA can step (U, V | up to 3)
+    // per-thread 8-B slots of the shared window buffer: RPT+1 window rows of NQ
+    // words; KEY-frame / INTRA threads keep their LR rows there instead (2 slots
+    // per LR row, PER+2 rows per plane): all planes at once when they fit,
+    // else two alternating plane sets -- which can need more slots than the
+    // window rows (4:2:0 chroma at s = 2: 24 > 18)
+    static constexpr int LRS = (PER + 2) * 2;
+    static constexpr bool LR_ALL = NPL * LRS <= (RPT + 1) * NQ;
+    static constexpr int SLOTS = (RPT + 1) * NQ > (LR_ALL ? NPL : 2) * LRS ? (RPT + 1) * NQ : (LR_ALL ? NPL : 2) * LRS;
 };
-constexpr int kResCols = 8 * kReconTX + 16;        // residual tile columns (one 16-B chunk of halo per side)
 
-template <int S>
+template <int S, bool CH = false>
 struct ReconSmem {
-    static constexpr int RROWS = kReconTY * ReconCfg<S>::PER + 2;      // residual tile LR rows
-    static constexpr size_t REF = (size_t)(ReconCfg<S>::RPT + 1) * ReconCfg<S>::NQ * kReconNT * 8;
-    static constexpr size_t RES = (size_t)3 * RROWS * kResCols * 2;
+    using Cfg = ReconCfg<S, CH>;
+    static constexpr int RROWS = kReconTY * Cfg::PER + 2;      // residual tile LR rows
+    static constexpr size_t REF = (size_t)Cfg::SLOTS * kReconNT * 8;
+    static constexpr size_t RES = (size_t)Cfg::NPL * RROWS * Cfg::RES_COLS * 2;
     static constexpr size_t BAR = REF + RES;                           // mbarrier of the residual tile
     static constexpr size_t BYTES = BAR + 16;
 };
@@ -135,21 +152,22 @@ __device__ __forceinline__ uint32_t mad_u32(uint32_t a, uint32_t b, uint32_t c) 
 __device__ __forceinline__ void cp_async8(void *dst, const void *src) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
-__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
 }
 
 // Stage the raw aligned 64-bit words covering reference bytes xs .. xs+BW of
 // one row into shared memory: dst[i * stride] is word i (struct-of-arrays
-// across the CTA's threads: conflict-free reads).  W and the word base are
-// multiples of 8, so every word lies wholly inside the row or wholly outside
-// it; an outside word stages the row's first / last word instead, and
-// recon_fix_row replicates its edge pixel (Z16) after the copy lands: every
-// global read stays an asynchronous copy, and none reads past the row.
-template <int S>
+// across the CTA's threads: conflict-free reads).  The plane width and the
+// word base are multiples of 8 (4:2:0 requires w % 16 == 0, so chroma planes
+// are too), so every word lies wholly inside the row or wholly outside it; an
+// outside word stages the row's first / last word instead, and recon_load_row
+// replicates its edge pixel (Z16) after the copy lands: every global read
+// stays an asynchronous copy, and none reads past the row.
+template <int S, bool CH>
 __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int W, bool interior, uint2 *dst,
                                                 int stride) {
-    using Cfg = ReconCfg<S>;
+    using Cfg = ReconCfg<S, CH>;
     const int xb = xs & ~7;
 #pragma unroll
     for (int i = 0; i < Cfg::NQ; i++) {
@@ -159,17 +177,18 @@ __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int 
 }
 // Load one staged window row (NQ words) into registers; for a non-interior
 // window replicate the edge pixel into the words that lie outside the row
-// (first word at xb).
-// (on = false: a KEY-frame / INTRA thread, whose warp weights are all 0 and
-// whose slots hold LR rows in flight: nothing is read, so no shared-memory race)
-template <int S>
+// (first word at xb).  (on = false: a KEY-frame / INTRA thread, whose warp
+// weights are all 0 and whose slots hold LR rows in flight: nothing is read,
+// so no shared-memory race.)
+template <int S, bool CH>
 __device__ __forceinline__ void recon_load_row(const uint2 *row, bool on, bool fix, int xb, int W,
-                                               uint2 (&q)[ReconCfg<S>::NQ]) {
+                                               uint2 (&q)[ReconCfg<S, CH>::NQ]) {
+    using Cfg = ReconCfg<S, CH>;
 #pragma unroll
-    for (int i = 0; i < ReconCfg<S>::NQ; i++) q[i] = on ? row[i * kReconNT] : make_uint2(0u, 0u);
+    for (int i = 0; i < Cfg::NQ; i++) q[i] = on ? row[i * kReconNT] : make_uint2(0u, 0u);
     if (fix) {
 #pragma unroll
-        for (int i = 0; i < ReconCfg<S>::NQ; i++) {
+        for (int i = 0; i < Cfg::NQ; i++) {
             const int st = xb + 8 * i;
             if (st < 0) {
                 const uint32_t v = prmt(q[i].x, 0u, 0x0000u);
@@ -182,16 +201,18 @@ __device__ __forceinline__ void recon_load_row(const uint2 *row, bool on, bool f
     }
 }
 
-// Horizontal bilinear pass over one staged reference row, scaled by 8.  Pixel
-// pairs are even/odd interleaved: pair 2g holds pixels (4g, 4g+2) and pair 2g+1
-// pixels (4g+1, 4g+3), so both operands of each pass come from one byte
-// permute of the aligned window word (no per-pair realignment):
-//   h8[2g]   = E_g (8-fx) + O_g fx + 4,  h8[2g+1] = O_g (8-fx) + E'_g fx + 4   (& ~7 per lane)
+// Horizontal bilinear pass over one staged reference row.  Pixel pairs are
+// even/odd interleaved: pair 2g holds pixels (4g, 4g+2) and pair 2g+1 pixels
+// (4g+1, 4g+3), so both operands of each pass come from one byte permute of
+// the aligned window word (no per-pair realignment):
+//   v[2g] = E_g (F-fx) + O_g fx + F/2,  v[2g+1] = O_g (F-fx) + E'_g fx + F/2  (F = 2^PB)
 // with E_g = [p4g, p4g+2], O_g = [p4g+1, p4g+3], E'_g = [p4g+2, p4g+4].
-template <int S>
-__device__ __forceinline__ void recon_hpass8(const uint2 (&q)[ReconCfg<S>::NQ], int m, uint32_t fxc, uint32_t fx,
-                                             uint32_t (&h)[ReconCfg<S>::NP]) {
-    using Cfg = ReconCfg<S>;
+// Luma keeps 8 floor(v/8) (v & ~7, the scale folded into the vertical pass);
+// chroma keeps floor(v/16) (every lane < 2^12).
+template <int S, bool CH>
+__device__ __forceinline__ void recon_hpass(const uint2 (&q)[ReconCfg<S, CH>::NQ], int m, uint32_t fxc, uint32_t fx,
+                                            uint32_t (&h)[ReconCfg<S, CH>::NP]) {
+    using Cfg = ReconCfg<S, CH>;
     constexpr int NG = Cfg::BW / 4;
     uint32_t w[2 * Cfg::NQ + 2];
 #pragma unroll
@@ -216,8 +237,13 @@ __device__ __forceinline__ void recon_hpass8(const uint2 (&q)[ReconCfg<S>::NQ], 
 #pragma unroll
     for (int g = 0; g < NG; g++) {
         const uint32_t E1 = __funnelshift_r(E[g], E[g + 1], 16);
-        h[2 * g] = (E[g] * fxc + O[g] * fx + 0x00040004u) & 0xFFF8FFF8u;
-        h[2 * g + 1] = (O[g] * fxc + E1 * fx + 0x00040004u) & 0xFFF8FFF8u;
+        if constexpr (CH) {
+            h[2 * g] = ((E[g] * fxc + O[g] * fx + 0x00080008u) >> 4) & 0x0FFF0FFFu;
+            h[2 * g + 1] = ((O[g] * fxc + E1 * fx + 0x00080008u) >> 4) & 0x0FFF0FFFu;
+        } else {
+            h[2 * g] = (E[g] * fxc + O[g] * fx + 0x00040004u) & 0xFFF8FFF8u;
+            h[2 * g + 1] = (O[g] * fxc + E1 * fx + 0x00040004u) & 0xFFF8FFF8u;
+        }
     }
 }
 // pixel (within the thread's row) of lane e of pair k (even/odd interleave)
@@ -225,42 +251,55 @@ __host__ __device__ constexpr int pair_px(int k, int e) { return 4 * (k >> 1) + 
 
 // LR rows of KEY frames / INTRA blocks (Z17) are staged per thread in the
 // thread's (otherwise unused) warp-window slots, two per LR row: the aligned
-// word of columns 8bx .. 8bx+7, and [columns 8bx-4 .. 8bx-1 | 8bx+8 .. 8bx+11]
-// (clamped to the row; the edge columns are replaced on use when outside, Z16).
-__device__ __forceinline__ void cp_async4(void *dst, const void *src) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-}
+// word of the block's LRB columns, and [the 4 columns left | the 4 columns
+// right] (clamped to the row; the edge columns are replaced on use when
+// outside, Z16).
+template <bool CH>
 __device__ __forceinline__ void recon_lr_row_stage(const uint8_t *plane, int row, int bx, int w, uint2 *dst) {
+    constexpr int LRB = CH ? 4 : 8;
     const uint8_t *p = plane + (size_t)row * w;
-    cp_async8(dst, p + 8 * bx);
+    if constexpr (CH) cp_async4(dst, p + LRB * bx);
+    else cp_async8(dst, p + LRB * bx);
     uint32_t *e = reinterpret_cast<uint32_t *>(dst + kReconNT);
-    cp_async4(e, p + max(8 * bx - 4, 0));
-    cp_async4(e + 1, p + min(8 * bx + 8, w - 4));
+    cp_async4(e, p + max(LRB * bx - 4, 0));
+    cp_async4(e + 1, p + min(LRB * bx + LRB, w - 4));
 }
-__device__ __forceinline__ void recon_lr_row_smem(const uint2 *src, bool left_in, bool right_in, int (&v)[10]) {
+template <bool CH>
+__device__ __forceinline__ void recon_lr_row_smem(const uint2 *src, bool left_in, bool right_in,
+                                                  int (&v)[(CH ? 4 : 8) + 2]) {
+    constexpr int LRB = CH ? 4 : 8;
     const uint2 q = src[0], e = src[kReconNT];
 #pragma unroll
     for (int i = 0; i < 4; i++) {
         v[1 + i] = (q.x >> (8 * i)) & 255;
-        v[5 + i] = (q.y >> (8 * i)) & 255;
+        if (!CH) v[5 + i] = (q.y >> (8 * i)) & 255;
     }
     v[0] = left_in ? (int)(e.x >> 24) : v[1];
-    v[9] = right_in ? (int)(e.y & 255) : v[8];
+    v[LRB + 1] = right_in ? (int)(e.y & 255) : v[LRB];
 }
 
-// Residual-row values for columns 8bx-1 .. 8bx+8 from the staged tile row `p`
-// (p points at tile column 8 tx, i.e. LR column 8bx - 8).
-__device__ __forceinline__ void recon_res_row_smem(const int16_t *p, bool left_in, bool right_in, int (&v)[10]) {
-    const uint4 m = *reinterpret_cast<const uint4 *>(p + 8);
-    const uint32_t qq[4] = {m.x, m.y, m.z, m.w};
+// Residual-row values for LR columns LRB bx - 1 .. LRB bx + LRB from the staged
+// tile row `p` (p points at tile column LRB tx, i.e. LR column LRB bx - 8).
+template <bool CH>
+__device__ __forceinline__ void recon_res_row_smem(const int16_t *p, bool left_in, bool right_in,
+                                                   int (&v)[(CH ? 4 : 8) + 2]) {
+    constexpr int LRB = CH ? 4 : 8;
+    uint32_t qq[LRB / 2];
+    if constexpr (CH) {
+        const uint2 m = *reinterpret_cast<const uint2 *>(p + 8);
+        qq[0] = m.x; qq[1] = m.y;
+    } else {
+        const uint4 m = *reinterpret_cast<const uint4 *>(p + 8);
+        qq[0] = m.x; qq[1] = m.y; qq[2] = m.z; qq[3] = m.w;
+    }
 #pragma unroll
-    for (int i = 0; i < 4; i++) {
+    for (int i = 0; i < LRB / 2; i++) {
         v[1 + 2 * i] = (int)(int16_t)(qq[i] & 0xFFFFu);
         v[2 + 2 * i] = __mulhi((int)qq[i], 65536);  // arithmetic >> 16 on the FMA pipe
     }
-    const int l = p[7], r = p[16];
+    const int l = p[7], r = p[8 + LRB];
     v[0] = left_in ? l : v[1];
-    v[9] = right_in ? r : v[8];
+    v[LRB + 1] = right_in ? r : v[LRB];
 }
 
 // Compile-time O6 taps.  For an axis coordinate X = S*m + ph + i:
@@ -277,13 +316,14 @@ __host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S)
 //   v    = 128 V[d] + w1 (V[d+1] - V[d])          (exact 2-D O6 sum, d = tap)
 //   s    = 4 (v + 8192 + 2^22) = 512 V[d] + 4 w1 (V[d+1] - V[d]) + KB
 // and r + 256 = s >> 16 (high half-word).
-template <int S, int WY>
-__device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[10], uint32_t (&u)[ReconCfg<S>::NP]) {
-    constexpr int BW = ReconCfg<S>::BW;
+template <int S, bool CH, int WY>
+__device__ __forceinline__ void recon_up_row(const int (&a)[ReconCfg<S, CH>::NLR], const int (&b)[ReconCfg<S, CH>::NLR],
+                                             uint32_t (&u)[ReconCfg<S, CH>::NP]) {
+    constexpr int BW = ReconCfg<S, CH>::BW, NLR = ReconCfg<S, CH>::NLR;
     constexpr int KB = 4 * 8192 + 4 * (256 << 14);
-    int V[10], base[10];
+    int V[NLR], base[NLR];
 #pragma unroll
-    for (int t = 0; t < 10; t++) {
+    for (int t = 0; t < NLR; t++) {
         V[t] = WY ? (128 - WY) * a[t] + WY * b[t] : 128 * a[t];
         base[t] = (int)mad_u32((uint32_t)V[t], 512u, (uint32_t)KB);
     }
@@ -300,17 +340,27 @@ __device__ __forceinline__ void recon_up_row(const int (&a)[10], const int (&b)[
     }
 }
 
-// Output rows: each thread stores its BW bytes per row as 8-B stores.  (Staging
-// the warp's row in shared memory and storing whole 16-B chunks -- the pattern
-// a store-only probe ran 2.2x faster, tools/mem_probe.cu -- measured slower in
+// Output rows: each thread stores its BW bytes per row as 8-B stores (4-B
+// stores when BW is not a multiple of 8: 4:2:0 chroma at s = 3).  (Staging the
+// warp's row in shared memory and storing whole 16-B chunks -- the pattern a
+// store-only probe ran 2.2x faster, tools/mem_probe.cu -- measured slower in
 // this kernel: +11% instructions for stores that were not its bottleneck.)
-template <int S>
-__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S>::BW / 4], bool on) {
+template <int S, bool CH>
+__device__ __forceinline__ void recon_store_row(uint8_t *dst, const uint32_t (&o)[ReconCfg<S, CH>::BW / 4], bool on) {
+    constexpr int BW = ReconCfg<S, CH>::BW;
+    if constexpr (BW % 8 == 0) {
 #pragma unroll
-    for (int q = 0; q < ReconCfg<S>::BW / 8; q++)
-        asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p st.global.v2.b32 [%0], {%1, %2}; }" ::"l"(dst + 8 * q),
-                     "r"(o[2 * q]), "r"(o[2 * q + 1]), "r"((uint32_t)on)
-                     : "memory");
+        for (int q = 0; q < BW / 8; q++)
+            asm volatile("{ .reg .pred p; setp.ne.u32 p, %3, 0; @p st.global.v2.b32 [%0], {%1, %2}; }" ::"l"(dst + 8 * q),
+                         "r"(o[2 * q]), "r"(o[2 * q + 1]), "r"((uint32_t)on)
+                         : "memory");
+    } else {
+#pragma unroll
+        for (int q = 0; q < BW / 4; q++)
+            asm volatile("{ .reg .pred p; setp.ne.u32 p, %2, 0; @p st.global.b32 [%0], %1; }" ::"l"(dst + 4 * q),
+                         "r"(o[q]), "r"((uint32_t)on)
+                         : "memory");
+    }
 }
 
 __device__ __forceinline__ uint32_t vmax_u16x2(uint32_t a, uint32_t b) {
@@ -385,44 +435,49 @@ __device__ __forceinline__ void recon_tile_copy(const uint8_t *src, uint8_t *dst
     }
 }
 
-template <int S>
-__global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
+template <int S, bool CH>
+__global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
     k_recon_step(const FrameDesc *fdesc, int n, int f, int s0) {
-    using Cfg = ReconCfg<S>;
-    using Sm = ReconSmem<S>;
-    constexpr int NP = Cfg::NP, RPT = Cfg::RPT, NQ = Cfg::NQ;
+    using Cfg = ReconCfg<S, CH>;
+    using Sm = ReconSmem<S, CH>;
+    constexpr int NP = Cfg::NP, RPT = Cfg::RPT, NQ = Cfg::NQ, LRB = Cfg::LRB, PB = Cfg::PB, NLR = Cfg::NLR;
+    constexpr int RC = Cfg::RES_COLS;
     const int sid = s0 + blockIdx.z;
     const FrameDesc fd = fdesc[(size_t)sid * n + f];
     if (fd.s != S) return;                              // CTA-uniform
-    const int w = fd.w, h = fd.h, H = h * S, W = w * S;
+    if (CH && fd.fmt != NS_FMT_I420) return;
+    const int w = fd.w, h = fd.h;
+    // this launch's plane geometry: full planes, or the 4:2:0 chroma planes
+    const int pw = CH ? w / 2 : w, ph = CH ? h / 2 : h, W = S * pw, H = S * ph;
     const int bx0 = blockIdx.x * kReconTX;              // first LR block column of the CTA
     const int Y0c = blockIdx.y * kReconTY * RPT;        // first HR row of the CTA
-    if (8 * bx0 >= w || Y0c >= H) return;               // CTA-uniform
+    if (LRB * bx0 >= pw || Y0c >= H) return;            // CTA-uniform
     const int tid = threadIdx.y * kReconTX + threadIdx.x;
-    const size_t lrp = (size_t)h * w, hrp = (size_t)H * W;
-    // planes stepped here: 3 (4:4:4), or the luma plane of a 4:2:0 frame (its
-    // chroma planes step in k_recon_c420)
-    const int np_ = fd.fmt == NS_FMT_I420 ? 1 : 3;
+    // planes: 3 (4:4:4), the luma plane of a 4:2:0 frame, or its two chroma planes
+    const size_t lrp = (size_t)h * w, hrp = (size_t)S * h * S * w;                   // full-size planes
+    const size_t plr = (size_t)ph * pw, phr = (size_t)H * W;                         // this launch's planes
+    const size_t lr0 = CH ? lrp : 0, hr0 = CH ? hrp : 0;                             // first plane's offset
+    const int np_ = CH ? 2 : (fd.fmt == NS_FMT_I420 ? 1 : 3);
     if (fd.gsave_src || (fd.anchor && fd.asrc)) {       // HR rings only (k_frame_desc)
-        const int x0 = 8 * S * bx0, x1 = min(8 * S * (bx0 + kReconTX), W), y1 = min(Y0c + kReconTY * RPT, H);
-        if (fd.gsave_src) recon_tile_copy(fd.gsave_src, fd.gsave_dst, hrp, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
-        if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc, fd.out, hrp, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
+        const int x0 = Cfg::BW * bx0, x1 = min(Cfg::BW * (bx0 + kReconTX), W), y1 = min(Y0c + kReconTY * RPT, H);
+        if (fd.gsave_src) recon_tile_copy(fd.gsave_src + hr0, fd.gsave_dst + hr0, phr, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
+        if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc + hr0, fd.out + hr0, phr, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
     }
     if (fd.anchor) return;                              // CTA-uniform: the anchor's SR bytes are in place
 
     extern __shared__ __align__(16) uint8_t recon_sm[];
     uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [RPT+1][NQ][NT] warp windows
-    int16_t *tres = reinterpret_cast<int16_t *>(recon_sm + Sm::REF);   // [3][RROWS][kResCols] residual tile
+    int16_t *tres = reinterpret_cast<int16_t *>(recon_sm + Sm::REF);   // [planes][RROWS][RC] residual tile
 
     // residual tile: tile row r <-> LR row Y0c/S - 1 + r (clamped, Z16), tile
-    // column t <-> LR column 8 bx0 - 8 + t; the part inside the row arrives as one
+    // column t <-> LR column LRB bx0 - 8 + t; the part inside the row arrives as one
     // bulk copy per (plane, row) issued by warp 0 (columns outside the row are
     // never read: the edge columns are clamped on use).  One bulk copy per row
     // instead of per-thread 16-B chunks: the chunk loop's index arithmetic was
     // ~6% of the kernel's instructions (ncu source counters).
     uint64_t *tbar = reinterpret_cast<uint64_t *>(recon_sm + Sm::BAR);
     if (!fd.key && tid < 32) {
-        const int col_lo = max(8 * bx0 - 8, 0), col_hi = min(8 * bx0 - 8 + kResCols, w);
+        const int col_lo = max(LRB * bx0 - 8, 0), col_hi = min(LRB * bx0 - 8 + RC, pw);
         const uint32_t bytes = (uint32_t)(col_hi - col_lo) * 2u;
         if (tid == 0) {
             mbar_init(tbar, 1);
@@ -432,39 +487,40 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
         __syncwarp();
         for (int e = tid; e < np_ * Sm::RROWS; e += 32) {
             const int c = e / Sm::RROWS, rr = e % Sm::RROWS;
-            const int row = min(max(Y0c / S - 1 + rr, 0), h - 1);
-            bulk_load(tres + (size_t)e * kResCols + (col_lo - (8 * bx0 - 8)),
-                      fd.res_f + c * lrp + (size_t)row * w + col_lo, bytes, tbar);
+            const int row = min(max(Y0c / S - 1 + rr, 0), ph - 1);
+            bulk_load(tres + (size_t)e * RC + (col_lo - (LRB * bx0 - 8)),
+                      fd.res_f + lr0 + c * plr + (size_t)row * pw + col_lo, bytes, tbar);
         }
     }
 
     const int bx = bx0 + threadIdx.x;
     const int Y0 = Y0c + threadIdx.y * RPT;
-    const bool valid = 8 * bx < w && Y0 < H;
+    const bool valid = LRB * bx < pw && Y0 < H;
     const int X0 = bx * Cfg::BW;
     ns_block_mv mv{};
     if (valid) mv = fd.mv_f[(size_t)(Y0 / Cfg::BW) * (w / 8) + bx];
     // KEY frames and INTRA blocks: up_s(LR[f]) (Z17) through the same arithmetic,
     // with a zero prediction (all warp weights 0) and LR rows instead of residual rows
     const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;
-    const uint8_t *ref = mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last;
-    // warp geometry (O7): m = s * mv in 1/8 HR pel
+    const uint8_t *ref = (mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last) + hr0;
+    // warp geometry (O7 / R9): m = s * mv in 1/2^PB HR pel of this plane
     const int mx = S * mv.mvx, my = S * mv.mvy;
-    const int xs = X0 + (mx >> 3);
-    const uint32_t fx = use_lr ? 0u : (uint32_t)(mx & 7), fy = use_lr ? 0u : (uint32_t)(my & 7);
-    const uint32_t fxc = use_lr ? 0u : 8u - fx, fyc = use_lr ? 0u : 8u - fy;  // lanes x SCALAR: no cross-lane terms
-    const int iy0 = Y0 + (my >> 3);
+    const int xs = X0 + (mx >> PB);
+    constexpr uint32_t F = 1u << PB;
+    const uint32_t fx = use_lr ? 0u : (uint32_t)(mx & (F - 1)), fy = use_lr ? 0u : (uint32_t)(my & (F - 1));
+    const uint32_t fxc = use_lr ? 0u : F - fx, fyc = use_lr ? 0u : F - fy;  // lanes x SCALAR: no cross-lane terms
+    const int iy0 = Y0 + (my >> PB);
     const bool interior = xs >= 0 && (xs & ~7) + 8 * NQ <= W;
     // Reference windows live in ONE buffer of RPT+1 rows: row r of plane c+1 is
     // staged right after plane c's warp pass has read row r, one commit group per
     // row, so before the pass over row r there are always exactly RPT groups newer
     // than row r's (wait_group RPT).  LR rows (use_lr threads) ride in the group
-    // of row 0: when all three planes fit the thread's slots (s = 3, 4) they are
-    // staged at once with plane 0 -- LR may be host memory read across PCIe
+    // of row 0: when all planes fit the thread's slots they are staged at once
+    // with plane 0 -- LR may be host memory read across PCIe
     // (ns_enhance_streams_host), so its latency is paid once, not per plane --
     // otherwise per plane, alternating between two slot sets.
-    constexpr int LRS = (Cfg::PER + 2) * 2;                 // slots per plane's LR rows
-    constexpr bool LR_ALL = 3 * LRS <= (RPT + 1) * NQ;
+    constexpr int LRS = Cfg::LRS;                           // slots per plane's LR rows
+    constexpr bool LR_ALL = Cfg::LR_ALL;
     auto lr_slots = [&](int c) { return (LR_ALL ? c : (c & 1)) * LRS * kReconNT; };
     uint2 *wbuf = rsm + tid;
     auto stage_row = [&](int c, int r) {
@@ -475,22 +531,27 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                 for (int cc = c; cc < (LR_ALL ? np_ : c + 1); cc++)
 #pragma unroll
                     for (int t = 0; t < Cfg::PER + 2; t++)
-                        recon_lr_row_stage(fd.lr_f + cc * lrp, min(max(Y0 / S - 1 + t, 0), h - 1), bx, w,
-                                           wbuf + lr_slots(cc) + t * 2 * kReconNT);
+                        recon_lr_row_stage<CH>(fd.lr_f + lr0 + cc * plr, min(max(Y0 / S - 1 + t, 0), ph - 1), bx, pw,
+                                               wbuf + lr_slots(cc) + t * 2 * kReconNT);
             }
             return;
         }
         const int rr = min(max(iy0 + r, 0), H - 1);
-        recon_row_stage<S>(ref + c * hrp + (size_t)rr * W, xs, W, interior, wbuf + r * NQ * kReconNT, kReconNT);
+        recon_row_stage<S, CH>(ref + c * phr + (size_t)rr * W, xs, W, interior, wbuf + r * NQ * kReconNT, kReconNT);
     };
     for (int r = 0; r <= RPT; r++) {
         stage_row(0, r);
         asm volatile("cp.async.commit_group;" ::: "memory");
     }
-    const bool left_in = bx > 0, right_in = 8 * bx + 8 < w;
+    const bool left_in = bx > 0, right_in = LRB * bx + LRB < pw;
     const int m = xs & 7;
     const bool fix = valid && !interior && !use_lr;
-    uint8_t *outp = fd.out + (size_t)Y0 * W + X0;
+    uint8_t *outp = fd.out + hr0 + (size_t)Y0 * W + X0;
+    // combine (see the top of this file): luma X = 64 (r + 256) + 8h0 (8-fy) + 8h1 fy + 32,
+    // chroma X = 16 (r + 256) + h0 (16-fy) + h1 fy + 8; floor(X / 2^SH) = pred + r + 256
+    constexpr uint32_t SH = CH ? 4 : 6;
+    constexpr uint32_t UMUL = 1u << SH, UADD = CH ? 0x00080008u : 0x00200020u;
+    constexpr uint32_t XLO = (256u << SH) * 0x00010001u, XHI = ((512u << SH) - 1) * 0x00010001u;
 
 #pragma unroll 1
     for (int c = 0; c < np_; c++) {
@@ -500,26 +561,26 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
             if (!fd.key) mbar_wait(tbar, 0);                    // the residual tile
         }
         // (use_lr threads run the warp pass on zero words: every weight is 0, so pred = 0)
-        const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * kResCols + 8 * threadIdx.x;
+        const int16_t *tp = tres + ((size_t)c * Sm::RROWS + threadIdx.y * Cfg::PER) * RC + LRB * threadIdx.x;
         const uint2 *lrb = wbuf + lr_slots(c);
-        uint8_t *outc = outp + c * hrp;
+        uint8_t *outc = outp + c * phr;
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
         {
             uint2 q[NQ];
-            recon_load_row<S>(wbuf, !use_lr, fix, xs & ~7, W, q);
-            recon_hpass8<S>(q, m, fxc, fx, hA);
+            recon_load_row<S, CH>(wbuf, !use_lr, fix, xs & ~7, W, q);
+            recon_hpass<S, CH>(q, m, fxc, fx, hA);
         }
         stage_row(c + 1, 0);
         asm volatile("cp.async.commit_group;" ::: "memory");
 #pragma unroll 1
         for (int it = 0; it < Cfg::PER; it++) {
-            int rv[3][10];  // LR rows it .. it + 2 of this thread
+            int rv[3][NLR];  // LR rows it .. it + 2 of this thread
             if (!use_lr) {
 #pragma unroll
-                for (int t = 0; t < 3; t++) recon_res_row_smem(tp + (it + t) * kResCols, left_in, right_in, rv[t]);
+                for (int t = 0; t < 3; t++) recon_res_row_smem<CH>(tp + (it + t) * RC, left_in, right_in, rv[t]);
             } else {
 #pragma unroll
-                for (int t = 0; t < 3; t++) recon_lr_row_smem(lrb + (it + t) * 2 * kReconNT, left_in, right_in, rv[t]);
+                for (int t = 0; t < 3; t++) recon_lr_row_smem<CH>(lrb + (it + t) * 2 * kReconNT, left_in, right_in, rv[t]);
             }
             auto one = [&](auto jc) {
                 constexpr int jj = decltype(jc)::value;
@@ -529,20 +590,20 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
                 uint32_t(&hc)[NP] = (jj & 1) ? hA : hB;
                 asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
                 uint2 q[NQ];
-                recon_load_row<S>(wbuf + (j + 1) * NQ * kReconNT, !use_lr, fix, xs & ~7, W, q);
+                recon_load_row<S, CH>(wbuf + (j + 1) * NQ * kReconNT, !use_lr, fix, xs & ~7, W, q);
                 uint32_t u[NP], x[NP], o[Cfg::BW / 4];
-                recon_up_row<S, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);   // independent of q: covers the load
-                recon_hpass8<S>(q, m, fxc, fx, hc);
+                recon_up_row<S, CH, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);   // independent of q: covers the load
+                recon_hpass<S, CH>(q, m, fxc, fx, hc);
                 stage_row(c + 1, j + 1);
                 asm volatile("cp.async.commit_group;" ::: "memory");
 #pragma unroll
                 for (int k = 0; k < NP; k++) {
-                    const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], 64u, 0x00200020u)));
-                    x[k] = __umulhi(vmin_u16x2(vmax_u16x2(X, 0x40004000u), 0x7FFF7FFFu), 1u << 26);  // >> 6
+                    const uint32_t X = mad_u32(hp[k], fyc, mad_u32(hc[k], fy, mad_u32(u[k], UMUL, UADD)));
+                    x[k] = __umulhi(vmin_u16x2(vmax_u16x2(X, XLO), XHI), 1u << (32 - SH));  // >> SH
                 }
 #pragma unroll
                 for (int q = 0; q < Cfg::BW / 4; q++) o[q] = prmt(x[2 * q], x[2 * q + 1], 0x6240u);
-                recon_store_row<S>(outc + (size_t)j * W, o, valid);
+                recon_store_row<S, CH>(outc + (size_t)j * W, o, valid);
             };
             static_for<S>(one);
             if constexpr (S & 1) {  // the period ended on an even row: its warp row is in hB
@@ -557,100 +618,19 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S>::MINB)
 // 256-KB array stays L1 (the window words of neighbouring threads overlap and
 // hit there): the maximum-shared carveout (28 KB of L1) vs this (60 KB) measured
 // 70.2 vs 62.8 ms of reconstruction per c4 step (tools/ab_libs.sh, one box).
-template <int S>
+template <int S, bool CH>
 constexpr int recon_carveout_pct() {
-    return (int)((ReconCfg<S>::MINB * (ReconSmem<S>::BYTES + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
+    return (int)((ReconCfg<S, CH>::MINB * (ReconSmem<S, CH>::BYTES + 1024) * 100 + 228 * 1024 - 1) / (228 * 1024));
 }
 
-template <int S>
+template <int S, bool CH>
 static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0) {
-    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S>>((int)ReconSmem<S>::BYTES, recon_carveout_pct<S>());
+    if (cudaError_t e = ensure_kernel_smem<k_recon_step<S, CH>>((int)ReconSmem<S, CH>::BYTES,
+                                                                 recon_carveout_pct<S, CH>());
         e != cudaSuccess)
         return e;
-    k_recon_step<S><<<g, dim3(kReconTX, kReconTY), ReconSmem<S>::BYTES, st>>>(fd, n, f, s0);
+    k_recon_step<S, CH><<<g, dim3(kReconTX, kReconTY), ReconSmem<S, CH>::BYTES, st>>>(fd, n, f, s0);
     return cudaGetLastError();
-}
-
-// ---------------------------------------------------------------- 4:2:0 chroma (NEXT-2)
-// One frame step of the U and V planes of the NS_FMT_I420 streams (readings R9,
-// R10; oracle or_reconstruct_i420).  An HR chroma pixel (X, Y) lies in the LR
-// block (X / 4s, Y / 4s); its motion is the block's luma vector read in 1/16
-// chroma pel, m = s mv: pred = 16-phase two-pass bilinear of the reference
-// chroma plane (edge replicated), plus up_s of the chroma residual plane, clamped;
-// KEY frames and INTRA blocks take up_s of the LR chroma plane.  A thread owns
-// two horizontally adjacent pixels (they share the block: 4s is even) of both
-// planes over kC420Rows rows, so the block's vector, the O6 taps and the warp
-// geometry are computed once per row for four outputs.  Plain integer code:
-// the chroma planes are half the luma plane's pixels.
-constexpr int kC420TX = 64, kC420TY = 2, kC420Rows = 4;
-
-__device__ __forceinline__ int c420_bilin16(const uint8_t *R, int PH, int PW, int X, int Y, int mx, int my) {
-    const int ix = X + (mx >> 4), fx = mx & 15, iy = Y + (my >> 4), fy = my & 15;
-    const int xa = min(max(ix, 0), PW - 1), xb = min(max(ix + 1, 0), PW - 1);
-    const int ya = min(max(iy, 0), PH - 1), yb = min(max(iy + 1, 0), PH - 1);
-    const int h0 = (R[(size_t)ya * PW + xa] * (16 - fx) + R[(size_t)ya * PW + xb] * fx + 8) >> 4;
-    const int h1 = (R[(size_t)yb * PW + xa] * (16 - fx) + R[(size_t)yb * PW + xb] * fx + 8) >> 4;
-    return (h0 * (16 - fy) + h1 * fy + 8) >> 4;
-}
-
-template <class T>
-__device__ __forceinline__ int c420_up(const T *P, int pw, int y0, int y1, int wy, int x0, int x1, int wx) {
-    const int v = (128 - wy) * ((128 - wx) * (int)P[(size_t)y0 * pw + x0] + wx * (int)P[(size_t)y0 * pw + x1]) +
-                  wy * ((128 - wx) * (int)P[(size_t)y1 * pw + x0] + wx * (int)P[(size_t)y1 * pw + x1]);
-    return (v + 8192) >> 14;   // floor((v + 8192) / 2^14) (arithmetic shift)
-}
-
-template <int S>
-__global__ void __launch_bounds__(kC420TX * kC420TY) k_recon_c420(const FrameDesc *fdesc, int n, int f, int s0) {
-    const int sid = s0 + blockIdx.z;
-    const FrameDesc fd = fdesc[(size_t)sid * n + f];
-    if (fd.s != S || fd.fmt != NS_FMT_I420) return;                 // CTA-uniform
-    const int w = fd.w, h = fd.h, H = S * h, W = S * w;
-    const int pw = w / 2, ph = h / 2, PW = W / 2, PH = H / 2;       // chroma planes (LR, HR)
-    const int X = 2 * (blockIdx.x * kC420TX + threadIdx.x);
-    const int Yb = (blockIdx.y * kC420TY + threadIdx.y) * kC420Rows;
-    if (X >= PW || Yb >= PH) return;
-    const size_t lrp = (size_t)h * w, hrp = (size_t)H * W, cl = lrp / 4, ch = hrp / 4;
-    const int Ye = min(Yb + kC420Rows, PH);
-    // HR rings: the GOLDEN save and the anchor copy of the chroma planes
-    auto copy2 = [&](const uint8_t *src, uint8_t *dst) {
-        for (int c = 0; c < 2; c++)
-            for (int Y = Yb; Y < Ye; Y++) {
-                const size_t o = hrp + c * ch + (size_t)Y * PW + X;
-                *reinterpret_cast<uint16_t *>(dst + o) = *reinterpret_cast<const uint16_t *>(src + o);
-            }
-    };
-    if (fd.gsave_src) copy2(fd.gsave_src, fd.gsave_dst);
-    if (fd.anchor) {
-        if (fd.asrc) copy2(fd.asrc, fd.out);
-        return;
-    }
-    constexpr int BLK = 4 * S;                                      // HR chroma pixels per LR block side
-    int xa[2], xb[2], wx[2];
-    for (int e = 0; e < 2; e++) up_tap_r(X + e, S, pw, xa[e], xb[e], wx[e]);
-    for (int Y = Yb; Y < Ye; Y++) {
-        const ns_block_mv mv = fd.mv_f[(size_t)(Y / BLK) * (w / 8) + X / BLK];
-        const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;
-        const uint8_t *ref = mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last;
-        int ya, yb, wy;
-        up_tap_r(Y, S, ph, ya, yb, wy);
-        for (int c = 0; c < 2; c++) {
-            uint8_t o[2];
-            for (int e = 0; e < 2; e++) {
-                int v;
-                if (use_lr) {
-                    v = c420_up(fd.lr_f + lrp + c * cl, pw, ya, yb, wy, xa[e], xb[e], wx[e]);
-                } else {
-                    const int r = c420_up(fd.res_f + lrp + c * cl, pw, ya, yb, wy, xa[e], xb[e], wx[e]);
-                    const int p = c420_bilin16(ref + hrp + c * ch, PH, PW, X + e, Y, S * mv.mvx, S * mv.mvy);
-                    v = min(max(p + r, 0), 255);
-                }
-                o[e] = (uint8_t)v;
-            }
-            *reinterpret_cast<uint16_t *>(fd.out + hrp + c * ch + (size_t)Y * PW + X) =
-                (uint16_t)(o[0] | (o[1] << 8));
-        }
-    }
 }
 
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
@@ -664,17 +644,15 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
         const int rpt = s == 2 ? ReconCfg<2>::RPT : s == 3 ? ReconCfg<3>::RPT : ReconCfg<4>::RPT;
         const int nrg = (max_lr_h[s] * s + rpt - 1) / rpt;  // groups of RPT HR rows
         dim3 g((nbx + kReconTX - 1) / kReconTX, (nrg + kReconTY - 1) / kReconTY, S);
-        const cudaError_t e = s == 2 ? recon_launch<2>(g, st, fd, n, f, s0)
-                              : s == 3 ? recon_launch<3>(g, st, fd, n, f, s0) : recon_launch<4>(g, st, fd, n, f, s0);
+        cudaError_t e = s == 2 ? recon_launch<2, false>(g, st, fd, n, f, s0)
+                        : s == 3 ? recon_launch<3, false>(g, st, fd, n, f, s0) : recon_launch<4, false>(g, st, fd, n, f, s0);
         if (e != cudaSuccess) return e;
         if (has_i420[s]) {  // the chroma planes of the 4:2:0 streams of this scale, same frame step
-            const int PW = max_lr_w[s] * s / 2, PH = max_lr_h[s] * s / 2;
-            dim3 gc((PW / 2 + kC420TX - 1) / kC420TX, (PH + kC420TY * kC420Rows - 1) / (kC420TY * kC420Rows), S);
-            dim3 bc(kC420TX, kC420TY);
-            if (s == 2) k_recon_c420<2><<<gc, bc, 0, st>>>(fd, n, f, s0);
-            else if (s == 3) k_recon_c420<3><<<gc, bc, 0, st>>>(fd, n, f, s0);
-            else k_recon_c420<4><<<gc, bc, 0, st>>>(fd, n, f, s0);
-            if (cudaError_t e2 = cudaGetLastError(); e2 != cudaSuccess) return e2;
+            const int nrc = (max_lr_h[s] / 2 * s + rpt - 1) / rpt;
+            dim3 gc(g.x, (nrc + kReconTY - 1) / kReconTY, S);
+            e = s == 2 ? recon_launch<2, true>(gc, st, fd, n, f, s0)
+                : s == 3 ? recon_launch<3, true>(gc, st, fd, n, f, s0) : recon_launch<4, true>(gc, st, fd, n, f, s0);
+            if (e != cudaSuccess) return e;
         }
     }
     return cudaGetLastError();

@@ -503,6 +503,9 @@ static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n
         if (c.scale < 2 || c.scale > 4) return fail(NS_EINVAL, "chunk %d: scale %d not in {2,3,4}", s, c.scale);
         if (c.format != NS_FMT_444 && c.format != NS_FMT_I420)
             return fail(NS_EINVAL, "chunk %d: format %d not NS_FMT_444 / NS_FMT_I420", s, c.format);
+        if (c.format == NS_FMT_I420 && (c.w % 16 || c.h % 16))
+            return fail(NS_EINVAL, "chunk %d: 4:2:0 needs w, h multiples of 16 (8 x 8 chroma blocks), got %dx%d", s,
+                        c.w, c.h);
         if (!c.lr || !c.res || !c.mv || !c.type) return fail(NS_EINVAL, "chunk %d: lr/res/mv/type must be non-NULL", s);
         if (!al16(c.res) || !al16(c.lr) || !al16(c.mv)) return fail(NS_EINVAL, "chunk %d: lr/res/mv must be 16-B aligned", s);
         if (c.gt && !al16(c.gt)) return fail(NS_EINVAL, "chunk %d: gt must be 16-B aligned", s);
@@ -800,6 +803,8 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
     for (int j = 0; j < n_jobs; j++)
         if (jobs[j].format != NS_FMT_444 && jobs[j].format != NS_FMT_I420)
             return fail(NS_EINVAL, "job %d: format %d invalid", j, jobs[j].format);
+        else if (jobs[j].format == NS_FMT_I420 && (jobs[j].w % 16 || jobs[j].h % 16))
+            return fail(NS_EINVAL, "job %d: 4:2:0 needs w, h multiples of 16", j);
     std::map<GroupKey, std::vector<int>> groups;
     for (int j = 0; j < n_jobs; j++)
         groups[GroupKey(jobs[j].h, jobs[j].w, jobs[j].model->C, jobs[j].model->s, jobs[j].model->n_blocks,

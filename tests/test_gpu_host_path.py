@@ -127,7 +127,7 @@ def test_host_path_i420_matches_device_path(ctx):
     results equal the device-input path byte for byte."""
     n, k = 10, 2
     cs = [synth.make_chunk_i420(7300 + i, w, h, s, n, types=synth.default_types(n, 4))
-          for i, (w, h, s) in enumerate([(64, 32, 2), (48, 24, 3), (64, 32, 2)])]
+          for i, (w, h, s) in enumerate([(64, 32, 2), (48, 32, 3), (64, 32, 2)])]
     outs = {}
     for path in ("device", "host"):
         dcs, hrs = [], []

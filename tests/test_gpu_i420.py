@@ -55,8 +55,8 @@ def _adversarial(c, seed):
     return c
 
 
-@pytest.mark.parametrize("s,w,h,adv", [(2, 64, 40, False), (3, 48, 32, False), (4, 32, 16, False),
-                                       (3, 264, 48, True), (2, 72, 40, True)])
+@pytest.mark.parametrize("s,w,h,adv", [(2, 64, 48, False), (3, 48, 32, False), (4, 32, 16, False),
+                                       (3, 272, 48, True), (2, 80, 32, True), (4, 288, 16, True)])
 def test_reconstruct_i420_bit_exact(ctx, s, w, h, adv):
     n = 9
     types = synth.default_types(n, 4)
@@ -84,8 +84,8 @@ def test_reconstruct_i420_bit_exact(ctx, s, w, h, adv):
     assert np.array_equal(dc.hr_golden.cpu().numpy(), egold)
 
 
-@pytest.mark.parametrize("B,C,s,w,h", [(2, 16, 2, 64, 48), (1, 32, 3, 136, 24), (1, 16, 4, 32, 16),
-                                       (1, 32, 3, 264, 256)])
+@pytest.mark.parametrize("B,C,s,w,h", [(2, 16, 2, 64, 48), (1, 32, 3, 144, 32), (1, 16, 4, 32, 16),
+                                       (1, 32, 3, 272, 256)])
 def test_sr_i420_vs_oracle(ctx, B, C, s, w, h):
     """ns_sr_anchors on 4:2:0 frames: the net on (Y, up2 U, up2 V), HR chroma
     by the rounded 2x2 average (R10); 264 x 256 spans several res-block and
@@ -110,7 +110,7 @@ def test_enhance_i420_and_444_mixed(ctx):
     split by format, frame steps run the luma kernel for both and the chroma
     kernel for the 4:2:0 ones; every stream against its oracle."""
     n, k = 10, 3
-    specs = [("i420", 64, 32, 2), ("444", 64, 32, 2), ("i420", 48, 24, 3), ("i420", 64, 32, 2)]
+    specs = [("i420", 64, 32, 2), ("444", 64, 32, 2), ("i420", 48, 32, 3), ("i420", 64, 32, 2)]
     dcs, hrs, refs = [], [], []
     rng = np.random.default_rng(9)
     for i, (fmt, w, h, s) in enumerate(specs):
@@ -212,3 +212,13 @@ def test_hybrid_encode_i420(ctx):
         ref = hr[h_.frame].cpu().numpy()[:H * W].reshape(H, W)
         d = y.astype(np.float64) - ref
         assert 10 * np.log10(255.0 ** 2 / max(float((d * d).mean()), 1e-9)) >= 30.0
+
+
+def test_i420_shape_rejected(ctx):
+    """4:2:0 frames need whole 8x8 chroma blocks: w, h multiples of 16."""
+    c = synth.make_chunk_i420(990, 40, 16, 3, 4, types=synth.default_types(4, None))
+    dc = _dev(c, last=np.zeros(_hr_size(c), np.uint8), gold=np.zeros(_hr_size(c), np.uint8))
+    hr = [torch.zeros(_hr_size(c), dtype=torch.uint8, device=DEV) for _ in range(4)]
+    with pytest.raises(ns.NsError) as ei:
+        ctx.reconstruct_chunk([dc], torch.zeros((1, 4), dtype=torch.uint8, device=DEV), [hr])
+    assert ei.value.status == ns.NS_EINVAL and "16" in str(ei.value)

@@ -1,0 +1,6 @@
+#!/bin/bash
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || { cat gpurun_out/build.log; exit 1; }
+timeout 900 python -m pytest tests/test_gpu_i420.py tests/test_gpu_host_path.py -q -x > gpurun_out/t_l_i420.log 2>&1; echo "TESTS rc=$?" >> gpurun_out/t_l_i420.log
+python bench.py --format i420 > gpurun_out/b_i420.json 2>gpurun_out/b_i420.err
+ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__inst_executed.sum --clock-control none -k regex:"k_recon" -s 40 -c 4 --csv python bench.py --format i420 --steps 1 --warmup 1 --no-cpu-baseline --e2e-steps 0 > gpurun_out/ncu_i420.csv 2>&1
+timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/t_l.log 2>&1; echo "TESTS rc=$?" >> gpurun_out/t_l.log
