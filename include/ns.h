@@ -67,6 +67,14 @@ typedef enum {
     NS_KEY = 0, NS_ALTREF = 1, NS_NORMAL = 2,
     NS_I = NS_KEY, NS_P = NS_ALTREF, NS_B = NS_NORMAL
 } ns_frame_type;
+/* Invisible frames (NEXT-2): VP9's alternative reference frames are "invisible
+   frames only used for interframe compression", shown later by an
+   overlay frame.  NS_INVISIBLE OR'ed into a type byte marks a frame that is
+   selected in its group, enhanced and kept as a reference exactly like a
+   visible one, but not displayed: the stats count and score only displayed
+   frames (reading R12).  Every call masks the type with NS_TYPE_MASK. */
+#define NS_INVISIBLE 0x80
+#define NS_TYPE_MASK 0x7F
 
 /* Reference index of a block ("reference index"). */
 typedef enum { NS_REF_LAST = 0, NS_REF_GOLDEN = 1, NS_REF_INTRA = 2 } ns_ref;
@@ -247,8 +255,8 @@ NS_API ns_status ns_reconstruct_chunk(ns_ctx *ctx, const ns_chunk *chunks, int S
    slot at their own frame step (the client "caches [SR anchors] in
    memory" and reuses them).
    is_anchor_out (DEVICE [S][n]) may be NULL.  stats: DEVICE [S][8] fp64 or
-   NULL: {frames, anchors, sum anchor score, total score, SSE vs gt (or -1),
-   PSNR vs gt (or -1), 0, 0}. */
+   NULL: {displayed frames, anchors, sum anchor score, total score, SSE vs gt
+   over the displayed frames (or -1), PSNR vs gt (or -1), 0, 0}. */
 NS_API ns_status ns_enhance_streams(ns_ctx *ctx, const ns_chunk *chunks, int S, const ns_select_params *p,
                              uint8_t *const *hr_out, uint8_t *is_anchor_out, double *stats, void *stream);
 

@@ -161,7 +161,7 @@ int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t 
                 uint8_t *op = out + (size_t)c * hr_plane;
                 for (size_t i = 0; i < lr_plane; i++) in[i] = lrp[i];
                 or_upsample(in, h, w, s, up_lr);
-                if (type[f] == OR_KEY) {
+                if ((type[f] & 0x7F) == OR_KEY) {
                     for (size_t i = 0; i < hr_plane; i++) op[i] = (uint8_t)up_lr[i];
                     continue;
                 }
@@ -179,7 +179,7 @@ int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t 
                     }
             }
         }
-        if (type[f] == OR_KEY || type[f] == OR_ALTREF) golden = out;
+        if ((type[f] & 0x7F) == OR_KEY || (type[f] & 0x7F) == OR_ALTREF) golden = out;  /* R12: 0x80 = invisible */
     }
     if (hr_last && n > 0) memmove(hr_last, hr + (size_t)(n - 1) * 3 * hr_plane, 3 * hr_plane);
     if (hr_golden && golden && golden != hr_golden) memmove(hr_golden, golden, 3 * hr_plane);
@@ -240,7 +240,7 @@ int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int
                 uint8_t *op = out + ho;
                 for (size_t i = 0; i < (size_t)ph * pw; i++) in[i] = lrp[i];
                 or_upsample(in, ph, pw, s, up_lr);
-                if (type[f] == OR_KEY) {
+                if ((type[f] & 0x7F) == OR_KEY) {
                     for (size_t i = 0; i < (size_t)PH * PW; i++) op[i] = (uint8_t)up_lr[i];
                     continue;
                 }
@@ -259,7 +259,7 @@ int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int
                     }
             }
         }
-        if (type[f] == OR_KEY || type[f] == OR_ALTREF) golden = out;
+        if ((type[f] & 0x7F) == OR_KEY || (type[f] & 0x7F) == OR_ALTREF) golden = out;  /* R12: 0x80 = invisible */
     }
     if (hr_last && n > 0) memmove(hr_last, hr + (size_t)(n - 1) * hrf, hrf);
     if (hr_golden && golden && golden != hr_golden) memmove(hr_golden, golden, hrf);

@@ -27,6 +27,16 @@ KEY_GAIN = (1 << 63) - 1          # "equal anchor gain" of key frames (P:170-176
 CARRY, FRESH = 0, 1
 
 
+INVISIBLE, TYPE_MASK = 0x80, 0x7F
+
+
+def frame_groups(types):
+    """Group of every frame: the type byte without the NS_INVISIBLE flag -- an
+    invisible ALTREF is still an alternative reference frame (reading
+    R12: invisibility changes what is displayed, not selection)."""
+    return [int(t) & TYPE_MASK for t in types]
+
+
 def calc_residual(types, score):
     """Alg. 1 CalcResidual (lines 15-20): running accumulated residual in
     decode order, cleared at KEY frames.  Returns (residuals, reset) where
@@ -98,6 +108,7 @@ def stream_gains(types, score, mode=CARRY):
     """Fig. 10 steps 1-2 for one stream: divide into G_key, G_altref, G_normal
      and estimate the gain of every frame.  Returns gain[f]
     (KEY_GAIN for key frames) and, per group, the greedy pick order."""
+    types = frame_groups(types)
     n = len(types)
     g_altref = [f for f in range(n) if types[f] == ALTREF]
     g_normal = [f for f in range(n) if types[f] == NORMAL]
@@ -115,6 +126,7 @@ def stream_gains(types, score, mode=CARRY):
 def stream_order(types, gain):
     """Fig. 10 step 3 within one stream: G_key first (ascending), then
     G_altref, then G_normal, each sorted by gain desc, frame asc (Z5)."""
+    types = frame_groups(types)
     n = len(types)
     keys = [f for f in range(n) if types[f] == KEY]
     alt = sorted((f for f in range(n) if types[f] == ALTREF), key=lambda f: (-gain[f], f))
@@ -176,6 +188,7 @@ def select_key(types, k):
     order = key frames ascending, then every other frame ascending; the anchors
     are the key frames among the first k (reading R6: k = n selects every key
     frame).  gain = KEY_GAIN for key frames, 0 otherwise."""
+    types = frame_groups(types)
     n = len(types)
     keys = [f for f in range(n) if types[f] == KEY]
     order = keys + [f for f in range(n) if types[f] != KEY]
@@ -189,6 +202,7 @@ def select_key_uniform(types, k):
     U = {floor(j * n / k) : 0 <= j < k}, the k equally spaced frames of the
     chunk (reading R5); order = key frames ascending, then the frames of U that
     are not key frames ascending, then the rest ascending; anchors = the first k."""
+    types = frame_groups(types)
     n = len(types)
     U = set((j * n) // k for j in range(k)) if k > 0 else set()
     keys = [f for f in range(n) if types[f] == KEY]
@@ -220,6 +234,7 @@ def merge_gathered(types, gains, sid, cost, budget):
     entries by (sid, frame), then G_altref, then G_normal, each by (gain desc,
     sid asc, frame asc); anchors = the longest prefix within budget (Z7).
     Returns per-row lists rank, is_anchor."""
+    types = [frame_groups(t) for t in types]
     rows = range(len(types))
     order = sorted(((i, f) for i in rows for f in range(len(types[i])) if types[i][f] == KEY),
                    key=lambda e: (sid[e[0]], e[1]))

@@ -22,6 +22,7 @@ LIB_PATH = os.environ.get("NS_LIB") or os.path.join(_HERE, "libneuroscaler.so")
 NS_OK, NS_EINVAL, NS_ECUDA, NS_ENOMEM, NS_EUNSUPPORTED = 0, -1, -2, -3, -4
 NS_KEY, NS_ALTREF, NS_NORMAL = 0, 1, 2
 NS_I, NS_P, NS_B = NS_KEY, NS_ALTREF, NS_NORMAL      # H.26x groups G_I, G_P, G_B
+NS_INVISIBLE, NS_TYPE_MASK = 0x80, 0x7F               # invisible frames, reading R12
 NS_REF_LAST, NS_REF_GOLDEN, NS_REF_INTRA = 0, 1, 2
 NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET, NS_GIVEN_ANCHORS = 0, 1, 2
 NS_CARRY, NS_FRESH = 0, 1

@@ -32,13 +32,13 @@ __global__ void k_golden_index(const StreamDesc *sd, int S, int n, const int16_t
     int g = -1;
     for (int f = 0; f < n; f++) {
         gold[(size_t)s * (n + 1) + f] = (int16_t)g;
-        if (T[f] == NS_KEY || T[f] == NS_ALTREF) g = f;
+        if ((T[f] & NS_TYPE_MASK) == NS_KEY || (T[f] & NS_TYPE_MASK) == NS_ALTREF) g = f;
     }
     gold[(size_t)s * (n + 1) + n] = (int16_t)g;
     if (!nxt) return;
     int gn = n;
     for (int f = n - 1; f >= 0; f--) {
-        const bool golden = T[f] == NS_KEY || T[f] == NS_ALTREF;
+        const bool golden = (T[f] & NS_TYPE_MASK) == NS_KEY || (T[f] & NS_TYPE_MASK) == NS_ALTREF;
         gsv[(size_t)s * n + f] = golden && nxt[(size_t)s * n + f] <= min(gn, n - 1);
         if (golden) gn = f;
     }
@@ -409,7 +409,7 @@ __global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *
     o.h = d.h;
     o.s = (int16_t)d.s;
     o.anchor = is_anchor[e] ? 1 : 0;
-    o.key = d.type[f] == NS_KEY;
+    o.key = (d.type[f] & NS_TYPE_MASK) == NS_KEY;
     o.fmt = d.fmt;
     fd[e] = o;
 }
@@ -697,14 +697,15 @@ __global__ void k_stats_meta(const StreamDesc *sd, int S, int n, const uint8_t *
                              double *stats) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S) return;
-    double a = 0, sa = 0, st = 0;
+    double a = 0, sa = 0, st = 0, shown = 0;
     for (int f = 0; f < n; f++) {
         const double v = (double)score[(size_t)s * n + f];
         st += v;
         if (is_anchor[(size_t)s * n + f]) { a += 1; sa += v; }
+        shown += (sd[s].type[f] & NS_INVISIBLE) ? 0 : 1;   // invisible frames are not displayed (R12)
     }
     double *o = stats + (size_t)s * 8;
-    o[0] = n; o[1] = a; o[2] = sa; o[3] = st;
+    o[0] = shown; o[1] = a; o[2] = sa; o[3] = st;
     o[4] = sd[s].gt ? 0.0 : -1.0;
     o[5] = -1.0; o[6] = 0; o[7] = 0;
 }
@@ -712,7 +713,7 @@ __global__ void k_stats_meta(const StreamDesc *sd, int S, int n, const uint8_t *
 __global__ void k_stats_sse(const StreamDesc *sd, int n, uint8_t *const *hr_tab, double *stats) {
     const int sf = blockIdx.x, sid = sf / n, f = sf % n;   // (stream, frame) on x: S*n may exceed 65535
     const StreamDesc d = sd[sid];
-    if (!d.gt) return;
+    if (!d.gt || (d.type[f] & NS_INVISIBLE)) return;   // quality over the displayed frames
     const size_t nvec = (size_t)d.hr_frame / 16;
     const uint4 *a = reinterpret_cast<const uint4 *>(hr_tab[d.hr_base + f]);
     const uint4 *b = reinterpret_cast<const uint4 *>(d.gt + (size_t)f * nvec * 16);
@@ -735,7 +736,7 @@ __global__ void k_stats_sse(const StreamDesc *sd, int n, uint8_t *const *hr_tab,
 __global__ void k_stats_final(const StreamDesc *sd, int S, int n, double *stats) {
     const int s = blockIdx.x * blockDim.x + threadIdx.x;
     if (s >= S || !sd[s].gt) return;
-    const double N = (double)sd[s].hr_frame * n;
+    const double N = (double)sd[s].hr_frame * stats[(size_t)s * 8 + 0];   // displayed frames
     const double sse = stats[(size_t)s * 8 + 4];
     double p = sse == 0.0 ? 100.0 : 10.0 * log10(255.0 * 255.0 / (sse / N));
     stats[(size_t)s * 8 + 5] = p > 100.0 ? 100.0 : p;

@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(kSelWarps * 32)
     uint8_t *T = sT[wi], *Reset = sReset[wi], *Done = sDone[wi];
     const int64_t *sc = score + (size_t)s * n;
     for (int f = lane; f < n; f += 32) {
-        T[f] = d.type[f];
+        T[f] = d.type[f] & NS_TYPE_MASK;   // an invisible frame keeps its group
         G[f] = (T[f] == NS_KEY) ? kKeyGain : 0;
         Done[f] = 0;
     }
@@ -207,7 +207,7 @@ __global__ void k_global_rank(const StreamDesc *sd, const uint8_t *type_flat, co
     const int s = e / n, f = e % n;
     auto types = [&](int q) -> const uint8_t * { return FLAT ? type_flat + (size_t)q * n : sd[q].type; };
     auto key = [&](int q) -> int { return FLAT ? sid[q] : q; };
-    const int t = types(s)[f];
+    const int t = types(s)[f] & NS_TYPE_MASK;
     const int ks = key(s);
     const int64_t g = gain[e];
     int cnt = rank_in[e];
@@ -221,7 +221,7 @@ __global__ void k_global_rank(const StreamDesc *sd, const uint8_t *type_flat, co
         while (lo < hi) {
             const int mid = (lo + hi) >> 1;
             const int f2 = O2[mid];
-            const int t2 = T2[f2];
+            const int t2 = T2[f2] & NS_TYPE_MASK;
             const int64_t g2 = G2[f2];
             const bool prec = (t2 < t) || (t2 == t && (g2 > g || (g2 == g && k2 < ks)));
             if (prec) lo = mid + 1;
@@ -246,11 +246,11 @@ __global__ void k_stream_rank(int N, int n, const int64_t *gain, const uint8_t *
     const int s = e / n, f = e % n;
     const uint8_t *T = type + (size_t)s * n;
     const int64_t *G = gain + (size_t)s * n;
-    const int t = T[f];
+    const int t = T[f] & NS_TYPE_MASK;
     const int64_t g = G[f];
     int cnt = 0;
     for (int f2 = 0; f2 < n; f2++) {
-        const int t2 = T[f2];
+        const int t2 = T[f2] & NS_TYPE_MASK;
         const int64_t g2 = G[f2];
         cnt += (t2 < t) || (t2 == t && (g2 > g || (g2 == g && f2 < f)));
     }

@@ -329,3 +329,34 @@ def test_select_h26x_groups(ctx):
             assert list(g[s]) == eg and list(r[s]) == er and list(a[s]) == ea, (k, s)
             if k >= 2:
                 assert a[s][0] and a[s][15]          # both I frames before any P or B
+
+
+def test_invisible_altrefs(ctx):
+    """NS_INVISIBLE ALTREFs (reading R12): selected and reconstructed as
+    references exactly like visible ones (the oracle on the same flagged chunk),
+    but the stats count and score only the displayed frames."""
+    n, k = 20, 3
+    m = ctx.model(1, 16, 2)
+    blob = synth.make_weights(31, 1, 16, 2)
+    m.set_weights(blob)
+    c = synth.make_chunk(3131, 48, 24, 2, n, types=synth.default_types(n, 5), with_gt=True)
+    c.type = np.where(c.type == synth.NS_ALTREF, c.type | ns.NS_INVISIBLE, c.type).astype(np.uint8)
+    shown = [f for f in range(n) if not c.type[f] & ns.NS_INVISIBLE]
+    assert len(shown) < n
+    dc = dev_chunk(ns, c, DEV, model=m, with_gt=True, state=True)
+    hr = alloc_hr(n, c, DEV)
+    ia = torch.zeros((1, n), dtype=torch.uint8, device=DEV)
+    st = torch.zeros((1, 8), dtype=torch.float64, device=DEV)
+    ctx.enhance_streams([dc], [hr], is_anchor_out=ia, stats=st, k=k)
+    torch.cuda.synchronize()
+    ref = oracle.enhance_chunk(c, blob, 1, 16, k)
+    assert list(ia.cpu().numpy()[0]) == ref["is_anchor"]
+    got = np.stack([t.cpu().numpy() for t in hr])
+    assert np.abs(got.astype(int) - ref["hr"].astype(int)).max() <= 2
+    exp, _, _ = oracle.reconstruct(c, ref["is_anchor"], got, np.zeros_like(got[0]), np.zeros_like(got[0]))
+    assert np.array_equal(got, exp)
+    s = st.cpu().numpy()[0]
+    assert s[0] == len(shown)
+    d = got[shown].astype(np.float64) - c.gt[shown].astype(np.float64)
+    mse = float((d * d).mean())
+    assert abs(s[5] - min(100.0, 10 * np.log10(255.0 ** 2 / mse))) < 1e-6
