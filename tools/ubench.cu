@@ -322,6 +322,9 @@ int main() {
     run_mma<256, false>(d);
     run_mma<32, true>(d);
     run_mma<96, true>(d);
+    run_mma<128, false>(d);
+    run_mma<128, true>(d);
+    run_mma<192, true>(d);
     run_mma<16, false, 4>(d);
     run_mma<32, false, 2>(d);
     run_mma<32, false, 4>(d);
