@@ -48,9 +48,10 @@ def lib():
         L.or_score.argtypes = [P, i, i, i, P, P]
         L.or_upsample.argtypes = [P, i, i, i, P]
         L.or_warp_plane.argtypes = [P, i, i, i, P, i, P]
-        L.or_reconstruct.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P]
+        L.or_reconstruct.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P, i]
         L.or_reconstruct.restype = i
-        L.or_reconstruct_i420.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P]
+        L.or_reconstruct_i420.argtypes = [i, i, i, i, P, P, P, P, P, P, P, P, i]
+        L.or_filter8.argtypes = [i, i, i]
         L.or_reconstruct_i420.restype = i
         L.or_conv3x3.argtypes = [P, i, i, i, P, P, i, P]
         L.or_pixel_shuffle.argtypes = [P, i, i, i, i, P]
@@ -113,7 +114,8 @@ def reconstruct(chunk, is_anchor, hr_anchor, hr_last=None, hr_golden=None, s=Non
     gold = None if hr_golden is None else np.array(hr_golden, np.uint8, copy=True, order="C")
     rc = lib().or_reconstruct(w, h, s, n, _p(np.ascontiguousarray(chunk.lr)),
                               _p(np.ascontiguousarray(chunk.res)), _p(np.ascontiguousarray(chunk.mv)),
-                              _p(np.ascontiguousarray(chunk.type)), _p(ia), _p(hr), _p(last), _p(gold))
+                              _p(np.ascontiguousarray(chunk.type)), _p(ia), _p(hr), _p(last), _p(gold),
+                              int(getattr(chunk, "interp", 0)))
     if rc != 0:
         raise RuntimeError(f"or_reconstruct failed: {rc}")
     return hr, last, gold
@@ -131,10 +133,16 @@ def reconstruct_i420(chunk, is_anchor, hr_anchor, hr_last=None, hr_golden=None, 
     gold = None if hr_golden is None else np.array(hr_golden, np.uint8, copy=True, order="C")
     rc = lib().or_reconstruct_i420(w, h, s, n, _p(np.ascontiguousarray(chunk.lr)),
                                    _p(np.ascontiguousarray(chunk.res)), _p(np.ascontiguousarray(chunk.mv)),
-                                   _p(np.ascontiguousarray(chunk.type)), _p(ia), _p(hr), _p(last), _p(gold))
+                                   _p(np.ascontiguousarray(chunk.type)), _p(ia), _p(hr), _p(last), _p(gold),
+                                   int(getattr(chunk, "interp", 0)))
     if rc != 0:
         raise RuntimeError(f"or_reconstruct_i420 failed: {rc}")
     return hr, last, gold
+
+
+def filter8(kernel: int) -> np.ndarray:
+    """The oracle's 8-tap table of one kernel (0 regular, 1 smooth, 2 sharp): int [16][8]."""
+    return np.array([[lib().or_filter8(kernel, p, t) for t in range(8)] for p in range(16)], np.int64)
 
 
 def i420_planes(flat: np.ndarray, h: int, w: int):

@@ -21,6 +21,8 @@
  *   or_warp_plane       O7: 1/8-pel two-pass bilinear warp of an HR plane (Z14)
  *   or_reconstruct      O8: reuse-based reconstruction of a chunk
  *   or_reconstruct_i420 O8 on YUV 4:2:0 frames, chroma MC at 1/16 pel (NEXT-2; R9)
+ *   (both take `interp`: 0 = the bilinear of O7 / R9, 1-4 = VP9's 8-tap
+ *    sub-pel filters, NEXT-2, reading R13)
  *   or_conv3x3          3x3 cross-correlation, zero padding 1 (EDSR conv, P:306 / [89])
  *   or_pixel_shuffle    PyTorch-order pixel shuffle (EDSR upsampler)
  *   or_sr_forward       O5: the whole SR DNN on one LR frame ("8 residual
@@ -33,9 +35,10 @@
 #include <string.h>
 #include <math.h>
 
-/* 8 bytes per 8x8 LR block: int16 mvx, int16 mvy (1/8 LR pel), uint8 ref, 3 pad.
+/* 8 bytes per 8x8 LR block: int16 mvx, int16 mvy (1/8 LR pel), uint8 ref,
+   uint8 filter (the block's 8-tap kernel when interp = 4), 2 pad.
    Layout restated from DESIGN.md "Data layout" (not included from include/). */
-typedef struct { int16_t mvx, mvy; uint8_t ref; uint8_t pad[3]; } or_mv;
+typedef struct { int16_t mvx, mvy; uint8_t ref; uint8_t filter; uint8_t pad[2]; } or_mv;
 enum { OR_KEY = 0, OR_ALTREF = 1, OR_NORMAL = 2 };
 enum { OR_LAST = 0, OR_GOLDEN = 1, OR_INTRA = 2 };
 
@@ -125,6 +128,72 @@ void or_warp_plane(const uint8_t *ref, int H, int W, int s, const or_mv *mv, int
         }
 }
 
+/* ---------------------------------------------------------------- 8-tap MC (NEXT-2, R13) */
+/* VP9's sub-pel interpolation kernels (libvpx vp9/common/vp9_filter.c:
+   sub_pel_filters_8, _8lp, _8s), 16 phases of 8 taps, each row summing to 128
+   (FILTER_BITS 7).  Index: [kernel][phase][tap], kernel 0 = EIGHTTAP
+   (regular), 1 = EIGHTTAP_SMOOTH, 2 = EIGHTTAP_SHARP (libvpx's order). */
+static const int OR_F8[3][16][8] = {
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {0, 1, -5, 126, 8, -3, 1, 0},
+     {-1, 3, -10, 122, 18, -6, 2, 0},   {-1, 4, -13, 118, 27, -9, 3, -1},
+     {-1, 4, -16, 112, 37, -11, 4, -1}, {-1, 5, -18, 105, 48, -14, 4, -1},
+     {-1, 5, -19, 97, 58, -16, 5, -1},  {-1, 6, -19, 88, 68, -18, 5, -1},
+     {-1, 6, -19, 78, 78, -19, 6, -1},  {-1, 5, -18, 68, 88, -19, 6, -1},
+     {-1, 5, -16, 58, 97, -19, 5, -1},  {-1, 4, -14, 48, 105, -18, 5, -1},
+     {-1, 4, -11, 37, 112, -16, 4, -1}, {-1, 3, -9, 27, 118, -13, 4, -1},
+     {0, 2, -6, 18, 122, -10, 3, -1},   {0, 1, -3, 8, 126, -5, 1, 0}},
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {-3, -1, 32, 64, 38, 1, -3, 0},
+     {-2, -2, 29, 63, 41, 2, -3, 0},    {-2, -2, 26, 63, 43, 4, -4, 0},
+     {-2, -3, 24, 62, 46, 5, -4, 0},    {-2, -3, 21, 60, 49, 7, -4, 0},
+     {-1, -4, 18, 59, 51, 9, -4, 0},    {-1, -4, 16, 57, 53, 12, -4, -1},
+     {-1, -4, 14, 55, 55, 14, -4, -1},  {-1, -4, 12, 53, 57, 16, -4, -1},
+     {0, -4, 9, 51, 59, 18, -4, -1},    {0, -4, 7, 49, 60, 21, -3, -2},
+     {0, -4, 5, 46, 62, 24, -3, -2},    {0, -4, 4, 43, 63, 26, -2, -2},
+     {0, -3, 2, 41, 63, 29, -2, -2},    {0, -3, 1, 38, 64, 32, -1, -3}},
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {-1, 3, -7, 127, 8, -3, 1, 0},
+     {-2, 5, -13, 125, 17, -6, 3, -1},  {-3, 7, -17, 121, 27, -10, 5, -2},
+     {-4, 9, -20, 115, 37, -13, 6, -2}, {-4, 10, -23, 108, 48, -16, 8, -3},
+     {-4, 10, -24, 100, 59, -19, 9, -3}, {-4, 11, -24, 90, 70, -21, 10, -4},
+     {-4, 11, -23, 80, 80, -23, 11, -4}, {-4, 10, -21, 70, 90, -24, 11, -4},
+     {-3, 9, -19, 59, 100, -24, 10, -4}, {-3, 8, -16, 48, 108, -23, 10, -4},
+     {-2, 6, -13, 37, 115, -20, 9, -4}, {-2, 5, -10, 27, 121, -17, 7, -3},
+     {-1, 3, -6, 17, 125, -13, 5, -2},  {0, 1, -3, 8, 127, -7, 3, -1}}};
+
+/* Read-only access for the pins (tests/test_oracle_eighttap.py). */
+int or_filter8(int kernel, int phase, int tap)
+{
+    if (kernel < 0 || kernel > 2 || phase < 0 || phase > 15 || tap < 0 || tap > 7) return -1000;
+    return OR_F8[kernel][phase][tap];
+}
+
+static int clip_pixel(int v) { return v < 0 ? 0 : (v > 255 ? 255 : v); }
+
+/* libvpx vpx_convolve8 semantics on the HR reference, positions in 1/16 pel
+   (q4): pixel (X, Y) with offset (qx, qy) samples x16 = 16 X + qx.  Horizontal
+   pass over the 8 rows iy-3 .. iy+4, each clip_pixel(ROUND_POWER_OF_TWO(
+   sum_k F[px][k] R[row][ix-3+k], 7)), then the vertical pass over those 8
+   values with F[py]; coordinates clamped to the plane (edge replicate, Z16). */
+static uint8_t warp_px8(const uint8_t *ref, int H, int W, int X, int Y, int qx, int qy, int kernel)
+{
+    const int64_t x16 = 16 * (int64_t)X + qx, y16 = 16 * (int64_t)Y + qy;
+    const int ix = (int)floor_div(x16, 16), px = (int)(x16 - 16 * (int64_t)ix);
+    const int iy = (int)floor_div(y16, 16), py = (int)(y16 - 16 * (int64_t)iy);
+    int t[8];
+    for (int r = 0; r < 8; r++) {
+        const int yy = clampi(iy - 3 + r, 0, H - 1);
+        int sum = 0;
+        for (int k = 0; k < 8; k++) sum += OR_F8[kernel][px][k] * ref[(size_t)yy * W + clampi(ix - 3 + k, 0, W - 1)];
+        t[r] = clip_pixel((int)floor_div(sum + 64, 128));
+    }
+    int sum = 0;
+    for (int r = 0; r < 8; r++) sum += OR_F8[kernel][py][r] * t[r];
+    return (uint8_t)clip_pixel((int)floor_div(sum + 64, 128));
+}
+
+/* The kernel a block uses: interp 1..3 -> kernel interp-1 for every block;
+   interp 4 (VP9's SWITCHABLE) -> the block's own filter byte (0..2). */
+static int block_kernel(int interp, const or_mv *b) { return interp == 4 ? b->filter : interp - 1; }
+
 /* ---------------------------------------------------------------- O8 reconstruct */
 /* Frame by frame in decode order (reuse previous SR frames guided by
    reference index, MV and residual; loss resets at an anchor; the
@@ -140,8 +209,9 @@ void or_warp_plane(const uint8_t *ref, int H, int W, int s, const or_mv *mv, int
    hr: [n][3][s*h][s*w]; lr, res: [n][3][h][w]; mv: [n][h/8][w/8]. */
 int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t *res,
                    const or_mv *mv, const uint8_t *type, const uint8_t *is_anchor,
-                   uint8_t *hr, uint8_t *hr_last, uint8_t *hr_golden)
+                   uint8_t *hr, uint8_t *hr_last, uint8_t *hr_golden, int interp)
 {
+    if (interp < 0 || interp > 4) return -2;
     const int H = s * h, W = s * w, bw = w / 8;
     const size_t lr_plane = (size_t)h * w, hr_plane = (size_t)H * W;
     int32_t *in = (int32_t *)malloc(lr_plane * sizeof(int32_t));
@@ -174,7 +244,11 @@ int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t 
                         if (b->ref == OR_INTRA) { op[i] = (uint8_t)up_lr[i]; continue; }
                         const uint8_t *r = (b->ref == OR_GOLDEN ? golden : last);
                         if (!r) { free(in); free(up_lr); free(up_res); free(pred); return -1; }
-                        int p = warp_px(r + (size_t)c * hr_plane, H, W, X, Y, s * b->mvx, s * b->mvy);
+                        if (interp == 4 && b->filter > 2) { free(in); free(up_lr); free(up_res); free(pred); return -2; }
+                        /* R13: luma q4 offset = 2 s mv (1/8 -> 1/16 pel) */
+                        int p = interp ? warp_px8(r + (size_t)c * hr_plane, H, W, X, Y, 2 * s * b->mvx, 2 * s * b->mvy,
+                                                  block_kernel(interp, b))
+                                       : warp_px(r + (size_t)c * hr_plane, H, W, X, Y, s * b->mvx, s * b->mvy);
                         op[i] = (uint8_t)clampi(p + up_res[i], 0, 255);
                     }
             }
@@ -215,8 +289,9 @@ static uint8_t warp_px16(const uint8_t *ref, int H, int W, int X, int Y, int mx,
    lr, res: [n][h*w*3/2]; hr: [n][s*h*s*w*3/2]; hr_last, hr_golden one HR frame. */
 int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int16_t *res,
                         const or_mv *mv, const uint8_t *type, const uint8_t *is_anchor,
-                        uint8_t *hr, uint8_t *hr_last, uint8_t *hr_golden)
+                        uint8_t *hr, uint8_t *hr_last, uint8_t *hr_golden, int interp)
 {
+    if (interp < 0 || interp > 4) return -2;
     const int H = s * h, W = s * w, bw = w / 8;
     const size_t lrf = (size_t)h * w * 3 / 2, hrf = (size_t)H * W * 3 / 2;
     int32_t *in = (int32_t *)malloc((size_t)h * w * sizeof(int32_t));
@@ -253,7 +328,11 @@ int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int
                         if (b->ref == OR_INTRA) { op[i] = (uint8_t)up_lr[i]; continue; }
                         const uint8_t *r = (b->ref == OR_GOLDEN ? golden : last);
                         if (!r) { free(in); free(up_lr); free(up_res); return -1; }
-                        int p = c ? warp_px16(r + ho, PH, PW, X, Y, s * b->mvx, s * b->mvy)
+                        if (interp == 4 && b->filter > 2) { free(in); free(up_lr); free(up_res); return -2; }
+                        /* R13: q4 offset = 2 s mv for luma, s mv for chroma (already 1/16 chroma pel, R9) */
+                        int p = interp ? warp_px8(r + ho, PH, PW, X, Y, (c ? 1 : 2) * s * b->mvx, (c ? 1 : 2) * s * b->mvy,
+                                                  block_kernel(interp, b))
+                              : c ? warp_px16(r + ho, PH, PW, X, Y, s * b->mvx, s * b->mvy)
                                   : warp_px(r + ho, PH, PW, X, Y, s * b->mvx, s * b->mvy);
                         op[i] = (uint8_t)clampi(p + up_res[i], 0, 255);
                     }

@@ -32,8 +32,28 @@ import numpy as np
 NS_KEY, NS_ALTREF, NS_NORMAL = 0, 1, 2
 NS_REF_LAST, NS_REF_GOLDEN, NS_REF_INTRA = 0, 1, 2
 
-# ns_block_mv in include/ns.h: { int16 mvx, mvy; uint8 ref; uint8 pad[3]; }
-MV_DTYPE = np.dtype([("mvx", "<i2"), ("mvy", "<i2"), ("ref", "u1"), ("pad", "u1", (3,))])
+# ns_block_mv in include/ns.h: { int16 mvx, mvy; uint8 ref; uint8 filter; uint8 pad[2]; }
+MV_DTYPE = np.dtype([("mvx", "<i2"), ("mvy", "<i2"), ("ref", "u1"), ("filter", "u1"), ("pad", "u1", (2,))])
+
+# Sub-pel interpolation of the synthetic codec (ns_chunk.interp): 0 = two-pass
+# bilinear; 1 / 2 / 3 = VP9's 8-tap regular / smooth / sharp kernel for every
+# block; 4 = per block (MV_DTYPE.filter: 0 regular, 1 smooth, 2 sharp).
+INTERP_BILINEAR, INTERP_REGULAR, INTERP_SMOOTH, INTERP_SHARP, INTERP_SWITCHABLE = 0, 1, 2, 3, 4
+# VP9's 8-tap kernels as published in libvpx (vp9_filter.c), phases 0..8; the
+# codec mirrors them for phases 9..15 (phase 16-p = phase p reversed).
+_VP9_HALF = {
+    0: [[0, 0, 0, 128, 0, 0, 0, 0], [0, 1, -5, 126, 8, -3, 1, 0], [-1, 3, -10, 122, 18, -6, 2, 0],
+        [-1, 4, -13, 118, 27, -9, 3, -1], [-1, 4, -16, 112, 37, -11, 4, -1], [-1, 5, -18, 105, 48, -14, 4, -1],
+        [-1, 5, -19, 97, 58, -16, 5, -1], [-1, 6, -19, 88, 68, -18, 5, -1], [-1, 6, -19, 78, 78, -19, 6, -1]],
+    1: [[0, 0, 0, 128, 0, 0, 0, 0], [-3, -1, 32, 64, 38, 1, -3, 0], [-2, -2, 29, 63, 41, 2, -3, 0],
+        [-2, -2, 26, 63, 43, 4, -4, 0], [-2, -3, 24, 62, 46, 5, -4, 0], [-2, -3, 21, 60, 49, 7, -4, 0],
+        [-1, -4, 18, 59, 51, 9, -4, 0], [-1, -4, 16, 57, 53, 12, -4, -1], [-1, -4, 14, 55, 55, 14, -4, -1]],
+    2: [[0, 0, 0, 128, 0, 0, 0, 0], [-1, 3, -7, 127, 8, -3, 1, 0], [-2, 5, -13, 125, 17, -6, 3, -1],
+        [-3, 7, -17, 121, 27, -10, 5, -2], [-4, 9, -20, 115, 37, -13, 6, -2], [-4, 10, -23, 108, 48, -16, 8, -3],
+        [-4, 10, -24, 100, 59, -19, 9, -3], [-4, 11, -24, 90, 70, -21, 10, -4], [-4, 11, -23, 80, 80, -23, 11, -4]],
+}
+VP9_KERNELS = np.array([h + [r[::-1] for r in h[7:0:-1]] for h in (_VP9_HALF[0], _VP9_HALF[1], _VP9_HALF[2])],
+                       np.int64)   # [kernel][phase 0..15][tap]
 
 # Six motion/texture profiles named after the paper's six Twitch categories
 # (P:275).  pan = (vx, vy) in 1/8 LR pel per frame; noise = amplitude of the
@@ -60,6 +80,7 @@ class Chunk:
     type: np.ndarray      # u8  [n]
     res_size: np.ndarray  # u32 [n] encoded-size proxy
     gt: np.ndarray | None = None  # u8 [n][3][s*h][s*w] (only with_gt=True)
+    interp: int = INTERP_BILINEAR  # the codec's sub-pel filter (ns_chunk.interp)
 
     @property
     def n(self) -> int:
@@ -234,9 +255,10 @@ def _box_down(img: np.ndarray, s: int) -> np.ndarray:
 def make_chunk(seed: int, w: int, h: int, scale: int, n: int, *, types=None,
                altref_every: int | None = 16, profile: int | None = None,
                intra_frac: float = 0.02, golden_frac: float = 0.15,
-               jitter: float = 0.3, with_gt: bool = False) -> Chunk:
+               jitter: float = 0.3, with_gt: bool = False, interp: int = INTERP_BILINEAR) -> Chunk:
     """Generate one stream's chunk.  Seeds follow SURVEY.md §8(d):
-    seed = stream_id + 1000 * config."""
+    seed = stream_id + 1000 * config.  interp: the codec's sub-pel filter
+    (INTERP_*); the default stream is bilinear and draws no extra randoms."""
     assert w % 8 == 0 and h % 8 == 0 and n >= 1
     rng = np.random.default_rng(seed)
     prof = PROFILES[(seed % len(PROFILES)) if profile is None else profile]
@@ -288,8 +310,16 @@ def make_chunk(seed: int, w: int, h: int, scale: int, n: int, *, types=None,
             mvy = np.clip(mvy, -32768, 32767)
             mvx[ref == NS_REF_INTRA] = 0
             mvy[ref == NS_REF_INTRA] = 0
-            pred_l = _codec_predict(lr[f - 1], mvx, mvy) if f > 0 else np.full((3, h, w), 128, np.int64)
-            pred_g = _codec_predict(lr[golden], mvx, mvy) if golden >= 0 and (ref == NS_REF_GOLDEN).any() else pred_l
+            if interp:
+                kb = _block_kernels(rng, interp, bh, bw)
+                mv[f]["filter"] = kb if interp == INTERP_SWITCHABLE else 0
+
+                def predict(r_):
+                    return _codec_predict8(r_, mvx, mvy, kb, 8, 2)
+            else:
+                predict = lambda r_: _codec_predict(r_, mvx, mvy)  # noqa: E731
+            pred_l = predict(lr[f - 1]) if f > 0 else np.full((3, h, w), 128, np.int64)
+            pred_g = predict(lr[golden]) if golden >= 0 and (ref == NS_REF_GOLDEN).any() else pred_l
             refpx = np.repeat(np.repeat(ref, 8, 0), 8, 1)[None]
             pred = np.where(refpx == NS_REF_GOLDEN, pred_g, pred_l)
             pred = np.where(refpx == NS_REF_INTRA, 128, pred)
@@ -305,7 +335,7 @@ def make_chunk(seed: int, w: int, h: int, scale: int, n: int, *, types=None,
     nz = np.abs(res.reshape(n, -1).astype(np.int64))
     res_size = (1 + (np.log2(1 + nz).sum(axis=1) / 8.0)).astype(np.uint32)
     return Chunk(w=w, h=h, scale=scale, lr=lr, res=res, mv=mv, type=types,
-                 res_size=res_size, gt=gt)
+                 res_size=res_size, gt=gt, interp=interp)
 
 
 def _codec_predict16(ref: np.ndarray, mvx_b: np.ndarray, mvy_b: np.ndarray) -> np.ndarray:
@@ -328,6 +358,40 @@ def _codec_predict16(ref: np.ndarray, mvx_b: np.ndarray, mvy_b: np.ndarray) -> n
     return out.transpose(0, 1, 3, 2, 4).reshape(C, H, W).astype(np.int64)
 
 
+def _codec_predict8(ref: np.ndarray, mvx_b: np.ndarray, mvy_b: np.ndarray, kern_b: np.ndarray, bs: int,
+                    q4: int) -> np.ndarray:
+    """Encoder-side 8-tap prediction of the synthetic codec (libvpx convolve8
+    semantics): the block's vector times q4 gives its offset in 1/16 pel (2 for
+    luma vectors in 1/8 pel, 1 for a 4:2:0 chroma plane), taps at -3..+4 around
+    the integer position, each pass rounded by 7 bits and clipped to a byte,
+    edge-replicated borders; blocks of bs x bs pixels, kernel per block."""
+    C, H, W = ref.shape
+    bh, bw = mvx_b.shape
+    ox16 = mvx_b.astype(np.int64) * q4
+    oy16 = mvy_b.astype(np.int64) * q4
+    ix, px = np.floor_divide(ox16, 16), np.mod(ox16, 16)
+    iy, py = np.floor_divide(oy16, 16), np.mod(oy16, 16)
+    m = int(max(np.abs(ix).max(initial=0), np.abs(iy).max(initial=0))) + 8
+    pad = np.pad(ref, ((0, 0), (m, m), (m, m)), mode="edge").astype(np.int64)
+    win = np.lib.stride_tricks.sliding_window_view(pad, (bs + 7, bs + 7), axis=(1, 2))
+    oy = (np.arange(bh) * bs)[:, None] + iy - 3 + m
+    ox = (np.arange(bw) * bs)[None, :] + ix - 3 + m
+    wv = win[:, oy, ox]                                    # [C][bh][bw][bs+7][bs+7]
+    fx = VP9_KERNELS[kern_b, px]                            # [bh][bw][8]
+    fy = VP9_KERNELS[kern_b, py]
+    taps = np.lib.stride_tricks.sliding_window_view(wv, 8, axis=4)   # [C][bh][bw][bs+7][bs][8]
+    hrow = np.clip(((taps * fx[None, :, :, None, None, :]).sum(-1) + 64) >> 7, 0, 255)   # [C][bh][bw][bs+7][bs]
+    vt = np.lib.stride_tricks.sliding_window_view(hrow, 8, axis=3)   # [C][bh][bw][bs][bs][8]
+    out = np.clip(((vt * fy[None, :, :, None, None, :]).sum(-1) + 64) >> 7, 0, 255)
+    return out.transpose(0, 1, 3, 2, 4).reshape(C, H, W).astype(np.int64)
+
+
+def _block_kernels(rng, interp: int, bh: int, bw: int) -> np.ndarray:
+    if interp == INTERP_SWITCHABLE:
+        return rng.integers(0, 3, (bh, bw)).astype(np.uint8)
+    return np.full((bh, bw), max(interp - 1, 0), np.uint8)
+
+
 @dataclasses.dataclass
 class ChunkI420:
     """One stream's chunk in YUV 4:2:0 (NEXT-2): per frame Y [h][w] then U, V
@@ -342,6 +406,7 @@ class ChunkI420:
     res_size: np.ndarray
     gt: np.ndarray | None = None   # u8 [n][s*h*s*w*3/2]
     fmt: str = "i420"
+    interp: int = INTERP_BILINEAR
 
     @property
     def n(self) -> int:
@@ -359,7 +424,7 @@ def to_i420(planes: np.ndarray) -> np.ndarray:
 
 def make_chunk_i420(seed: int, w: int, h: int, scale: int, n: int, *, types=None, altref_every: int | None = 16,
                     profile: int | None = None, intra_frac: float = 0.02, golden_frac: float = 0.15,
-                    jitter: float = 0.3, with_gt: bool = False) -> ChunkI420:
+                    jitter: float = 0.3, with_gt: bool = False, interp: int = INTERP_BILINEAR) -> ChunkI420:
     """The synthetic codec loop of make_chunk in YUV 4:2:0: luma exactly as
     there, chroma planes at half resolution predicted with the block's luma
     vector read in 1/16 chroma pel (_codec_predict16)."""
@@ -417,6 +482,9 @@ def make_chunk_i420(seed: int, w: int, h: int, scale: int, n: int, *, types=None
             mvy = np.clip(mvy, -32768, 32767)
             mvx[ref == NS_REF_INTRA] = 0
             mvy[ref == NS_REF_INTRA] = 0
+            if interp:
+                kb = _block_kernels(rng, interp, bh, bw)
+                mv[f]["filter"] = kb if interp == INTERP_SWITCHABLE else 0
             pred = np.empty(P * 3 // 2, np.int64)
             refpx_y = np.repeat(np.repeat(ref, 8, 0), 8, 1)
             refpx_c = np.repeat(np.repeat(ref, 4, 0), 4, 1)
@@ -424,8 +492,12 @@ def make_chunk_i420(seed: int, w: int, h: int, scale: int, n: int, *, types=None
                 if rp_ < 0 or not (ref == which).any():
                     continue
                 ry, rc = planes(lr[rp_])
-                py = _codec_predict(ry, mvx, mvy)[0]
-                pc = _codec_predict16(rc, mvx, mvy)
+                if interp:
+                    py = _codec_predict8(ry, mvx, mvy, kb, 8, 2)[0]
+                    pc = _codec_predict8(rc, mvx, mvy, kb, 4, 1)
+                else:
+                    py = _codec_predict(ry, mvx, mvy)[0]
+                    pc = _codec_predict16(rc, mvx, mvy)
                 cur = np.concatenate([py.ravel(), pc.reshape(-1)])
                 sel = np.concatenate([(refpx_y == which).ravel(), np.tile((refpx_c == which).ravel(), 2)])
                 pred[sel] = cur[sel]
@@ -441,7 +513,8 @@ def make_chunk_i420(seed: int, w: int, h: int, scale: int, n: int, *, types=None
             golden = f
     nz = np.abs(res.astype(np.int64))
     res_size = (1 + (np.log2(1 + nz).sum(axis=1) / 8.0)).astype(np.uint32)
-    return ChunkI420(w=w, h=h, scale=scale, lr=lr, res=res, mv=mv, type=types, res_size=res_size, gt=gt)
+    return ChunkI420(w=w, h=h, scale=scale, lr=lr, res=res, mv=mv, type=types, res_size=res_size, gt=gt,
+                     interp=interp)
 
 
 def _to_bf16_bits(x: np.ndarray) -> np.ndarray:
