@@ -79,12 +79,34 @@ typedef enum {
 /* Reference index of a block ("reference index"). */
 typedef enum { NS_REF_LAST = 0, NS_REF_GOLDEN = 1, NS_REF_INTRA = 2 } ns_ref;
 
-/* One 8x8 LR block's motion vector (1/8 LR pel) and reference. 8 bytes. */
+/* One 8x8 LR block's motion vector (1/8 LR pel) and reference. 8 bytes.
+   A codec's larger partitions (VP9 16x16 .. 64x64) are their vector repeated
+   on every 8x8 block they cover (reading R14). */
 typedef struct {
     int16_t mvx, mvy;
     uint8_t ref;        /* ns_ref */
-    uint8_t pad[3];
+    uint8_t filter;     /* NS_INTERP_SWITCHABLE chunks: this block's 8-tap kernel,
+                           0 EIGHTTAP, 1 EIGHTTAP_SMOOTH, 2 EIGHTTAP_SHARP (values
+                           above 2 read as 0); ignored otherwise               */
+    uint8_t pad[2];
 } ns_block_mv;
+
+/* Sub-pel motion compensation of a stream (ns_chunk.interp; SURVEY §8(f)
+   NEXT-2, reading R13).  P:89 names "lightweight bilinear interpolation":
+   NS_INTERP_BILINEAR (0, the default) is the two-pass bilinear of reading
+   Z14 (R9 for 4:2:0 chroma).  The others are VP9's own sub-pel filters
+   (libvpx vpx_convolve8 semantics), so a reused frame is predicted the way
+   the decoder predicted its LR frame: positions in 1/16 pel (2 s mv for luma,
+   s mv for 4:2:0 chroma), 8 taps at -3..+4, each pass rounded by 7 bits and
+   clipped to a byte, edges replicated.  SWITCHABLE takes the kernel per block
+   (ns_block_mv.filter), as VP9's per-block interp_filter. */
+enum {
+    NS_INTERP_BILINEAR = 0,
+    NS_INTERP_EIGHTTAP = 1,         /* libvpx sub_pel_filters_8   */
+    NS_INTERP_EIGHTTAP_SMOOTH = 2,  /* libvpx sub_pel_filters_8lp */
+    NS_INTERP_EIGHTTAP_SHARP = 3,   /* libvpx sub_pel_filters_8s  */
+    NS_INTERP_SWITCHABLE = 4
+};
 
 typedef struct ns_ctx ns_ctx;
 typedef struct ns_model ns_model;
@@ -122,6 +144,7 @@ typedef struct {
                                   May be NULL under the same condition.            */
     const uint8_t *gt;         /* optional [n][3][s*h][s*w] ground truth for stats   */
     int32_t format;            /* NS_FMT_444 (0, the layouts above) | NS_FMT_I420   */
+    int32_t interp;            /* NS_INTERP_* (0 = bilinear); the codec's MC filter */
 } ns_chunk;
 
 /* Anchor selection mode (§5.1 top-k per chunk; §5.2 global budget).

@@ -191,8 +191,9 @@ static uint8_t warp_px8(const uint8_t *ref, int H, int W, int X, int Y, int qx, 
 }
 
 /* The kernel a block uses: interp 1..3 -> kernel interp-1 for every block;
-   interp 4 (VP9's SWITCHABLE) -> the block's own filter byte (0..2). */
-static int block_kernel(int interp, const or_mv *b) { return interp == 4 ? b->filter : interp - 1; }
+   interp 4 (VP9's SWITCHABLE) -> the block's own filter byte (0..2; larger
+   values read as 0, include/ns.h). */
+static int block_kernel(int interp, const or_mv *b) { return interp == 4 ? (b->filter > 2 ? 0 : b->filter) : interp - 1; }
 
 /* ---------------------------------------------------------------- O8 reconstruct */
 /* Frame by frame in decode order (reuse previous SR frames guided by
@@ -244,7 +245,6 @@ int or_reconstruct(int w, int h, int s, int n, const uint8_t *lr, const int16_t 
                         if (b->ref == OR_INTRA) { op[i] = (uint8_t)up_lr[i]; continue; }
                         const uint8_t *r = (b->ref == OR_GOLDEN ? golden : last);
                         if (!r) { free(in); free(up_lr); free(up_res); free(pred); return -1; }
-                        if (interp == 4 && b->filter > 2) { free(in); free(up_lr); free(up_res); free(pred); return -2; }
                         /* R13: luma q4 offset = 2 s mv (1/8 -> 1/16 pel) */
                         int p = interp ? warp_px8(r + (size_t)c * hr_plane, H, W, X, Y, 2 * s * b->mvx, 2 * s * b->mvy,
                                                   block_kernel(interp, b))
@@ -328,7 +328,6 @@ int or_reconstruct_i420(int w, int h, int s, int n, const uint8_t *lr, const int
                         if (b->ref == OR_INTRA) { op[i] = (uint8_t)up_lr[i]; continue; }
                         const uint8_t *r = (b->ref == OR_GOLDEN ? golden : last);
                         if (!r) { free(in); free(up_lr); free(up_res); return -1; }
-                        if (interp == 4 && b->filter > 2) { free(in); free(up_lr); free(up_res); return -2; }
                         /* R13: q4 offset = 2 s mv for luma, s mv for chroma (already 1/16 chroma pel, R9) */
                         int p = interp ? warp_px8(r + ho, PH, PW, X, Y, (c ? 1 : 2) * s * b->mvx, (c ? 1 : 2) * s * b->mvy,
                                                   block_kernel(interp, b))

@@ -28,6 +28,9 @@ NS_TOPK_PER_STREAM, NS_GLOBAL_BUDGET, NS_GIVEN_ANCHORS = 0, 1, 2
 NS_CARRY, NS_FRESH = 0, 1
 NS_SEL_NEUROSCALER, NS_SEL_KEY, NS_SEL_KEY_UNIFORM = 0, 1, 2
 NS_FMT_444, NS_FMT_I420 = 0, 1
+# sub-pel motion compensation (ns_chunk.interp; reading R13)
+NS_INTERP_BILINEAR, NS_INTERP_EIGHTTAP, NS_INTERP_EIGHTTAP_SMOOTH, NS_INTERP_EIGHTTAP_SHARP, NS_INTERP_SWITCHABLE = \
+    0, 1, 2, 3, 4
 
 P = ctypes.c_void_p
 
@@ -35,7 +38,8 @@ P = ctypes.c_void_p
 class NsChunk(ctypes.Structure):
     _fields_ = [("w", ctypes.c_int32), ("h", ctypes.c_int32), ("scale", ctypes.c_int32), ("n_frames", ctypes.c_int32),
                 ("lr", P), ("res", P), ("mv", P), ("type", P), ("res_size", P), ("model", P),
-                ("hr_last", P), ("hr_golden", P), ("gt", P), ("format", ctypes.c_int32)]
+                ("hr_last", P), ("hr_golden", P), ("gt", P), ("format", ctypes.c_int32),
+                ("interp", ctypes.c_int32)]
 
 
 class NsSelectParams(ctypes.Structure):
@@ -190,6 +194,7 @@ class DeviceChunk:
     hr_golden: "object" = None
     gt: "object" = None        # uint8 [n,3,sH,sW]
     format: int = NS_FMT_444   # NS_FMT_I420: lr/res [n, h*w*3/2], HR frames s*h*s*w*3/2 bytes
+    interp: int = NS_INTERP_BILINEAR  # the codec's sub-pel filter (NS_INTERP_*)
 
     @property
     def n(self) -> int:
@@ -198,11 +203,11 @@ class DeviceChunk:
     def to_c(self) -> NsChunk:
         return NsChunk(self.w, self.h, self.scale, self.n, _ptr(self.lr), _ptr(self.res), _ptr(self.mv),
                        _ptr(self.type), _ptr(self.res_size), self.model.handle if self.model else None,
-                       _ptr(self.hr_last), _ptr(self.hr_golden), _ptr(self.gt), int(self.format))
+                       _ptr(self.hr_last), _ptr(self.hr_golden), _ptr(self.gt), int(self.format), int(self.interp))
 
     @staticmethod
     def from_numpy(lr, res, mv, types, w, h, scale, device, res_size=None, gt=None, model=None,
-                   hr_last=None, hr_golden=None, format=NS_FMT_444) -> "DeviceChunk":
+                   hr_last=None, hr_golden=None, format=NS_FMT_444, interp=NS_INTERP_BILINEAR) -> "DeviceChunk":
         """Copies host arrays (mv as a structured or raw 8-byte array) to `device`."""
         import torch
         mvb = np.ascontiguousarray(mv).view(np.uint8).reshape(mv.shape[0], h // 8, w // 8, 8)
@@ -210,12 +215,12 @@ class DeviceChunk:
         rs = None if res_size is None else t(np.asarray(res_size).astype(np.int32))
         return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
                            model=model, res_size=rs, gt=None if gt is None else t(gt),
-                           hr_last=hr_last, hr_golden=hr_golden, format=format)
+                           hr_last=hr_last, hr_golden=hr_golden, format=format, interp=interp)
 
 
     @staticmethod
     def pinned_from_numpy(lr, res, mv, types, w, h, scale, res_size=None, model=None,
-                          hr_last=None, hr_golden=None, format=NS_FMT_444) -> "DeviceChunk":
+                          hr_last=None, hr_golden=None, format=NS_FMT_444, interp=NS_INTERP_BILINEAR) -> "DeviceChunk":
         """Host chunk for ns_enhance_streams_host: inputs in page-locked host
         memory (torch pinned tensors); hr_last / hr_golden stay on the device."""
         import torch
@@ -223,7 +228,8 @@ class DeviceChunk:
         t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
         rs = None if res_size is None else t(np.asarray(res_size).astype(np.int32))
         return DeviceChunk(w=w, h=h, scale=scale, lr=t(lr), res=t(res), mv=t(mvb), type=t(np.asarray(types, np.uint8)),
-                           model=model, res_size=rs, hr_last=hr_last, hr_golden=hr_golden, format=format)
+                           model=model, res_size=rs, hr_last=hr_last, hr_golden=hr_golden, format=format,
+                           interp=interp)
 
 
 class Model:

@@ -316,11 +316,12 @@ __host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S)
 //   v    = 128 V[d] + w1 (V[d+1] - V[d])          (exact 2-D O6 sum, d = tap)
 //   s    = 4 (v + 8192 + 2^22) = 512 V[d] + 4 w1 (V[d+1] - V[d]) + KB
 // and r + 256 = s >> 16 (high half-word).
-template <int S, bool CH, int WY>
+// (UOFF: the lane offset, r + UOFF; 256 here, 384 in k_recon8)
+template <int S, bool CH, int WY, int UOFF = 256>
 __device__ __forceinline__ void recon_up_row(const int (&a)[ReconCfg<S, CH>::NLR], const int (&b)[ReconCfg<S, CH>::NLR],
                                              uint32_t (&u)[ReconCfg<S, CH>::NP]) {
     constexpr int BW = ReconCfg<S, CH>::BW, NLR = ReconCfg<S, CH>::NLR;
-    constexpr int KB = 4 * 8192 + 4 * (256 << 14);
+    constexpr int KB = 4 * 8192 + 4 * (UOFF << 14);
     int V[NLR], base[NLR];
 #pragma unroll
     for (int t = 0; t < NLR; t++) {
@@ -411,6 +412,7 @@ __global__ void k_frame_desc(const StreamDesc *sd, int S, int n, const uint8_t *
     o.anchor = is_anchor[e] ? 1 : 0;
     o.key = (d.type[f] & NS_TYPE_MASK) == NS_KEY;
     o.fmt = d.fmt;
+    o.interp = d.interp;
     fd[e] = o;
 }
 
@@ -464,6 +466,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
         if (fd.anchor && fd.asrc) recon_tile_copy(fd.asrc + hr0, fd.out + hr0, phr, W, x0, x1, Y0c, y1, tid, kReconNT, np_);
     }
     if (fd.anchor) return;                              // CTA-uniform: the anchor's SR bytes are in place
+    if (fd.interp != NS_INTERP_BILINEAR) return;        // CTA-uniform: an 8-tap stream steps in k_recon8
 
     extern __shared__ __align__(16) uint8_t recon_sm[];
     uint2 *rsm = reinterpret_cast<uint2 *>(recon_sm);                  // [RPT+1][NQ][NT] warp windows
@@ -614,6 +617,247 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
     }
 }
 
+// ---------------------------------------------------------------- 8-tap MC (NEXT-2, R13)
+// Streams whose codec predicts with VP9's 8-tap sub-pel filters (ns_chunk.interp,
+// include/ns.h): the reused frame is predicted the way the decoder predicted
+// its LR frame -- libvpx convolve8 on the HR reference at 1/16 pel (2 s mv for
+// luma, s mv for 4:2:0 chroma), 8 taps at -3..+4, each pass rounded by 7 bits
+// and clipped to a byte, edges replicated -- then the O8 combine with up_s of
+// the residual, exactly as in k_recon_step.
+//
+// A thread owns 4 LR columns (4s HR pixels; half a luma block, a whole chroma
+// block) over 4s HR rows, so its motion vector is uniform.  Its reference
+// window rows (4s + 7 bytes, 4s + 7 rows) stream through a shared-memory ring
+// by cp.async; each row's horizontal pass is kept in registers (8 rows, 16-bit
+// lanes holding two pixels, even/odd interleaved as in k_recon_step) and the
+// vertical pass of output row j runs as soon as window row j + 7 is filtered.
+// 16-bit lanes: a pass sums 8 taps of bytes with a bias of 128 * 128 + 64 per
+// lane, sum + bias in [2678, 62858] for every kernel (the sharpest phase has
+// positive taps 182, negative 54), so the packed multiply-adds never carry
+// across lanes; the clamp to [128 * 128, 384 * 128 - 1] is the byte clip.
+//
+// VP9's kernels (libvpx vp9_filter.c: sub_pel_filters_8, _8lp, _8s), a
+// transcription of its own (the oracle keeps another).
+__constant__ int16_t c_vp9_f8[3][16][8] = {
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {0, 1, -5, 126, 8, -3, 1, 0},
+     {-1, 3, -10, 122, 18, -6, 2, 0},   {-1, 4, -13, 118, 27, -9, 3, -1},
+     {-1, 4, -16, 112, 37, -11, 4, -1}, {-1, 5, -18, 105, 48, -14, 4, -1},
+     {-1, 5, -19, 97, 58, -16, 5, -1},  {-1, 6, -19, 88, 68, -18, 5, -1},
+     {-1, 6, -19, 78, 78, -19, 6, -1},  {-1, 5, -18, 68, 88, -19, 6, -1},
+     {-1, 5, -16, 58, 97, -19, 5, -1},  {-1, 4, -14, 48, 105, -18, 5, -1},
+     {-1, 4, -11, 37, 112, -16, 4, -1}, {-1, 3, -9, 27, 118, -13, 4, -1},
+     {0, 2, -6, 18, 122, -10, 3, -1},   {0, 1, -3, 8, 126, -5, 1, 0}},
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {-3, -1, 32, 64, 38, 1, -3, 0},
+     {-2, -2, 29, 63, 41, 2, -3, 0},    {-2, -2, 26, 63, 43, 4, -4, 0},
+     {-2, -3, 24, 62, 46, 5, -4, 0},    {-2, -3, 21, 60, 49, 7, -4, 0},
+     {-1, -4, 18, 59, 51, 9, -4, 0},    {-1, -4, 16, 57, 53, 12, -4, -1},
+     {-1, -4, 14, 55, 55, 14, -4, -1},  {-1, -4, 12, 53, 57, 16, -4, -1},
+     {0, -4, 9, 51, 59, 18, -4, -1},    {0, -4, 7, 49, 60, 21, -3, -2},
+     {0, -4, 5, 46, 62, 24, -3, -2},    {0, -4, 4, 43, 63, 26, -2, -2},
+     {0, -3, 2, 41, 63, 29, -2, -2},    {0, -3, 1, 38, 64, 32, -1, -3}},
+    {{0, 0, 0, 128, 0, 0, 0, 0},        {-1, 3, -7, 127, 8, -3, 1, 0},
+     {-2, 5, -13, 125, 17, -6, 3, -1},  {-3, 7, -17, 121, 27, -10, 5, -2},
+     {-4, 9, -20, 115, 37, -13, 6, -2}, {-4, 10, -23, 108, 48, -16, 8, -3},
+     {-4, 10, -24, 100, 59, -19, 9, -3}, {-4, 11, -24, 90, 70, -21, 10, -4},
+     {-4, 11, -23, 80, 80, -23, 11, -4}, {-4, 10, -21, 70, 90, -24, 11, -4},
+     {-3, 9, -19, 59, 100, -24, 10, -4}, {-3, 8, -16, 48, 108, -23, 10, -4},
+     {-2, 6, -13, 37, 115, -20, 9, -4}, {-2, 5, -10, 27, 121, -17, 7, -3},
+     {-1, 3, -6, 17, 125, -13, 5, -2},  {0, 1, -3, 8, 127, -7, 3, -1}}};
+
+constexpr int kR8TX = 32, kR8TY = 4, kR8NT = kR8TX * kR8TY;
+template <int S>
+struct R8Cfg {
+    static constexpr int TW = 4 * S;                  // HR pixels per thread row (4 LR columns)
+    static constexpr int NPT = TW / 2;                // 16-bit pairs per row
+    static constexpr int R = 4 * S;                   // HR rows per thread
+    static constexpr int NW = R + 7;                  // window rows
+    static constexpr int NQ = (7 + TW + 7 + 7) / 8;   // aligned 8-B words per window row
+    static constexpr int LA = 6;                      // window rows in flight
+    static constexpr int NR = LA + 1;                 // ring slots (row i + LA lands in row i - 1's)
+    static constexpr int JMAX = pair_px(NPT - 1, 0) + 7;  // last pair source P_j of a row
+    static constexpr int GMAX = JMAX / 4 + 1;         // aligned 4-byte groups a row's pass touches
+    static constexpr size_t SMEM = (size_t)NR * NQ * kR8NT * 8;
+    static_assert(4 * (GMAX + 1) + 7 <= 8 * NQ + 8, "window words cover every pass source");
+};
+constexpr uint32_t kR8Bias = (128u * 128u + 64u) * 0x00010001u;
+constexpr uint32_t kR8Lo = (128u * 128u) * 0x00010001u, kR8Hi = (384u * 128u - 1u) * 0x00010001u;
+
+template <int S, bool CH>
+__global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n, int f, int s0) {
+    using Cfg = R8Cfg<S>;
+    constexpr int TW = Cfg::TW, NPT = Cfg::NPT, R = Cfg::R, NW = Cfg::NW, NQ = Cfg::NQ, LA = Cfg::LA, NR = Cfg::NR;
+    constexpr int GMAX = Cfg::GMAX;
+    const int sid = s0 + blockIdx.z;
+    const FrameDesc fd = fdesc[(size_t)sid * n + f];
+    if (fd.s != S || fd.interp == NS_INTERP_BILINEAR || fd.anchor) return;   // CTA-uniform
+    if (CH && fd.fmt != NS_FMT_I420) return;
+    const int w = fd.w, h = fd.h;
+    const int pw = CH ? w / 2 : w, ph = CH ? h / 2 : h, W = S * pw, H = S * ph;
+    const int gx0 = blockIdx.x * kR8TX;                 // first 4-LR-column group of the CTA
+    const int Y0c = blockIdx.y * kR8TY * R;
+    if (4 * gx0 >= pw || Y0c >= H) return;              // CTA-uniform
+    __shared__ int16_t s_f8[3 * 16 * 8];
+    extern __shared__ __align__(16) uint8_t r8_sm[];
+    const int tid = threadIdx.y * kR8TX + threadIdx.x;
+    for (int i = tid; i < 3 * 16 * 8; i += kR8NT) s_f8[i] = (&c_vp9_f8[0][0][0])[i];
+    __syncthreads();
+    const int gx = gx0 + threadIdx.x;
+    const int Y0 = Y0c + threadIdx.y * R;
+    if (4 * gx >= pw || Y0 >= H) return;                // (no barrier below)
+
+    const size_t lrp = (size_t)h * w, hrp = (size_t)S * h * S * w;
+    const size_t plr = (size_t)ph * pw, phr = (size_t)H * W;
+    const size_t lr0 = CH ? lrp : 0, hr0 = CH ? hrp : 0;
+    const int np_ = CH ? 2 : (fd.fmt == NS_FMT_I420 ? 1 : 3);
+    // the block's vector: luma blocks are 8 LR columns (two threads), chroma blocks 4
+    const int bxm = CH ? gx : gx >> 1, bym = CH ? Y0 / (4 * S) : Y0 / (8 * S);
+    const ns_block_mv mv = fd.mv_f[(size_t)bym * (w / 8) + bxm];
+    const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;   // KEY / INTRA: up_s(LR) (Z17)
+    const int kern = fd.interp == NS_INTERP_SWITCHABLE ? (mv.filter > 2 ? 0 : mv.filter) : fd.interp - 1;
+    const int qx = (CH ? 1 : 2) * S * mv.mvx, qy = (CH ? 1 : 2) * S * mv.mvy;   // 1/16 HR pel
+    const int X0 = gx * TW;
+    const int xs = X0 + (qx >> 4) - 3, ys = Y0 + (qy >> 4) - 3;   // window origin (tap -3)
+    uint32_t fx[8], fy[8];
+#pragma unroll
+    for (int t = 0; t < 8; t++) {
+        fx[t] = (uint32_t)(int)s_f8[(kern * 16 + (qx & 15)) * 8 + t];
+        fy[t] = (uint32_t)(int)s_f8[(kern * 16 + (qy & 15)) * 8 + t];
+    }
+    const int xb = xs & ~7, m = xs & 7;
+    const bool interior = xb >= 0 && xb + 8 * NQ <= W;
+    const uint8_t *ref = (mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last) + hr0;
+    uint2 *ring = reinterpret_cast<uint2 *>(r8_sm) + tid;
+    const int c0 = 4 * gx, cl = max(c0 - 1, 0), cr = min(c0 + 4, pw - 1);
+
+#pragma unroll 1
+    for (int c = 0; c < np_; c++) {
+        const uint8_t *refc = ref + c * phr;
+        auto stage = [&](int i) {
+            if (!use_lr && i < NW) {
+                const uint8_t *row = refc + (size_t)min(max(ys + i, 0), H - 1) * W;
+                uint2 *dst = ring + (i % NR) * NQ * kR8NT;
+#pragma unroll
+                for (int q = 0; q < NQ; q++)
+                    cp_async8(dst + q * kR8NT, row + (interior ? xb + 8 * q : min(max(xb + 8 * q, 0), W - 8)));
+            }
+            asm volatile("cp.async.commit_group;" ::: "memory");
+        };
+#pragma unroll
+        for (int i = 0; i < LA; i++) stage(i);
+        const int16_t *resc = fd.res_f + lr0 + c * plr;
+        const uint8_t *lrc = fd.lr_f + lr0 + c * plr;
+        uint8_t *outc = fd.out + hr0 + c * phr + (size_t)Y0 * W + X0;
+        uint32_t T[8][NPT];
+        int rv[3][6];
+        auto load_lr_rows = [&](int it) {   // LR rows it .. it+2 of this thread (row Y0/S - 1 + it), clamped (Z16)
+#pragma unroll
+            for (int t = 0; t < 3; t++) {
+                const int row = min(max(Y0 / S - 1 + it + t, 0), ph - 1);
+                if (use_lr) {
+                    const uint8_t *p = lrc + (size_t)row * pw;
+                    const uint32_t q4 = *reinterpret_cast<const uint32_t *>(p + c0);
+#pragma unroll
+                    for (int e = 0; e < 4; e++) rv[t][1 + e] = (q4 >> (8 * e)) & 255;
+                    rv[t][0] = p[cl];
+                    rv[t][5] = p[cr];
+                } else {
+                    const int16_t *p = resc + (size_t)row * pw;
+                    const uint2 q4 = *reinterpret_cast<const uint2 *>(p + c0);
+                    rv[t][1] = (int)(int16_t)(q4.x & 0xFFFFu); rv[t][2] = (int)(int16_t)(q4.x >> 16);
+                    rv[t][3] = (int)(int16_t)(q4.y & 0xFFFFu); rv[t][4] = (int)(int16_t)(q4.y >> 16);
+                    rv[t][0] = p[cl];
+                    rv[t][5] = p[cr];
+                }
+            }
+        };
+        auto row_i = [&](auto ic) {
+            constexpr int i = decltype(ic)::value;
+            // window row i: landed when at most LA - 1 newer groups are pending
+            asm volatile("cp.async.wait_group %0;" ::"n"(LA - 1) : "memory");
+            uint2 q[NQ];
+            const uint2 *src = ring + (i % NR) * NQ * kR8NT;
+#pragma unroll
+            for (int k = 0; k < NQ; k++) q[k] = use_lr ? make_uint2(0u, 0u) : src[k * kR8NT];
+            if (!interior) {   // words wholly outside the row replicate its edge pixel (Z16)
+#pragma unroll
+                for (int k = 0; k < NQ; k++) {
+                    const int st = xb + 8 * k;
+                    if (st < 0) { const uint32_t v = prmt(q[k].x, 0u, 0x0000u); q[k] = make_uint2(v, v); }
+                    else if (st >= W) { const uint32_t v = prmt(q[k].y, 0u, 0x3333u); q[k] = make_uint2(v, v); }
+                }
+            }
+            stage(i + LA);
+            // horizontal pass: P_j = [w(j), w(j + 2)] from the aligned 4-byte groups
+            uint32_t wv[2 * NQ + 2];
+#pragma unroll
+            for (int k = 0; k < NQ; k++) { wv[2 * k] = q[k].x; wv[2 * k + 1] = q[k].y; }
+            wv[2 * NQ] = 0;
+            wv[2 * NQ + 1] = 0;
+            if (m >= 4) {
+#pragma unroll
+                for (int k = 0; k < 2 * NQ + 1; k++) wv[k] = wv[k + 1];
+            }
+            const uint32_t sh = 8u * (uint32_t)(m & 3);
+            uint32_t E[GMAX + 1], O[GMAX + 1];
+#pragma unroll
+            for (int g = 0; g <= GMAX; g++) {
+                const uint32_t a = __funnelshift_r(wv[g], wv[g + 1], sh);
+                E[g] = prmt(a, 0u, 0x4240u);
+                O[g] = prmt(a, 0u, 0x4341u);
+            }
+            auto P = [&](int j) -> uint32_t {
+                const int g = j >> 2;
+                switch (j & 3) {
+                    case 0: return E[g];
+                    case 1: return O[g];
+                    case 2: return __funnelshift_r(E[g], E[g + 1], 16);
+                    default: return __funnelshift_r(O[g], O[g + 1], 16);
+                }
+            };
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                const int x0 = pair_px(k, 0);
+                uint32_t acc = kR8Bias;
+#pragma unroll
+                for (int t = 0; t < 8; t++) acc = mad_u32(P(x0 + t), fx[t], acc);
+                acc = vmin_u16x2(vmax_u16x2(acc, kR8Lo), kR8Hi);
+                T[i % 8][k] = ((acc - kR8Lo) >> 7) & 0x00FF00FFu;
+            }
+            if constexpr (i >= 7) {
+                constexpr int j = i - 7, it = j / S, jj = j % S;
+                if constexpr (jj == 0) load_lr_rows(it);
+                constexpr int ta = tap_d<S>(jj) + 1;
+                uint32_t u[NPT], x[NPT], o[TW / 4];
+                recon_up_row<S, true, tap_w1<S>(jj), 384>(rv[ta], rv[ta + 1], u);   // r + 384 per lane
+#pragma unroll
+                for (int k = 0; k < NPT; k++) {
+                    uint32_t acc = kR8Bias;
+#pragma unroll
+                    for (int r = 0; r < 8; r++) acc = mad_u32(T[(j + r) % 8][k], fy[r], acc);
+                    acc = vmin_u16x2(vmax_u16x2(acc, kR8Lo), kR8Hi);
+                    const uint32_t pv = use_lr ? 0x00800080u : (acc >> 7) & 0x01FF01FFu;   // pred + 128
+                    x[k] = vmin_u16x2(vmax_u16x2(pv + u[k], 0x02000200u), 0x02FF02FFu);      // pred + r + 512, clamped
+                }
+#pragma unroll
+                for (int qq = 0; qq < TW / 4; qq++) o[qq] = prmt(x[2 * qq], x[2 * qq + 1], 0x6240u);
+                uint8_t *dst = outc + (size_t)j * W;
+                if constexpr (TW % 16 == 0) {
+#pragma unroll
+                    for (int qq = 0; qq < TW / 16; qq++)
+                        *reinterpret_cast<uint4 *>(dst + 16 * qq) = make_uint4(o[4 * qq], o[4 * qq + 1], o[4 * qq + 2], o[4 * qq + 3]);
+                } else if constexpr (TW % 8 == 0) {
+#pragma unroll
+                    for (int qq = 0; qq < TW / 8; qq++) *reinterpret_cast<uint2 *>(dst + 8 * qq) = make_uint2(o[2 * qq], o[2 * qq + 1]);
+                } else {
+#pragma unroll
+                    for (int qq = 0; qq < TW / 4; qq++) *reinterpret_cast<uint32_t *>(dst + 4 * qq) = o[qq];
+                }
+            }
+        };
+        static_for<NW>(row_i);
+    }
+}
+
 // Carveout: just enough shared memory for MINB resident CTAs, the rest of the
 // 256-KB array stays L1 (the window words of neighbouring threads overlap and
 // hit there): the maximum-shared carveout (28 KB of L1) vs this (60 KB) measured
@@ -633,10 +877,18 @@ static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, in
     return cudaGetLastError();
 }
 
+template <int S, bool CH>
+static cudaError_t recon8_launch(int max_pw, int max_ph, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0,
+                                 int nstreams) {
+    dim3 g((max_pw / 4 + kR8TX - 1) / kR8TX, (max_ph * S / R8Cfg<S>::R + kR8TY - 1) / kR8TY, nstreams);
+    k_recon8<S, CH><<<g, dim3(kR8TX, kR8TY), R8Cfg<S>::SMEM, st>>>(fd, n, f, s0);
+    return cudaGetLastError();
+}
+
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              const int *has_i420, cudaStream_t st, int s0) {
+                              const int *has_i420, const int *e8, cudaStream_t st, int s0) {
     int nl = 0;
-    for (int s = 2; s <= 4; s++) nl += (max_lr_w[s] > 0) + (has_i420[s] != 0);
+    for (int s = 2; s <= 4; s++) nl += (max_lr_w[s] > 0) + (has_i420[s] != 0) + (e8[s] & 1) + ((e8[s] >> 1) & 1);
     KScope ks(F_RECON, st, nl);
     for (int s = 2; s <= 4; s++) {
         if (max_lr_w[s] <= 0) continue;
@@ -652,6 +904,19 @@ cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const in
             dim3 gc(g.x, (nrc + kReconTY - 1) / kReconTY, S);
             e = s == 2 ? recon_launch<2, true>(gc, st, fd, n, f, s0)
                 : s == 3 ? recon_launch<3, true>(gc, st, fd, n, f, s0) : recon_launch<4, true>(gc, st, fd, n, f, s0);
+            if (e != cudaSuccess) return e;
+        }
+        // 8-tap streams (after k_recon_step, which did their HR-ring copies)
+        const int W8 = max_lr_w[s], H8 = max_lr_h[s];
+        if (e8[s] & 1) {
+            e = s == 2 ? recon8_launch<2, false>(W8, H8, st, fd, n, f, s0, S)
+                : s == 3 ? recon8_launch<3, false>(W8, H8, st, fd, n, f, s0, S) : recon8_launch<4, false>(W8, H8, st, fd, n, f, s0, S);
+            if (e != cudaSuccess) return e;
+        }
+        if (e8[s] & 2) {
+            e = s == 2 ? recon8_launch<2, true>(W8 / 2, H8 / 2, st, fd, n, f, s0, S)
+                : s == 3 ? recon8_launch<3, true>(W8 / 2, H8 / 2, st, fd, n, f, s0, S)
+                         : recon8_launch<4, true>(W8 / 2, H8 / 2, st, fd, n, f, s0, S);
             if (e != cudaSuccess) return e;
         }
     }

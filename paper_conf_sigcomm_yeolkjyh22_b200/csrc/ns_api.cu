@@ -506,6 +506,8 @@ static ns_status check_chunks(const ns_chunk *ch, int S, bool need_model, int *n
         if (c.format == NS_FMT_I420 && (c.w % 16 || c.h % 16))
             return fail(NS_EINVAL, "chunk %d: 4:2:0 needs w, h multiples of 16 (8 x 8 chroma blocks), got %dx%d", s,
                         c.w, c.h);
+        if (c.interp < NS_INTERP_BILINEAR || c.interp > NS_INTERP_SWITCHABLE)
+            return fail(NS_EINVAL, "chunk %d: interp %d not an NS_INTERP_* value", s, c.interp);
         if (!c.lr || !c.res || !c.mv || !c.type) return fail(NS_EINVAL, "chunk %d: lr/res/mv/type must be non-NULL", s);
         if (!al16(c.res) || !al16(c.lr) || !al16(c.mv)) return fail(NS_EINVAL, "chunk %d: lr/res/mv must be 16-B aligned", s);
         if (c.gt && !al16(c.gt)) return fail(NS_EINVAL, "chunk %d: gt must be 16-B aligned", s);
@@ -614,6 +616,7 @@ static ns_status stage_streams(ns_ctx *c, const ns_chunk *ch, int S, int n, uint
         d.job_goff = pl.job_goff ? pl.job_goff[s] : 0;
         d.use_res_size = use_res_size ? 1 : 0;
         d.fmt = k.format;
+        d.interp = k.interp;
         d.lr_frame = (int64_t)lr_frame_elems(k);
         d.hr_frame = (int64_t)hr_frame_bytes(k);
         d.acache = pl.acache ? pl.acache[s] : nullptr;
@@ -843,6 +846,7 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
 // [s0, s0 + cnt), and the chunk-end state (all streams).
 struct ReconGeom {
     int mw[5] = {0, 0, 0, 0, 0}, mh[5] = {0, 0, 0, 0, 0}, i420[5] = {0, 0, 0, 0, 0};
+    int e8[5] = {0, 0, 0, 0, 0};   // bit 0: an 8-tap stream of that scale, bit 1: an 8-tap 4:2:0 one
     size_t maxhr = 0;
 };
 static ReconGeom recon_geom(const ns_chunk *ch, int s0, int cnt) {
@@ -851,6 +855,7 @@ static ReconGeom recon_geom(const ns_chunk *ch, int s0, int cnt) {
         gm.mw[ch[s].scale] = std::max(gm.mw[ch[s].scale], ch[s].w);
         gm.mh[ch[s].scale] = std::max(gm.mh[ch[s].scale], ch[s].h);
         gm.i420[ch[s].scale] |= ch[s].format == NS_FMT_I420;
+        if (ch[s].interp != NS_INTERP_BILINEAR) gm.e8[ch[s].scale] |= ch[s].format == NS_FMT_I420 ? 3 : 1;
         gm.maxhr = std::max(gm.maxhr, hr_frame_bytes(ch[s]));
     }
     return gm;
@@ -864,7 +869,7 @@ static ns_status recon_prepare(ns_ctx *c, const Staged &g, int S, int n, const u
 }
 static ns_status recon_steps(ns_ctx *c, const ns_chunk *ch, int s0, int cnt, int n, cudaStream_t st) {
     const ReconGeom gm = recon_geom(ch, s0, cnt);
-    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, cnt, n, f, gm.mw, gm.mh, gm.i420, st, s0));
+    for (int f = 0; f < n; f++) NS_CUDA(launch_recon_step(c->fdesc, cnt, n, f, gm.mw, gm.mh, gm.i420, gm.e8, st, s0));
     return NS_OK;
 }
 static ns_status recon_finish(ns_ctx *c, const Staged &g, const ns_chunk *ch, int S, int n, cudaStream_t st) {

@@ -33,6 +33,7 @@ struct StreamDesc {
     int32_t use_res_size;
     int32_t job_goff;      // first job slot of the stream's SR shape group
     int32_t fmt;           // NS_FMT_444 | NS_FMT_I420
+    int32_t interp;        // NS_INTERP_* (k_recon_step: bilinear streams; k_recon8: the 8-tap ones)
     int64_t lr_frame;      // elements per LR / residual frame: 3 h w, or h w 3/2 (I420)
     int64_t hr_frame;      // bytes per HR frame: 3 H W, or H W 3/2 (I420)
     uint8_t *acache;       // HR rings: the group's anchor cache (job slot j at acache + (j - job_goff) * stride)
@@ -57,8 +58,9 @@ struct __align__(16) FrameDesc {
     int32_t w, h;              // LR size
     int16_t s;                 // scale
     uint8_t anchor, key;       // is_anchor[f], type[f] == KEY
-    int32_t fmt;               // NS_FMT_444 | NS_FMT_I420 (k_recon_step: luma only; k_recon_c420: chroma)
-    int32_t pad1, pad2;
+    int32_t fmt;               // NS_FMT_444 | NS_FMT_I420
+    int32_t interp;            // NS_INTERP_*: 0 -> k_recon_step, else k_recon8
+    int32_t pad2;
 };
 static_assert(sizeof(FrameDesc) == 96, "FrameDesc is one 96-B record");
 
@@ -149,10 +151,12 @@ cudaError_t launch_frame_desc(const StreamDesc *d_sd, int S, int n, const uint8_
                               uint8_t *const *d_hr_table, const int16_t *gold_idx, const uint8_t *gsv,
                               const uint8_t *const *asrc, FrameDesc *fd, cudaStream_t st);
 // max_lr_w / max_lr_h: [5] per scale; has_i420[5]: a 4:2:0 stream of that scale
-// (its chroma planes then step in k_recon_c420 in the same frame step)
-// streams [s0, s0 + S) of the frame-descriptor table
+// (its chroma planes then step in k_recon_step<s, true> in the same frame
+// step); e8[5]: bit 0 an 8-tap stream of that scale (k_recon8), bit 1 an
+// 8-tap 4:2:0 one (k_recon8<s, true> for its chroma).  Streams [s0, s0 + S)
+// of the frame-descriptor table.
 cudaError_t launch_recon_step(const FrameDesc *fd, int S, int n, int f, const int *max_lr_w, const int *max_lr_h,
-                              const int *has_i420, cudaStream_t st, int s0 = 0);
+                              const int *has_i420, const int *e8, cudaStream_t st, int s0 = 0);
 cudaError_t launch_state_copy(const StreamDesc *d_sd, int S, int n, uint8_t *const *d_hr_table,
                               const int16_t *gold_idx, const uint8_t *gsv, size_t max_hr_bytes, cudaStream_t st);
 cudaError_t launch_stats(const StreamDesc *d_sd, int S, int n, const uint8_t *is_anchor, const int64_t *score,

@@ -17,7 +17,7 @@ def dev_chunk(ns, c: "synth.Chunk", device, model=None, with_gt=False, res_size=
     return ns.DeviceChunk.from_numpy(c.lr, c.res, c.mv, c.type, c.w, c.h, c.scale, device,
                                      res_size=c.res_size if res_size else None,
                                      gt=c.gt if with_gt else None, model=model,
-                                     hr_last=hr_last, hr_golden=hr_golden)
+                                     hr_last=hr_last, hr_golden=hr_golden, interp=getattr(c, "interp", 0))
 
 
 def alloc_hr(n, c, device, fill=0):

@@ -145,11 +145,16 @@ def test_switchable_is_per_block_kernel():
             assert np.array_equal(got[sl], per[kb[by, bx]][sl])
 
 
-def test_invalid_interp_rejected():
+def test_invalid_interp_rejected_and_filter_byte_range():
     c = _two_frame(16, 16, 2, 0, 0, 5)
     with pytest.raises(RuntimeError):
         oracle.reconstruct(c, [0, 0], np.zeros((2, 3, 32, 32), np.uint8), np.zeros((3, 32, 32), np.uint8))
+    # a switchable block's filter byte above 2 reads as EIGHTTAP (include/ns.h)
+    rng = np.random.default_rng(2)
+    last = rng.integers(0, 256, (3, 32, 32)).astype(np.uint8)
     c = _two_frame(16, 16, 2, 3, 1, 4)
-    c.mv["filter"] = 3
-    with pytest.raises(RuntimeError):
-        oracle.reconstruct(c, [0, 0], np.zeros((2, 3, 32, 32), np.uint8), np.zeros((3, 32, 32), np.uint8))
+    c.mv["filter"] = 7
+    a = oracle.reconstruct(c, [0, 0], np.zeros((2, 3, 32, 32), np.uint8), last, last.copy())[0]
+    b = oracle.reconstruct(_two_frame(16, 16, 2, 3, 1, 1), [0, 0], np.zeros((2, 3, 32, 32), np.uint8), last,
+                           last.copy())[0]
+    assert np.array_equal(a, b)
