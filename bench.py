@@ -50,27 +50,32 @@ def cfg_of(args):
     return c
 
 
-def workload_config(cfg, world, select="topk", fmt="444"):
+INTERPS = {"bilinear": 0, "regular": 1, "smooth": 2, "sharp": 3, "switchable": 4}
+
+
+def workload_config(cfg, world, select="topk", fmt="444", interp="bilinear"):
     """The `config` object both arms print (same workload, same keys)."""
     S, s, w, h = cfg["streams"], cfg["scale"], cfg["w"], cfg["h"]
     sel = ("top-k per stream" if select == "topk" else
            f"global budget k*S*N = {cfg['k'] * S * world} anchors over all GPUs' streams (§5.2, NEXT-1)")
     fm = "" if fmt == "444" else ", YUV 4:2:0 (NEXT-2)"
+    if interp != "bilinear":
+        fm += f", VP9 8-tap MC ({interp}, NEXT-2)"
     return {"workload": f"{cfg['name']}: {S} concurrent {w}x{h}->{s * w}x{s * h} x{s} streams per GPU, "
                         f"B{cfg['n_blocks']}/C{cfg['n_ch']}, n={cfg['n']}, k={cfg['k']} ({sel}){fm}",
             "streams_per_gpu": S, "frames_per_step_per_gpu": S * cfg["n"], "parallelism": f"streams x{world}",
-            "select": select, "format": fmt}
+            "select": select, "format": fmt, "interp": interp}
 
 
 def _gen(a):
     seed, w, h, s, n, alt = a[:6]
     mk = synth.make_chunk_i420 if len(a) > 6 and a[6] == "i420" else synth.make_chunk
-    return mk(seed, w, h, s, n, types=synth.default_types(n, alt))
+    return mk(seed, w, h, s, n, types=synth.default_types(n, alt), interp=a[7] if len(a) > 7 else 0)
 
 
-def gen_pool(cfg, n_distinct, rank, fmt="444"):
+def gen_pool(cfg, n_distinct, rank, fmt="444", interp=0):
     seeds = [1000 * 4 + rank * 100000 + i for i in range(n_distinct)]
-    args = [(sd, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"], fmt) for sd in seeds]
+    args = [(sd, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"], fmt, interp) for sd in seeds]
     procs = min(len(args), max(1, (os.cpu_count() or 1)))
     if procs > 1:
         import multiprocessing as mp
@@ -142,7 +147,7 @@ def cpu_sample(cfg, chunk, blob):
     oracle.sr_forward(np.ascontiguousarray(chunk.lr[0][:, :rows]), blob, B, C, s)
     t_sr = (time.perf_counter() - t0) * h / rows
     sub = synth.Chunk(w=w, h=h, scale=s, lr=chunk.lr[:3], res=chunk.res[:3], mv=chunk.mv[:3],
-                      type=chunk.type[:3].copy(), res_size=chunk.res_size[:3])
+                      type=chunk.type[:3].copy(), res_size=chunk.res_size[:3], interp=getattr(chunk, "interp", 0))
     hr = np.zeros((3, 3, s * h, s * w), np.uint8)
     t0 = time.perf_counter()
     oracle.reconstruct(sub, [1, 0, 0], hr)
@@ -167,7 +172,8 @@ def run_reference(args):
     cfg = cfg_of(args)
     if cfg["w"] is None:  # c5: the sample is one 720p->4K stream-chunk of the mixed fleet
         cfg.update(w=1280, h=720)
-    chunk = _gen((4000, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"]))
+    chunk = _gen((4000, cfg["w"], cfg["h"], cfg["scale"], cfg["n"], cfg["altref_every"], "444",
+                  INTERPS[args.interp]))
     blob = synth.make_weights(4000, cfg["n_blocks"], cfg["n_ch"], cfg["scale"])
     vals = []
     for i in range(args.warmup + args.steps):
@@ -179,7 +185,7 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": dict(workload_config(cfg, args.gpus), sample="one stream-chunk of the workload per step "
+            "config": dict(workload_config(cfg, args.gpus, interp=args.interp), sample="one stream-chunk of the workload per step "
                                                                     "(see cpu_baseline.sample), scaled to frames/s"),
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["cores"], "kind": "oracle", "sample": r["sample"]},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -238,6 +244,8 @@ def main():
     ap.add_argument("--ring", type=int, default=3, help="config 5: HR frames per stream (ring)")
     ap.add_argument("--format", default="444", choices=["444", "i420"],
                     help="frame format of the streams (i420: YUV 4:2:0, NEXT-2)")
+    ap.add_argument("--interp", default="bilinear", choices=list(INTERPS),
+                    help="the streams' sub-pel MC: bilinear (Z14) or VP9 8-tap (NEXT-2, R13)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N > 1 (gloo + NS_BENCH_SHARE_GPU=1: N ranks on one GPU)")
     ap.add_argument("--encode", action="store_true",
@@ -270,7 +278,8 @@ def main():
 
     t_gen = time.time()
     i420 = args.format == "i420"
-    pool = gen_pool(cfg, P, rank, args.format)
+    interp_c = INTERPS[args.interp]
+    pool = gen_pool(cfg, P, rank, args.format, interp_c)
     t_gen = time.time() - t_gen
 
     host_pool = ns.Context.host_pool_bytes(w, h, n, k, S) if args.e2e_steps > 0 else 0
@@ -303,7 +312,8 @@ def main():
     state = torch.zeros((S, 2) + HRF, dtype=torch.uint8, device=dev)
     fmt_c = ns.NS_FMT_I420 if i420 else ns.NS_FMT_444
     chunks = [ns.DeviceChunk(w=w, h=h, scale=s, lr=lr_d[si], res=res_d[si], mv=mv_d[si], type=ty_d[si],
-                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1], format=fmt_c)
+                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1], format=fmt_c,
+                             interp=interp_c)
               for si in range(S)]
     hr_out = [[hr[si, f] for f in range(n)] for si in range(S)]
     ia = torch.zeros((S, n), dtype=torch.uint8, device=dev)
@@ -399,12 +409,17 @@ def main():
     dom = max((f for f in rl if "bound" in rl[f]), key=lambda f: rl[f]["ms_per_step"])
     d = rl[dom]
     traffic = None
+    tkey = dom
+    per_launch = (fl.get(dom) or by.get(dom)) / max(1, d["launches_per_step"])
+    if dom == "recon" and args.interp != "bilinear":
+        # 8-tap streams step in k_recon8, one working launch per frame step (the
+        # bilinear kernel's launches of the same family return at once)
+        tkey, per_launch = "recon8", by[dom] / n
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(dom)
-    per_launch = (fl.get(dom) or by.get(dom)) / max(1, d["launches_per_step"])
+        traffic = json.load(open(tp)).get(tkey)
     roofline = {"bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
-                "frac": d["frac"], "traffic": traffic, "kernel": dom,
+                "frac": d["frac"], "traffic": traffic, "kernel": "k_recon8" if tkey == "recon8" else dom,
                 "per_launch_algorithmic": per_launch,
                 "peak_source": f"{pk['src']} ({'bf16 sustained' if d['bound'] == 'tensor' else 'HBM copy'})"}
 
@@ -414,7 +429,8 @@ def main():
     # anchors' LR frames; then the step's result (stats, anchor map) is read back.
     e2e = None
     if args.e2e_steps > 0:
-        hpool = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, w, h, s, format=fmt_c) for c in pool]
+        hpool = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, w, h, s, format=fmt_c, interp=interp_c)
+                 for c in pool]
         hchunks = []
         for si in range(S):
             hc = dataclasses.replace(hpool[si % P], model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1])
@@ -473,7 +489,8 @@ def main():
                 "vs_baseline": None, "dtype": "bf16",
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
-                "config": dict(workload_config(cfg, world, args.select, args.format), balance=bool(args.balance),
+                "config": dict(workload_config(cfg, world, args.select, args.format, args.interp),
+                               balance=bool(args.balance),
                                l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,

@@ -8,7 +8,7 @@ for L in ${LIBS:-default}; do
     env:*) unset NS_LIB; export ${L#env:} ;;
     *) export NS_LIB=$PWD/$L ;;
   esac
-  python bench.py --steps ${STEPS:-5} --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/ab.json 2>gpurun_out/ab.err
+  python bench.py --steps ${STEPS:-5} --warmup 3 --no-cpu-baseline --e2e-steps 0 $BENCH_ARGS > gpurun_out/ab.json 2>gpurun_out/ab.err
   python - "$L" <<'PY'
 import json, sys
 l = [x for x in open("gpurun_out/ab.json") if x.startswith("{")]
