@@ -365,8 +365,10 @@ def main():
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize(dev)
     e0.record(stream)
+    th0 = time.perf_counter()
     for _ in range(args.steps):
         step()
+    host_ms = (time.perf_counter() - th0) * 1000.0 / args.steps   # host time to enqueue a step (no sync inside)
     e1.record(stream)
     torch.cuda.synchronize(dev)
     ns.profile_enable(False)
@@ -497,6 +499,7 @@ def main():
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
                              "anchors_per_step": int(ia_np.sum())},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+                "host_enqueue_ms_per_step": host_ms,
                 "hybrid_encode": hybrid,
                 # real-time check: one n-frame chunk of every stream (n/60 s of
                 # 60 fps video) must finish within its own duration
