@@ -244,6 +244,9 @@ def main():
     ap.add_argument("--ring", type=int, default=3, help="config 5: HR frames per stream (ring)")
     ap.add_argument("--format", default="444", choices=["444", "i420"],
                     help="frame format of the streams (i420: YUV 4:2:0, NEXT-2)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "peer"],
+                    help="--balance: moved anchors by NCCL point-to-point copies, or read/written in place by the "
+                         "importing GPU's SR kernels through CUDA IPC peer mappings")
     ap.add_argument("--interp", default="bilinear", choices=list(INTERPS),
                     help="the streams' sub-pel MC: bilinear (Z14) or VP9 8-tap (NEXT-2, R13)")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
@@ -343,7 +346,7 @@ def main():
             anchors_all = [[int(f) for f in np.nonzero(anc_h[i])[0]] for i in range(len(sid_h))]
             shard.balanced_sr_and_reconstruct(ctx, chunks, models_all, sids, anc, hr_out, anchors_all,
                                               [x // S for x in sid_h], sid_h, allr["cost"].cpu().tolist(),
-                                              shape_all=allr["shape"].cpu().tolist())
+                                              shape_all=allr["shape"].cpu().tolist(), transport=args.transport)
             ia.copy_(anc)
         elif args.select == "global":
             anc, _ = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream)
@@ -496,7 +499,7 @@ def main():
                 "data": f"synthetic ({P} generated streams replicated to {S} distinct device buffers per GPU; "
                         f"random-init per-stream weights of the NAS 'high' architecture)",
                 "config": dict(workload_config(cfg, world, args.select, args.format, args.interp),
-                               balance=bool(args.balance),
+                               balance=bool(args.balance), transport=args.transport if args.balance else None,
                                l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,

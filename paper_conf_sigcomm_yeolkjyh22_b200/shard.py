@@ -178,8 +178,23 @@ def plan_anchor_moves(anchors, owner, cost, world):
     return moves
 
 
+def _ipc_share(t):
+    """Picklable description of tensor t's memory for another process on this
+    host: CUDA IPC for device memory (the peer maps it: NVLink peer memory on a
+    multi-GPU node, the same GPU when ranks share one), shared memory for host
+    tensors (the gloo tests)."""
+    import torch.multiprocessing  # noqa: F401  (registers the tensor reductions)
+    from multiprocessing.reduction import ForkingPickler
+    return bytes(ForkingPickler.dumps(t))
+
+
+def _ipc_open(desc):
+    import pickle
+    return pickle.loads(desc)
+
+
 def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anchors_all, owner_all, sid_all, cost_all,
-                                group=None, stream=None, shape_all=None, device=None):
+                                group=None, stream=None, shape_all=None, device=None, transport="nccl"):
     """SR on this GPU's share of the balanced anchor set, then reconstruction of
     this GPU's streams (ns_sr_anchors + ns_reconstruct_chunk).  anchors_all /
     owner_all / sid_all / cost_all describe every gathered stream row (host
@@ -207,6 +222,41 @@ def balanced_sr_and_reconstruct(ctx, chunks, models, sid, is_anchor, hr_out, anc
         for f in anchors_all[row]:
             if (s, f) not in exported:
                 jobs.append((models[s], chunks[li].lr[f], hr_out[li][f]))
+    if transport == "peer" and dist_on:
+        # Peer memory (§5.2 (2) without staging copies): every exporter publishes
+        # its moved anchors' LR frame and HR slot; the importer maps them and runs
+        # SR straight from the exporter's LR into the exporter's HR slot -- the SR
+        # kernels read and write the peer's memory (k_prep_lr loads the LR frame,
+        # the upsampler epilogue and border fix-up store the HR frame), so the
+        # transfer rides inside the kernels instead of separate NCCL copies.
+        if chunks and chunks[0].lr.is_cuda:
+            torch.cuda.current_stream().synchronize()   # this rank's inputs and HR slots are settled
+        offer = {}
+        for i, f, src, dst in moves:
+            if src == me:
+                s = sid_all[i]
+                offer[(i, f)] = (_ipc_share(chunks[local[s]].lr[f]), _ipc_share(hr_out[local[s]][f]))
+        offers = [None] * world
+        dist.all_gather_object(offers, offer, group=group)
+        mapped = []
+        for i, f, src, dst in moves:
+            if dst == me:
+                lr, hr = (_ipc_open(d) for d in offers[src][(i, f)])
+                mapped.append((lr, hr))
+                jobs.append((models[sid_all[i]], lr, hr))
+        if jobs:
+            ctx.sr_anchors(jobs, stream=stream)
+            if mapped and mapped[0][0].is_cuda:
+                (stream if stream is not None else torch.cuda.current_stream()).synchronize()
+        dist.barrier(group=group)             # every moved anchor's HR is in its owner's slot
+        del mapped
+        if chunks:
+            ctx.reconstruct_chunk(chunks, is_anchor, hr_out, stream=stream)
+        return moves
+    if dist_on and moves and dist.get_backend(group) == "gloo" and (
+            (chunks and chunks[0].lr.is_cuda) or (device is not None and torch.device(device).type == "cuda")):
+        raise ValueError("point-to-point copies of device tensors need the nccl backend; "
+                         "with gloo use transport='peer'")
     imports = []
     ops = []
     for i, f, src, dst in moves:          # LR out / in, in the global move order on every rank

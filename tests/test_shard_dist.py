@@ -172,8 +172,10 @@ class _FakeCtx:
         self.recon_calls += 1
 
 
-def _lb_worker(rank, world, port, q):
+def _lb_worker(rank, world, port, q, transport="nccl"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if transport == "peer":   # host tensors shared by file name (the CUDA analogue is CUDA IPC)
+        mp.set_sharing_strategy("file_system")
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from types import SimpleNamespace
@@ -192,7 +194,7 @@ def _lb_worker(rank, world, port, q):
         ia = torch.zeros((len(mine), n), dtype=torch.uint8)
         ctx = _FakeCtx()
         moves = shard.balanced_sr_and_reconstruct(ctx, chunks, models, mine, ia, hr_out, anchors_all, owner_all,
-                                                  sid_all, cost_all)
+                                                  sid_all, cost_all, transport=transport)
         ok = True
         for li, s in enumerate(mine):
             for f in anchors_all[s]:
@@ -203,11 +205,14 @@ def _lb_worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-def test_gloo_world2_balanced_sr_exchange():
+@pytest.mark.parametrize("transport", ["nccl", "peer"])
+def test_gloo_world2_balanced_sr_exchange(transport):
+    """transport nccl: point-to-point copies; peer: the importer writes the
+    exporter's HR slots through a mapping of its memory (no copies)."""
     world, port = 2, _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_lb_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_lb_worker, args=(r, world, port, q, transport)) for r in range(world)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=120) for _ in range(world))
@@ -221,10 +226,12 @@ def test_gloo_world2_balanced_sr_exchange():
     assert rc0 == rc1 == 1
 
 
-def _lb_worker_mixed(rank, world, port, q):
+def _lb_worker_mixed(rank, world, port, q, transport="nccl"):
     """Mixed resolutions (c5-like fleets) and a rank that owns no stream: the
     imported anchors' buffers take their source stream's shape (shape_all)."""
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if transport == "peer":
+        mp.set_sharing_strategy("file_system")
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from types import SimpleNamespace
@@ -246,7 +253,7 @@ def _lb_worker_mixed(rank, world, port, q):
         ia = torch.zeros((len(mine), n), dtype=torch.uint8)
         ctx = _FakeCtx()
         moves = shard.balanced_sr_and_reconstruct(ctx, chunks, models, mine, ia, hr_out, anchors_all, owner_all,
-                                                  sid_all, cost_all, shape_all=shapes, device="cpu")
+                                                  sid_all, cost_all, shape_all=shapes, device="cpu", transport=transport)
         ok = True
         for li, s in enumerate(mine):
             for f in anchors_all[s]:
@@ -257,11 +264,12 @@ def _lb_worker_mixed(rank, world, port, q):
         dist.destroy_process_group()
 
 
-def test_gloo_world2_balanced_mixed_shapes_empty_rank():
+@pytest.mark.parametrize("transport", ["nccl", "peer"])
+def test_gloo_world2_balanced_mixed_shapes_empty_rank(transport):
     world, port = 2, _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_lb_worker_mixed, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_lb_worker_mixed, args=(r, world, port, q, transport)) for r in range(world)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=120) for _ in range(world))
