@@ -86,33 +86,66 @@ def gen_pool(cfg, n_distinct, rank, fmt="444", interp=0):
 
 # ---------------------------------------------------------------- clocks
 class Clocks:
+    """nvidia-smi sampling of the SM clock and throttle reasons.  The sampler is
+    started before the warm-up (its start-up -- process launch and NVML init --
+    stalls the driver for milliseconds and must not land in a short timed
+    region); every line is stamped on arrival and only the samples taken
+    during [begin(), end()] (plus the first one after, which covers the region's
+    last 200 ms) are kept."""
     FIELDS = "clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown," \
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap"
 
     def __init__(self, gpu_index):
         self.idx = gpu_index
         self.p = None
+        self.lines = []
+        self.t0 = self.t1 = None
 
     def start(self):
+        import threading
         try:
             self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
                                        "-i", str(self.idx), "-lms", "200"], stdout=subprocess.PIPE,
                                       stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.p = None
+            return
+
+        def reader():
+            for line in self.p.stdout:
+                self.lines.append((time.time(), line))
+        self.th = threading.Thread(target=reader, daemon=True)
+        self.th.start()
+        deadline = time.time() + 5.0        # settled once the first sample is out
+        while time.time() < deadline and not self.lines:
+            time.sleep(0.02)
+
+    def begin(self):
+        self.t0 = time.time()
+
+    def end(self):
+        self.t1 = time.time()
+        if self.p:   # wait for one sample after the region
+            deadline = self.t1 + 1.0
+            while time.time() < deadline and not any(t > self.t1 for t, _ in self.lines):
+                time.sleep(0.02)
 
     def stop(self):
         if not self.p:
             return None
         self.p.terminate()
         try:
-            out, _ = self.p.communicate(timeout=5)
+            self.p.wait(timeout=5)
         except Exception:
             self.p.kill()
-            out, _ = self.p.communicate()
+        self.th.join(timeout=5)
+        t0 = self.t0 if self.t0 is not None else 0.0
+        t1 = self.t1 if self.t1 is not None else float("inf")
+        inside = [ln for t, ln in self.lines if t0 <= t <= t1]
+        after = [ln for t, ln in self.lines if t > t1][:1]
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in out.strip().splitlines():
+        for line in inside + after:
             parts = [x.strip() for x in line.split(",")]
             if len(parts) < 6:
                 continue
@@ -355,32 +388,38 @@ def main():
         else:
             ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, k=k, stream=stream)
 
+    clocks = Clocks(int(os.environ.get("CUDA_VISIBLE_DEVICES", str(local)).split(",")[local])
+                    if os.environ.get("CUDA_VISIBLE_DEVICES") else local)
+    clocks.start()
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
-    clocks = Clocks(int(os.environ.get("CUDA_VISIBLE_DEVICES", str(local)).split(",")[local])
-                    if os.environ.get("CUDA_VISIBLE_DEVICES") else local)
-    clocks.start()
     ns.launch_count(reset=True)
-    ns.profile_enable(True)
+    prof_on = os.environ.get("NS_BENCH_NOPROF") != "1"
+    ns.profile_enable(prof_on)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev_steps = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     torch.cuda.synchronize(dev)
+    clocks.begin()
     e0.record(stream)
     host_t = []
-    for _ in range(args.steps):
+    for i in range(args.steps):
         th0 = time.perf_counter()
         step()
+        ev_steps[i].record(stream)
         host_t.append((time.perf_counter() - th0) * 1000.0)
+    e1.record(stream)      # before any host work: a short step list may already be done on the GPU
     # host time to enqueue one step: the first call after the synchronize is pure
     # enqueue work (later ones may wait for a staging slot the GPU still reads)
     host_ms = {"first": host_t[0], "median": float(np.median(host_t))}
-    e1.record(stream)
     torch.cuda.synchronize(dev)
+    clocks.end()
     ns.profile_enable(False)
     launches = ns.launch_count()
     ms = e0.elapsed_time(e1)
+    step_ms = [e0.elapsed_time(ev_steps[0])] + [ev_steps[i - 1].elapsed_time(ev_steps[i]) for i in range(1, args.steps)]
     clk = clocks.stop()
     prof = ns.profile_read()
     ms = shard.max_over_ranks(ms)      # job time = the slowest rank (device-timed)
@@ -415,22 +454,24 @@ def main():
     sr_fams = [f for f in ("sr_prep", "sr_head", "sr_body", "sr_end", "sr_up", "sr_tail") if f in rl]
     sr_ms = sum(rl[f]["ms_per_step"] for f in sr_fams)
     sr_tf = sum(fl.values()) / (sr_ms / 1000.0) / 1e12 if sr_ms else 0.0
-    dom = max((f for f in rl if "bound" in rl[f]), key=lambda f: rl[f]["ms_per_step"])
-    d = rl[dom]
-    traffic = None
-    tkey = dom
-    per_launch = (fl.get(dom) or by.get(dom)) / max(1, d["launches_per_step"])
-    if dom == "recon" and args.interp != "bilinear":
-        # 8-tap streams step in k_recon8, one working launch per frame step (the
-        # bilinear kernel's launches of the same family return at once)
-        tkey, per_launch = "recon8", by[dom] / n
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        traffic = json.load(open(tp)).get(tkey)
-    roofline = {"bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
-                "frac": d["frac"], "traffic": traffic, "kernel": "k_recon8" if tkey == "recon8" else dom,
-                "per_launch_algorithmic": per_launch,
-                "peak_source": f"{pk['src']} ({'bf16 sustained' if d['bound'] == 'tensor' else 'HBM copy'})"}
+    dom = max((f for f in rl if "bound" in rl[f]), key=lambda f: rl[f]["ms_per_step"], default=None)
+    roofline = None   # (NS_BENCH_NOPROF=1, a diagnostic run: no per-family timing)
+    if dom is not None:
+        d = rl[dom]
+        traffic = None
+        tkey = dom
+        per_launch = (fl.get(dom) or by.get(dom)) / max(1, d["launches_per_step"])
+        if dom == "recon" and args.interp != "bilinear":
+            # 8-tap streams step in k_recon8, one working launch per frame step (the
+            # bilinear kernel's launches of the same family return at once)
+            tkey, per_launch = "recon8", by[dom] / n
+        tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+        if os.path.exists(tp):
+            traffic = json.load(open(tp)).get(tkey)
+        roofline = {"bound": d["bound"], "achieved": d["achieved"], "peak": d["peak"], "unit": d["unit"],
+                    "frac": d["frac"], "traffic": traffic, "kernel": "k_recon8" if tkey == "recon8" else dom,
+                    "per_launch_algorithmic": per_launch,
+                    "peak_source": f"{pk['src']} ({'bf16 sustained' if d['bound'] == 'tensor' else 'HBM copy'})"}
 
     # e2e: the public host-input call (ns_enhance_streams_host): every step the
     # library uploads each stream's res/mv/type from pinned host memory (stream
@@ -506,7 +547,7 @@ def main():
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
                              "anchors_per_step": int(ia_np.sum())},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
-                "host_enqueue_ms_per_step": host_ms,
+                "host_enqueue_ms_per_step": host_ms, "step_ms": [round(x, 3) for x in step_ms],
                 "hybrid_encode": hybrid,
                 # real-time check: one n-frame chunk of every stream (n/60 s of
                 # 60 fps video) must finish within its own duration
@@ -625,22 +666,24 @@ def run_c5(args):
     def step():
         ctx.enhance_streams(chunks, rows, is_anchor_out=ia, stats=stats, k=k, stream=stream)
 
+    clocks = Clocks(local)
+    clocks.start()
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
-    clocks = Clocks(local)
-    clocks.start()
     ns.launch_count(reset=True)
     ns.profile_enable(True)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize(dev)
+    clocks.begin()
     e0.record(stream)
     for _ in range(args.steps):
         step()
     e1.record(stream)
     torch.cuda.synchronize(dev)
+    clocks.end()
     ns.profile_enable(False)
     launches = ns.launch_count()
     ms_local = e0.elapsed_time(e1)
