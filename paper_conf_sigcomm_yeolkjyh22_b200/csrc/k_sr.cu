@@ -1074,12 +1074,25 @@ __device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>:
                                               uint8_t *so, int p) {
     constexpr int wy = UpTapC<S, I>::w1;
     constexpr int base = UpCols<NB, S>::base(I);
-    int pa[3][3], pb[3][3];
+    // O6 is separable with exact integer weights: the vertical pass first,
+    // va[c][t] = (128 - wy) a + wy b per LR column t of the 3 taps, then per output
+    // ((128 - wx) va[ox] + wx va[ox + 1] + 8192) >> 14 -- the same sum as
+    // horizontal-first (distributivity, no intermediate rounding), 3 column
+    // values per plane instead of 2 per output; sub-rows with wy = 0 read one
+    // LR row only.
+    int va[3][3];
 #pragma unroll
     for (int c = 0; c < 3; c++) {
-        const uint8_t *La = lr + (ra * 3 + c) * kLrBoxW, *Lb = lr + (rb * 3 + c) * kLrBoxW;
-        pa[c][0] = La[cm]; pa[c][1] = La[c0]; pa[c][2] = La[cp];
-        pb[c][0] = Lb[cm]; pb[c][1] = Lb[c0]; pb[c][2] = Lb[cp];
+        const uint8_t *La = lr + (ra * 3 + c) * kLrBoxW;
+        const int a0 = La[cm], a1 = La[c0], a2 = La[cp];
+        if constexpr (wy == 0) {
+            va[c][0] = 128 * a0; va[c][1] = 128 * a1; va[c][2] = 128 * a2;
+        } else {
+            const uint8_t *Lb = lr + (rb * 3 + c) * kLrBoxW;
+            va[c][0] = (128 - wy) * a0 + wy * Lb[cm];
+            va[c][1] = (128 - wy) * a1 + wy * Lb[c0];
+            va[c][2] = (128 - wy) * a2 + wy * Lb[cp];
+        }
     }
 #pragma unroll
     for (int j = 0; j < S; j++) {
@@ -1087,9 +1100,7 @@ __device__ __forceinline__ void uptail_subrow(const uint32_t (&v)[UpCols<NB, S>:
         const int wx = (128 * ((2 * j + 1 - S) - 2 * S * (ox - 1)) + S) / (2 * S);
 #pragma unroll
         for (int c = 0; c < 3; c++) {
-            const int ha = (128 - wx) * pa[c][ox] + wx * pa[c][ox + 1];
-            const int hb = (128 - wx) * pb[c][ox] + wx * pb[c][ox + 1];
-            const int U = ((128 - wy) * ha + wy * hb + 8192) >> 14;
+            const int U = (wx ? (128 - wx) * va[c][ox] + wx * va[c][ox + 1] : 128 * va[c][ox]) + 8192 >> 14;
             const int n = (I * S + j) * 3 + c;
             so[c * (kTile * S) + p * S + j] = (uint8_t)f2u8_floor_sat((float)U + (__uint_as_float(v[n - base]) + bh[n - 3 * S * I]));
         }
