@@ -435,6 +435,7 @@ def main():
     pk = peaks()
     fl, by = algorithmic(cfg, types, ia_np, S, n, args.format)
     rl = {}
+    busy = prof.pop("any", None)   # union over all families: device time with library work running
     for fam, (nl, ng, tms) in prof.items():
         if nl == 0 or tms <= 0:
             continue
@@ -548,6 +549,7 @@ def main():
                              "anchors_per_step": int(ia_np.sum())},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
                 "host_enqueue_ms_per_step": host_ms, "step_ms": [round(x, 3) for x in step_ms],
+                "device_busy_ms_per_step": busy[2] / args.steps if busy else None,
                 "hybrid_encode": hybrid,
                 # real-time check: one n-frame chunk of every stream (n/60 s of
                 # 60 fps video) must finish within its own duration
@@ -689,6 +691,7 @@ def run_c5(args):
     ms_local = e0.elapsed_time(e1)
     clk = clocks.stop()
     prof = ns.profile_read()
+    prof.pop("any", None)
     ms = shard.max_over_ranks(ms_local)
     px4k_local = sum(n * 9 * x["w"] * x["h"] for x in mine) / K4_PX      # 4K-equivalent frames per step
     tot = torch.tensor([px4k_local, float(S), float(sum(n for _ in mine))], dtype=torch.float64,

@@ -355,7 +355,10 @@ NS_API uint64_t ns_launch_count(int reset);
    every launch wrapper brackets its kernel(s) with CUDA events on the call's
    stream.  ns_profile_enable(1) clears and starts, (0) stops (records are kept).
    ns_profile_read synchronises the recorded events and fills one entry per
-   family (out must hold >= 16 entries); returns the number written or < 0. */
+   family (out must hold >= 16 entries) -- total_ms is the union of the
+   family's event intervals -- plus, when out holds more, an entry "any": the
+   union over all families (device time in which some library work ran);
+   returns the number written or < 0. */
 typedef struct {
     char name[24];
     uint64_t launches;     /* kernels launched                         */

@@ -470,7 +470,28 @@ extern "C" int ns_profile_read(ns_prof_entry *out, int max) {
         if (!v.empty() && hi > lo) tot += hi - lo;
         out[f].total_ms = tot;
     }
-    return (int)F_COUNT;
+    if (max <= (int)F_COUNT) return (int)F_COUNT;
+    // entry F_COUNT, "any": the union over every family -- the device time in
+    // which at least one library scope was running (step time minus it = idle)
+    std::vector<std::pair<double, double>> all;
+    for (auto &v : iv) all.insert(all.end(), v.begin(), v.end());
+    std::sort(all.begin(), all.end());
+    double tot = 0.0, lo = 0.0, hi = -1e300;
+    for (auto &x : all) {
+        if (x.first > hi) {
+            if (hi > lo) tot += hi - lo;
+            lo = x.first;
+            hi = x.second;
+        } else if (x.second > hi) {
+            hi = x.second;
+        }
+    }
+    if (!all.empty() && hi > lo) tot += hi - lo;
+    memset(&out[F_COUNT], 0, sizeof(ns_prof_entry));
+    snprintf(out[F_COUNT].name, sizeof(out[F_COUNT].name), "any");
+    for (int f = 0; f < F_COUNT; f++) { out[F_COUNT].launches += out[f].launches; out[F_COUNT].scopes += out[f].scopes; }
+    out[F_COUNT].total_ms = tot;
+    return (int)F_COUNT + 1;
 }
 
 // ------------------------------------------------------------------ validation
