@@ -22,9 +22,9 @@ def ctx():
     c.close()
 
 
-def _streams(seed0, shapes, n, keys):
-    return [synth.make_chunk(seed0 + i, w, h, s, n, types=synth.default_types(n, keys)) for i, (w, h, s) in
-            enumerate(shapes)]
+def _streams(seed0, shapes, n, keys, interp=0):
+    return [synth.make_chunk(seed0 + i, w, h, s, n, types=synth.default_types(n, keys), interp=interp)
+            for i, (w, h, s) in enumerate(shapes)]
 
 
 def _run_both(ctx, chunks, specs, n_calls=2, **kw):
@@ -48,12 +48,13 @@ def _run_both(ctx, chunks, specs, n_calls=2, **kw):
             st = torch.zeros((len(cs), 8), dtype=torch.float64, device=DEV)
             if path == "device":
                 dc = [ns.DeviceChunk.from_numpy(c.lr, c.res, c.mv, c.type, c.w, c.h, c.scale, DEV, model=models[i],
-                                                hr_last=state[i][0], hr_golden=state[i][1]) for i, c in enumerate(cs)]
+                                                hr_last=state[i][0], hr_golden=state[i][1], interp=c.interp)
+                      for i, c in enumerate(cs)]
                 ctx.enhance_streams(dc, hr, is_anchor_out=ia, stats=st, **kw)
                 moved = None
             else:
                 hc = [ns.DeviceChunk.pinned_from_numpy(c.lr, c.res, c.mv, c.type, c.w, c.h, c.scale, model=models[i],
-                                                       hr_last=state[i][0], hr_golden=state[i][1])
+                                                       hr_last=state[i][0], hr_golden=state[i][1], interp=c.interp)
                       for i, c in enumerate(cs)]
                 moved = ctx.enhance_streams_host(hc, hr, is_anchor_out=ia, stats=st, **kw)
             torch.cuda.synchronize()
@@ -90,6 +91,14 @@ def test_host_path_matches_device_path_topk():
             assert outs["host"][call]["moved"] == exp
     finally:
         c.close()
+
+
+def test_host_path_8tap_matches_device_path(ctx):
+    """8-tap streams (R13) through the host-input call equal the device path."""
+    shapes = [(64, 32, 2), (48, 24, 3), (32, 16, 4)]
+    chunks = [_streams(5500, shapes, 8, 3, interp=4)]
+    outs = _run_both(ctx, chunks, [(1, 16)] * 3, n_calls=1, k=2)
+    _assert_same(outs)
 
 
 def test_host_path_matches_device_path_many_streams(ctx):

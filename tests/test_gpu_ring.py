@@ -31,13 +31,13 @@ def ctx():
     c.close()
 
 
-def _streams(ctx, specs, n, seed0, altref=4):
+def _streams(ctx, specs, n, seed0, altref=4, interp=0):
     out = []
     for i, (B, C, s, w, h) in enumerate(specs):
         types = synth.default_types(n, altref)
         if i % 2 == 1 and n > 6:
             types[n // 2] = synth.NS_KEY          # a KEY frame inside the chunk
-        c = synth.make_chunk(seed0 + i, w, h, s, n, types=types)
+        c = synth.make_chunk(seed0 + i, w, h, s, n, types=types, interp=interp if i % 2 == 0 else 0)
         m = ctx.model(B, C, s)
         blob = synth.make_weights(seed0 + i, B, C, s)
         m.set_weights(blob)
@@ -86,6 +86,29 @@ def test_ring_equals_full_table(ctx, R):
             assert np.array_equal(ring[si][r], full[si][f_last]), (si, r, f_last)
         assert np.array_equal(st_r[si][0], st_f[si][0]), si     # hr_last
         assert np.array_equal(st_r[si][1], st_f[si][1]), si     # hr_golden
+
+
+def test_ring_equals_full_table_8tap(ctx):
+    """Rings with 8-tap streams (R13; k_recon8 reads the GOLDEN copies and the
+    anchor-cache copies the bilinear kernel makes) next to bilinear ones."""
+    specs = [(2, 16, 2, 64, 32), (1, 32, 3, 48, 24), (1, 16, 3, 48, 24), (1, 16, 4, 32, 16)]
+    n, R = 13, 3
+    streams = _streams(ctx, specs, n, 8300, interp=4)
+    full, ia_f, st_f = _run(ctx, streams, 0, k=4)
+    ring, ia_r, st_r = _run(ctx, streams, R, k=4)
+    assert np.array_equal(ia_f, ia_r)
+    for si, (c, m, blob, (B, C)) in enumerate(streams):
+        for r in range(R):
+            f_last = max(f for f in range(n) if f % R == r)
+            assert np.array_equal(ring[si][r], full[si][f_last]), (si, r, f_last)
+        assert np.array_equal(st_r[si][0], st_f[si][0]) and np.array_equal(st_r[si][1], st_f[si][1]), si
+    # and the full run is the oracle's reconstruction from its own anchors (non-anchor frames exact)
+    rng = np.random.default_rng(17)
+    for si, (c, m, blob, _) in enumerate(streams):
+        last, gold = (x.cpu().numpy() for x in _state(c, rng))
+        got = np.stack(full[si])
+        exp, _, _ = oracle.reconstruct(c, list(ia_f[si]), got, last, gold)
+        assert np.array_equal(got, exp), si
 
 
 def test_ring_full_table_matches_oracle(ctx):
