@@ -316,12 +316,11 @@ __host__ __device__ constexpr int tap_w1(int k) { return (128 * ((2 * k + 1 - S)
 //   v    = 128 V[d] + w1 (V[d+1] - V[d])          (exact 2-D O6 sum, d = tap)
 //   s    = 4 (v + 8192 + 2^22) = 512 V[d] + 4 w1 (V[d+1] - V[d]) + KB
 // and r + 256 = s >> 16 (high half-word).
-// (UOFF: the lane offset, r + UOFF; 256 here, 384 in k_recon8)
-template <int S, bool CH, int WY, int UOFF = 256>
+template <int S, bool CH, int WY>
 __device__ __forceinline__ void recon_up_row(const int (&a)[ReconCfg<S, CH>::NLR], const int (&b)[ReconCfg<S, CH>::NLR],
                                              uint32_t (&u)[ReconCfg<S, CH>::NP]) {
     constexpr int BW = ReconCfg<S, CH>::BW, NLR = ReconCfg<S, CH>::NLR;
-    constexpr int KB = 4 * 8192 + 4 * (UOFF << 14);
+    constexpr int KB = 4 * 8192 + 4 * (256 << 14);
     int V[NLR], base[NLR];
 #pragma unroll
     for (int t = 0; t < NLR; t++) {
@@ -626,11 +625,15 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
 // the residual, exactly as in k_recon_step.
 //
 // A thread owns 4 LR columns (4s HR pixels; half a luma block, a whole chroma
-// block) over 4s HR rows, so its motion vector is uniform.  Its reference
-// window rows (4s + 7 bytes, 4s + 7 rows) stream through a shared-memory ring
-// by cp.async; each row's horizontal pass is kept in registers (8 rows, 16-bit
-// lanes holding two pixels, even/odd interleaved as in k_recon_step) and the
+// block) over one block row (8s luma / 4s chroma HR rows), so its motion
+// vector and kernel are uniform.  Its reference window rows (4s + 7 bytes,
+// R + 7 rows) stream through a shared-memory ring by cp.async; each row's
+// horizontal pass (16-bit lanes holding two pixels, even/odd interleaved as in
+// k_recon_step) goes into a per-thread shared-memory ring of 8 rows, and the
 // vertical pass of output row j runs as soon as window row j + 7 is filtered.
+// (Keeping those 8 rows in registers needs the row loop fully unrolled: 5.9K
+// instructions that miss the instruction cache, 167 registers, 3 CTAs per SM
+// -- 204 vs 147 ms per c4 step.)
 // 16-bit lanes: a pass sums 8 taps of bytes with a bias of 128 * 128 + 64 per
 // lane, sum + bias in [2678, 62858] for every kernel (the sharpest phase has
 // positive taps 182, negative 54), so the packed multiply-adds never carry
@@ -665,26 +668,57 @@ __constant__ int16_t c_vp9_f8[3][16][8] = {
      {-1, 3, -6, 17, 125, -13, 5, -2},  {0, 1, -3, 8, 127, -7, 3, -1}}};
 
 constexpr int kR8TX = 32, kR8TY = 4, kR8NT = kR8TX * kR8TY;
-template <int S>
-struct R8Cfg {
-    static constexpr int TW = 4 * S;                  // HR pixels per thread row (4 LR columns)
-    static constexpr int NPT = TW / 2;                // 16-bit pairs per row
-    static constexpr int R = 4 * S;                   // HR rows per thread
-    static constexpr int NW = R + 7;                  // window rows
-    static constexpr int NQ = (7 + TW + 7 + 7) / 8;   // aligned 8-B words per window row
-    static constexpr int LA = 6;                      // window rows in flight
-    static constexpr int NR = LA + 1;                 // ring slots (row i + LA lands in row i - 1's)
-    static constexpr int JMAX = pair_px(NPT - 1, 0) + 7;  // last pair source P_j of a row
-    static constexpr int GMAX = JMAX / 4 + 1;         // aligned 4-byte groups a row's pass touches
-    static constexpr size_t SMEM = (size_t)NR * NQ * kR8NT * 8;
-    static_assert(4 * (GMAX + 1) + 7 <= 8 * NQ + 8, "window words cover every pass source");
-};
+#ifndef NS_R8_LA
+#define NS_R8_LA 4     // window rows in flight per thread
+#endif
+#ifndef NS_R8_UNROLL
+#define NS_R8_UNROLL 1 // row-loop unroll of k_recon8
+#endif
+#define NS_PRAGMA_(x) _Pragma(#x)
+#define NS_UNROLL_(n) NS_PRAGMA_(unroll n)
 constexpr uint32_t kR8Bias = (128u * 128u + 64u) * 0x00010001u;
 constexpr uint32_t kR8Lo = (128u * 128u) * 0x00010001u, kR8Hi = (384u * 128u - 1u) * 0x00010001u;
 
+// One LR row of a k_recon8 thread's 6 O6 source columns (4 own + one each
+// side, clamped, Z16): LR bytes (KEY / INTRA) or the residual.
+template <bool LR>
+__device__ __forceinline__ void r8_lr_row(const void *plane, int row, int pw, int c0, int cl, int cr, int (&v)[6]) {
+    if constexpr (LR) {
+        const uint8_t *p = static_cast<const uint8_t *>(plane) + (size_t)row * pw;
+        const uint32_t q4 = *reinterpret_cast<const uint32_t *>(p + c0);
+#pragma unroll
+        for (int e = 0; e < 4; e++) v[1 + e] = (q4 >> (8 * e)) & 255;
+        v[0] = p[cl];
+        v[5] = p[cr];
+    } else {
+        const int16_t *p = static_cast<const int16_t *>(plane) + (size_t)row * pw;
+        const uint2 q4 = *reinterpret_cast<const uint2 *>(p + c0);
+        v[1] = (int)(int16_t)(q4.x & 0xFFFFu); v[2] = (int)(int16_t)(q4.x >> 16);
+        v[3] = (int)(int16_t)(q4.y & 0xFFFFu); v[4] = (int)(int16_t)(q4.y >> 16);
+        v[0] = p[cl];
+        v[5] = p[cr];
+    }
+}
+
+template <int S, bool CH>
+struct R8Cfg {
+    static constexpr int TW = 4 * S;                  // HR pixels per thread row (4 LR columns)
+    static constexpr int NPT = TW / 2;                // 16-bit pairs per row
+    static constexpr int R = CH ? 4 * S : 8 * S;      // HR rows per thread: one block row (uniform vector)
+    static constexpr int NW = R + 7;                  // window rows
+    static constexpr int NQ = (7 + TW + 7 + 7) / 8;   // aligned 8-B words per window row
+    static constexpr int JMAX = pair_px(NPT - 1, 0) + 7;  // last pair source P_j of a row
+    static constexpr int GMAX = JMAX / 4 + 1;         // aligned 4-byte groups a row's pass touches
+    static_assert(4 * (GMAX + 1) + 7 <= 8 * NQ + 8, "window words cover every pass source");
+    static constexpr int LA = NS_R8_LA, NR = LA + 1;  // window rows in flight; ring slots
+    static constexpr size_t WIN = (size_t)NR * NQ * kR8NT * 8;             // [NR][NQ][NT] 8-B words
+    static constexpr size_t TRING = (size_t)8 * (NPT / 2) * kR8NT * 8;     // [8][NPT/2][NT] pass rows
+    static constexpr size_t SMEM = WIN + TRING;
+};
+
 template <int S, bool CH>
 __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n, int f, int s0) {
-    using Cfg = R8Cfg<S>;
+    using Cfg = R8Cfg<S, CH>;
     constexpr int TW = Cfg::TW, NPT = Cfg::NPT, R = Cfg::R, NW = Cfg::NW, NQ = Cfg::NQ, LA = Cfg::LA, NR = Cfg::NR;
     constexpr int GMAX = Cfg::GMAX;
     const int sid = s0 + blockIdx.z;
@@ -693,7 +727,7 @@ __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n,
     if (CH && fd.fmt != NS_FMT_I420) return;
     const int w = fd.w, h = fd.h;
     const int pw = CH ? w / 2 : w, ph = CH ? h / 2 : h, W = S * pw, H = S * ph;
-    const int gx0 = blockIdx.x * kR8TX;                 // first 4-LR-column group of the CTA
+    const int gx0 = blockIdx.x * kR8TX;
     const int Y0c = blockIdx.y * kR8TY * R;
     if (4 * gx0 >= pw || Y0c >= H) return;              // CTA-uniform
     __shared__ int16_t s_f8[3 * 16 * 8];
@@ -709,14 +743,13 @@ __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n,
     const size_t plr = (size_t)ph * pw, phr = (size_t)H * W;
     const size_t lr0 = CH ? lrp : 0, hr0 = CH ? hrp : 0;
     const int np_ = CH ? 2 : (fd.fmt == NS_FMT_I420 ? 1 : 3);
-    // the block's vector: luma blocks are 8 LR columns (two threads), chroma blocks 4
-    const int bxm = CH ? gx : gx >> 1, bym = CH ? Y0 / (4 * S) : Y0 / (8 * S);
+    const int bxm = CH ? gx : gx >> 1, bym = Y0 / R;
     const ns_block_mv mv = fd.mv_f[(size_t)bym * (w / 8) + bxm];
-    const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;   // KEY / INTRA: up_s(LR) (Z17)
+    const bool use_lr = fd.key || mv.ref == NS_REF_INTRA;
     const int kern = fd.interp == NS_INTERP_SWITCHABLE ? (mv.filter > 2 ? 0 : mv.filter) : fd.interp - 1;
-    const int qx = (CH ? 1 : 2) * S * mv.mvx, qy = (CH ? 1 : 2) * S * mv.mvy;   // 1/16 HR pel
+    const int qx = (CH ? 1 : 2) * S * mv.mvx, qy = (CH ? 1 : 2) * S * mv.mvy;
     const int X0 = gx * TW;
-    const int xs = X0 + (qx >> 4) - 3, ys = Y0 + (qy >> 4) - 3;   // window origin (tap -3)
+    const int xs = X0 + (qx >> 4) - 3, ys = Y0 + (qy >> 4) - 3;
     uint32_t fx[8], fy[8];
 #pragma unroll
     for (int t = 0; t < 8; t++) {
@@ -726,59 +759,49 @@ __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n,
     const int xb = xs & ~7, m = xs & 7;
     const bool interior = xb >= 0 && xb + 8 * NQ <= W;
     const uint8_t *ref = (mv.ref == NS_REF_GOLDEN ? fd.ref_gold : fd.ref_last) + hr0;
-    uint2 *ring = reinterpret_cast<uint2 *>(r8_sm) + tid;
+    uint2 *ring = reinterpret_cast<uint2 *>(r8_sm) + tid;                         // [NR][NQ][NT]
+    uint2 *tring = reinterpret_cast<uint2 *>(r8_sm + Cfg::WIN) + tid;            // [8][NPT/2][NT]
     const int c0 = 4 * gx, cl = max(c0 - 1, 0), cr = min(c0 + 4, pw - 1);
+    const int lr_row0 = Y0 / S - 1;
 
 #pragma unroll 1
     for (int c = 0; c < np_; c++) {
         const uint8_t *refc = ref + c * phr;
+        int st_slot = 0, rd_slot = 0;
         auto stage = [&](int i) {
             if (!use_lr && i < NW) {
                 const uint8_t *row = refc + (size_t)min(max(ys + i, 0), H - 1) * W;
-                uint2 *dst = ring + (i % NR) * NQ * kR8NT;
+                uint2 *dst = ring + st_slot * NQ * kR8NT;
 #pragma unroll
                 for (int q = 0; q < NQ; q++)
                     cp_async8(dst + q * kR8NT, row + (interior ? xb + 8 * q : min(max(xb + 8 * q, 0), W - 8)));
             }
+            st_slot = st_slot == NR - 1 ? 0 : st_slot + 1;
             asm volatile("cp.async.commit_group;" ::: "memory");
         };
 #pragma unroll
         for (int i = 0; i < LA; i++) stage(i);
-        const int16_t *resc = fd.res_f + lr0 + c * plr;
-        const uint8_t *lrc = fd.lr_f + lr0 + c * plr;
-        uint8_t *outc = fd.out + hr0 + c * phr + (size_t)Y0 * W + X0;
-        uint32_t T[8][NPT];
-        int rv[3][6];
-        auto load_lr_rows = [&](int it) {   // LR rows it .. it+2 of this thread (row Y0/S - 1 + it), clamped (Z16)
-#pragma unroll
-            for (int t = 0; t < 3; t++) {
-                const int row = min(max(Y0 / S - 1 + it + t, 0), ph - 1);
-                if (use_lr) {
-                    const uint8_t *p = lrc + (size_t)row * pw;
-                    const uint32_t q4 = *reinterpret_cast<const uint32_t *>(p + c0);
-#pragma unroll
-                    for (int e = 0; e < 4; e++) rv[t][1 + e] = (q4 >> (8 * e)) & 255;
-                    rv[t][0] = p[cl];
-                    rv[t][5] = p[cr];
-                } else {
-                    const int16_t *p = resc + (size_t)row * pw;
-                    const uint2 q4 = *reinterpret_cast<const uint2 *>(p + c0);
-                    rv[t][1] = (int)(int16_t)(q4.x & 0xFFFFu); rv[t][2] = (int)(int16_t)(q4.x >> 16);
-                    rv[t][3] = (int)(int16_t)(q4.y & 0xFFFFu); rv[t][4] = (int)(int16_t)(q4.y >> 16);
-                    rv[t][0] = p[cl];
-                    rv[t][5] = p[cr];
-                }
-            }
+        const void *src_c = use_lr ? static_cast<const void *>(fd.lr_f + lr0 + c * plr)
+                                   : static_cast<const void *>(fd.res_f + lr0 + c * plr);
+        auto lr_row = [&](int k, int (&v)[6]) {
+            const int row = min(max(lr_row0 + k, 0), ph - 1);
+            if (use_lr) r8_lr_row<true>(src_c, row, pw, c0, cl, cr, v);
+            else r8_lr_row<false>(src_c, row, pw, c0, cl, cr, v);
         };
-        auto row_i = [&](auto ic) {
-            constexpr int i = decltype(ic)::value;
-            // window row i: landed when at most LA - 1 newer groups are pending
+        int rv[3][6];
+        lr_row(0, rv[0]);
+        lr_row(1, rv[1]);
+        lr_row(2, rv[2]);
+        uint8_t *outc = fd.out + hr0 + c * phr + (size_t)Y0 * W + X0;
+        NS_UNROLL_(NS_R8_UNROLL)
+        for (int i = 0; i < NW; i++) {
             asm volatile("cp.async.wait_group %0;" ::"n"(LA - 1) : "memory");
             uint2 q[NQ];
-            const uint2 *src = ring + (i % NR) * NQ * kR8NT;
+            const uint2 *src = ring + rd_slot * NQ * kR8NT;
+            rd_slot = rd_slot == NR - 1 ? 0 : rd_slot + 1;
 #pragma unroll
             for (int k = 0; k < NQ; k++) q[k] = use_lr ? make_uint2(0u, 0u) : src[k * kR8NT];
-            if (!interior) {   // words wholly outside the row replicate its edge pixel (Z16)
+            if (!interior) {
 #pragma unroll
                 for (int k = 0; k < NQ; k++) {
                     const int st = xb + 8 * k;
@@ -787,7 +810,6 @@ __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n,
                 }
             }
             stage(i + LA);
-            // horizontal pass: P_j = [w(j), w(j + 2)] from the aligned 4-byte groups
             uint32_t wv[2 * NQ + 2];
 #pragma unroll
             for (int k = 0; k < NQ; k++) { wv[2 * k] = q[k].x; wv[2 * k + 1] = q[k].y; }
@@ -814,47 +836,79 @@ __global__ void __launch_bounds__(kR8NT) k_recon8(const FrameDesc *fdesc, int n,
                     default: return __funnelshift_r(O[g], O[g + 1], 16);
                 }
             };
+            uint2 *trow = tring + (i & 7) * (NPT / 2) * kR8NT;
 #pragma unroll
-            for (int k = 0; k < NPT; k++) {
-                const int x0 = pair_px(k, 0);
-                uint32_t acc = kR8Bias;
+            for (int k2 = 0; k2 < NPT / 2; k2++) {
+                uint32_t tv[2];
 #pragma unroll
-                for (int t = 0; t < 8; t++) acc = mad_u32(P(x0 + t), fx[t], acc);
-                acc = vmin_u16x2(vmax_u16x2(acc, kR8Lo), kR8Hi);
-                T[i % 8][k] = ((acc - kR8Lo) >> 7) & 0x00FF00FFu;
-            }
-            if constexpr (i >= 7) {
-                constexpr int j = i - 7, it = j / S, jj = j % S;
-                if constexpr (jj == 0) load_lr_rows(it);
-                constexpr int ta = tap_d<S>(jj) + 1;
-                uint32_t u[NPT], x[NPT], o[TW / 4];
-                recon_up_row<S, true, tap_w1<S>(jj), 384>(rv[ta], rv[ta + 1], u);   // r + 384 per lane
-#pragma unroll
-                for (int k = 0; k < NPT; k++) {
+                for (int e = 0; e < 2; e++) {
+                    const int x0 = pair_px(2 * k2 + e, 0);
                     uint32_t acc = kR8Bias;
 #pragma unroll
-                    for (int r = 0; r < 8; r++) acc = mad_u32(T[(j + r) % 8][k], fy[r], acc);
+                    for (int t = 0; t < 8; t++) acc = mad_u32(P(x0 + t), fx[t], acc);
                     acc = vmin_u16x2(vmax_u16x2(acc, kR8Lo), kR8Hi);
-                    const uint32_t pv = use_lr ? 0x00800080u : (acc >> 7) & 0x01FF01FFu;   // pred + 128
-                    x[k] = vmin_u16x2(vmax_u16x2(pv + u[k], 0x02000200u), 0x02FF02FFu);      // pred + r + 512, clamped
+                    tv[e] = ((acc - kR8Lo) >> 7) & 0x00FF00FFu;
                 }
+                trow[k2 * kR8NT] = make_uint2(tv[0], tv[1]);
+            }
+            if (i < 7) continue;
+            const int j = i - 7, jj = j % S;
+            if (jj == 0 && j > 0) {   // a new O6 period: shift the source rows in
 #pragma unroll
-                for (int qq = 0; qq < TW / 4; qq++) o[qq] = prmt(x[2 * qq], x[2 * qq + 1], 0x6240u);
-                uint8_t *dst = outc + (size_t)j * W;
-                if constexpr (TW % 16 == 0) {
+                for (int t = 0; t < 6; t++) { rv[0][t] = rv[1][t]; rv[1][t] = rv[2][t]; }
+                lr_row(j / S + 2, rv[2]);
+            }
+            const int ta = tap_d<S>(jj) + 1, wy = tap_w1<S>(jj);
+            int V[6], base[6];
 #pragma unroll
-                    for (int qq = 0; qq < TW / 16; qq++)
-                        *reinterpret_cast<uint4 *>(dst + 16 * qq) = make_uint4(o[4 * qq], o[4 * qq + 1], o[4 * qq + 2], o[4 * qq + 3]);
-                } else if constexpr (TW % 8 == 0) {
+            for (int t = 0; t < 6; t++) {
+                const int a = ta ? rv[1][t] : rv[0][t], b = ta ? rv[2][t] : rv[1][t];
+                V[t] = (128 - wy) * a + wy * b;
+                base[t] = (int)mad_u32((uint32_t)V[t], 512u, (uint32_t)(4 * 8192 + 4 * (384 << 14)));
+            }
+            uint32_t acc[NPT];
 #pragma unroll
-                    for (int qq = 0; qq < TW / 8; qq++) *reinterpret_cast<uint2 *>(dst + 8 * qq) = make_uint2(o[2 * qq], o[2 * qq + 1]);
-                } else {
+            for (int k = 0; k < NPT; k++) acc[k] = kR8Bias;
 #pragma unroll
-                    for (int qq = 0; qq < TW / 4; qq++) *reinterpret_cast<uint32_t *>(dst + 4 * qq) = o[qq];
+            for (int r = 0; r < 8; r++) {
+                const uint2 *tr = tring + ((j + r) & 7) * (NPT / 2) * kR8NT;
+#pragma unroll
+                for (int k2 = 0; k2 < NPT / 2; k2++) {
+                    const uint2 tv = tr[k2 * kR8NT];
+                    acc[2 * k2] = mad_u32(tv.x, fy[r], acc[2 * k2]);
+                    acc[2 * k2 + 1] = mad_u32(tv.y, fy[r], acc[2 * k2 + 1]);
                 }
             }
-        };
-        static_for<NW>(row_i);
+            uint32_t x[NPT], o[TW / 4];
+#pragma unroll
+            for (int k = 0; k < NPT; k++) {
+                uint32_t sv[2];
+#pragma unroll
+                for (int e = 0; e < 2; e++) {
+                    const int px = pair_px(k, e);
+                    const int d = tap_d<S>(px) + 1, w1 = tap_w1<S>(px);
+                    sv[e] = (uint32_t)(w1 ? base[d] + (4 * w1) * (V[d + 1] - V[d]) : base[d]);
+                }
+                const uint32_t u = prmt(sv[0], sv[1], 0x7632u);
+                const uint32_t a = vmin_u16x2(vmax_u16x2(acc[k], kR8Lo), kR8Hi);
+                const uint32_t pv = use_lr ? 0x00800080u : (a >> 7) & 0x01FF01FFu;
+                x[k] = vmin_u16x2(vmax_u16x2(pv + u, 0x02000200u), 0x02FF02FFu);
+            }
+#pragma unroll
+            for (int qq = 0; qq < TW / 4; qq++) o[qq] = prmt(x[2 * qq], x[2 * qq + 1], 0x6240u);
+            uint8_t *dst = outc + (size_t)j * W;
+            if constexpr (TW % 16 == 0) {
+#pragma unroll
+                for (int qq = 0; qq < TW / 16; qq++)
+                    *reinterpret_cast<uint4 *>(dst + 16 * qq) = make_uint4(o[4 * qq], o[4 * qq + 1], o[4 * qq + 2], o[4 * qq + 3]);
+            } else if constexpr (TW % 8 == 0) {
+#pragma unroll
+                for (int qq = 0; qq < TW / 8; qq++) *reinterpret_cast<uint2 *>(dst + 8 * qq) = make_uint2(o[2 * qq], o[2 * qq + 1]);
+            } else {
+#pragma unroll
+                for (int qq = 0; qq < TW / 4; qq++) *reinterpret_cast<uint32_t *>(dst + 4 * qq) = o[qq];
+            }
+        }
     }
 }
 
@@ -880,8 +934,10 @@ static cudaError_t recon_launch(dim3 g, cudaStream_t st, const FrameDesc *fd, in
 template <int S, bool CH>
 static cudaError_t recon8_launch(int max_pw, int max_ph, cudaStream_t st, const FrameDesc *fd, int n, int f, int s0,
                                  int nstreams) {
-    dim3 g((max_pw / 4 + kR8TX - 1) / kR8TX, (max_ph * S / R8Cfg<S>::R + kR8TY - 1) / kR8TY, nstreams);
-    k_recon8<S, CH><<<g, dim3(kR8TX, kR8TY), R8Cfg<S>::SMEM, st>>>(fd, n, f, s0);
+    using Cfg = R8Cfg<S, CH>;
+    if (cudaError_t e = ensure_kernel_smem<k_recon8<S, CH>>((int)Cfg::SMEM); e != cudaSuccess) return e;
+    dim3 g((max_pw / 4 + kR8TX - 1) / kR8TX, (max_ph * S / Cfg::R + kR8TY - 1) / kR8TY, nstreams);
+    k_recon8<S, CH><<<g, dim3(kR8TX, kR8TY), Cfg::SMEM, st>>>(fd, n, f, s0);
     return cudaGetLastError();
 }
 
