@@ -172,6 +172,24 @@ __device__ __forceinline__ void tmem_st1(uint32_t taddr, float v) {
     asm volatile("tcgen05.st.sync.aligned.32x32b.x1.b32 [%0], {%1};" ::"r"(taddr), "f"(v) : "memory");
 }
 __device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+// N consecutive columns from v[0..N) in at most two stores (.x8 / .x4 / .x2 / .x1).
+template <int N>
+__device__ __forceinline__ void tmem_st_run(uint32_t taddr, const float *v) {
+    if constexpr (N >= 8) {
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), "f"(v[0]),
+                     "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]) : "memory");
+        tmem_st_run<N - 8>(taddr + 8, v + 8);
+    } else if constexpr (N >= 4) {
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x4.b32 [%0], {%1,%2,%3,%4};" ::"r"(taddr), "f"(v[0]), "f"(v[1]),
+                     "f"(v[2]), "f"(v[3]) : "memory");
+        tmem_st_run<N - 4>(taddr + 4, v + 4);
+    } else if constexpr (N >= 2) {
+        asm volatile("tcgen05.st.sync.aligned.32x32b.x2.b32 [%0], {%1,%2};" ::"r"(taddr), "f"(v[0]), "f"(v[1]) : "memory");
+        tmem_st_run<N - 2>(taddr + 2, v + 2);
+    } else if constexpr (N == 1) {
+        tmem_st1(taddr, v[0]);
+    }
+}
 
 __device__ __forceinline__ int mod5(int v) { return ((v % 5) + 5) % 5; }
 
@@ -1291,8 +1309,7 @@ __global__ void __launch_bounds__(Up2Cfg<CIN, NB, S>::NWARPS * 32, 1)
                 // before the block is free, and no bias add below.  The first five
                 // retirements read blocks zeroed at allocation and add it here.
                 const bool addb = q < 5;
-#pragma unroll
-                for (int i = 0; i < 3 * S; i++) tmem_st1(acc + (uint32_t)(3 * S * g + i), bh[i]);
+                tmem_st_run<3 * S>(acc + (uint32_t)(3 * S * g), bh);
                 tmem_wait_st();
                 tc_fence_before();
                 mbar_arrive(edone(k));
