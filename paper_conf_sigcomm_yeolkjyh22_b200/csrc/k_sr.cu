@@ -112,7 +112,10 @@ struct RotCfg {
     static constexpr uint32_t BIAS_BYTES = NB * 4u;
     static constexpr uint32_t W_REGION = round_up(B_BYTES + BIAS_BYTES, 1024);
     static constexpr uint32_t SLOT_BYTES = kHalo * CIN * 2u;
-    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 1024);
+    // 128-B slots (bulk-copy rows need 16 B): with 1-KB rounding the C = 32
+    // conv (the end conv) took 59.5 KB and 3 CTAs per SM; 56.8 KB fits 4,
+    // as many as its TMEM (128 columns each) allows
+    static constexpr uint32_t SLOT = round_up(SLOT_BYTES, 128);
     static constexpr int NSLOT = 3;  // input ring; the barrier array is laid out [0,3) ring, 3 weights, 4 MMA
     static constexpr uint32_t TMEM_COLS = tmem_cols_for(3 * NB);
     static constexpr uint32_t SMEM = W_REGION + NSLOT * SLOT + 128;
@@ -1668,7 +1671,7 @@ constexpr int kRotRows = 180;  // rows per CTA strip of the rotated conv and upt
 template <int CIN, int NB, int EPI>
 static cudaError_t conv_rot(int fam, const CUtensorMap &tm, ConvArgs args, int nj, cudaStream_t st) {
     using Cfg = RotCfg<CIN, NB>;
-    if (cudaError_t e = ensure_kernel_smem<k_conv_rot<CIN, NB, EPI>>(Cfg::SMEM); e != cudaSuccess) return e;
+    if (cudaError_t e = ensure_kernel_smem<k_conv_rot<CIN, NB, EPI>>(Cfg::SMEM, 100); e != cudaSuccess) return e;
     args.n_xtiles = (args.W + kTile - 1) / kTile;
     args.rows_per_cta = kRotRows;
     dim3 grid(args.n_xtiles, (args.H + kRotRows - 1) / kRotRows, nj);
