@@ -250,7 +250,8 @@ NS_API ns_status ns_select_merge(ns_ctx *ctx, int S, int n, const int64_t *gain,
                                  int32_t *rank, uint8_t *is_anchor, void *stream);
 
 /* SR on a host-supplied job list (jobs: HOST array [n_jobs]).  Jobs may mix
-   models and resolutions; they are grouped by shape internally. */
+   models and resolutions; they are grouped by shape internally.  lr and
+   hr_out must be 16-B aligned (as the chunk buffers). */
 NS_API ns_status ns_sr_anchors(ns_ctx *ctx, const ns_sr_job *jobs, int n_jobs, void *stream);
 
 /* Reuse-based reconstruction of every non-anchor frame of S chunks (§2, §6.1).

@@ -1529,32 +1529,42 @@ __device__ __forceinline__ int up2_px(const uint8_t *P, int ph, int pw, int y, i
     return (v + 8192) >> 14;
 }
 
+// One thread per 4 consecutive LR pixels (w % 8 == 0): 4-byte loads per plane,
+// four 16-B x0 stores and 4-byte lr8 stores (a thread per pixel with byte
+// accesses ran at 0.5 of HBM).
 __global__ void k_prep_lr(const SrJob *jobs, int j0, const int32_t *job_count, int h, int w, uint16_t *x0,
                           uint8_t *lr8, int wp, int fmt) {
     const int slot = blockIdx.y, job = j0 + slot;
     if (job_count && job >= *job_count) return;
-    const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-    if (idx >= h * w) return;
-    const int y = idx / w, x = idx % w;
+    const int idx4 = blockIdx.x * blockDim.x + threadIdx.x, w4 = w / 4;
+    if (idx4 >= h * w4) return;
+    const int y = idx4 / w4, x = 4 * (idx4 % w4);
     const uint8_t *L = jobs[job].lr;
-    const size_t plane = (size_t)h * w;
-    int p0 = L[idx], p1, p2;
+    const size_t plane = (size_t)h * w, idx = (size_t)y * w + x;
+    uint32_t q[3];
+    q[0] = __ldg(reinterpret_cast<const unsigned int *>(L + idx));
     if (fmt == NS_FMT_I420) {
-        p1 = up2_px(L + plane, h / 2, w / 2, y, x);
-        p2 = up2_px(L + plane + plane / 4, h / 2, w / 2, y, x);
+#pragma unroll
+        for (int c = 1; c < 3; c++) {
+            const uint8_t *P = L + plane + (size_t)(c - 1) * (plane / 4);
+            q[c] = 0;
+#pragma unroll
+            for (int e = 0; e < 4; e++) q[c] |= (uint32_t)up2_px(P, h / 2, w / 2, y, x + e) << (8 * e);
+        }
     } else {
-        p1 = L[plane + idx];
-        p2 = L[2 * plane + idx];
+        q[1] = __ldg(reinterpret_cast<const unsigned int *>(L + plane + idx));
+        q[2] = __ldg(reinterpret_cast<const unsigned int *>(L + 2 * plane + idx));
     }
-    uint4 o0;
-    o0.x = pack_bf16((float)p0 - 128.f, (float)p1 - 128.f);
-    o0.y = pack_bf16((float)p2 - 128.f, 0.f);
-    o0.z = 0; o0.w = 0;
-    *reinterpret_cast<uint4 *>(x0 + (((size_t)slot * h + y) * w + x) * 8) = o0;  // channel group 0 only
+    uint4 *o = reinterpret_cast<uint4 *>(x0 + (((size_t)slot * h + y) * w + x) * 8);   // channel group 0 only
+#pragma unroll
+    for (int e = 0; e < 4; e++) {
+        const float p0 = (float)((q[0] >> (8 * e)) & 255), p1 = (float)((q[1] >> (8 * e)) & 255),
+                    p2 = (float)((q[2] >> (8 * e)) & 255);
+        o[e] = make_uint4(pack_bf16(p0 - 128.f, p1 - 128.f), pack_bf16(p2 - 128.f, 0.f), 0u, 0u);
+    }
     uint8_t *l8 = lr8 + ((size_t)slot * h + y) * 3 * wp + x;
-    l8[0] = (uint8_t)p0;
-    l8[wp] = (uint8_t)p1;
-    l8[2 * wp] = (uint8_t)p2;
+#pragma unroll
+    for (int c = 0; c < 3; c++) *reinterpret_cast<uint32_t *>(l8 + (size_t)c * wp) = q[c];
 }
 
 // NS_FMT_I420 output: the net's full-resolution HR [3][H][W] (hr_tmp) -> jobs[].hr
@@ -1731,7 +1741,7 @@ static cudaError_t run_net(const SrArena *a, int n_blocks, const SrJob *jobs, in
     const int h = a->h, w = a->w, s = a->s;
     cudaError_t e;
     {
-        dim3 g((h * w + 255) / 256, nj);
+        dim3 g((h * (w / 4) + 255) / 256, nj);
         KScope ks(F_SR_PREP, st);
         k_prep_lr<<<g, 256, 0, st>>>(jobs, j0, job_count, h, w, a->x0, a->lr8, a->wp, a->fmt);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;

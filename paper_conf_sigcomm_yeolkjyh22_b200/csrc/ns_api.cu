@@ -818,6 +818,7 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
     for (int j = 0; j < n_jobs; j++) {
         const ns_sr_job &J = jobs[j];
         if (!J.model || !J.lr || !J.hr_out) return fail(NS_EINVAL, "job %d: NULL model/lr/hr_out", j);
+        if (!al16(J.lr) || !al16(J.hr_out)) return fail(NS_EINVAL, "job %d: lr/hr_out must be 16-B aligned", j);
         if (!J.model->has_weights) return fail(NS_EINVAL, "job %d: model has no weights", j);
         if (J.w < 8 || J.h < 8 || J.w % 8 || J.h % 8) return fail(NS_EINVAL, "job %d: w=%d h=%d must be multiples of 8", j, J.w, J.h);
     }

@@ -147,6 +147,9 @@ def test_sr_jobs_rejected(ctx, model):
     lr = torch.zeros((3, 16, 36), dtype=torch.uint8, device=DEV)
     hr = torch.zeros((3, 32, 72), dtype=torch.uint8, device=DEV)
     _expect(ns.NS_EINVAL, ctx.sr_anchors, [(model, lr, hr)], msg="multiples of 8")
+    lr_buf = torch.zeros(3 * 16 * 32 + 4, dtype=torch.uint8, device=DEV)
+    hr_ok = torch.zeros((3, 32, 64), dtype=torch.uint8, device=DEV)
+    _expect(ns.NS_EINVAL, ctx.sr_anchors, [(model, lr_buf[4:].view(3, 16, 32), hr_ok)], msg="aligned")
     L = ns.lib()
     assert L.ns_sr_anchors(ctypes.c_void_p(ctx.handle), None, 2, None) == ns.NS_EINVAL
 
