@@ -163,6 +163,17 @@ class Clocks:
 
 
 # ---------------------------------------------------------------- CPU oracle
+def cpu_model():
+    """The host CPU the oracle ran on (lscpu's "Model name", from /proc/cpuinfo)."""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return f"{line.split(':', 1)[1].strip()} ({os.cpu_count()} logical CPUs)"
+    except OSError:
+        pass
+    return None
+
+
 def cpu_sample(cfg, chunk, blob):
     """Times the oracle as it stands on a bounded sample of one stream-chunk and
     converts to the metric: chunk time = score+select (whole chunk) + k x SR
@@ -187,7 +198,7 @@ def cpu_sample(cfg, chunk, blob):
     t_rec = (time.perf_counter() - t0) / 2
     t_chunk = t_sel + k * t_sr + (n - k) * t_rec
     threads = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
-    return dict(value=n / t_chunk, unit=UNIT, cores=threads, kind="oracle",
+    return dict(value=n / t_chunk, unit=UNIT, cores=threads, kind="oracle", cpu=cpu_model(),
                 sample=f"1 stream-chunk of {cfg['name']} ({w}x{h}->x{s}, n={n}, k={k}): score+select on the full "
                        f"chunk ({t_sel:.2f}s), SR on a {w}x{rows} LR strip scaled by pixels ({t_sr:.1f}s/frame, fp64 "
                        f"OpenMP), reconstruction of 2 non-anchor frames ({t_rec:.2f}s/frame, 1 thread)",
@@ -220,7 +231,8 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": dict(workload_config(cfg, args.gpus, interp=args.interp), sample="one stream-chunk of the workload per step "
                                                                     "(see cpu_baseline.sample), scaled to frames/s"),
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["cores"], "kind": "oracle", "sample": r["sample"]},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["cores"], "kind": "oracle", "sample": r["sample"],
+                             "cpu": r["cpu"]},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -552,7 +564,7 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not i420:
         r = cpu_sample(cfg, pool[0], synth.make_weights(4000, B, C, s))
-        cpu = {kk: r[kk] for kk in ("value", "unit", "cores", "kind", "sample")}
+        cpu = {kk: r[kk] for kk in ("value", "unit", "cores", "kind", "sample", "cpu")}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,

@@ -1,0 +1,122 @@
+"""GPU parity in the bench's own launch configuration (BASELINE.json configs[3],
+c4): 64 concurrent 1280x720 -> 3840x2160 (x3) streams, 60-frame chunks, k = 5,
+in ONE ns_enhance_streams call -- distinct per-stream content-aware models,
+inputs in 64 distinct device buffers (8 generated contents, as bench.py lays
+them out), SR batched 16 anchors at a time across streams on two alternating SR
+streams, and every frame step one launch over all 64 streams.
+
+Checked against the oracle (same bars as tests/test_gpu_parity.py):
+  * the anchor map of every stream (bit-exact);
+  * SR on sampled windows -- both frame corners, res-block strip starts
+    (y = 240, 480) and a CTA x-seam -- of anchors of streams that land in
+    different SR batches (max-abs <= 2);
+  * reconstruction of whole 60-frame 4K chunks bit-exact given the GPU's anchor
+    bytes (two streams), and the first frames of two more streams that share
+    content with them but not weights.
+"""
+import multiprocessing as mp
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from helpers import oracle_sr_crops
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+ns = pytest.importorskip("paper_conf_sigcomm_yeolkjyh22_b200")
+
+DEV = "cuda:0"
+SR_MAX_ABS = 2
+S, P = 64, 8
+
+
+def _gen(seed):
+    cfg = synth.CONFIGS[4]
+    return synth.make_chunk(seed, cfg["w"], cfg["h"], cfg["scale"], cfg["n"],
+                            types=synth.default_types(cfg["n"], cfg["altref_every"]))
+
+
+@pytest.fixture(scope="module")
+def c4():
+    cfg = synth.CONFIGS[4]
+    B, C, s, n, k, h, w = (cfg[x] for x in ("n_blocks", "n_ch", "scale", "n", "k", "h", "w"))
+    seeds = [7400 + i for i in range(P)]
+    with mp.get_context("fork").Pool(min(P, os.cpu_count() or 1)) as pool:
+        pool_chunks = pool.map(_gen, seeds)
+    torch.cuda.empty_cache()
+    ctx = ns.Context(0, pool_bytes=12 << 30)
+    blobs = [synth.make_weights(7400 + si, B, C, s) for si in range(S)]
+    models = []
+    for si in range(S):
+        m = ctx.model(B, C, s)
+        m.set_weights(blobs[si])
+        models.append(m)
+    dev = torch.device(DEV)
+    lr_d = torch.empty((S, n, 3, h, w), dtype=torch.uint8, device=dev)
+    res_d = torch.empty((S, n, 3, h, w), dtype=torch.int16, device=dev)
+    mv_d = torch.empty((S, n, h // 8, w // 8, 8), dtype=torch.uint8, device=dev)
+    ty_d = torch.empty((S, n), dtype=torch.uint8, device=dev)
+    for si in range(S):
+        c = pool_chunks[si % P]
+        lr_d[si].copy_(torch.from_numpy(c.lr))
+        res_d[si].copy_(torch.from_numpy(c.res))
+        mv_d[si].copy_(torch.from_numpy(np.ascontiguousarray(c.mv).view(np.uint8).reshape(n, h // 8, w // 8, 8)))
+        ty_d[si].copy_(torch.from_numpy(c.type))
+    hr = torch.empty((S, n, 3, s * h, s * w), dtype=torch.uint8, device=dev)
+    state = torch.zeros((S, 2, 3, s * h, s * w), dtype=torch.uint8, device=dev)
+    chunks = [ns.DeviceChunk(w=w, h=h, scale=s, lr=lr_d[si], res=res_d[si], mv=mv_d[si], type=ty_d[si],
+                             model=models[si], hr_last=state[si, 0], hr_golden=state[si, 1])
+              for si in range(S)]
+    hr_out = [[hr[si, f] for f in range(n)] for si in range(S)]
+    ia = torch.zeros((S, n), dtype=torch.uint8, device=dev)
+    stats = torch.zeros((S, 8), dtype=torch.float64, device=dev)
+    ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, k=k)
+    torch.cuda.synchronize()
+    yield dict(cfg=cfg, pool=pool_chunks, blobs=blobs, hr=hr, ia=ia.cpu().numpy(), stats=stats.cpu().numpy())
+    del chunks, hr_out, hr, state, lr_d, res_d, mv_d, ty_d
+    ctx.close()
+    torch.cuda.empty_cache()
+
+
+def test_c4_selection_every_stream(c4):
+    n, k = c4["cfg"]["n"], c4["cfg"]["k"]
+    for p, c in enumerate(c4["pool"]):
+        _, _, exp = oracle.select_topk(list(c.type), [int(v) for v in oracle.score(c.res)], k)
+        for si in range(p, S, P):
+            assert list(c4["ia"][si]) == exp, si
+    assert c4["ia"].sum() == S * k
+    # stats: frames and anchors per stream (the bench's per-stream stats row)
+    assert np.all(c4["stats"][:, 0] == n) and np.all(c4["stats"][:, 1] == k)
+
+
+def test_c4_sr_windows_across_batches(c4):
+    cfg = c4["cfg"]
+    B, C, s, h, w = cfg["n_blocks"], cfg["n_ch"], cfg["scale"], cfg["h"], cfg["w"]
+    # 16 jobs per SR batch, stream by stream: streams 0, 21, 42, 63 land in batches 0, 6, 13, 19
+    wins = [(0, 0, 16, 24), (232, 240, 16, 24), (472, 500, 16, 24), (h - 16, w - 24, 16, 24)]
+    worst = 0
+    for si in (0, 21, 42, 63):
+        c = c4["pool"][si % P]
+        f = [f for f in range(cfg["n"]) if c4["ia"][si, f]][1]          # a non-KEY anchor
+        got = c4["hr"][si, f].cpu().numpy()
+        for (Y0, X0, HH, WW), patch in oracle_sr_crops(c.lr[f], c4["blobs"][si], B, C, s, wins):
+            d = np.abs(got[:, Y0:Y0 + HH, X0:X0 + WW].astype(int) - patch.astype(int))
+            worst = max(worst, int(d.max()))
+    assert worst <= SR_MAX_ABS, worst
+
+
+def test_c4_reconstruction_given_gpu_anchors(c4):
+    n = c4["cfg"]["n"]
+    for si, frames in ((0, n), (63, n), (8, 4), (47, 4)):
+        c = c4["pool"][si % P]
+        got = c4["hr"][si, :frames].cpu().numpy()
+        if frames < n:  # a prefix of the chunk: frames 0..frames-1 depend only on earlier frames
+            c = synth.Chunk(w=c.w, h=c.h, scale=c.scale, lr=c.lr[:frames], res=c.res[:frames], mv=c.mv[:frames],
+                            type=c.type[:frames].copy(), res_size=c.res_size[:frames])
+        z = np.zeros_like(got[0])
+        exp, _, _ = oracle.reconstruct(c, list(c4["ia"][si, :frames]), got, z, z)
+        assert np.array_equal(got, exp), si
