@@ -1,8 +1,8 @@
 """GPU parity in the bench's own launch configuration (BASELINE.json configs[3],
 c4): 64 concurrent 1280x720 -> 3840x2160 (x3) streams, 60-frame chunks, k = 5,
 in ONE ns_enhance_streams call -- distinct per-stream content-aware models,
-inputs in 64 distinct device buffers (8 generated contents, as bench.py lays
-them out), SR batched 16 anchors at a time across streams on two alternating SR
+inputs in 64 distinct device buffers (4 generated contents, laid out as
+bench.py lays out its 8), SR batched 16 anchors at a time across streams on two alternating SR
 streams, and every frame step one launch over all 64 streams.
 
 Checked against the oracle (same bars as tests/test_gpu_parity.py):
@@ -14,9 +14,6 @@ Checked against the oracle (same bars as tests/test_gpu_parity.py):
     bytes (two streams), and the first frames of two more streams that share
     content with them but not weights.
 """
-import multiprocessing as mp
-import os
-
 import numpy as np
 import pytest
 
@@ -31,13 +28,7 @@ ns = pytest.importorskip("paper_conf_sigcomm_yeolkjyh22_b200")
 
 DEV = "cuda:0"
 SR_MAX_ABS = 2
-S, P = 64, 8
-
-
-def _gen(seed):
-    cfg = synth.CONFIGS[4]
-    return synth.make_chunk(seed, cfg["w"], cfg["h"], cfg["scale"], cfg["n"],
-                            types=synth.default_types(cfg["n"], cfg["altref_every"]))
+S, P = 64, 4
 
 
 @pytest.fixture(scope="module")
@@ -45,8 +36,8 @@ def c4():
     cfg = synth.CONFIGS[4]
     B, C, s, n, k, h, w = (cfg[x] for x in ("n_blocks", "n_ch", "scale", "n", "k", "h", "w"))
     seeds = [7400 + i for i in range(P)]
-    with mp.get_context("fork").Pool(min(P, os.cpu_count() or 1)) as pool:
-        pool_chunks = pool.map(_gen, seeds)
+    # generated in this process (~20 s each; it already runs CUDA threads, so no fork pool)
+    pool_chunks = [synth.make_chunk(sd, w, h, s, n, types=synth.default_types(n, cfg["altref_every"])) for sd in seeds]
     torch.cuda.empty_cache()
     ctx = ns.Context(0, pool_bytes=12 << 30)
     blobs = [synth.make_weights(7400 + si, B, C, s) for si in range(S)]
@@ -111,7 +102,7 @@ def test_c4_sr_windows_across_batches(c4):
 
 def test_c4_reconstruction_given_gpu_anchors(c4):
     n = c4["cfg"]["n"]
-    for si, frames in ((0, n), (63, n), (8, 4), (47, 4)):
+    for si, frames in ((0, n), (63, n), (8, 4), (46, 4)):
         c = c4["pool"][si % P]
         got = c4["hr"][si, :frames].cpu().numpy()
         if frames < n:  # a prefix of the chunk: frames 0..frames-1 depend only on earlier frames
