@@ -456,10 +456,14 @@ def main():
         if fam in fl:
             a = fl[fam] / (tot / 1000.0) / 1e12
             ent.update(bound="tensor", achieved=a, unit="TFLOP/s", peak=pk["bf16_sus"], frac=a / pk["bf16_sus"])
-            if fam == "sr_up":  # executed work of the composed 5x5 conv (fewer FLOPs than defined)
+            if fam == "sr_up":
+                # the composed upsampler o shuffle o tail (one 5x5 conv at LR) executes fewer FLOPs than the
+                # two defined convs: its tensor utilisation is the executed work; the algorithmic rate is kept
+                # beside it (> 1 of peak by construction, not a utilisation)
                 ex = int(ia.sum()) * cfg["h"] * cfg["w"] * 2.0 * 25 * C * 3 * s * s
-                ent["executed_tflops"] = ex / (tot / 1000.0) / 1e12
-                ent["executed_frac"] = ent["executed_tflops"] / pk["bf16_sus"]
+                e_tf = ex / (tot / 1000.0) / 1e12
+                ent.update(achieved=e_tf, frac=e_tf / pk["bf16_sus"], work="executed FLOPs of the composed 5x5 conv",
+                           algorithmic_tflops=a, algorithmic_frac=a / pk["bf16_sus"])
         elif fam in by:
             a = by[fam] / (tot / 1000.0) / 1e9
             ent.update(bound="hbm", achieved=a, unit="GB/s", peak=pk["hbm"], frac=a / pk["hbm"])
@@ -578,7 +582,9 @@ def main():
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
-                             "anchors_per_step": int(ia_np.sum())},
+                             "anchors_per_step": int(ia_np.sum()),
+                             "work": "algorithmic FLOPs of the defined convs over the summed SR family times "
+                                     "(the families overlap on two SR streams)"},
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
                 "host_enqueue_ms_per_step": host_ms, "step_ms": [round(x, 3) for x in step_ms],
                 "e2e_package": e2e_pkg,
