@@ -179,24 +179,25 @@ __device__ __forceinline__ void recon_row_stage(const uint8_t *row, int xs, int 
 // window replicate the edge pixel into the words that lie outside the row
 // (first word at xb).  (on = false: a KEY-frame / INTRA thread, whose warp
 // weights are all 0 and whose slots hold LR rows in flight: nothing is read,
-// so no shared-memory race.)
+// so no shared-memory race.)  wfix is warp-uniform (some lane's window leaves
+// the row): the replication is one byte permute per half-word with the
+// selector chosen per word -- identity inside the row, byte 0 (the row's first
+// pixel) left of it, byte 7 (its last) right of it -- so the row body carries
+// 2 NQ permutes behind one uniform branch instead of per-word branches (the
+// recon loop is instruction-cache sensitive: DESIGN.md §7).
 template <int S, bool CH>
-__device__ __forceinline__ void recon_load_row(const uint2 *row, bool on, bool fix, int xb, int W,
+__device__ __forceinline__ void recon_load_row(const uint2 *row, bool on, bool wfix, int xb, int W,
                                                uint2 (&q)[ReconCfg<S, CH>::NQ]) {
     using Cfg = ReconCfg<S, CH>;
 #pragma unroll
     for (int i = 0; i < Cfg::NQ; i++) q[i] = on ? row[i * kReconNT] : make_uint2(0u, 0u);
-    if (fix) {
+    if (wfix) {
 #pragma unroll
         for (int i = 0; i < Cfg::NQ; i++) {
             const int st = xb + 8 * i;
-            if (st < 0) {
-                const uint32_t v = prmt(q[i].x, 0u, 0x0000u);
-                q[i] = make_uint2(v, v);
-            } else if (st >= W) {
-                const uint32_t v = prmt(q[i].y, 0u, 0x3333u);
-                q[i] = make_uint2(v, v);
-            }
+            const uint32_t sx = st < 0 ? 0x0000u : (st >= W ? 0x7777u : 0x3210u);
+            const uint32_t sy = st < 0 ? 0x0000u : (st >= W ? 0x7777u : 0x7654u);
+            q[i] = make_uint2(prmt(q[i].x, q[i].y, sx), prmt(q[i].x, q[i].y, sy));
         }
     }
 }
@@ -547,7 +548,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
     }
     const bool left_in = bx > 0, right_in = LRB * bx + LRB < pw;
     const int m = xs & 7;
-    const bool fix = valid && !interior && !use_lr;
+    const bool wfix = __any_sync(0xffffffffu, valid && !interior && !use_lr);  // warp-uniform
     uint8_t *outp = fd.out + hr0 + (size_t)Y0 * W + X0;
     // combine (see the top of this file): luma X = 64 (r + 256) + 8h0 (8-fy) + 8h1 fy + 32,
     // chroma X = 16 (r + 256) + h0 (16-fy) + h1 fy + 8; floor(X / 2^SH) = pred + r + 256
@@ -569,7 +570,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
         uint32_t hA[NP], hB[NP];   // warp rows j (prev) and j + 1 (cur), ping-pong by row parity
         {
             uint2 q[NQ];
-            recon_load_row<S, CH>(wbuf, !use_lr, fix, xs & ~7, W, q);
+            recon_load_row<S, CH>(wbuf, !use_lr, wfix, xs & ~7, W, q);
             recon_hpass<S, CH>(q, m, fxc, fx, hA);
         }
         stage_row(c + 1, 0);
@@ -592,7 +593,7 @@ __global__ void __launch_bounds__(kReconNT, ReconCfg<S, CH>::MINB)
                 uint32_t(&hc)[NP] = (jj & 1) ? hA : hB;
                 asm volatile("cp.async.wait_group %0;" ::"n"(RPT) : "memory");
                 uint2 q[NQ];
-                recon_load_row<S, CH>(wbuf + (j + 1) * NQ * kReconNT, !use_lr, fix, xs & ~7, W, q);
+                recon_load_row<S, CH>(wbuf + (j + 1) * NQ * kReconNT, !use_lr, wfix, xs & ~7, W, q);
                 uint32_t u[NP], x[NP], o[Cfg::BW / 4];
                 recon_up_row<S, CH, tap_w1<S>(jj)>(rv[ta], rv[ta + 1], u);   // independent of q: covers the load
                 recon_hpass<S, CH>(q, m, fxc, fx, hc);
