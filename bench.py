@@ -279,7 +279,8 @@ def main():
     ap.add_argument("--distinct", type=int, default=8, help="distinct generated streams (replicated on device)")
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--sr-batch", type=int, default=int(os.environ.get("NS_SR_BATCH", "16")))
+    ap.add_argument("--sr-batch", type=int, default=int(os.environ.get("NS_SR_BATCH", "0")),
+                    help="anchors per SR batch (pool sizing; the library reads NS_SR_BATCH); 0 = per frame shape")
     ap.add_argument("--balance", action="store_true",
                     help="with --select global: anchor-level load balancing across GPUs (shard.plan_anchor_moves; "
                          "LR out / HR back point-to-point), then ns_sr_anchors + ns_reconstruct_chunk")
@@ -332,7 +333,8 @@ def main():
 
     host_pool = ns.Context.host_pool_bytes(w, h, n, k, S) if args.e2e_steps > 0 else 0
     # two SR arenas: batches alternate between two streams (ns_api.cu run_sr_group)
-    ctx = ns.Context(local, pool_bytes=int((2.4 * ns_arena_gb(cfg, args.sr_batch, args.format) + 2) * (1 << 30)) +
+    nb = sr_jobs(h, w, torch.cuda.get_device_properties(dev).multi_processor_count, args.sr_batch)
+    ctx = ns.Context(local, pool_bytes=int((2.4 * ns_arena_gb(cfg, nb, args.format) + 2) * (1 << 30)) +
                      host_pool)
     # per-stream content-aware models: distinct weights per stream
     models = []
@@ -578,7 +580,7 @@ def main():
                         f"random-init per-stream weights of the NAS 'high' architecture)",
                 "config": dict(workload_config(cfg, world, args.select, args.format, args.interp),
                                balance=bool(args.balance), transport=args.transport if args.balance else None,
-                               l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=args.sr_batch,
+                               l2="inputs larger than L2 (~130 GB touched per step)", sr_batch=nb,
                                gen_s=round(t_gen, 1)),
                 "roofline": roofline, "rooflines": rl,
                 "sr_total": {"ms_per_step": sr_ms, "achieved_tflops": sr_tf, "frac": sr_tf / pk["bf16_sus"],
@@ -682,7 +684,8 @@ def run_c5(args):
     S = len(mine)
     # pool: SR arenas (two per shape) + the anchor cache (k anchors per stream)
     acache = sum(len(v) * k * 3 * (s * w) * (s * h) for (w, h), v in by_shape.items())
-    arenas = sum(2.4 * ns_arena_gb(dict(cfg, w=w, h=h), args.sr_batch) for (w, h) in shapes)
+    sms = torch.cuda.get_device_properties(dev).multi_processor_count
+    arenas = sum(2.4 * ns_arena_gb(dict(cfg, w=w, h=h), sr_jobs(h, w, sms, args.sr_batch)) for (w, h) in shapes)
     ctx = ns.Context(local, pool_bytes=int((arenas + 2) * (1 << 30)) + acache + (256 << 20))
     chunks, rows, hr_bufs, states = [], [], [], []
     for (w, h) in shapes:
@@ -766,6 +769,15 @@ def run_c5(args):
     ctx.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def sr_jobs(h, w, sms, fixed=None):
+    """Anchors per SR batch of one frame shape, as the library picks them
+    (csrc/k_sr.cu sr_batch_jobs): about two waves of the fused residual block."""
+    if fixed:
+        return fixed
+    per_job = -(-h // 240) * ((-(-w // 126) + 1) // 2)
+    return min(64, max(16, 2 * sms // max(per_job, 1)))
 
 
 def ns_arena_gb(cfg, nb, fmt="444"):

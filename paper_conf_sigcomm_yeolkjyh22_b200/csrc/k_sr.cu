@@ -1699,6 +1699,17 @@ static cudaError_t uptail(const CUtensorMap &tm, ConvArgs args, int nj, cudaStre
 // 288 CTAs per 16-job launch, 1.95 waves of 148 SMs, so a launch that runs
 // alone (no overlap) wastes little as well: 240.
 constexpr int kRbRows = 240;  // rows per CTA strip of the fused res-block
+
+// Jobs (anchors) per SR batch of one frame shape: about two waves of the fused
+// residual block, the dominant SR kernel (one CTA per SM; ceil(h / kRbRows)
+// strips x ceil(tiles / 2) CTAs per job) -- 16 at 720p (18 CTAs per job, 288
+// per launch on 148 SMs), 49 at 360p (6 per job) instead of a fixed 16, whose
+// 96-CTA launches left a third of the GPU idle on c5's 360p half -- clamped to
+// [16, 64] (arena memory).
+int sr_batch_jobs(int h, int w, int sms) {
+    const int per_job = ((h + kRbRows - 1) / kRbRows) * ((((w + kRbOut - 1) / kRbOut) + 1) / 2);
+    return std::min(64, std::max(16, 2 * sms / std::max(per_job, 1)));
+}
 template <int C>
 static cudaError_t resblock(const CUtensorMap &tm, const RbArgs &args0, int nj, cudaStream_t st) {
     using Cfg = RbCfg<C>;

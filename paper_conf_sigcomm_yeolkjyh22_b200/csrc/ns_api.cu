@@ -166,10 +166,12 @@ static int overlap_parts_default() {
     return v > 0 ? v : 1;
 }
 
+// anchors per SR batch: 0 = per frame shape (sr_batch_jobs); NS_SR_BATCH in the
+// environment fixes it (tuning experiments only)
 static int sr_batch_default() {
     const char *e = getenv("NS_SR_BATCH");
     const int v = e ? atoi(e) : 0;
-    return v > 0 ? v : 16;
+    return v > 0 ? v : 0;
 }
 
 struct ArenaEntry {
@@ -207,7 +209,7 @@ struct ns_ctx {
     SrJob *jobs;
     uint16_t *blob_stage;  // device staging for host weight blobs
     size_t blob_stage_elems;
-    int sr_batch = sr_batch_default();  // anchors per SR batch (arena size)
+    int sr_batch = sr_batch_default();  // anchors per SR batch (arena size); 0 = per shape
     std::deque<ArenaEntry> arenas;   // deque: entries never move
     // host-input path (ns_enhance_streams_host): copy stream, two input staging
     // buffers (group ping-pong) and the anchor-LR gather staging, carved from
@@ -758,13 +760,24 @@ extern "C" ns_status ns_select_merge(ns_ctx *c, int S, int n, const int64_t *gai
 }
 
 // ------------------------------------------------------------------ SR
-static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int fmt, int idx, const SrArena **out) {
+// idx 0: the shape's first arena, sized for sr_batch_jobs (halved down to 16 if
+// the pool cannot hold two of that size); idx 1: the second, with the first one's job count
+// (batches alternate between them), or none if the pool has no room for it.
+static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int fmt, int idx, int nb_req, const SrArena **out) {
     for (auto &e : c->arenas)
         if (e.h == h && e.w == w && e.C == C && e.s == s && e.fmt == fmt && e.idx == idx) {
             *out = &e.a;
             return NS_OK;
         }
-    const size_t bytes = sr_arena_bytes(h, w, C, s, c->sr_batch, fmt);
+    int nb = nb_req;
+    if (idx == 0) {
+        int dev = 0, sms = 148;
+        if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        nb = c->sr_batch > 0 ? c->sr_batch : sr_batch_jobs(h, w, sms);
+        // (room for both arenas, so batches keep alternating between two streams)
+        while (nb > 16 && c->used + 2 * sr_arena_bytes(h, w, C, s, nb, fmt) + 512 > c->pool_bytes) nb = std::max(16, nb / 2);
+    }
+    const size_t bytes = sr_arena_bytes(h, w, C, s, nb, fmt);
     if (idx > 0 && c->used + bytes + 256 > c->pool_bytes) {  // no room for a second arena: one stream
         *out = nullptr;
         return NS_OK;
@@ -772,9 +785,9 @@ static ns_status get_arena(ns_ctx *c, int h, int w, int C, int s, int fmt, int i
     uint8_t *mem = pool_take(c, bytes);
     if (!mem)
         return fail(NS_ENOMEM, "SR arena for %dx%d C%d x%d (%d jobs) needs %zu bytes; pool has %zu free", w, h, C, s,
-                    c->sr_batch, bytes, c->pool_bytes - c->used);
+                    nb, bytes, c->pool_bytes - c->used);
     ArenaEntry e{h, w, C, s, fmt, idx, {}};
-    if (sr_arena_init(&e.a, h, w, C, s, c->sr_batch, fmt, mem) != 0)
+    if (sr_arena_init(&e.a, h, w, C, s, nb, fmt, mem) != 0)
         return fail(NS_ECUDA, "cuTensorMapEncodeTiled failed for the SR arena");
     c->arenas.push_back(e);
     *out = &c->arenas.back().a;
@@ -790,10 +803,10 @@ static ns_status run_sr_group(ns_ctx *c, const GroupKey &key, const SrJob *d_job
     int h, w, C, s, B, fmt;
     std::tie(h, w, C, s, B, fmt) = key;
     const SrArena *a[2] = {nullptr, nullptr};
-    ns_status r = get_arena(c, h, w, C, s, fmt, 0, &a[0]);
+    ns_status r = get_arena(c, h, w, C, s, fmt, 0, 0, &a[0]);
     if (r != NS_OK) return r;
     const int nbatch = (max_jobs + a[0]->nb - 1) / a[0]->nb;
-    if (nbatch > 1 && (r = get_arena(c, h, w, C, s, fmt, 1, &a[1])) != NS_OK) return r;
+    if (nbatch > 1 && (r = get_arena(c, h, w, C, s, fmt, 1, a[0]->nb, &a[1])) != NS_OK) return r;
     const bool two = a[1] != nullptr;
     if (two) {
         NS_CUDA(cudaEventRecord(c->ev_fork, st));
@@ -840,8 +853,8 @@ extern "C" ns_status ns_sr_anchors(ns_ctx *c, const ns_sr_job *jobs, int n_jobs,
         int h, w, C, s, B, fmt;
         std::tie(h, w, C, s, B, fmt) = kv.first;
         const SrArena *a0 = nullptr, *a1 = nullptr;
-        if ((r = get_arena(c, h, w, C, s, fmt, 0, &a0)) != NS_OK) return r;
-        if ((int)kv.second.size() > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, &a1)) != NS_OK) return r;
+        if ((r = get_arena(c, h, w, C, s, fmt, 0, 0, &a0)) != NS_OK) return r;
+        if ((int)kv.second.size() > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, a0->nb, &a1)) != NS_OK) return r;
     }
     for (auto &kv : groups) {
         const auto &idx = kv.second;
@@ -995,8 +1008,8 @@ static ns_status enhance_impl(ns_ctx *c, const ns_chunk *ch, int S, int n, const
             int h, w, C, s, B, fmt;
             std::tie(h, w, C, s, B, fmt) = gkey[gi];
             const SrArena *a0 = nullptr, *a1 = nullptr;
-            if ((r = get_arena(c, h, w, C, s, fmt, 0, &a0)) != NS_OK) return r;
-            if (gcount[gi] > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, &a1)) != NS_OK) return r;
+            if ((r = get_arena(c, h, w, C, s, fmt, 0, 0, &a0)) != NS_OK) return r;
+            if (gcount[gi] > a0->nb && (r = get_arena(c, h, w, C, s, fmt, 1, a0->nb, &a1)) != NS_OK) return r;
         }
     const bool any_ring = std::find(ring.begin(), ring.end(), 1) != ring.end();
     std::vector<uint8_t *> acache(S, nullptr);

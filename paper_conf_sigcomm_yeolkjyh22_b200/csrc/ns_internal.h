@@ -175,6 +175,7 @@ struct SrArena {
     CUtensorMap tm_x0, tm_h0, tm_hb, tm_tb, tm_tb5, tm_hb5;   // *5: 132-px boxes (5x5 conv)
     CUtensorMap tm_lr8;                // box: kLrBoxW px x 3 planes x 3 rows
 };
+int sr_batch_jobs(int h, int w, int sms);  // jobs per SR batch of one shape (k_sr.cu)
 size_t sr_arena_bytes(int h, int w, int C, int s, int nb, int fmt);
 int sr_arena_init(SrArena *a, int h, int w, int C, int s, int nb, int fmt, uint8_t *mem);  // 0 ok
 // Runs the whole net on jobs [j0, j0+nj) of a device job table (all of one
