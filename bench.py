@@ -384,10 +384,17 @@ def main():
                 m.set_weights(synth.make_weights(4000 + r * 100000 + si, B, C, s))
                 models_all[r * S + si] = m
 
+    # the global selection's per-stream rows, built once (no host->device copy or
+    # host synchronisation inside a step)
+    sid_d = torch.tensor(sids, dtype=torch.int32, device=dev)
+    cost_d = torch.tensor(cost, dtype=torch.int64, device=dev)
+    shape_d = torch.tensor([[w, h, s]] * S, dtype=torch.int32, device=dev)
+    counts = shard.row_counts(S, dev) if args.select == "global" else None
+
     def step():
         if args.select == "global" and args.balance:
-            anc, _, allr = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream,
-                                                            return_all=True)
+            anc, _, allr = shard.select_global_across_ranks(ctx, chunks, sid_d, cost_d, budget, stream=stream,
+                                                            return_all=True, shape=shape_d, counts=counts)
             anc_h = allr["anchor"].cpu().numpy()
             sid_h = allr["sid"].cpu().tolist()
             anchors_all = [[int(f) for f in np.nonzero(anc_h[i])[0]] for i in range(len(sid_h))]
@@ -396,7 +403,8 @@ def main():
                                               shape_all=allr["shape"].cpu().tolist(), transport=args.transport)
             ia.copy_(anc)
         elif args.select == "global":
-            anc, _ = shard.select_global_across_ranks(ctx, chunks, sids, cost, budget, stream=stream)
+            anc, _ = shard.select_global_across_ranks(ctx, chunks, sid_d, cost_d, budget, stream=stream,
+                                                      shape=shape_d, counts=counts)
             ctx.enhance_streams(chunks, hr_out, is_anchor_out=ia, stats=stats, stream=stream,
                                 mode=ns.NS_GIVEN_ANCHORS, anchor_in=anc, cost=cost, budget=budget)
         else:

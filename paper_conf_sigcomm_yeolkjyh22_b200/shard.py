@@ -73,22 +73,23 @@ def gather_stats(stats, group=None):
 
 
 # ---------------------------------------------------------------- NEXT-1: global selection across GPUs
-def gather_rows(tensors, group=None):
+def gather_rows(tensors, group=None, counts=None):
     """all_gather of per-rank tensors whose first dimension (streams) differs
     between ranks: every tensor is padded to the largest S_r, gathered, and the
     valid rows concatenated rank-major.  Returns (gathered tensors, row offset
     of this rank).  One small exchange per chunk (<= 30k
-    entries); NCCL on GPUs, gloo on CPU.  Data movement only."""
+    entries); NCCL on GPUs, gloo on CPU.  Data movement only.  counts: every
+    rank's row count when the caller already knows them (they are fixed for a
+    run): skips the count exchange and its host synchronisation."""
     import torch
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
         return list(tensors), 0
     world, me = dist.get_world_size(group), dist.get_rank(group)
     dev = tensors[0].device
-    cnt = torch.tensor([tensors[0].shape[0]], dtype=torch.int64, device=dev)
-    cnts = [torch.zeros_like(cnt) for _ in range(world)]
-    dist.all_gather(cnts, cnt, group=group)
-    cnts = [int(c.item()) for c in cnts]
+    if counts is None:
+        counts = row_counts(tensors[0].shape[0], dev, group)
+    cnts = list(counts)
     smax = max(cnts)
     out = []
     for t in tensors:
@@ -100,8 +101,21 @@ def gather_rows(tensors, group=None):
     return out, sum(cnts[:me])
 
 
+def row_counts(S, device, group=None):
+    """Every rank's stream count (one all_gather; host-synchronising): compute
+    once per run and pass to gather_rows / select_global_across_ranks."""
+    import torch
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return [int(S)]
+    cnt = torch.tensor([int(S)], dtype=torch.int64, device=device)
+    cnts = [torch.zeros_like(cnt) for _ in range(dist.get_world_size(group))]
+    dist.all_gather(cnts, cnt, group=group)
+    return [int(c.item()) for c in cnts]
+
+
 def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_res_size=False, group=None,
-                               stream=None, return_all=False, n=None, device=None):
+                               stream=None, return_all=False, n=None, device=None, shape=None, counts=None):
     """§5.2 global anchor selection over the streams of every GPU:
     (1) per-stream gains and ranks on this GPU (ns_select_anchors, Alg. 1);
     (2) all_gather of gain / rank / type / sid / cost rows (gather_rows);
@@ -110,7 +124,10 @@ def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_
     [S_local, n] (device u8) for ns_enhance_streams(mode=NS_GIVEN_ANCHORS,
     anchor_in=..., cost=cost, budget=budget), and the global rank rows.
     A rank may own no streams (chunks == []): it then passes n and device, and
-    still takes part in the gather and the merge."""
+    still takes part in the gather and the merge.  sid / cost may be lists or
+    device tensors, shape an [S, 3] device tensor of (w, h, scale), counts the
+    ranks' stream counts (row_counts): a caller that passes them once-built
+    keeps every host->device copy and host synchronisation out of its steps."""
     import torch
     from . import NS_TOPK_PER_STREAM
     S = len(chunks)
@@ -125,13 +142,15 @@ def select_global_across_ranks(ctx, chunks, sid, cost, budget, fresh=False, use_
         types = torch.stack([c.type for c in chunks])
     else:
         types = torch.zeros((0, n), dtype=torch.uint8, device=dev)
-    sid_t = torch.as_tensor(list(sid), dtype=torch.int32).reshape(-1).to(dev)
-    cost_t = torch.as_tensor(list(cost), dtype=torch.int64).reshape(-1).to(dev)
+    sid_t = sid if isinstance(sid, torch.Tensor) else torch.as_tensor(list(sid), dtype=torch.int32).reshape(-1).to(dev)
+    cost_t = (cost if isinstance(cost, torch.Tensor) else
+              torch.as_tensor(list(cost), dtype=torch.int64).reshape(-1).to(dev))
     # (w, h, scale) of every row: the anchor exchange sizes each moved frame by
     # its own stream's shape (mixed-resolution fleets)
-    shape_t = torch.as_tensor([[c.w, c.h, c.scale] for c in chunks], dtype=torch.int32).reshape(-1, 3).to(dev)
+    shape_t = shape if shape is not None else torch.as_tensor(
+        [[c.w, c.h, c.scale] for c in chunks], dtype=torch.int32).reshape(-1, 3).to(dev)
     (g_all, r_all, t_all, s_all, c_all, sh_all), off = gather_rows([gain, rank, types, sid_t, cost_t, shape_t],
-                                                                   group)
+                                                                   group, counts)
     rank_out = torch.empty_like(r_all)
     anc_all = torch.empty_like(t_all)
     ctx.select_merge(g_all, r_all, t_all, s_all, c_all, budget, rank_out, anc_all, stream=stream)
